@@ -1,0 +1,82 @@
+// kernels.h -- internal launcher declarations shared by the .cu kernel files and the
+// host driver (rgsqr.cpp).  Not part of the public C-ABI (include/rgsqr.h).
+#pragma once
+#include <cstddef>
+#include <cstdint>
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+namespace rg {
+
+// ---- scale.cu (section 3.5)
+cudaError_t launch_colnorm(const float* A, int64_t lda, int64_t m, int n, double* partial, double* norm2,
+                           cudaStream_t st);
+cudaError_t launch_colscale(const double* norm2, int n, int do_scale, float* scale, int* status, int col0,
+                            cudaStream_t st);
+size_t colnorm_partial_doubles(int64_t m, int n);
+cudaError_t launch_scale_cast(const float* A, int64_t lda, float* Q, int64_t ldq, uint16_t* Qh, uint16_t* Ql,
+                              int64_t ldh, int64_t m, int n, const float* scale, int bf16, cudaStream_t st);
+cudaError_t launch_unscale_r(float* R, int64_t ldr, int n, const float* scale, cudaStream_t st);
+
+// ---- panel.cu (eq 8 + Alg 2)
+struct PanelLaunch {
+    float* Q;
+    int64_t ldq;
+    uint16_t* Qh;
+    uint16_t* Ql;
+    int64_t ldh;
+    int64_t m;
+    int nc;
+    float* R;
+    int64_t ldr;
+    float* ws;
+    int* counters;
+    int distributed;
+    int bf16;
+    int col0;
+    int* status;
+};
+int panel_levels(int ntiles, int* lvl_n);
+size_t panel_ws_floats(int64_t m);
+size_t panel_counters(int64_t m);
+cudaError_t launch_panel(const PanelLaunch& pl, cudaStream_t st);
+cudaError_t launch_panel_apply(const PanelLaunch& pl, const float* Gq, cudaStream_t st);
+cudaError_t launch_panel_stack(const float* Rall, int P, int nc, float* R, int64_t ldr, float* Qblocks, int* status,
+                               int col0, cudaStream_t st);
+
+// ---- gemm_tc.cu (Alg 1 lines 8-9 on tcgen05)
+cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int splits, const CUtensorMap& q1,
+                             const CUtensorMap& a2, const CUtensorMap& q1_lo, const CUtensorMap& a2_lo, float* P,
+                             int64_t ldp, int64_t p_stride, int kb_total, int kb_per_split, int bf16,
+                             cudaStream_t st);
+cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, const CUtensorMap& q1_mn,
+                               const CUtensorMap& r12, const CUtensorMap& q1_mn_lo, const CUtensorMap& r12_lo,
+                               float* C, int64_t ldc, void* Ch, void* Cl, int64_t ldh, int bf16, cudaStream_t st);
+cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, int splits, int h, int w, float* R,
+                               int64_t ldr, float* Rf, int64_t ldf, uint16_t* Rh, uint16_t* Rl, int64_t ldh, int bf16,
+                               cudaStream_t st);
+cudaError_t launch_proj_finish(const float* Rf, int64_t ldf, int h, int w, float* R, int64_t ldr, uint16_t* Rh,
+                               uint16_t* Rl, int64_t ldh, int bf16, cudaStream_t st);
+
+// ---- blas.cu (CGLS vectors, triangular inverse, small products)
+cudaError_t launch_gemv_n(const float* A, int64_t lda, int64_t m, int n, const double* x, double* y, double* work,
+                          cudaStream_t st);
+size_t gemv_n_work_doubles(int64_t m, int n);
+cudaError_t launch_gemv_t(const float* A, int64_t lda, int64_t m, int n, const double* r, double* s, double* work,
+                          cudaStream_t st);
+size_t gemv_t_work_doubles(int64_t m, int n);
+cudaError_t launch_trinv_upper(const float* R, int64_t ldr, int n, double* Rinv, cudaStream_t st);
+cudaError_t launch_trmv(const double* Rinv, int n, const double* x, double* y, int transpose, cudaStream_t st);
+cudaError_t launch_cgls_init(const float* b, int64_t m, int n, double* r, double* x, cudaStream_t st);
+cudaError_t launch_sqnorm(const double* v, int64_t len, double* sc, int idx, cudaStream_t st);
+cudaError_t launch_cgls_xr(double* x, const double* t, double* r, const double* q, int64_t m, int n, double* sc,
+                           cudaStream_t st);
+cudaError_t launch_cgls_p(const double* s, double* p, int n, double* sc, int first, cudaStream_t st);
+cudaError_t launch_gaussian_philox(int64_t total, uint64_t seed, double* out64, float* out32, cudaStream_t st);
+size_t probe_work_doubles(int64_t m, int n, int p);
+cudaError_t launch_orth_probe(const float* Q, int64_t ldq, int64_t m, int n, const double* G, double* work,
+                              double* out, cudaStream_t st);
+cudaError_t launch_trmm_upper(const float* A, int64_t lda, const float* B, int64_t ldb, float* C, int64_t ldc, int n,
+                              cudaStream_t st);
+
+}  // namespace rg

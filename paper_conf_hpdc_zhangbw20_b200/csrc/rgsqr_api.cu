@@ -1,0 +1,737 @@
+// rgsqr_api.cu -- host driver and C-ABI (include/rgsqr.h) of the B200 RGSQR library.
+//
+// rgsqr_factor runs Algorithm 1 as a static, depth-first plan:
+//   colnorm -> colscale -> scale/cast (section 3.5)
+//   for each node of the recursion tree (left to right):
+//     leaf   : panel (eq 8 + Alg 2, fp32)                               [+ allgather/stack]
+//     inner  : K1 R12 = Q1^T A2 (tcgen05, split-K) -> reduce -> R, R12h   [+ allreduce]
+//              K2 A2 -= Q1 R12 (tcgen05, fused fp32 RMW + 16-bit shadow)
+//   unscale R (R <- R P^{-1}, exact)
+// The plan (tensor maps, grid shapes, split factors) is built once per (shape, pointers,
+// options) and captured into a CUDA graph, so a call is one graph launch.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <climits>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../../include/rgsqr.h"
+#include "kernels.h"
+
+// ------------------------------------------------------------------ NCCL (dlopen)
+typedef struct ncclComm* ncclComm_t;
+typedef struct {
+    char internal[128];
+} ncclUniqueId;
+typedef enum { ncclSuccess = 0 } ncclResult_t;
+typedef enum { ncclInt8 = 0, ncclFloat32 = 7, ncclFloat64 = 8 } ncclDataType_t;
+typedef enum { ncclSum = 0 } ncclRedOp_t;
+
+namespace {
+struct NcclApi {
+    void* lib = nullptr;
+    ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                              cudaStream_t) = nullptr;
+    ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+};
+NcclApi g_nccl;
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn g_encode = nullptr;
+
+int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+
+int rgsqr_split(int64_t n) {  // reading #1: h = roundup(n/2, 32), clamped
+    int64_t h = ((n / 2) + 31) / 32 * 32;
+    if (h >= n) h = n / 2;
+    if (h < 1) h = 1;
+    return (int)h;
+}
+
+bool encode_map(CUtensorMap* map, const void* base, int64_t inner, int64_t outer, int64_t ld_elems, int box_inner,
+                int box_outer, bool bf16) {
+    if (!g_encode) return false;
+    cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld_elems * 2)};
+    cuuint32_t box[2] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = g_encode(map, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2,
+                          const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                          CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+int pick_bn(int w) { return w <= 32 ? 32 : w <= 64 ? 64 : w <= 128 ? 128 : 256; }
+
+enum ProfClass { PC_UPDATE = 0, PC_PROJ = 1, PC_PANEL = 2, PC_SCALE = 3, PC_CGLS = 4, PC_OTHER = 5, PC_N = 6 };
+
+}  // namespace
+
+// ------------------------------------------------------------------ device buffers
+static int g_alloc_epoch = 0;  // bumped whenever any workspace buffer moves (plans/graphs embed addresses)
+
+struct DevBuf {
+    void* p = nullptr;
+    size_t bytes = 0;
+    bool ensure(size_t b) {
+        if (b <= bytes) return true;
+        ++g_alloc_epoch;
+        if (p) cudaFree(p);
+        p = nullptr;
+        bytes = 0;
+        if (cudaMalloc(&p, b) != cudaSuccess) return false;
+        bytes = b;
+        return true;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        bytes = 0;
+    }
+    template <class T>
+    T* as() const {
+        return reinterpret_cast<T*>(p);
+    }
+};
+
+struct Op {
+    enum Kind { PANEL, PROJ, UPDATE } kind;
+    int c0, h, w;  // PANEL: c0, w = columns.  PROJ/UPDATE: Q1 = [c0, c0+h), A2 = [c0+h, c0+h+w)
+    int bn = 0, tiles_i = 0, tiles_j = 0, splits = 0, kb_total = 0, kb_per_split = 0;
+    CUtensorMap ma, mb, ma_lo, mb_lo;
+};
+
+struct Plan {
+    // key
+    int64_t m = 0, n = 0, lda = 0, ldq = 0, ldr = 0;
+    const float* A = nullptr;
+    float* Q = nullptr;
+    float* R = nullptr;
+    int nb = 0, bf16 = 0, split = 0, scale = 1, nranks = 1, rank = 0;
+    int epoch = -1;          // g_alloc_epoch the plan was built against
+    // derived
+    int64_t ldh = 0, ldr12 = 0;
+    std::vector<Op> ops;
+    size_t p_floats = 0;
+    cudaGraphExec_t exec = nullptr;
+};
+
+struct rg_handle_s {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    cudaStream_t capture_stream = nullptr;  // private stream used only to capture plans into graphs
+    ncclComm_t comm = nullptr;
+    int rank = 0, nranks = 1;
+    int64_t last_info = -1;
+    // workspace
+    DevBuf qh, ql, P, r12h, r12l, r12f, partial, norm2, scale, status, pws, pcnt, rgather, rstackq;
+    DevBuf stageA, stageQ, stageR, stageB, stageX;  // host-pointer staging
+    DevBuf cg;                                      // CGLS vectors
+    DevBuf aux;                                     // misc (orthogonalize / lowrank)
+    int* status_host = nullptr;                     // pinned
+    int ws_generation = 0;
+    std::unique_ptr<Plan> plan;
+    // profiling
+    bool prof = false;
+    double prof_ms[PC_N] = {0};
+    int64_t prof_launches[PC_N] = {0};
+    double prof_flops[PC_N] = {0};
+    double prof_bytes[PC_N] = {0};
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> ev_pool;
+    struct PendingEv {
+        int cls;
+        cudaEvent_t a, b;
+        double flops, bytes;
+    };
+    std::vector<PendingEv> pending;
+    size_t ev_next = 0;
+};
+
+namespace {
+
+#define RG_CUDA(x)                                                                   \
+    do {                                                                             \
+        cudaError_t _e = (x);                                                        \
+        if (_e != cudaSuccess) {                                                     \
+            fprintf(stderr, "[rgsqr] CUDA error %s at %s:%d: %s\n", cudaGetErrorName(_e), __FILE__, __LINE__, \
+                    cudaGetErrorString(_e));                                         \
+            return RG_CUDA_ERROR;                                                    \
+        }                                                                            \
+    } while (0)
+
+// profiling brackets ------------------------------------------------------------
+struct ProfScope {
+    rg_handle h;
+    int cls;
+    double flops, bytes;
+    cudaEvent_t b = nullptr, e = nullptr;
+    ProfScope(rg_handle h_, int cls_, double flops_ = 0, double bytes_ = 0)
+        : h(h_), cls(cls_), flops(flops_), bytes(bytes_) {
+        if (!h->prof) return;
+        if (h->ev_next >= h->ev_pool.size()) {
+            cudaEvent_t x, y;
+            cudaEventCreate(&x);
+            cudaEventCreate(&y);
+            h->ev_pool.push_back({x, y});
+        }
+        b = h->ev_pool[h->ev_next].first;
+        e = h->ev_pool[h->ev_next].second;
+        h->ev_next++;
+        cudaEventRecord(b, h->stream);
+    }
+    ~ProfScope() {
+        if (!h->prof) return;
+        cudaEventRecord(e, h->stream);
+        h->pending.push_back({cls, b, e, flops, bytes});
+    }
+};
+
+void prof_collect(rg_handle h) {
+    if (!h->prof || h->pending.empty()) return;
+    cudaStreamSynchronize(h->stream);
+    for (auto& p : h->pending) {
+        float ms = 0;
+        cudaEventElapsedTime(&ms, p.a, p.b);
+        h->prof_ms[p.cls] += ms;
+        h->prof_launches[p.cls] += 1;
+        h->prof_flops[p.cls] += p.flops;
+        h->prof_bytes[p.cls] += p.bytes;
+    }
+    h->pending.clear();
+    h->ev_next = 0;
+}
+
+bool ensure_encode() {
+    if (g_encode) return true;
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn)
+        return false;
+    g_encode = reinterpret_cast<EncodeTiledFn>(fn);
+    return true;
+}
+
+enum PtrSide { SIDE_DEVICE, SIDE_HOST };
+PtrSide ptr_side(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return SIDE_HOST;
+    }
+    return (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) ? SIDE_DEVICE : SIDE_HOST;
+}
+
+// ------------------------------------------------------------------ plan construction
+void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb) {
+    if (ncols <= nb) {
+        Op o{};
+        o.kind = Op::PANEL;
+        o.c0 = c0;
+        o.w = ncols;
+        ops.push_back(o);
+        return;
+    }
+    const int h = rgsqr_split(ncols), w = ncols - h;
+    build_ops(ops, c0, h, nb);
+    Op p{};
+    p.kind = Op::PROJ;
+    p.c0 = c0;
+    p.h = h;
+    p.w = w;
+    ops.push_back(p);
+    Op u = p;
+    u.kind = Op::UPDATE;
+    ops.push_back(u);
+    build_ops(ops, c0 + h, w, nb);
+}
+
+int make_plan(rg_handle h, Plan& pl) {
+    if (!ensure_encode()) return RG_CUDA_ERROR;
+    const int64_t m = pl.m;
+    const int n = (int)pl.n;
+    pl.ldh = round_up(std::max<int64_t>(m, 8), 8);
+    pl.ops.clear();
+    build_ops(pl.ops, 0, n, pl.nb);
+    int max_h = 0, max_w = 0;
+    size_t pmax = 0;
+    for (auto& o : pl.ops)
+        if (o.kind != Op::PANEL) {
+            max_h = std::max(max_h, o.h);
+            max_w = std::max(max_w, o.w);
+        }
+    pl.ldr12 = round_up(std::max(max_h, 8), 8);
+    const uint16_t* qh = h->qh.as<uint16_t>();
+    const uint16_t* ql = h->ql.as<uint16_t>();
+    const uint16_t* r12h = h->r12h.as<uint16_t>();
+    const uint16_t* r12l = h->r12l.as<uint16_t>();
+    const bool bf = pl.bf16 != 0;
+    for (auto& o : pl.ops) {
+        if (o.kind == Op::PANEL) continue;
+        const uint16_t* q1 = qh + (int64_t)o.c0 * pl.ldh;
+        const uint16_t* a2 = qh + (int64_t)(o.c0 + o.h) * pl.ldh;
+        const uint16_t* q1l = pl.split ? ql + (int64_t)o.c0 * pl.ldh : q1;
+        const uint16_t* a2l = pl.split ? ql + (int64_t)(o.c0 + o.h) * pl.ldh : a2;
+        o.bn = pick_bn(o.w);
+        if (o.kind == Op::PROJ) {
+            o.tiles_i = (o.h + 127) / 128;
+            o.tiles_j = (o.w + o.bn - 1) / o.bn;
+            o.kb_total = (int)((m + 63) / 64);
+            const int tiles = o.tiles_i * o.tiles_j;
+            int splits = std::max(1, (2 * 148 + tiles / 2) / tiles);
+            splits = std::min(splits, std::max(1, o.kb_total / 4));
+            o.kb_per_split = (o.kb_total + splits - 1) / splits;
+            o.splits = (o.kb_total + o.kb_per_split - 1) / o.kb_per_split;
+            pmax = std::max(pmax, (size_t)o.splits * o.tiles_j * o.bn * o.tiles_i * 128);
+            bool ok = encode_map(&o.ma, q1, m, o.h, pl.ldh, 64, 128, bf) &&
+                      encode_map(&o.mb, a2, m, o.w, pl.ldh, 64, o.bn, bf) &&
+                      encode_map(&o.ma_lo, q1l, m, o.h, pl.ldh, 64, 128, bf) &&
+                      encode_map(&o.mb_lo, a2l, m, o.w, pl.ldh, 64, o.bn, bf);
+            if (!ok) return RG_CUDA_ERROR;
+        } else {
+            bool ok = encode_map(&o.ma, q1, m, o.h, pl.ldh, 64, 64, bf) &&
+                      encode_map(&o.mb, r12h, o.h, o.w, pl.ldr12, 64, o.bn, bf) &&
+                      encode_map(&o.ma_lo, q1l, m, o.h, pl.ldh, 64, 64, bf) &&
+                      encode_map(&o.mb_lo, pl.split ? r12l : r12h, o.h, o.w, pl.ldr12, 64, o.bn, bf);
+            if (!ok) return RG_CUDA_ERROR;
+        }
+    }
+    pl.p_floats = pmax;
+    (void)max_w;
+    return RG_OK;
+}
+
+// grow every workspace buffer the plan needs; returns false on allocation failure
+bool ensure_workspace(rg_handle h, int64_t m, int64_t n, int split) {
+    const int64_t ldh = round_up(std::max<int64_t>(m, 8), 8);
+    const size_t qh_bytes = (size_t)ldh * n * 2;
+    // projection partials: bounded by splits * padded tiles; computed generously here
+    const int64_t hmax = n / 2 + 32, wmax = n / 2 + 32;
+    bool ok = h->qh.ensure(qh_bytes) && (!split || h->ql.ensure(qh_bytes)) &&
+              h->r12h.ensure((size_t)round_up(hmax, 8) * wmax * 2 + 4096) &&
+              (!split || h->r12l.ensure((size_t)round_up(hmax, 8) * wmax * 2 + 4096)) &&
+              h->r12f.ensure((size_t)hmax * wmax * 4 + 4096) &&
+              h->partial.ensure(rg::colnorm_partial_doubles(m, (int)n) * 8 + 64) && h->norm2.ensure(n * 8 + 64) &&
+              h->scale.ensure(n * 4 + 64) && h->status.ensure(64) &&
+              h->pws.ensure(rg::panel_ws_floats(m) * 4 + 4096) && h->pcnt.ensure(rg::panel_counters(m) * 4 + 64) &&
+              h->rgather.ensure((size_t)64 * 32 * 32 * 4) && h->rstackq.ensure((size_t)64 * 32 * 32 * 4);
+    return ok;
+}
+
+int nccl_allreduce(rg_handle h, void* buf, size_t count, ncclDataType_t t) {
+    if (h->nranks <= 1 || !h->comm) return RG_OK;
+    if (g_nccl.AllReduce(buf, buf, count, t, ncclSum, h->comm, h->stream) != ncclSuccess) return RG_NCCL_ERROR;
+    return RG_OK;
+}
+
+// enqueue one RGSQR pass on h->stream (no sync).  A -> Q (may alias), R (ldr).
+int enqueue_rgsqr(rg_handle h, Plan& pl) {
+    cudaStream_t st = h->stream;
+    const int64_t m = pl.m;
+    const int n = (int)pl.n;
+    uint16_t* qh = h->qh.as<uint16_t>();
+    uint16_t* ql = pl.split ? h->ql.as<uint16_t>() : nullptr;
+    int* status = h->status.as<int>();
+    const bool dist = h->nranks > 1 && h->comm;
+    {
+        ProfScope _s(h, PC_SCALE, 0, (double)m * n * (pl.split ? 16 : 14));
+        RG_CUDA(rg::launch_colnorm(pl.A, pl.lda, m, n, h->partial.as<double>(), h->norm2.as<double>(), st));
+        int rc = nccl_allreduce(h, h->norm2.p, n, ncclFloat64);
+        if (rc) return rc;
+        RG_CUDA(rg::launch_colscale(h->norm2.as<double>(), n, pl.scale, h->scale.as<float>(), status, 0, st));
+        RG_CUDA(rg::launch_scale_cast(pl.A, pl.lda, pl.Q, pl.ldq, qh, ql, pl.ldh, m, n, h->scale.as<float>(), pl.bf16,
+                                      st));
+        RG_CUDA(cudaMemset2DAsync(pl.R, pl.ldr * sizeof(float), 0, n * sizeof(float), n, st));
+    }
+    for (auto& o : pl.ops) {
+        if (o.kind == Op::PANEL) {
+            ProfScope _s(h, PC_PANEL, 2.0 * m * o.w * o.w, (double)m * o.w * (pl.split ? 16 : 14));
+            rg::PanelLaunch p{};
+            p.Q = pl.Q + (int64_t)o.c0 * pl.ldq;
+            p.ldq = pl.ldq;
+            p.Qh = qh + (int64_t)o.c0 * pl.ldh;
+            p.Ql = ql ? ql + (int64_t)o.c0 * pl.ldh : nullptr;
+            p.ldh = pl.ldh;
+            p.m = m;
+            p.nc = o.w;
+            p.ws = h->pws.as<float>();
+            p.counters = h->pcnt.as<int>();
+            p.bf16 = pl.bf16;
+            p.col0 = o.c0;
+            p.status = status;
+            if (!dist) {
+                p.R = pl.R + o.c0 + (int64_t)o.c0 * pl.ldr;
+                p.ldr = pl.ldr;
+                p.distributed = 0;
+                RG_CUDA(rg::launch_panel(p, st));
+            } else {
+                // local TSQR -> gather the P local R's -> redundant stack MGS -> apply own block
+                float* rg_all = h->rgather.as<float>();
+                p.R = rg_all + (int64_t)h->rank * o.w * o.w;
+                p.ldr = o.w;
+                p.distributed = 1;
+                RG_CUDA(rg::launch_panel(p, st));
+                if (g_nccl.AllGather(p.R, rg_all, (size_t)o.w * o.w, ncclFloat32, h->comm, st) != ncclSuccess)
+                    return RG_NCCL_ERROR;
+                float* qb = h->rstackq.as<float>();
+                RG_CUDA(rg::launch_panel_stack(rg_all, h->nranks, o.w, pl.R + o.c0 + (int64_t)o.c0 * pl.ldr, pl.ldr,
+                                               qb, status, o.c0, st));
+                RG_CUDA(rg::launch_panel_apply(p, qb + (int64_t)h->rank * 32 * 32, st));
+            }
+        } else if (o.kind == Op::PROJ) {
+            ProfScope _s(h, PC_PROJ, 2.0 * m * o.h * o.w * (pl.split ? 3 : 1),
+                             (double)m * (o.h + o.w) * (pl.split ? 4 : 2));
+            float* P = h->P.as<float>();
+            const int64_t ldp = (int64_t)o.tiles_i * 128;
+            const int64_t pstride = ldp * o.tiles_j * o.bn;
+            RG_CUDA(rg::launch_proj_gemm(o.bn, pl.split != 0, o.tiles_i, o.tiles_j, o.splits, o.ma, o.mb, o.ma_lo,
+                                         o.mb_lo, P, ldp, pstride, o.kb_total, o.kb_per_split, pl.bf16, st));
+            float* Rblk = pl.R + o.c0 + (int64_t)(o.c0 + o.h) * pl.ldr;
+            uint16_t* r12l = pl.split ? h->r12l.as<uint16_t>() : nullptr;
+            if (!dist) {
+                RG_CUDA(rg::launch_proj_reduce(P, ldp, pstride, o.splits, o.h, o.w, Rblk, pl.ldr, nullptr, 0,
+                                               h->r12h.as<uint16_t>(), r12l, pl.ldr12, pl.bf16, st));
+            } else {
+                float* rf = h->r12f.as<float>();
+                RG_CUDA(rg::launch_proj_reduce(P, ldp, pstride, o.splits, o.h, o.w, nullptr, 0, rf, o.h, nullptr,
+                                               nullptr, 0, pl.bf16, st));
+                int rc = nccl_allreduce(h, rf, (size_t)o.h * o.w, ncclFloat32);
+                if (rc) return rc;
+                RG_CUDA(rg::launch_proj_finish(rf, o.h, o.h, o.w, Rblk, pl.ldr, h->r12h.as<uint16_t>(), r12l, pl.ldr12,
+                                               pl.bf16, st));
+            }
+        } else {
+            ProfScope _s(h, PC_UPDATE, 2.0 * m * o.h * o.w * (pl.split ? 3 : 1),
+                             (double)m * o.h * (pl.split ? 4 : 2) + (double)m * o.w * (pl.split ? 12 : 10));
+            float* C = pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq;
+            uint16_t* Ch = qh + (int64_t)(o.c0 + o.h) * pl.ldh;
+            uint16_t* Cl = ql ? ql + (int64_t)(o.c0 + o.h) * pl.ldh : nullptr;
+            RG_CUDA(rg::launch_update_gemm(o.bn, pl.split != 0, m, o.w, o.h, o.ma, o.mb, o.ma_lo, o.mb_lo, C, pl.ldq, Ch,
+                                           Cl, pl.ldh, pl.bf16, st));
+        }
+    }
+    {
+        ProfScope _s(h, PC_OTHER);
+        RG_CUDA(rg::launch_unscale_r(pl.R, pl.ldr, n, pl.scale ? h->scale.as<float>() : nullptr, st));
+    }
+    return RG_OK;
+}
+
+int reset_status(rg_handle h) {
+    static const int init[4] = {INT_MAX, INT_MAX, 0, 0};
+    RG_CUDA(cudaMemcpyAsync(h->status.p, init, sizeof(init), cudaMemcpyHostToDevice, h->stream));
+    return RG_OK;
+}
+
+int check_status(rg_handle h) {
+    RG_CUDA(cudaMemcpyAsync(h->status_host, h->status.p, 4 * sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    RG_CUDA(cudaStreamSynchronize(h->stream));
+    h->last_info = -1;
+    if (h->status_host[1] != INT_MAX) {
+        h->last_info = h->status_host[1];
+        return RG_NONFINITE;
+    }
+    if (h->status_host[0] != INT_MAX) {
+        h->last_info = h->status_host[0];
+        return RG_BREAKDOWN;
+    }
+    return RG_OK;
+}
+
+// run one RGSQR pass (device pointers), with plan caching + CUDA graph replay
+int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq, float* R,
+              int64_t ldr, const rg_opts& o, int split) {
+    if (!ensure_workspace(h, m, n, split)) return RG_ALLOC;
+    const int nb = (o.nb <= 0 || o.nb > 32) ? 32 : o.nb;
+    Plan* pl = h->plan.get();
+    const bool same = pl && pl->m == m && pl->n == n && pl->lda == lda && pl->ldq == ldq && pl->ldr == ldr &&
+                      pl->A == A && pl->Q == Q && pl->R == R && pl->nb == nb && pl->bf16 == o.precision &&
+                      pl->split == split && pl->scale == o.scale && pl->nranks == h->nranks &&
+                      pl->rank == h->rank && pl->epoch == g_alloc_epoch;
+    if (!same) {
+        if (pl && pl->exec) cudaGraphExecDestroy(pl->exec);
+        h->plan.reset(new Plan());
+        pl = h->plan.get();
+        pl->m = m; pl->n = n; pl->lda = lda; pl->ldq = ldq; pl->ldr = ldr;
+        pl->A = A; pl->Q = Q; pl->R = R;
+        pl->nb = nb; pl->bf16 = o.precision; pl->split = split; pl->scale = o.scale;
+        pl->nranks = h->nranks; pl->rank = h->rank;
+        int rc = make_plan(h, *pl);
+        if (rc) return rc;
+        if (!h->P.ensure(pl->p_floats * 4 + 4096)) return RG_ALLOC;
+        pl->epoch = g_alloc_epoch;  // P may have moved: the graph is captured below, after this
+    }
+    int rc = reset_status(h);
+    if (rc) return rc;
+    const bool use_graph = !h->prof && getenv("RGSQR_NO_GRAPH") == nullptr;
+    if (!use_graph) return enqueue_rgsqr(h, *pl);
+    if (!pl->exec) {
+        // capture on the private stream (the user's may be the legacy stream, which cannot
+        // capture); the instantiated graph is then launched on the user's stream
+        cudaGraph_t g;
+        cudaStream_t user = h->stream;
+        h->stream = h->capture_stream;
+        RG_CUDA(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
+        rc = enqueue_rgsqr(h, *pl);
+        cudaError_t ce = cudaStreamEndCapture(h->stream, &g);
+        h->stream = user;
+        if (rc) {
+            if (ce == cudaSuccess) cudaGraphDestroy(g);
+            return rc;
+        }
+        RG_CUDA(ce);
+        cudaError_t ie = cudaGraphInstantiate(&pl->exec, g, 0);
+        cudaGraphDestroy(g);
+        RG_CUDA(ie);
+    }
+    RG_CUDA(cudaGraphLaunch(pl->exec, h->stream));
+    return RG_OK;
+}
+
+
+}  // namespace
+
+// ====================================================================== C-ABI
+extern "C" {
+
+void rg_opts_default(rg_opts* o) {
+    if (!o) return;
+    o->precision = 0;
+    o->nb = 32;
+    o->scale = 1;
+    o->reortho = -1;
+    o->split = 0;
+    o->sync = 1;
+}
+
+const char* rg_version(void) { return "rgsqr 0.1 sm_100a tcgen05/TMA"; }
+
+const char* rg_status_string(int s) {
+    if (s < 0) return "invalid argument";
+    switch (s) {
+        case RG_OK: return "ok";
+        case RG_BREAKDOWN: return "breakdown: zero or non-finite column norm (rank deficient)";
+        case RG_NOT_CONVERGED: return "not converged";
+        case RG_NONFINITE: return "non-finite input";
+        case RG_CUDA_ERROR: return "CUDA error";
+        case RG_NCCL_ERROR: return "NCCL error";
+        case RG_NO_DEVICE: return "no sm_100 CUDA device";
+        case RG_ALLOC: return "allocation failed";
+        default: return "unknown status";
+    }
+}
+
+int rg_create(rg_handle* out, int device, void* stream) {
+    if (!out) return -1;
+    *out = nullptr;
+    int count = 0;
+    if (cudaGetDeviceCount(&count) != cudaSuccess || device < 0 || device >= count) {
+        cudaGetLastError();
+        return RG_NO_DEVICE;
+    }
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, device) != cudaSuccess || prop.major != 10) return RG_NO_DEVICE;
+    if (cudaSetDevice(device) != cudaSuccess) return RG_NO_DEVICE;
+    rg_handle h = new rg_handle_s();
+    h->device = device;
+    h->stream = reinterpret_cast<cudaStream_t>(stream);
+    if (cudaMallocHost(&h->status_host, 64) != cudaSuccess) {
+        delete h;
+        return RG_ALLOC;
+    }
+    if (cudaStreamCreateWithFlags(&h->capture_stream, cudaStreamNonBlocking) != cudaSuccess) {
+        cudaFreeHost(h->status_host);
+        delete h;
+        return RG_CUDA_ERROR;
+    }
+    if (!ensure_encode()) {
+        cudaFreeHost(h->status_host);
+        delete h;
+        return RG_CUDA_ERROR;
+    }
+    *out = h;
+    return RG_OK;
+}
+
+int rg_set_stream(rg_handle h, void* stream) {
+    if (!h) return -1;
+    if (h->plan && h->plan->exec) {
+        cudaGraphExecDestroy(h->plan->exec);
+        h->plan->exec = nullptr;
+    }
+    h->stream = reinterpret_cast<cudaStream_t>(stream);
+    return RG_OK;
+}
+
+int rg_destroy(rg_handle h) {
+    if (!h) return -1;
+    cudaSetDevice(h->device);
+    cudaStreamSynchronize(h->stream);
+    if (h->plan && h->plan->exec) cudaGraphExecDestroy(h->plan->exec);
+    DevBuf* bufs[] = {&h->qh, &h->ql, &h->P, &h->r12h, &h->r12l, &h->r12f, &h->partial, &h->norm2, &h->scale,
+                      &h->status, &h->pws, &h->pcnt, &h->rgather, &h->rstackq, &h->stageA, &h->stageQ,
+                      &h->stageR, &h->stageB, &h->stageX, &h->cg, &h->aux};
+    for (auto* b : bufs) b->release();
+    for (auto& e : h->ev_pool) {
+        cudaEventDestroy(e.first);
+        cudaEventDestroy(e.second);
+    }
+    if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
+    if (h->status_host) cudaFreeHost(h->status_host);
+    if (h->capture_stream) cudaStreamDestroy(h->capture_stream);
+    delete h;
+    return RG_OK;
+}
+
+int64_t rg_last_info(rg_handle h) { return h ? h->last_info : -1; }
+
+int rg_nccl_load(const char* path) {
+    if (g_nccl.lib) return RG_OK;
+    void* lib = dlopen(path ? path : "libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!lib) return RG_NCCL_ERROR;
+    g_nccl.GetUniqueId = (decltype(g_nccl.GetUniqueId))dlsym(lib, "ncclGetUniqueId");
+    g_nccl.CommInitRank = (decltype(g_nccl.CommInitRank))dlsym(lib, "ncclCommInitRank");
+    g_nccl.CommDestroy = (decltype(g_nccl.CommDestroy))dlsym(lib, "ncclCommDestroy");
+    g_nccl.AllReduce = (decltype(g_nccl.AllReduce))dlsym(lib, "ncclAllReduce");
+    g_nccl.AllGather = (decltype(g_nccl.AllGather))dlsym(lib, "ncclAllGather");
+    if (!g_nccl.GetUniqueId || !g_nccl.CommInitRank || !g_nccl.AllReduce || !g_nccl.AllGather) {
+        dlclose(lib);
+        return RG_NCCL_ERROR;
+    }
+    g_nccl.lib = lib;
+    return RG_OK;
+}
+
+int rg_comm_unique_id(void* id128) {
+    if (!id128) return -1;
+    if (!g_nccl.lib && rg_nccl_load(nullptr) != RG_OK) return RG_NCCL_ERROR;
+    ncclUniqueId id;
+    if (g_nccl.GetUniqueId(&id) != ncclSuccess) return RG_NCCL_ERROR;
+    memcpy(id128, &id, sizeof(id));
+    return RG_OK;
+}
+
+int rg_comm_init(rg_handle h, const void* id128, int rank, int nranks) {
+    if (!h) return -1;
+    if (!id128) return -2;
+    if (nranks < 1 || nranks > 64) return -4;
+    if (rank < 0 || rank >= nranks) return -3;
+    if (!g_nccl.lib && rg_nccl_load(nullptr) != RG_OK) return RG_NCCL_ERROR;
+    ncclUniqueId id;
+    memcpy(&id, id128, sizeof(id));
+    cudaSetDevice(h->device);
+    ncclComm_t c = nullptr;
+    if (g_nccl.CommInitRank(&c, nranks, id, rank) != ncclSuccess) return RG_NCCL_ERROR;
+    if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
+    h->comm = c;
+    h->rank = rank;
+    h->nranks = nranks;
+    if (h->plan && h->plan->exec) {
+        cudaGraphExecDestroy(h->plan->exec);
+        h->plan->exec = nullptr;
+    }
+    h->plan.reset();
+    return RG_OK;
+}
+
+int rg_profile_enable(rg_handle h, int enable) {
+    if (!h) return -1;
+    h->prof = enable != 0;
+    return RG_OK;
+}
+int rg_profile_reset(rg_handle h) {
+    if (!h) return -1;
+    prof_collect(h);
+    for (int i = 0; i < PC_N; ++i) {
+        h->prof_ms[i] = 0;
+        h->prof_launches[i] = 0;
+        h->prof_flops[i] = 0;
+        h->prof_bytes[i] = 0;
+    }
+    return RG_OK;
+}
+int rg_profile_get(rg_handle h, int cls, double* ms, int64_t* launches, double* flops, double* bytes) {
+    if (!h) return -1;
+    if (cls < 0 || cls >= PC_N) return -2;
+    prof_collect(h);
+    if (ms) *ms = h->prof_ms[cls];
+    if (launches) *launches = h->prof_launches[cls];
+    if (flops) *flops = h->prof_flops[cls];
+    if (bytes) *bytes = h->prof_bytes[cls];
+    return RG_OK;
+}
+
+int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq,
+                 float* R, int64_t ldr, const rg_opts* opts) {
+    if (!h) return -1;
+    rg_opts o;
+    if (opts) o = *opts; else rg_opts_default(&o);
+    if (m_local < 1 || (h->nranks <= 1 && m_local < n)) return -2;
+    if (n < 1 || n > 65535) return -3;
+    if (!A) return -4;
+    if (lda < m_local) return -5;
+    if (!Q) return -6;
+    if (ldq < m_local) return -7;
+    if (!R) return -8;
+    if (ldr < n) return -9;
+    if (o.precision != 0 && o.precision != 1) return -10;
+    cudaSetDevice(h->device);
+    const bool host = ptr_side(A) == SIDE_HOST;
+    if (host && (ptr_side(Q) != SIDE_HOST || ptr_side(R) != SIDE_HOST)) return -6;
+    const float* dA = A;
+    float* dQ = Q;
+    float* dR = R;
+    int64_t dlda = lda, dldq = ldq, dldr = ldr;
+    if (host) {
+        // stage: A -> device Q buffer (factor in place), results copied back
+        if (!h->stageQ.ensure((size_t)m_local * n * 4) || !h->stageR.ensure((size_t)n * n * 4)) return RG_ALLOC;
+        dQ = h->stageQ.as<float>();
+        dR = h->stageR.as<float>();
+        dldq = m_local;
+        dldr = n;
+        RG_CUDA(cudaMemcpy2DAsync(dQ, m_local * 4, A, lda * 4, m_local * 4, n, cudaMemcpyHostToDevice, h->stream));
+        dA = dQ;
+        dlda = m_local;
+    }
+    int rc = RG_OK;
+    int passes = 1 + std::max(0, o.reortho);
+    for (int p = 0; p < passes && rc == RG_OK; ++p) {
+        if (p == 0) {
+            rc = run_rgsqr(h, m_local, n, dA, dlda, dQ, dldq, dR, dldr, o, o.split);
+        } else {
+            // refinement pass: [Q2, R2] = RGSQR(Q) in split precision, R <- R2 R
+            if (!h->aux.ensure((size_t)2 * n * n * 4)) return RG_ALLOC;
+            float* R2 = h->aux.as<float>();
+            float* Rt = R2 + n * n;
+            if (rc == RG_OK && o.sync) rc = check_status(h);
+            if (rc) break;
+            rc = run_rgsqr(h, m_local, n, dQ, dldq, dQ, dldq, R2, n, o, 1);
+            if (rc) break;
+            RG_CUDA(rg::launch_trmm_upper(R2, n, dR, dldr, Rt, n, (int)n, h->stream));
+            RG_CUDA(cudaMemcpy2DAsync(dR, dldr * 4, Rt, n * 4, n * 4, n, cudaMemcpyDeviceToDevice, h->stream));
+        }
+    }
+    if (rc) return rc;
+    if (host) {
+        RG_CUDA(cudaMemcpy2DAsync(Q, ldq * 4, dQ, dldq * 4, m_local * 4, n, cudaMemcpyDeviceToHost, h->stream));
+        RG_CUDA(cudaMemcpy2DAsync(R, ldr * 4, dR, dldr * 4, n * 4, n, cudaMemcpyDeviceToHost, h->stream));
+    }
+    if (o.sync || host) rc = check_status(h);
+    prof_collect(h);
+    return rc;
+}
+
+}  // extern "C"

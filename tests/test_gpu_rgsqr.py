@@ -1,0 +1,156 @@
+"""GPU parity of rgsqr_factor (C-ABI) against the fp64 oracle (-m gpu).
+
+Tolerances (BASELINE north_star, restated in DESIGN.md "Tolerances"):
+  backward error ||A - QR||_F / ||A||_F <= 5e-3, orthogonality ||I - Q^T Q||_F <= 1e-2 sqrt(n)
+  before reorthogonalisation on well-conditioned inputs (reading #11).  Distance to the
+  unique QR (oracle Householder, positive diagonal): ||R - R*||_F/||R*||_F <= 10 kappa * be.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def rg():
+    import paper_conf_hpdc_zhangbw20_b200 as rg
+    return rg
+
+
+def _dev(A):
+    """numpy (m, n) -> column-major CUDA fp32 tensor (strides (1, m))."""
+    return torch.from_numpy(np.ascontiguousarray(np.asarray(A, dtype=np.float32).T)).cuda().t()
+
+
+def _run(rg, A32, **kw):
+    Ad = _dev(A32)
+    Q, R = rg.rgsqr_factor(Ad, opts=rg.make_opts(**kw))
+    torch.cuda.synchronize()
+    return Q.cpu().numpy().astype(np.float64), R.cpu().numpy().astype(np.float64)
+
+
+def _check_qr(A32, Q, R, kappa=10.0, orth_scale=1e-2):
+    A = np.asarray(A32, dtype=np.float64)
+    m, n = A.shape
+    assert np.all(np.isfinite(Q)) and np.all(np.isfinite(R))
+    assert np.all(np.tril(R, -1) == 0)
+    assert np.all(np.diag(R) > 0)
+    be = oracle.backward_error(A, Q, R)
+    orth = oracle.orthogonality(Q)
+    assert be <= 5e-3, be
+    assert orth <= orth_scale * np.sqrt(n), orth
+    Qo, Ro, _ = oracle.householder(A)
+    dr = np.linalg.norm(R - Ro) / np.linalg.norm(Ro)
+    assert dr <= max(10 * kappa * be, 1e-5), (dr, be)
+    return be, orth, dr
+
+
+@pytest.mark.parametrize("m,n", [(64, 1), (100, 7), (256, 32), (1000, 32), (1024, 64), (1025, 96), (4099, 64),
+                                 (3000, 200), (8192, 256), (777, 333)])
+def test_rgsqr_gaussian_parity(rg, m, n):
+    A = synth.gaussian(m, n, seed=synth.SEED_BASE + m + n).astype(np.float32)
+    Q, R = _run(rg, A)
+    _check_qr(A, Q, R, kappa=np.linalg.cond(A))
+
+
+def test_rgsqr_config1(rg):
+    """BASELINE config 1: 1024 x 64, cond ~ 10 (geometric spectrum), vs the fp64 oracle."""
+    A = synth.svd_matrix(1024, 64, "geometric", 10.0, seed=synth.SEED_BASE + 0).astype(np.float32)
+    Q, R = _run(rg, A)
+    be, orth, dr = _check_qr(A, Q, R, kappa=10.0)
+    assert be < 2e-4  # fp16 updates, fp32 panel: SURVEY [EMU] ~4e-5
+
+
+def test_rgsqr_single_panel_is_fp32_accurate(rg):
+    """n <= 32: the whole call is one fp32 TSQR/MGS panel (no tensor cores)."""
+    A = synth.gaussian(5000, 32, seed=3).astype(np.float32)
+    Q, R = _run(rg, A)
+    A64 = A.astype(np.float64)
+    assert oracle.backward_error(A64, Q, R) < 1e-6
+    assert oracle.orthogonality(Q) < 1e-5
+
+
+def test_rgsqr_bf16(rg):
+    A = synth.gaussian(2048, 128, seed=4).astype(np.float32)
+    Q, R = _run(rg, A, precision="bf16")
+    _check_qr(A, Q, R, kappa=np.linalg.cond(A), orth_scale=5e-2)
+
+
+def test_rgsqr_scaling_invariance(rg):
+    """AP = Q (R P) for power-of-two P (section 3.5): Q identical, R column-scaled."""
+    A = synth.gaussian(2048, 96, seed=5).astype(np.float32)
+    g = synth.rng(6)
+    p = (2.0 ** g.integers(-20, 21, size=96)).astype(np.float32)
+    Q1, R1 = _run(rg, A)
+    Q2, R2 = _run(rg, A * p)
+    np.testing.assert_array_equal(Q1, Q2)
+    np.testing.assert_allclose(R2, R1 * p, rtol=1e-6, atol=0)
+
+
+def test_rgsqr_badly_scaled_columns(rg):
+    """Columns far outside the fp16 range factor correctly thanks to scaling."""
+    A = synth.gaussian(4096, 64, seed=7).astype(np.float32)
+    A[:, ::3] *= 1e6
+    A[:, 1::3] *= 1e-6
+    Q, R = _run(rg, A)
+    Ar = A.astype(np.float64)
+    assert oracle.backward_error(Ar, Q, R) < 5e-3
+    assert oracle.orthogonality(Q) < 1e-2 * 8
+
+
+def test_rgsqr_deterministic(rg):
+    A = synth.gaussian(4096, 128, seed=8).astype(np.float32)
+    Q1, R1 = _run(rg, A)
+    Q2, R2 = _run(rg, A)
+    np.testing.assert_array_equal(Q1, Q2)
+    np.testing.assert_array_equal(R1, R2)
+
+
+def test_rgsqr_inplace_and_lda(rg):
+    A = synth.gaussian(1000, 64, seed=9).astype(np.float32)
+    big = np.zeros((1024 + 13, 64), dtype=np.float32)
+    big[:1000] = A
+    Bd = _dev(big)
+    view = Bd[:1000]
+    Q, R = rg.rgsqr_factor(view, Q=view)
+    torch.cuda.synchronize()
+    Qn = Bd.cpu().numpy()[:1000].astype(np.float64)
+    _check_qr(A, Qn, R.cpu().numpy().astype(np.float64), kappa=np.linalg.cond(A))
+    np.testing.assert_array_equal(Bd.cpu().numpy()[1000:], 0)
+
+
+def test_rgsqr_host_pointers(rg):
+    A = np.asfortranarray(synth.gaussian(3000, 96, seed=10).astype(np.float32))
+    Q, R = rg.rgsqr_factor(A)
+    _check_qr(A, Q.astype(np.float64), R.astype(np.float64), kappa=np.linalg.cond(A))
+
+
+def test_rgsqr_breakdown_status(rg):
+    A = synth.gaussian(512, 40, seed=11).astype(np.float32)
+    A[:, 17] = 0.0
+    with pytest.raises(rg.RGError) as e:
+        _run(rg, A)
+    assert e.value.status == rg.RG_BREAKDOWN
+    A = synth.gaussian(512, 40, seed=11).astype(np.float32)
+    A[3, 5] = np.nan
+    with pytest.raises(rg.RGError) as e:
+        _run(rg, A)
+    assert e.value.status == rg.RG_NONFINITE and e.value.info == 5
+
+
+def test_rgsqr_invalid_arguments(rg):
+    import ctypes
+    h = rg.default_handle()
+    L = rg.lib()
+    o = rg.make_opts()
+    A = torch.zeros(10, 20, device="cuda")
+    p = ctypes.c_void_p(A.data_ptr())
+    assert L.rgsqr_factor(h.ptr, 10, 20, p, 10, p, 10, p, 20, ctypes.byref(o)) == -2   # m < n
+    assert L.rgsqr_factor(h.ptr, 20, 0, p, 20, p, 20, p, 20, ctypes.byref(o)) == -3
+    assert L.rgsqr_factor(h.ptr, 20, 10, None, 20, p, 20, p, 20, ctypes.byref(o)) == -4
+    assert L.rgsqr_factor(h.ptr, 20, 10, p, 19, p, 20, p, 20, ctypes.byref(o)) == -5
+    assert L.rgsqr_factor(h.ptr, 20, 10, p, 20, p, 20, p, 9, ctypes.byref(o)) == -9
