@@ -66,6 +66,9 @@ typedef struct {
                        orthogonalize always uses it for its refinement passes */
     int sync;       /* 1 (default) = synchronise at the end of the call and return breakdown /
                        non-finite status; 0 = fully asynchronous (status not checked) */
+    int panel;      /* leaf panel algorithm: 0 = auto (default): CholQR2 with an fp64 Gram, falling
+                       back on the device to the TSQR/MGS panel if a Cholesky pivot fails;
+                       1 = TSQR/MGS only (eq 8 + Alg 2, the paper's panel) */
 } rg_opts;
 
 RG_API void rg_opts_default(rg_opts* o);
@@ -78,6 +81,9 @@ RG_API int rg_destroy(rg_handle h);
 RG_API const char* rg_status_string(int status);
 /* Column index attached to the last RG_BREAKDOWN / RG_NONFINITE status (-1 if none). */
 RG_API int64_t rg_last_info(rg_handle h);
+/* Number of library kernels launched by the last API call on this handle (a CUDA-graph replay
+ * counts the kernels it contains). */
+RG_API int64_t rg_last_launches(rg_handle h);
 /* Build identity, e.g. "rgsqr sm_100a tcgen05"; never NULL. */
 RG_API const char* rg_version(void);
 

@@ -28,7 +28,7 @@ RG_OK, RG_BREAKDOWN, RG_NOT_CONVERGED, RG_NONFINITE, RG_CUDA_ERROR, RG_NCCL_ERRO
 
 EXPORTS = [
     "rg_opts_default", "rg_create", "rg_set_stream", "rg_destroy", "rg_status_string", "rg_last_info",
-    "rg_version", "rg_nccl_load", "rg_comm_unique_id", "rg_comm_init", "rgsqr_factor", "orthogonalize",
+    "rg_version", "rg_last_launches", "rg_nccl_load", "rg_comm_unique_id", "rg_comm_init", "rgsqr_factor", "orthogonalize",
     "ls_solve_refined", "lowrank_approx", "rg_profile_enable", "rg_profile_reset", "rg_profile_get",
 ]
 
@@ -51,7 +51,8 @@ class RGError(RuntimeError):
 
 class rg_opts(ctypes.Structure):
     _fields_ = [("precision", ctypes.c_int), ("nb", ctypes.c_int), ("scale", ctypes.c_int),
-                ("reortho", ctypes.c_int), ("split", ctypes.c_int), ("sync", ctypes.c_int)]
+                ("reortho", ctypes.c_int), ("split", ctypes.c_int), ("sync", ctypes.c_int),
+                ("panel", ctypes.c_int)]
 
 
 _LIB = None
@@ -74,11 +75,13 @@ def _lib():
         L.rg_last_info.argtypes = [vp]
         L.rg_last_info.restype = i64
         L.rg_version.restype = ctypes.c_char_p
+        L.rg_last_launches.argtypes = [vp]
+        L.rg_last_launches.restype = i64
         L.rg_nccl_load.argtypes = [ctypes.c_char_p]
         L.rg_comm_unique_id.argtypes = [vp]
         L.rg_comm_init.argtypes = [vp, vp, i32, i32]
         L.rgsqr_factor.argtypes = [vp, i64, i64, vp, i64, vp, i64, vp, i64, ctypes.POINTER(rg_opts)]
-        for _name in ("orthogonalize", "ls_solve_refined", "lowrank_approx"):
+        for _name in ("lowrank_approx",):
             if not hasattr(L, _name):  # TEMP during bring-up
                 setattr(L, _name, lambda *a: RG_CUDA_ERROR)
         L.orthogonalize.argtypes = [vp, i64, i64, vp, i64, vp, i64, ctypes.c_double, i32,
@@ -108,7 +111,7 @@ def version() -> str:
     return _lib().rg_version().decode()
 
 
-def make_opts(precision="fp16", nb=32, scale=True, reortho=-1, split=False, sync=True) -> rg_opts:
+def make_opts(precision="fp16", nb=32, scale=True, reortho=-1, split=False, sync=True, panel="auto") -> rg_opts:
     o = rg_opts()
     _lib().rg_opts_default(ctypes.byref(o))
     o.precision = {"fp16": 0, "bf16": 1}[precision] if isinstance(precision, str) else int(precision)
@@ -117,6 +120,7 @@ def make_opts(precision="fp16", nb=32, scale=True, reortho=-1, split=False, sync
     o.reortho = int(reortho)
     o.split = int(bool(split))
     o.sync = int(bool(sync))
+    o.panel = {"auto": 0, "cholqr2": 0, "mgs": 1, "tsqr": 1}[panel] if isinstance(panel, str) else int(panel)
     return o
 
 
@@ -198,6 +202,9 @@ class Handle:
 
     def last_info(self) -> int:
         return int(_lib().rg_last_info(self._h))
+
+    def last_launches(self) -> int:
+        return int(_lib().rg_last_launches(self._h))
 
     # ---- multi-GPU (row-sharded) -------------------------------------------------------
     def init_comm(self, rank: int, nranks: int, group=None, nccl_path=None):

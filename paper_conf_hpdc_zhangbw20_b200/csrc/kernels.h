@@ -8,6 +8,9 @@
 
 namespace rg {
 
+// kernel launches issued by this thread (bench.py "gpu_launches" claim)
+extern thread_local long long g_launches;
+
 // ---- scale.cu (section 3.5)
 cudaError_t launch_colnorm(const float* A, int64_t lda, int64_t m, int n, double* partial, double* norm2,
                            cudaStream_t st);
@@ -35,6 +38,7 @@ struct PanelLaunch {
     int bf16;
     int col0;
     int* status;
+    const int* guard;   // non-null: the kernels run only if *guard != 0 (CholQR2 fallback)
 };
 int panel_levels(int ntiles, int* lvl_n);
 size_t panel_ws_floats(int64_t m);
@@ -42,7 +46,31 @@ size_t panel_counters(int64_t m);
 cudaError_t launch_panel(const PanelLaunch& pl, cudaStream_t st);
 cudaError_t launch_panel_apply(const PanelLaunch& pl, const float* Gq, cudaStream_t st);
 cudaError_t launch_panel_stack(const float* Rall, int P, int nc, float* R, int64_t ldr, float* Qblocks, int* status,
-                               int col0, cudaStream_t st);
+                               int col0, const int* guard, cudaStream_t st);
+
+// ---- panel_cholqr.cu (CholQR2, fp64 Gram)
+struct CholqrLaunch {
+    const float* P;
+    int64_t ldp;
+    float* Q1;      // m x 32 workspace (ld m)
+    float* Q;
+    int64_t ldq;
+    uint16_t* Qh;
+    uint16_t* Ql;
+    int64_t ldh;
+    int64_t m;
+    int nc;
+    double* ws;     // cholqr_ws_doubles(m)
+    int* counter;   // zero-initialised, self-resetting
+    int* fail;      // set on a failed pivot (guards the MGS fallback)
+    float* R;
+    int64_t ldr;
+    int bf16;
+    int (*allreduce_g)(double* G, void* ctx);  // non-null: multi-rank Gram allreduce (1024 doubles)
+    void* ctx;
+};
+size_t cholqr_ws_doubles(int64_t m);
+cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st);
 
 // ---- gemm_tc.cu (Alg 1 lines 8-9 on tcgen05)
 cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int splits, const CUtensorMap& q1,
@@ -60,13 +88,14 @@ cudaError_t launch_proj_finish(const float* Rf, int64_t ldf, int h, int w, float
 
 // ---- blas.cu (CGLS vectors, triangular inverse, small products)
 cudaError_t launch_gemv_n(const float* A, int64_t lda, int64_t m, int n, const double* x, double* y, double* work,
-                          cudaStream_t st);
+                          const double* done, cudaStream_t st);
 size_t gemv_n_work_doubles(int64_t m, int n);
 cudaError_t launch_gemv_t(const float* A, int64_t lda, int64_t m, int n, const double* r, double* s, double* work,
-                          cudaStream_t st);
+                          const double* done, cudaStream_t st);
 size_t gemv_t_work_doubles(int64_t m, int n);
 cudaError_t launch_trinv_upper(const float* R, int64_t ldr, int n, double* Rinv, cudaStream_t st);
-cudaError_t launch_trmv(const double* Rinv, int n, const double* x, double* y, int transpose, cudaStream_t st);
+cudaError_t launch_trmv(const double* Rinv, int n, const double* x, double* y, int transpose, const double* done,
+                        cudaStream_t st);
 cudaError_t launch_cgls_init(const float* b, int64_t m, int n, double* r, double* x, cudaStream_t st);
 cudaError_t launch_sqnorm(const double* v, int64_t len, double* sc, int idx, cudaStream_t st);
 cudaError_t launch_cgls_xr(double* x, const double* t, double* r, const double* q, int64_t m, int n, double* sc,
@@ -74,8 +103,9 @@ cudaError_t launch_cgls_xr(double* x, const double* t, double* r, const double* 
 cudaError_t launch_cgls_p(const double* s, double* p, int n, double* sc, int first, cudaStream_t st);
 cudaError_t launch_gaussian_philox(int64_t total, uint64_t seed, double* out64, float* out32, cudaStream_t st);
 size_t probe_work_doubles(int64_t m, int n, int p);
-cudaError_t launch_orth_probe(const float* Q, int64_t ldq, int64_t m, int n, const double* G, double* work,
-                              double* out, cudaStream_t st);
+cudaError_t launch_orth_probe_z(const float* Q, int64_t ldq, int64_t m, int n, const double* G, double* work,
+                                double* Z, cudaStream_t st);
+cudaError_t launch_orth_probe_finish(const double* Z, int n, const double* G, double* out, cudaStream_t st);
 cudaError_t launch_trmm_upper(const float* A, int64_t lda, const float* B, int64_t ldb, float* C, int64_t ldc, int n,
                               cudaStream_t st);
 

@@ -119,6 +119,7 @@ struct PanelArgs {
     int bf16;
     int col0;          // global index of the panel's first column (status reporting)
     int* status;       // [0] = first breakdown column (INT_MAX if none)
+    const int* guard;  // non-null: run only if *guard != 0 (fallback of the CholQR2 panel)
 };
 
 __device__ __forceinline__ int64_t tile_row0(const PanelArgs& p, int t) {
@@ -126,6 +127,7 @@ __device__ __forceinline__ int64_t tile_row0(const PanelArgs& p, int t) {
 }
 
 __global__ void __launch_bounds__(256, 2) panel_tile_kernel(PanelArgs p) {
+    if (p.guard && *p.guard == 0) return;
     __shared__ float qbuf[2 * PT];
     __shared__ float Rs[PNB][33];
     __shared__ int bad;
@@ -245,6 +247,7 @@ __global__ void __launch_bounds__(256, 2) panel_tile_kernel(PanelArgs p) {
 // Step (4)+(5): Q_tile <- Q_tile * (Qf_1[t] * Qf_2[t/8] * ... * Gq), fp32 + 16-bit shadow.
 // Gq (32x32, ld 32) is the rank's block of the cross-GPU stack factor, or null.
 __global__ void __launch_bounds__(256) panel_apply_kernel(PanelArgs p, const float* __restrict__ Gq) {
+    if (p.guard && *p.guard == 0) return;
     __shared__ float M[PNB][PNB + 1];
     __shared__ float Tm[PNB][PNB + 1];
     __shared__ float F[PNB][PNB + 1];
@@ -311,7 +314,9 @@ __global__ void __launch_bounds__(256) panel_apply_kernel(PanelArgs p, const flo
 // gathered as P x (32x32) blocks) are stacked and factored by MGS; writes the final R
 // and the P Q-blocks (each 32x32) of the stack factor.
 __global__ void __launch_bounds__(256) panel_stack_kernel(const float* __restrict__ Rall, int P, int nc, float* R,
-                                                          int64_t ldr, float* Qblocks, int* status, int col0) {
+                                                          int64_t ldr, float* Qblocks, int* status, int col0,
+                                                          const int* guard) {
+    if (guard && *guard == 0) return;
     __shared__ float qbuf[2 * PT];
     __shared__ float Rs[PNB][33];
     __shared__ int bad;
@@ -410,11 +415,14 @@ cudaError_t launch_panel(const PanelLaunch& pl, cudaStream_t st) {
     p.bf16 = pl.bf16;
     p.col0 = pl.col0;
     p.status = pl.status;
+    p.guard = pl.guard;
+    ++g_launches;
     panel_tile_kernel<<<p.ntiles, 256, 0, st>>>(p);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     if (pl.distributed) return cudaSuccess;  // caller gathers R, then calls launch_panel_apply
     if (p.levels > 0) {
+        ++g_launches;
         panel_apply_kernel<<<p.ntiles, 256, 0, st>>>(p, nullptr);
         e = cudaGetLastError();
     }
@@ -444,13 +452,16 @@ cudaError_t launch_panel_apply(const PanelLaunch& pl, const float* Gq, cudaStrea
         off += (int64_t)lvl_n[l - 1] * PNB * PNB;
     }
     p.bf16 = pl.bf16;
+    p.guard = pl.guard;
+    ++g_launches;
     panel_apply_kernel<<<p.ntiles, 256, 0, st>>>(p, Gq);
     return cudaGetLastError();
 }
 
 cudaError_t launch_panel_stack(const float* Rall, int P, int nc, float* R, int64_t ldr, float* Qblocks, int* status,
-                               int col0, cudaStream_t st) {
-    panel_stack_kernel<<<1, 256, 0, st>>>(Rall, P, nc, R, ldr, Qblocks, status, col0);
+                               int col0, const int* guard, cudaStream_t st) {
+    ++g_launches;
+    panel_stack_kernel<<<1, 256, 0, st>>>(Rall, P, nc, R, ldr, Qblocks, status, col0, guard);
     return cudaGetLastError();
 }
 

@@ -94,6 +94,7 @@ struct DevBuf {
         p = nullptr;
         bytes = 0;
         if (cudaMalloc(&p, b) != cudaSuccess) return false;
+        cudaMemset(p, 0, b);  // counters / flags rely on zero-initialised workspace
         bytes = b;
         return true;
     }
@@ -121,12 +122,13 @@ struct Plan {
     const float* A = nullptr;
     float* Q = nullptr;
     float* R = nullptr;
-    int nb = 0, bf16 = 0, split = 0, scale = 1, nranks = 1, rank = 0;
+    int nb = 0, bf16 = 0, split = 0, scale = 1, nranks = 1, rank = 0, panel = 0;
     int epoch = -1;          // g_alloc_epoch the plan was built against
     // derived
     int64_t ldh = 0, ldr12 = 0;
     std::vector<Op> ops;
     size_t p_floats = 0;
+    long long launches = 0;  // kernels per pass (counted while enqueueing)
     cudaGraphExec_t exec = nullptr;
 };
 
@@ -138,12 +140,17 @@ struct rg_handle_s {
     int rank = 0, nranks = 1;
     int64_t last_info = -1;
     // workspace
+    DevBuf cq_q1, cq_ws, cq_flags;                  // CholQR2 panel workspace (flags: counter, fail)
     DevBuf qh, ql, P, r12h, r12l, r12f, partial, norm2, scale, status, pws, pcnt, rgather, rstackq;
     DevBuf stageA, stageQ, stageR, stageB, stageX;  // host-pointer staging
     DevBuf cg;                                      // CGLS vectors
+    DevBuf lsQ, lsR, rinv, probeG, probeW;          // ls_solve_refined / orthogonalize workspace
+    cudaGraphExec_t cgls_exec = nullptr;            // captured block of CGLS iterations
+    const void* cgls_key[4] = {nullptr, nullptr, nullptr, nullptr};
+    int64_t cgls_key_mn[3] = {0, 0, 0};
     DevBuf aux;                                     // misc (orthogonalize / lowrank)
     int* status_host = nullptr;                     // pinned
-    int ws_generation = 0;
+    long long last_launches = 0;                    // kernels launched by the last API call
     std::unique_ptr<Plan> plan;
     // profiling
     bool prof = false;
@@ -327,7 +334,9 @@ bool ensure_workspace(rg_handle h, int64_t m, int64_t n, int split) {
               h->partial.ensure(rg::colnorm_partial_doubles(m, (int)n) * 8 + 64) && h->norm2.ensure(n * 8 + 64) &&
               h->scale.ensure(n * 4 + 64) && h->status.ensure(64) &&
               h->pws.ensure(rg::panel_ws_floats(m) * 4 + 4096) && h->pcnt.ensure(rg::panel_counters(m) * 4 + 64) &&
-              h->rgather.ensure((size_t)64 * 32 * 32 * 4) && h->rstackq.ensure((size_t)64 * 32 * 32 * 4);
+              h->rgather.ensure((size_t)64 * 32 * 32 * 4) && h->rstackq.ensure((size_t)64 * 32 * 32 * 4) &&
+              h->cq_q1.ensure((size_t)std::max<int64_t>(m, 8) * 32 * 4) &&
+              h->cq_ws.ensure(rg::cholqr_ws_doubles(m) * 8 + 256) && h->cq_flags.ensure(64);
     return ok;
 }
 
@@ -338,7 +347,14 @@ int nccl_allreduce(rg_handle h, void* buf, size_t count, ncclDataType_t t) {
 }
 
 // enqueue one RGSQR pass on h->stream (no sync).  A -> Q (may alias), R (ldr).
+int enqueue_rgsqr_impl(rg_handle h, Plan& pl);
 int enqueue_rgsqr(rg_handle h, Plan& pl) {
+    const long long before = rg::g_launches;
+    int rc = enqueue_rgsqr_impl(h, pl);
+    pl.launches = rg::g_launches - before;
+    return rc;
+}
+int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     cudaStream_t st = h->stream;
     const int64_t m = pl.m;
     const int n = (int)pl.n;
@@ -372,8 +388,38 @@ int enqueue_rgsqr(rg_handle h, Plan& pl) {
             p.bf16 = pl.bf16;
             p.col0 = o.c0;
             p.status = status;
+            float* Rdiag = pl.R + o.c0 + (int64_t)o.c0 * pl.ldr;
+            int* cq_fail = h->cq_flags.as<int>() + 1;
+            if (pl.panel == 0) {
+                // CholQR2 (fp64 Gram); the MGS/TSQR kernels below run only if a pivot failed
+                rg::CholqrLaunch c{};
+                c.P = p.Q;
+                c.ldp = pl.ldq;
+                c.Q1 = h->cq_q1.as<float>();
+                c.Q = p.Q;
+                c.ldq = pl.ldq;
+                c.Qh = p.Qh;
+                c.Ql = p.Ql;
+                c.ldh = pl.ldh;
+                c.m = m;
+                c.nc = o.w;
+                c.ws = h->cq_ws.as<double>();
+                c.counter = h->cq_flags.as<int>();
+                c.fail = cq_fail;
+                c.R = Rdiag;
+                c.ldr = pl.ldr;
+                c.bf16 = pl.bf16;
+                if (dist) {
+                    c.allreduce_g = [](double* G, void* ctx) {
+                        return nccl_allreduce(reinterpret_cast<rg_handle>(ctx), G, 1024, ncclFloat64);
+                    };
+                    c.ctx = h;
+                }
+                RG_CUDA(rg::launch_panel_cholqr(c, st));
+                p.guard = cq_fail;
+            }
             if (!dist) {
-                p.R = pl.R + o.c0 + (int64_t)o.c0 * pl.ldr;
+                p.R = Rdiag;
                 p.ldr = pl.ldr;
                 p.distributed = 0;
                 RG_CUDA(rg::launch_panel(p, st));
@@ -387,8 +433,7 @@ int enqueue_rgsqr(rg_handle h, Plan& pl) {
                 if (g_nccl.AllGather(p.R, rg_all, (size_t)o.w * o.w, ncclFloat32, h->comm, st) != ncclSuccess)
                     return RG_NCCL_ERROR;
                 float* qb = h->rstackq.as<float>();
-                RG_CUDA(rg::launch_panel_stack(rg_all, h->nranks, o.w, pl.R + o.c0 + (int64_t)o.c0 * pl.ldr, pl.ldr,
-                                               qb, status, o.c0, st));
+                RG_CUDA(rg::launch_panel_stack(rg_all, h->nranks, o.w, Rdiag, pl.ldr, qb, status, o.c0, p.guard, st));
                 RG_CUDA(rg::launch_panel_apply(p, qb + (int64_t)h->rank * 32 * 32, st));
             }
         } else if (o.kind == Op::PROJ) {
@@ -460,7 +505,7 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
     const bool same = pl && pl->m == m && pl->n == n && pl->lda == lda && pl->ldq == ldq && pl->ldr == ldr &&
                       pl->A == A && pl->Q == Q && pl->R == R && pl->nb == nb && pl->bf16 == o.precision &&
                       pl->split == split && pl->scale == o.scale && pl->nranks == h->nranks &&
-                      pl->rank == h->rank && pl->epoch == g_alloc_epoch;
+                      pl->rank == h->rank && pl->panel == o.panel && pl->epoch == g_alloc_epoch;
     if (!same) {
         if (pl && pl->exec) cudaGraphExecDestroy(pl->exec);
         h->plan.reset(new Plan());
@@ -468,7 +513,7 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
         pl->m = m; pl->n = n; pl->lda = lda; pl->ldq = ldq; pl->ldr = ldr;
         pl->A = A; pl->Q = Q; pl->R = R;
         pl->nb = nb; pl->bf16 = o.precision; pl->split = split; pl->scale = o.scale;
-        pl->nranks = h->nranks; pl->rank = h->rank;
+        pl->nranks = h->nranks; pl->rank = h->rank; pl->panel = o.panel;
         int rc = make_plan(h, *pl);
         if (rc) return rc;
         if (!h->P.ensure(pl->p_floats * 4 + 4096)) return RG_ALLOC;
@@ -476,8 +521,13 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
     }
     int rc = reset_status(h);
     if (rc) return rc;
+    h->last_launches += 0;
     const bool use_graph = !h->prof && getenv("RGSQR_NO_GRAPH") == nullptr;
-    if (!use_graph) return enqueue_rgsqr(h, *pl);
+    if (!use_graph) {
+        rc = enqueue_rgsqr(h, *pl);
+        h->last_launches += pl->launches;
+        return rc;
+    }
     if (!pl->exec) {
         // capture on the private stream (the user's may be the legacy stream, which cannot
         // capture); the instantiated graph is then launched on the user's stream
@@ -498,17 +548,102 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
         RG_CUDA(ie);
     }
     RG_CUDA(cudaGraphLaunch(pl->exec, h->stream));
+    h->last_launches += pl->launches;
     return RG_OK;
 }
 
 
+
+// R <- R2 R (both upper triangular n x n), via a scratch copy
+int trmm_into(rg_handle h, const float* R2, int64_t ld2, float* R, int64_t ldr, int n) {
+    if (!h->aux.ensure((size_t)n * n * 4 + 256)) return RG_ALLOC;
+    float* Rt = h->aux.as<float>();
+    RG_CUDA(rg::launch_trmm_upper(R2, ld2, R, ldr, Rt, n, n, h->stream));
+    RG_CUDA(cudaMemcpy2DAsync(R, ldr * 4, Rt, (size_t)n * 4, (size_t)n * 4, n, cudaMemcpyDeviceToDevice, h->stream));
+    return RG_OK;
+}
+
+// Hutchinson estimate of ||I - Q^T Q||_F with 8 fixed Philox probes (fp64), synchronous.
+int orth_estimate(rg_handle h, const float* Q, int64_t ldq, int64_t m, int n, double* est) {
+    const size_t pw = rg::probe_work_doubles(m, n, 8) + (size_t)n * 8 + 16;
+    if (!h->probeG.ensure((size_t)n * 8 * 8 + 64) || !h->probeW.ensure(pw * 8)) return RG_ALLOC;
+    double* G = h->probeG.as<double>();
+    double* Z = h->probeW.as<double>();
+    double* W = Z + (size_t)n * 8;
+    double* out = W + rg::probe_work_doubles(m, n, 8);
+    RG_CUDA(rg::launch_gaussian_philox((int64_t)n * 8, 0x5EEDCAFEULL, G, nullptr, h->stream));
+    RG_CUDA(rg::launch_orth_probe_z(Q, ldq, m, n, G, W, Z, h->stream));
+    int rc = nccl_allreduce(h, Z, (size_t)n * 8, ncclFloat64);
+    if (rc) return rc;
+    RG_CUDA(rg::launch_orth_probe_finish(Z, n, G, out, h->stream));
+    double v = 0;
+    RG_CUDA(cudaMemcpyAsync(&v, out, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    RG_CUDA(cudaStreamSynchronize(h->stream));
+    *est = sqrt(v);
+    return RG_OK;
+}
+
+// run RGSQR + `extra` split-precision reorthogonalisation passes; Q (ldq) and R (ldr) outputs
+int factor_with_reortho(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq, float* R,
+                        int64_t ldr, const rg_opts& o, int extra) {
+    int rc = run_rgsqr(h, m, n, A, lda, Q, ldq, R, ldr, o, o.split);
+    for (int p = 0; p < extra && rc == RG_OK; ++p) {
+        if (o.sync) {
+            rc = check_status(h);
+            if (rc) return rc;
+        }
+        if (!h->lsR.ensure((size_t)n * n * 4 + 256)) return RG_ALLOC;
+        float* R2 = h->lsR.as<float>();
+        rc = run_rgsqr(h, m, n, Q, ldq, Q, ldq, R2, n, o, 1);
+        if (rc) return rc;
+        rc = trmm_into(h, R2, n, R, ldr, (int)n);
+    }
+    return rc;
+}
+
+// CGLS iterations (Alg 3 corrected, readings #5-#7) on device vectors; R^{-1} explicit (fp64).
+int enqueue_cgls_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int n, int iters, double* base) {
+    cudaStream_t st = h->stream;
+    double* sc = base;
+    double* Rinv = h->rinv.as<double>();
+    double* x = sc + 16;
+    double* p = x + n;
+    double* s = p + n;
+    double* t = s + n;
+    double* sv = t + n;
+    double* r = sv + n;
+    double* q = r + m;
+    double* work = q + m;
+    const double* done = sc + 6;
+    for (int k = 0; k < iters; ++k) {
+        ProfScope _s(h, PC_CGLS, 4.0 * m * n, 8.0 * m * n);
+        RG_CUDA(rg::launch_trmv(Rinv, n, p, t, 0, done, st));                 // t = R \ p
+        RG_CUDA(rg::launch_gemv_n(A, lda, m, n, t, q, work, done, st));         // line 11: q = A t
+        RG_CUDA(rg::launch_sqnorm(q, m, sc, 1, st));                           // line 12: delta
+        int rc = nccl_allreduce(h, sc + 1, 1, ncclFloat64);
+        if (rc) return rc;
+        RG_CUDA(rg::launch_cgls_xr(x, t, r, q, m, n, sc, st));                 // lines 13-15
+        RG_CUDA(rg::launch_gemv_t(A, lda, m, n, r, sv, work, done, st));        // A^T r
+        rc = nccl_allreduce(h, sv, n, ncclFloat64);
+        if (rc) return rc;
+        RG_CUDA(rg::launch_trmv(Rinv, n, sv, s, 1, done, st));                // line 16: s = R^-T A^T r
+        RG_CUDA(rg::launch_cgls_p(s, p, n, sc, 0, st));                        // lines 17-21
+    }
+    return RG_OK;
+}
+
 }  // namespace
+
+namespace rg {
+thread_local long long g_launches = 0;
+}
 
 // ====================================================================== C-ABI
 extern "C" {
 
 void rg_opts_default(rg_opts* o) {
     if (!o) return;
+    o->panel = 0;
     o->precision = 0;
     o->nb = 32;
     o->scale = 1;
@@ -583,7 +718,10 @@ int rg_destroy(rg_handle h) {
     if (h->plan && h->plan->exec) cudaGraphExecDestroy(h->plan->exec);
     DevBuf* bufs[] = {&h->qh, &h->ql, &h->P, &h->r12h, &h->r12l, &h->r12f, &h->partial, &h->norm2, &h->scale,
                       &h->status, &h->pws, &h->pcnt, &h->rgather, &h->rstackq, &h->stageA, &h->stageQ,
-                      &h->stageR, &h->stageB, &h->stageX, &h->cg, &h->aux};
+                      &h->stageR, &h->stageB, &h->stageX, &h->cg, &h->aux,
+                      &h->lsQ, &h->lsR, &h->rinv, &h->probeG, &h->probeW, &h->cq_q1, &h->cq_ws,
+                      &h->cq_flags};
+    if (h->cgls_exec) cudaGraphExecDestroy(h->cgls_exec);
     for (auto* b : bufs) b->release();
     for (auto& e : h->ev_pool) {
         cudaEventDestroy(e.first);
@@ -597,6 +735,8 @@ int rg_destroy(rg_handle h) {
 }
 
 int64_t rg_last_info(rg_handle h) { return h ? h->last_info : -1; }
+
+int64_t rg_last_launches(rg_handle h) { return h ? (int64_t)h->last_launches : -1; }
 
 int rg_nccl_load(const char* path) {
     if (g_nccl.lib) return RG_OK;
@@ -689,6 +829,7 @@ int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_
     if (ldr < n) return -9;
     if (o.precision != 0 && o.precision != 1) return -10;
     cudaSetDevice(h->device);
+    h->last_launches = 0;
     const bool host = ptr_side(A) == SIDE_HOST;
     if (host && (ptr_side(Q) != SIDE_HOST || ptr_side(R) != SIDE_HOST)) return -6;
     const float* dA = A;
@@ -732,6 +873,194 @@ int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_
     if (o.sync || host) rc = check_status(h);
     prof_collect(h);
     return rc;
+}
+
+
+int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda, float* R, int64_t ldr,
+                  double orth_tol, int max_passes, int* passes_out, double* orth_est_out, const rg_opts* opts) {
+    if (!h) return -1;
+    rg_opts o;
+    if (opts) o = *opts; else rg_opts_default(&o);
+    if (m_local < 1 || (h->nranks <= 1 && m_local < n)) return -2;
+    if (n < 1 || n > 65535) return -3;
+    if (!A) return -4;
+    if (lda < m_local) return -5;
+    if (R && ldr < n) return -7;
+    if (max_passes < 1) return -9;
+    cudaSetDevice(h->device);
+    h->last_launches = 0;
+    const bool host = ptr_side(A) == SIDE_HOST;
+    float* dA = A;
+    int64_t dlda = lda;
+    if (host) {
+        if (!h->stageQ.ensure((size_t)m_local * n * 4)) return RG_ALLOC;
+        dA = h->stageQ.as<float>();
+        dlda = m_local;
+        RG_CUDA(cudaMemcpy2DAsync(dA, m_local * 4, A, lda * 4, m_local * 4, n, cudaMemcpyHostToDevice, h->stream));
+    }
+    if (!h->stageR.ensure((size_t)n * n * 4 + 256)) return RG_ALLOC;
+    float* dR = h->stageR.as<float>();   // accumulated R (n x n, ld n)
+    int rc = run_rgsqr(h, m_local, n, dA, dlda, dA, dlda, dR, n, o, o.split);
+    int passes = 1;
+    double est = -1.0;
+    while (rc == RG_OK && passes < max_passes) {
+        if (o.sync || orth_tol > 0) {
+            rc = check_status(h);
+            if (rc) break;
+        }
+        if (orth_tol > 0) {
+            rc = orth_estimate(h, dA, dlda, m_local, (int)n, &est);
+            if (rc || est <= orth_tol) break;
+        }
+        // [Q2, R2] = RGSQR(Q) with split-precision GEMMs (reading #9); R <- R2 R
+        if (!h->lsR.ensure((size_t)n * n * 4 + 256)) return RG_ALLOC;
+        float* R2 = h->lsR.as<float>();
+        rc = run_rgsqr(h, m_local, n, dA, dlda, dA, dlda, R2, n, o, 1);
+        if (rc) break;
+        rc = trmm_into(h, R2, n, dR, n, (int)n);
+        ++passes;
+        est = -1.0;
+    }
+    if (rc) return rc;
+    if (o.sync || host || orth_tol > 0 || orth_est_out) rc = check_status(h);
+    if (rc) return rc;
+    if ((orth_tol > 0 || orth_est_out) && est < 0) {
+        rc = orth_estimate(h, dA, dlda, m_local, (int)n, &est);
+        if (rc) return rc;
+    }
+    if (R) RG_CUDA(cudaMemcpy2DAsync(R, ldr * 4, dR, n * 4, n * 4, n,
+                                     host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, h->stream));
+    if (host)
+        RG_CUDA(cudaMemcpy2DAsync(A, lda * 4, dA, dlda * 4, m_local * 4, n, cudaMemcpyDeviceToHost, h->stream));
+    if (host || o.sync) RG_CUDA(cudaStreamSynchronize(h->stream));
+    if (passes_out) *passes_out = passes;
+    if (orth_est_out) *orth_est_out = est;
+    prof_collect(h);
+    if (orth_tol > 0 && est > orth_tol) return RG_NOT_CONVERGED;
+    return RG_OK;
+}
+
+int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_t lda, const float* b, double* x,
+                     double tol, int maxit, int* iters_out, double* relres_out, const rg_opts* opts) {
+    if (!h) return -1;
+    rg_opts o;
+    if (opts) o = *opts; else rg_opts_default(&o);
+    if (m_local < 1 || (h->nranks <= 1 && m_local < n)) return -2;
+    if (n < 1 || n > 16384) return -3;
+    if (!A) return -4;
+    if (lda < m_local) return -5;
+    if (!b) return -6;
+    if (!x) return -7;
+    if (!(tol >= 0)) return -8;
+    if (maxit < 0) return -9;
+    cudaSetDevice(h->device);
+    h->last_launches = 0;
+    const bool host = ptr_side(A) == SIDE_HOST;
+    const float* dA = A;
+    const float* db = b;
+    int64_t dlda = lda;
+    if (host) {
+        if (!h->stageA.ensure((size_t)m_local * n * 4) || !h->stageB.ensure((size_t)m_local * 4 + 64)) return RG_ALLOC;
+        RG_CUDA(cudaMemcpy2DAsync(h->stageA.p, m_local * 4, A, lda * 4, m_local * 4, n, cudaMemcpyHostToDevice,
+                                  h->stream));
+        RG_CUDA(cudaMemcpyAsync(h->stageB.p, b, m_local * 4, cudaMemcpyHostToDevice, h->stream));
+        dA = h->stageA.as<float>();
+        db = h->stageB.as<float>();
+        dlda = m_local;
+    }
+    // ---- QR preconditioner: RGSQR (+ reortho passes, reading #8)
+    if (!h->lsQ.ensure((size_t)m_local * n * 4) || !h->stageR.ensure((size_t)n * n * 4 + 256)) return RG_ALLOC;
+    float* Qw = h->lsQ.as<float>();
+    float* Rw = h->stageR.as<float>();
+    const int extra = o.reortho < 0 ? 1 : o.reortho;
+    int rc = factor_with_reortho(h, m_local, n, dA, dlda, Qw, m_local, Rw, n, o, extra);
+    if (rc) return rc;
+    rc = check_status(h);
+    if (rc) return rc;
+    // ---- explicit R^{-1} (fp64)
+    if (!h->rinv.ensure((size_t)n * n * 8 + 64)) return RG_ALLOC;
+    RG_CUDA(rg::launch_trinv_upper(Rw, n, (int)n, h->rinv.as<double>(), h->stream));
+    // ---- CGLS state: sc[16] | x p s t sv (n each) | r q (m each) | gemv work
+    const size_t work = std::max(rg::gemv_n_work_doubles(m_local, (int)n), rg::gemv_t_work_doubles(m_local, (int)n));
+    if (!h->cg.ensure((16 + 5 * (size_t)n + 2 * (size_t)m_local + work) * 8 + 256)) return RG_ALLOC;
+    double* base = h->cg.as<double>();
+    double* sc = base;
+    double* xd = sc + 16;
+    double* p = xd + n;
+    double* s = p + n;
+    double* sv = s + 2 * n;
+    double* r = sv + n;
+    double* wk = r + 2 * m_local;
+    {
+        double init[16] = {0};
+        init[8] = tol;
+        RG_CUDA(cudaMemcpyAsync(sc, init, sizeof(init), cudaMemcpyHostToDevice, h->stream));
+    }
+    RG_CUDA(rg::launch_cgls_init(db, m_local, (int)n, r, xd, h->stream));          // lines 4-5
+    RG_CUDA(rg::launch_gemv_t(dA, dlda, m_local, (int)n, r, sv, wk, nullptr, h->stream));
+    rc = nccl_allreduce(h, sv, n, ncclFloat64);
+    if (rc) return rc;
+    RG_CUDA(rg::launch_trmv(h->rinv.as<double>(), (int)n, sv, s, 1, nullptr, h->stream));  // line 6 (corrected)
+    RG_CUDA(rg::launch_cgls_p(s, p, (int)n, sc, 1, h->stream));                    // lines 7-9
+    // ---- iterations in captured blocks of `blk`, convergence flag read between blocks
+    const int blk = 8;
+    int done_iters = 0;
+    double hsc[16];
+    const bool use_graph = !h->prof && getenv("RGSQR_NO_GRAPH") == nullptr;
+    while (done_iters < maxit) {
+        const int cnt = std::min(blk, maxit - done_iters);
+        if (use_graph && cnt == blk) {
+            const bool same = h->cgls_exec && h->cgls_key[0] == dA && h->cgls_key[1] == base &&
+                              h->cgls_key[2] == h->rinv.p && h->cgls_key_mn[0] == m_local && h->cgls_key_mn[1] == n &&
+                              h->cgls_key_mn[2] == dlda;
+            if (!same) {
+                if (h->cgls_exec) cudaGraphExecDestroy(h->cgls_exec);
+                h->cgls_exec = nullptr;
+                cudaGraph_t g;
+                cudaStream_t user = h->stream;
+                h->stream = h->capture_stream;
+                RG_CUDA(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
+                const long long before = rg::g_launches;
+                rc = enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, blk, base);
+                h->cgls_key_mn[2] = dlda;
+                cudaError_t ce = cudaStreamEndCapture(h->stream, &g);
+                h->stream = user;
+                if (rc) return rc;
+                RG_CUDA(ce);
+                cudaError_t ie = cudaGraphInstantiate(&h->cgls_exec, g, 0);
+                cudaGraphDestroy(g);
+                RG_CUDA(ie);
+                h->cgls_key[0] = dA;
+                h->cgls_key[1] = base;
+                h->cgls_key[2] = h->rinv.p;
+                h->cgls_key_mn[0] = m_local;
+                h->cgls_key_mn[1] = n;
+                h->cgls_key[3] = (const void*)(intptr_t)(rg::g_launches - before);
+            }
+            RG_CUDA(cudaGraphLaunch(h->cgls_exec, h->stream));
+            h->last_launches += (long long)(intptr_t)h->cgls_key[3];
+        } else {
+            const long long before = rg::g_launches;
+            rc = enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, cnt, base);
+            h->last_launches += rg::g_launches - before;
+            if (rc) return rc;
+        }
+        done_iters += cnt;
+        RG_CUDA(cudaMemcpyAsync(hsc, sc, sizeof(hsc), cudaMemcpyDeviceToHost, h->stream));
+        RG_CUDA(cudaStreamSynchronize(h->stream));
+        if (hsc[6] != 0.0) break;
+    }
+    if (done_iters == 0) {
+        RG_CUDA(cudaMemcpyAsync(hsc, sc, sizeof(hsc), cudaMemcpyDeviceToHost, h->stream));
+        RG_CUDA(cudaStreamSynchronize(h->stream));
+    }
+    RG_CUDA(cudaMemcpyAsync(x, xd, n * 8, host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, h->stream));
+    RG_CUDA(cudaStreamSynchronize(h->stream));
+    if (iters_out) *iters_out = (int)hsc[7];
+    if (relres_out) *relres_out = hsc[4] > 0 ? hsc[5] / hsc[4] : 0.0;
+    prof_collect(h);
+    if (!(hsc[6] != 0.0) && maxit > 0 && !(hsc[5] <= tol * hsc[4])) return RG_NOT_CONVERGED;
+    return RG_OK;
 }
 
 }  // extern "C"

@@ -159,15 +159,18 @@ cudaError_t launch_colnorm(const float* A, int64_t lda, int64_t m, int n, double
                            cudaStream_t st) {
     const int chunks = (int)((m + kNormChunk - 1) / kNormChunk);
     dim3 grid(n, chunks);
+    ++g_launches;
     colnorm_partial_kernel<<<grid, 256, 0, st>>>(A, lda, m, n, partial);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
+    ++g_launches;
     colnorm_sum_kernel<<<(n + 127) / 128, 128, 0, st>>>(partial, chunks, n, norm2);
     return cudaGetLastError();
 }
 
 cudaError_t launch_colscale(const double* norm2, int n, int do_scale, float* scale, int* status, int col0,
                             cudaStream_t st) {
+    ++g_launches;
     colscale_kernel<<<(n + 127) / 128, 128, 0, st>>>(norm2, n, do_scale, scale, status, col0);
     return cudaGetLastError();
 }
@@ -184,6 +187,7 @@ cudaError_t launch_scale_cast(const float* A, int64_t lda, float* Q, int64_t ldq
     int bx = (int)(per_col < target ? per_col : target);
     if (bx < 1) bx = 1;
     dim3 grid(bx, n);
+    ++g_launches;
     scale_cast_kernel<<<grid, 256, 0, st>>>(A, lda, Q, ldq, Qh, Ql, ldh, m, n, scale, bf16);
     return cudaGetLastError();
 }
@@ -192,6 +196,7 @@ cudaError_t launch_unscale_r(float* R, int64_t ldr, int n, const float* scale, c
     const int64_t total = (int64_t)n * n;
     int blocks = (int)((total + 255) / 256);
     if (blocks > 148 * 8) blocks = 148 * 8;
+    ++g_launches;
     unscale_r_kernel<<<blocks, 256, 0, st>>>(R, ldr, n, scale);
     return cudaGetLastError();
 }

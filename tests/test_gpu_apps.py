@@ -1,0 +1,93 @@
+"""GPU parity of ls_solve_refined and orthogonalize (C-ABI) against the fp64 oracle (-m gpu).
+
+Tolerances (north_star): refined LS ||x - x*||/||x*|| <= 1e-5 for cond <= 1e4 (x* = the
+oracle's solution of the fp32-rounded problem); orthogonality <= 1e-5 after
+reorthogonalisation.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def rg():
+    import paper_conf_hpdc_zhangbw20_b200 as rg
+    return rg
+
+
+def _dev(A):
+    return torch.from_numpy(np.ascontiguousarray(np.asarray(A, dtype=np.float32).T)).cuda().t()
+
+
+@pytest.mark.parametrize("kind,kappa", [("geometric", 1e2), ("geometric", 1e4), ("arithmetic", 1e4),
+                                        ("cluster", 1e4)])
+@pytest.mark.parametrize("consistent", [False, True])
+def test_ls_refined_parity(rg, kind, kappa, consistent):
+    m, n = 8192, 256
+    A = synth.svd_matrix(m, n, kind, kappa, seed=31).astype(np.float32)
+    b = synth.rhs(A.astype(np.float64), seed=31, consistent=consistent).astype(np.float32)
+    x_star, _ = oracle.ls_qr(A.astype(np.float64), b.astype(np.float64))
+    x = torch.zeros(n, dtype=torch.float64, device="cuda")
+    x, it, rel, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), x, tol=1e-10, maxit=200)
+    xe = x.cpu().numpy()
+    fe = np.linalg.norm(xe - x_star) / np.linalg.norm(x_star)
+    assert st == rg.RG_OK, (st, it, rel)
+    assert fe <= 1e-5, (fe, it)
+    assert it <= 60   # reortho'd R: kappa(A R^-1) ~ 1 (reading #8; SURVEY [EMU] ~10-18)
+
+
+def test_ls_refined_4x2_closed_form(rg):
+    A = np.array([[1, 1], [1, 2], [1, 3], [1, 4]], dtype=np.float32)
+    b = np.array([1, 3, 2, 5], dtype=np.float32)
+    x, it, rel, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), tol=1e-13)
+    np.testing.assert_allclose(x.cpu().numpy(), [0.0, 1.1], atol=1e-9)
+
+
+def test_ls_host_pointers(rg):
+    A = np.asfortranarray(synth.svd_matrix(4096, 64, "geometric", 1e3, seed=2).astype(np.float32))
+    b = synth.rhs(A.astype(np.float64), seed=2, consistent=False).astype(np.float32)
+    x = np.zeros(64)
+    x, it, rel, st = rg.ls_solve_refined(A, b, x)
+    x_star, _ = oracle.ls_qr(A.astype(np.float64), b.astype(np.float64))
+    assert np.linalg.norm(x - x_star) / np.linalg.norm(x_star) <= 1e-5
+
+
+def test_ls_paper_faithful_mode_converges_slower(rg):
+    """reortho = 0 (paper-faithful, one RGSQR pass): CGLS still converges, with more iterations."""
+    A = synth.svd_matrix(8192, 128, "geometric", 1e4, seed=5).astype(np.float32)
+    b = synth.rhs(A.astype(np.float64), seed=5, consistent=True).astype(np.float32)
+    _, it0, _, st0 = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), opts=rg.make_opts(reortho=0),
+                                         maxit=400)
+    _, it1, _, st1 = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), opts=rg.make_opts(reortho=1))
+    assert st1 == rg.RG_OK
+    assert it1 <= it0
+
+
+@pytest.mark.parametrize("kappa", [1.0, 1e3, 1e4])
+def test_orthogonalize_parity(rg, kappa):
+    m, n = 16384, 256
+    A = (synth.gaussian(m, n, seed=7) if kappa == 1.0 else
+         synth.svd_matrix(m, n, "geometric", kappa, seed=7)).astype(np.float32)
+    Ad = _dev(A)
+    R = torch.zeros(n, n, device="cuda").t()
+    Q, R, passes, est = rg.orthogonalize(Ad, R, orth_tol=1e-5, max_passes=3)
+    Qn = Q.cpu().numpy().astype(np.float64)
+    orth = oracle.orthogonality(Qn)
+    assert orth <= 1e-5, (orth, passes, est)
+    be = oracle.backward_error(A.astype(np.float64), Qn, R.cpu().numpy().astype(np.float64))
+    assert be <= 5e-3
+    assert 1 <= passes <= 3
+    assert abs(est - orth) <= 0.5 * orth + 1e-7   # Hutchinson estimate is close
+
+
+def test_orthogonalize_fixed_two_passes(rg):
+    A = synth.gaussian(2 ** 16, 256, seed=8).astype(np.float32)
+    Ad = _dev(A)
+    Q, _, passes, est = rg.orthogonalize(Ad, None, orth_tol=0.0, max_passes=2)
+    assert passes == 2
+    assert oracle.orthogonality(Q.cpu().numpy().astype(np.float64)) <= 1e-5

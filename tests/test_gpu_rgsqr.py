@@ -49,12 +49,23 @@ def _check_qr(A32, Q, R, kappa=10.0, orth_scale=1e-2):
     return be, orth, dr
 
 
+@pytest.mark.parametrize("panel", ["auto", "mgs"])
 @pytest.mark.parametrize("m,n", [(64, 1), (100, 7), (256, 32), (1000, 32), (1024, 64), (1025, 96), (4099, 64),
-                                 (3000, 200), (8192, 256), (777, 333)])
-def test_rgsqr_gaussian_parity(rg, m, n):
+                                 (3000, 200), (8192, 256), (777, 333), (70000, 40)])
+def test_rgsqr_gaussian_parity(rg, m, n, panel):
     A = synth.gaussian(m, n, seed=synth.SEED_BASE + m + n).astype(np.float32)
-    Q, R = _run(rg, A)
+    Q, R = _run(rg, A, panel=panel)
     _check_qr(A, Q, R, kappa=np.linalg.cond(A))
+
+
+@pytest.mark.parametrize("kappa", [1e2, 1e4, 1e6])
+def test_rgsqr_ill_conditioned_backward_error(rg, kappa):
+    """Backward error independent of cond(A) (Fig 3); orthogonality grows ~kappa u_h."""
+    A = synth.svd_matrix(4096, 128, "geometric", kappa, seed=21).astype(np.float32)
+    Q, R = _run(rg, A)
+    A64 = A.astype(np.float64)
+    assert oracle.backward_error(A64, Q, R) < 5e-3
+    assert np.all(np.diag(R) > 0)
 
 
 def test_rgsqr_config1(rg):
@@ -65,10 +76,11 @@ def test_rgsqr_config1(rg):
     assert be < 2e-4  # fp16 updates, fp32 panel: SURVEY [EMU] ~4e-5
 
 
-def test_rgsqr_single_panel_is_fp32_accurate(rg):
-    """n <= 32: the whole call is one fp32 TSQR/MGS panel (no tensor cores)."""
+@pytest.mark.parametrize("panel", ["auto", "mgs"])
+def test_rgsqr_single_panel_is_fp32_accurate(rg, panel):
+    """n <= 32: the whole call is one fp32 panel (no tensor cores)."""
     A = synth.gaussian(5000, 32, seed=3).astype(np.float32)
-    Q, R = _run(rg, A)
+    Q, R = _run(rg, A, panel=panel)
     A64 = A.astype(np.float64)
     assert oracle.backward_error(A64, Q, R) < 1e-6
     assert oracle.orthogonality(Q) < 1e-5
