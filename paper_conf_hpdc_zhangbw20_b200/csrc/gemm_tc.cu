@@ -5,14 +5,19 @@
 //
 // fp16 (or bf16) operands, fp32 accumulation in TMEM (reading #3), issued
 // with tcgen05.mma by one thread, operands staged by TMA into 128B-swizzled shared memory
-// through an mbarrier ring.  K1 is split over m (deterministic two-stage reduction, no
-// float atomics, reading #19); K2 fuses the fp32 read-modify-write of A2 and the fp16
-// shadow write of the updated A2 into the TMEM epilogue.
+// through an mbarrier ring.  Persistent, warp-specialised kernel:
+//   warp 0      TMA producer            warp 1   MMA issuer (one elected lane)
+//   warp 2      TMEM allocator          warp 3   idle
+//   warps 4..   epilogue warpgroup(s): TMEM -> registers -> per-warp smem transpose ->
+//               16-byte global accesses (4 consecutive rows of one column per lane)
+// Two TMEM accumulator buffers (when they fit) let the epilogue of one tile overlap the
+// MMAs of the next.  K1 is split over m with a deterministic two-stage reduction (no float
+// atomics, reading #19); K2 fuses the fp32 read-modify-write of A2 and the 16-bit shadow
+// write of the updated A2 into the epilogue.
 //
-// Split precision (reading #9, used by reorthogonalisation passes): each operand X is held
-// as hi = fp16(X) and lo = fp16((X - hi) * 2^11); the kernels then issue three MMA groups
-// hi*hi into accumulator 0 and hi*lo + lo*hi into accumulator 1 and combine
-// D = D0 + D1 * 2^-11 in the epilogue.
+// Split precision (reading #9, reorthogonalisation passes): operands are held as
+// hi = fp16(X) and lo = fp16((X - hi) 2^11); three MMA groups accumulate hi*hi into
+// accumulator 0 and hi*lo + lo*hi into accumulator 1; D = D0 + 2^-11 D1 in the epilogue.
 #include <cuda.h>
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
@@ -26,25 +31,30 @@ namespace rg {
 constexpr int kBM = 128;    // UMMA M (rows of the accumulator = TMEM lanes)
 constexpr int kBK = 64;     // k extent of one pipeline stage (one 128B swizzle row of fp16)
 constexpr int kUK = 16;     // UMMA K for kind::f16
-constexpr int kThreads = 128;
+constexpr int kEpiLd = 36;  // per-warp transpose buffer row stride (floats, 16B aligned)
 
-template <int BN, int STAGES, bool SPLIT>
-struct GemmSmem {
+template <int BN, int STAGES, bool SPLIT, int EPI_WG>
+struct GemmCfg {
     static constexpr int kABytes = kBM * kBK * 2;           // 16 KB
     static constexpr int kBBytes = BN * kBK * 2;
     static constexpr int kOps = SPLIT ? 2 : 1;               // hi (+ lo) copies of each operand
     static constexpr int kStageBytes = kOps * (kABytes + kBBytes);
     static constexpr int kDataBytes = STAGES * kStageBytes;
-    static constexpr int kBarOffset = kDataBytes;
-    static constexpr int kTotal = kDataBytes + 1024 /*barriers*/ + 1024 /*alignment slack*/;
-};
-
-template <int N>
-struct TmemCols {
-    static constexpr uint32_t value = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : N <= 256 ? 256 : 512;
+    static constexpr int kEpiWarps = 4 * EPI_WG;
+    static constexpr int kEpiBytes = kEpiWarps * 32 * kEpiLd * 4;
+    static constexpr int kBarOffset = kDataBytes + kEpiBytes;
+    static constexpr int kTotal = kBarOffset + 512 + 1024;   // barriers + 1 KB alignment slack
+    static constexpr int kThreads = 128 + 32 * kEpiWarps;
+    static constexpr int kAccCols = SPLIT ? 2 * BN : BN;
+    static constexpr int kAcc = (2 * kAccCols <= 512) ? 2 : 1;  // TMEM accumulator buffers
+    static constexpr uint32_t kTmemCols = (kAcc * kAccCols <= 32) ? 32 : (kAcc * kAccCols <= 64) ? 64
+                                        : (kAcc * kAccCols <= 128) ? 128 : (kAcc * kAccCols <= 256) ? 256 : 512;
 };
 
 struct GemmArgs {
+    // work decomposition
+    int units;             // total work units
+    int tiles_i, tiles_j;  // output tiles (MODE 0: i = Q1 col tiles; MODE 1: i = row tiles)
     // K1 (projection): partial output P[z][j*ldp + i], K range in 64-row blocks
     float* P;
     int64_t ldp;           // leading dim of one partial (>= padded h)
@@ -61,6 +71,8 @@ struct GemmArgs {
     int w;
     int kb_h;              // ceil(h / 64)
     int bf16;
+    int vec_ok;            // C / Ch / Cl accesses may use 16-byte (8-byte) vectors
+    int overwrite;         // K2 only: C = D instead of C -= D (plain product, lowrank_approx)
 };
 
 __device__ __forceinline__ uint16_t f2h_bits(float x, int bf16) {
@@ -80,33 +92,44 @@ __device__ __forceinline__ float h2f_bits(uint16_t u, int bf16) {
     return __half2float(h);
 }
 
-// MODE 0 = K1 projection (A, B K-major; grid = (tiles_i, tiles_j, splits))
-// MODE 1 = K2 update     (A MN-major, B K-major; grid = (row tiles, col tiles))
-template <int MODE, int BN, int STAGES, bool SPLIT>
-__global__ void __launch_bounds__(kThreads, 1)
+// unit -> (t0 = first row of the M tile, tj = N tile index, z = split, [kb0, kb1))
+template <int MODE>
+__device__ __forceinline__ void unit_coords(const GemmArgs& a, int u, int& t0, int& tj, int& z, int& kb0, int& kb1) {
+    if (MODE == 0) {
+        const int tiles = a.tiles_i * a.tiles_j;
+        z = u / tiles;
+        const int rem = u % tiles;
+        t0 = (rem % a.tiles_i) * kBM;
+        tj = rem / a.tiles_i;
+        kb0 = z * a.kb_per_split;
+        kb1 = min(kb0 + a.kb_per_split, a.kb_total);
+    } else {
+        z = 0;
+        t0 = (u / a.tiles_j) * kBM;
+        tj = u % a.tiles_j;
+        kb0 = 0;
+        kb1 = a.kb_h;
+    }
+}
+
+// MODE 0 = K1 projection (A, B K-major), MODE 1 = K2 update (A MN-major, B K-major)
+template <int MODE, int BN, int STAGES, bool SPLIT, int EPI_WG>
+__global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const __grid_constant__ CUtensorMap tmA_lo, const __grid_constant__ CUtensorMap tmB_lo,
                    GemmArgs args) {
-    using L = GemmSmem<BN, STAGES, SPLIT>;
-    constexpr uint32_t kTmemCols = TmemCols<(SPLIT ? 2 : 1) * BN>::value;
+    using C = GemmCfg<BN, STAGES, SPLIT, EPI_WG>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint64_t* full_bar = reinterpret_cast<uint64_t*>(smem + L::kBarOffset);
+    float* epi_buf = reinterpret_cast<float*>(smem + C::kDataBytes);
+    uint64_t* full_bar = reinterpret_cast<uint64_t*>(smem + C::kBarOffset);
     uint64_t* empty_bar = full_bar + STAGES;
-    uint64_t* accum_bar = empty_bar + STAGES;
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(accum_bar + 1);
+    uint64_t* tfull_bar = empty_bar + STAGES;
+    uint64_t* tempty_bar = tfull_bar + 2;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty_bar + 2);
 
     const int warp = threadIdx.x >> 5;
-    int kb_begin, kb_end;
-    if (MODE == 0) {
-        kb_begin = blockIdx.z * args.kb_per_split;
-        kb_end = min(kb_begin + args.kb_per_split, args.kb_total);
-    } else {
-        kb_begin = 0;
-        kb_end = args.kb_h;
-    }
-    const int tile0 = blockIdx.x * kBM;   // i (K1: Q1 column) or r (K2: row)
-    const int tile1 = blockIdx.y * BN;    // j (A2 column)
+    const int lane = threadIdx.x & 31;
 
     if (threadIdx.x == 0) {
         tma_prefetch_desc(&tmA);
@@ -119,155 +142,246 @@ __global__ void __launch_bounds__(kThreads, 1)
             mbar_init(&full_bar[s], 1);
             mbar_init(&empty_bar[s], 1);
         }
-        mbar_init(accum_bar, 1);
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(&tfull_bar[a], 1);
+            mbar_init(&tempty_bar[a], C::kEpiWarps);
+        }
         fence_barrier_init();
     }
-    if (warp == 2) tmem_alloc<kTmemCols>(tmem_slot);
+    if (warp == 2) tmem_alloc<C::kTmemCols>(tmem_slot);
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
-    if (warp == 0 && elect_one()) {
-        // ---------------- TMA producer
-        for (int kb = kb_begin; kb < kb_end; ++kb) {
-            const int it = kb - kb_begin;
-            const int s = it % STAGES;
-            const uint32_t round = it / STAGES;
-            mbar_wait(&empty_bar[s], (round & 1u) ^ 1u);
-            uint8_t* sa = smem + s * L::kStageBytes;
-            uint8_t* sb = sa + L::kABytes;
-            mbar_arrive_expect_tx(&full_bar[s], L::kStageBytes);
-            if (MODE == 0) {
-                tma_load_2d(sa, &tmA, &full_bar[s], kb * kBK, tile0);
-                tma_load_2d(sb, &tmB, &full_bar[s], kb * kBK, tile1);
-                if (SPLIT) {
-                    tma_load_2d(sb + L::kBBytes, &tmA_lo, &full_bar[s], kb * kBK, tile0);
-                    tma_load_2d(sb + L::kBBytes + L::kABytes, &tmB_lo, &full_bar[s], kb * kBK, tile1);
-                }
-            } else {
-                // MN-major A: two 64(row) x 64(k) boxes, the second at +8 KB (LBO)
-                tma_load_2d(sa, &tmA, &full_bar[s], tile0, kb * kBK);
-                tma_load_2d(sa + L::kABytes / 2, &tmA, &full_bar[s], tile0 + 64, kb * kBK);
-                tma_load_2d(sb, &tmB, &full_bar[s], kb * kBK, tile1);
-                if (SPLIT) {
-                    uint8_t* sal = sb + L::kBBytes;
-                    tma_load_2d(sal, &tmA_lo, &full_bar[s], tile0, kb * kBK);
-                    tma_load_2d(sal + L::kABytes / 2, &tmA_lo, &full_bar[s], tile0 + 64, kb * kBK);
-                    tma_load_2d(sal + L::kABytes, &tmB_lo, &full_bar[s], kb * kBK, tile1);
-                }
-            }
-        }
-    } else if (warp == 1 && elect_one()) {
-        // ---------------- MMA issuer (single thread)
-        const uint32_t idesc = umma_idesc_f16(kBM, BN, MODE == 1 ? 1u : 0u, 0u, (uint32_t)args.bf16);
-        for (int kb = kb_begin; kb < kb_end; ++kb) {
-            const int it = kb - kb_begin;
-            const int s = it % STAGES;
-            const uint32_t round = it / STAGES;
-            mbar_wait(&full_bar[s], round & 1u);
-            tc_fence_after();
-            const uint32_t sa = smem_u32(smem + s * L::kStageBytes);
-            const uint32_t sb = sa + L::kABytes;
-            const uint32_t sal = sb + L::kBBytes;
-            const uint32_t sbl = sal + L::kABytes;
-#pragma unroll
-            for (int kk = 0; kk < kBK / kUK; ++kk) {
-                uint64_t ad, adl;
-                if (MODE == 0) {
-                    ad = umma_desc_sw128(sa + kk * 32, 16, 1024);
-                    adl = umma_desc_sw128(sal + kk * 32, 16, 1024);
-                } else {
-                    ad = umma_desc_sw128(sa + kk * 2048, L::kABytes / 2, 1024);
-                    adl = umma_desc_sw128(sal + kk * 2048, L::kABytes / 2, 1024);
-                }
-                const uint64_t bd = umma_desc_sw128(sb + kk * 32, 16, 1024);
-                const uint32_t acc = (it > 0 || kk > 0) ? 1u : 0u;
-                umma_f16(tmem_base, ad, bd, idesc, acc);
-                if (SPLIT) {
-                    const uint64_t bdl = umma_desc_sw128(sbl + kk * 32, 16, 1024);
-                    umma_f16(tmem_base + BN, ad, bdl, idesc, acc);   // hi * lo
-                    umma_f16(tmem_base + BN, adl, bd, idesc, 1u);    // lo * hi
-                }
-            }
-            umma_commit(&empty_bar[s]);
-        }
-        umma_commit(accum_bar);
-    }
-
-    // ---------------- epilogue: all 4 warps, thread <-> accumulator row (TMEM lane)
-    __syncwarp();
-    mbar_wait(accum_bar, 0);
-    tc_fence_after();
-    const int row = warp * 32 + (threadIdx.x & 31);
-    const uint32_t lane_addr = tmem_base + (static_cast<uint32_t>(warp * 32) << 16);
-    const bool empty_range = kb_end <= kb_begin;
-#pragma unroll 1
-    for (int c = 0; c < BN; c += 32) {
-        uint32_t v[32];
-        tmem_ld32(lane_addr + c, v);
-        float d[32];
-        tmem_ld_wait();
-#pragma unroll
-        for (int jj = 0; jj < 32; ++jj) d[jj] = empty_range ? 0.f : __uint_as_float(v[jj]);
-        if (SPLIT) {
-            uint32_t u[32];
-            tmem_ld32(lane_addr + BN + c, u);
-            tmem_ld_wait();
-#pragma unroll
-            for (int jj = 0; jj < 32; ++jj)
-                d[jj] += empty_range ? 0.f : __uint_as_float(u[jj]) * (1.0f / 2048.0f);
-        }
-        if (MODE == 0) {
-            float* out = args.P + blockIdx.z * args.p_stride + (int64_t)(tile1 + c) * args.ldp + tile0 + row;
-#pragma unroll
-            for (int jj = 0; jj < 32; ++jj) out[(int64_t)jj * args.ldp] = d[jj];
-        } else {
-            const int64_t r = (int64_t)tile0 + row;
-            if (r < args.m) {
-                float* cp = args.C + r;
-                float old[32];
-#pragma unroll
-                for (int jj = 0; jj < 32; ++jj) {
-                    const int j = tile1 + c + jj;
-                    old[jj] = (j < args.w) ? cp[(int64_t)j * args.ldc] : 0.f;
-                }
-#pragma unroll
-                for (int jj = 0; jj < 32; ++jj) {
-                    const int j = tile1 + c + jj;
-                    if (j < args.w) {
-                        const float nv = old[jj] - d[jj];
-                        cp[(int64_t)j * args.ldc] = nv;
-                        if (args.Ch) {
-                            const uint16_t hb = f2h_bits(nv, args.bf16);
-                            reinterpret_cast<uint16_t*>(args.Ch)[r + (int64_t)j * args.ldh] = hb;
-                            if (args.Cl) {
-                                const float lo = (nv - h2f_bits(hb, args.bf16)) * 2048.0f;
-                                reinterpret_cast<uint16_t*>(args.Cl)[r + (int64_t)j * args.ldh] =
-                                    f2h_bits(lo, args.bf16);
-                            }
+    if (warp == 0) {
+        if (elect_one()) {
+            // ---------------- TMA producer
+            int it = 0;
+            for (int u = blockIdx.x; u < args.units; u += gridDim.x) {
+                int t0, tj, z, kb0, kb1;
+                unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
+                const int t1 = tj * BN;
+                for (int kb = kb0; kb < kb1; ++kb, ++it) {
+                    const int s = it % STAGES;
+                    const uint32_t round = it / STAGES;
+                    mbar_wait(&empty_bar[s], (round & 1u) ^ 1u);
+                    uint8_t* sa = smem + s * C::kStageBytes;
+                    uint8_t* sb = sa + C::kABytes;
+                    mbar_arrive_expect_tx(&full_bar[s], C::kStageBytes);
+                    if (MODE == 0) {
+                        tma_load_2d(sa, &tmA, &full_bar[s], kb * kBK, t0);
+                        tma_load_2d(sb, &tmB, &full_bar[s], kb * kBK, t1);
+                        if (SPLIT) {
+                            tma_load_2d(sb + C::kBBytes, &tmA_lo, &full_bar[s], kb * kBK, t0);
+                            tma_load_2d(sb + C::kBBytes + C::kABytes, &tmB_lo, &full_bar[s], kb * kBK, t1);
+                        }
+                    } else {
+                        // MN-major A: two 64(row) x 64(k) boxes, the second at +8 KB (LBO)
+                        tma_load_2d(sa, &tmA, &full_bar[s], t0, kb * kBK);
+                        tma_load_2d(sa + C::kABytes / 2, &tmA, &full_bar[s], t0 + 64, kb * kBK);
+                        tma_load_2d(sb, &tmB, &full_bar[s], kb * kBK, t1);
+                        if (SPLIT) {
+                            uint8_t* sal = sb + C::kBBytes;
+                            tma_load_2d(sal, &tmA_lo, &full_bar[s], t0, kb * kBK);
+                            tma_load_2d(sal + C::kABytes / 2, &tmA_lo, &full_bar[s], t0 + 64, kb * kBK);
+                            tma_load_2d(sal + C::kABytes, &tmB_lo, &full_bar[s], kb * kBK, t1);
                         }
                     }
                 }
             }
         }
+        __syncwarp();
+    } else if (warp == 1) {
+        if (elect_one()) {
+            // ---------------- MMA issuer (single thread)
+            const uint32_t idesc = umma_idesc_f16(kBM, BN, MODE == 1 ? 1u : 0u, 0u, (uint32_t)args.bf16);
+            int it = 0, cnt = 0;
+            for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+                int t0, tj, z, kb0, kb1;
+                unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
+                const int acc = cnt % C::kAcc;
+                const uint32_t aphase = (uint32_t)(cnt / C::kAcc) & 1u;
+                mbar_wait(&tempty_bar[acc], aphase ^ 1u);
+                tc_fence_after();
+                const uint32_t dtm = tmem_base + acc * C::kAccCols;
+                for (int kb = kb0; kb < kb1; ++kb, ++it) {
+                    const int s = it % STAGES;
+                    const uint32_t round = it / STAGES;
+                    mbar_wait(&full_bar[s], round & 1u);
+                    tc_fence_after();
+                    const uint32_t sa = smem_u32(smem + s * C::kStageBytes);
+                    const uint32_t sb = sa + C::kABytes;
+                    const uint32_t sal = sb + C::kBBytes;
+                    const uint32_t sbl = sal + C::kABytes;
+#pragma unroll
+                    for (int kk = 0; kk < kBK / kUK; ++kk) {
+                        uint64_t ad, adl;
+                        if (MODE == 0) {
+                            ad = umma_desc_sw128(sa + kk * 32, 16, 1024);
+                            adl = umma_desc_sw128(sal + kk * 32, 16, 1024);
+                        } else {
+                            ad = umma_desc_sw128(sa + kk * 2048, C::kABytes / 2, 1024);
+                            adl = umma_desc_sw128(sal + kk * 2048, C::kABytes / 2, 1024);
+                        }
+                        const uint64_t bd = umma_desc_sw128(sb + kk * 32, 16, 1024);
+                        const uint32_t accum = (kb > kb0 || kk > 0) ? 1u : 0u;
+                        umma_f16(dtm, ad, bd, idesc, accum);
+                        if (SPLIT) {
+                            const uint64_t bdl = umma_desc_sw128(sbl + kk * 32, 16, 1024);
+                            umma_f16(dtm + BN, ad, bdl, idesc, accum);   // hi * lo
+                            umma_f16(dtm + BN, adl, bd, idesc, 1u);      // lo * hi
+                        }
+                    }
+                    umma_commit(&empty_bar[s]);
+                }
+                umma_commit(&tfull_bar[acc]);
+            }
+        }
+        __syncwarp();
+    } else if (warp >= 4) {
+        // ---------------- epilogue warps: ew = TMEM lane quarter, wg = column interleave
+        const int ew = warp & 3;
+        const int wg = (warp - 4) >> 2;
+        float* tb = epi_buf + (warp - 4) * 32 * kEpiLd;
+        const uint32_t lane_off = static_cast<uint32_t>(ew * 32) << 16;
+        const int q = lane & 7;       // row quad within the warp's 32 rows
+        const int jsub = lane >> 3;   // column within a group of 4
+        int cnt = 0;
+        for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+            int t0, tj, z, kb0, kb1;
+            unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
+            const int t1 = tj * BN;
+            const int acc = cnt % C::kAcc;
+            const uint32_t aphase = (uint32_t)(cnt / C::kAcc) & 1u;
+            const int64_t row0 = (int64_t)t0 + ew * 32 + 4 * q;   // first of this lane's 4 rows
+            constexpr int kChunks = BN / 32;
+            bool waited = false;
+            for (int ch = wg; ch < kChunks; ch += EPI_WG) {
+                const int c = ch * 32;
+                // ---- K2: prefetch the fp32 C values of this chunk before touching TMEM
+                float4 old[8];
+                if (MODE == 1 && !args.overwrite) {
+#pragma unroll
+                    for (int k = 0; k < 8; ++k) {
+                        const int j = t1 + c + k * 4 + jsub;
+                        const float* cp = args.C + row0 + (int64_t)j * args.ldc;
+                        if (j < args.w && row0 + 3 < args.m && args.vec_ok) {
+                            old[k] = __ldcs(reinterpret_cast<const float4*>(cp));
+                        } else {
+                            old[k].x = (j < args.w && row0 + 0 < args.m) ? cp[0] : 0.f;
+                            old[k].y = (j < args.w && row0 + 1 < args.m) ? cp[1] : 0.f;
+                            old[k].z = (j < args.w && row0 + 2 < args.m) ? cp[2] : 0.f;
+                            old[k].w = (j < args.w && row0 + 3 < args.m) ? cp[3] : 0.f;
+                        }
+                    }
+                }
+                if (!waited) {
+                    mbar_wait(&tfull_bar[acc], aphase);
+                    tc_fence_after();
+                    waited = true;
+                }
+                const uint32_t dtm = tmem_base + acc * C::kAccCols + lane_off;
+                uint32_t v[32];
+                tmem_ld32(dtm + c, v);
+                tmem_ld_wait();
+                float d[32];
+#pragma unroll
+                for (int jj = 0; jj < 32; ++jj) d[jj] = __uint_as_float(v[jj]);
+                if (SPLIT) {
+                    tmem_ld32(dtm + BN + c, v);
+                    tmem_ld_wait();
+#pragma unroll
+                    for (int jj = 0; jj < 32; ++jj) d[jj] += __uint_as_float(v[jj]) * (1.0f / 2048.0f);
+                }
+                if (ch + EPI_WG >= kChunks) {
+                    // last TMEM read of this accumulator by this warp: release it early
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&tempty_bar[acc]);
+                }
+                // ---- transpose through smem: tb[j][row] (row = lane)
+#pragma unroll
+                for (int jj = 0; jj < 32; ++jj) tb[jj * kEpiLd + lane] = d[jj];
+                __syncwarp();
+#pragma unroll
+                for (int k = 0; k < 8; ++k) {
+                    const int jl = k * 4 + jsub;
+                    const int j = t1 + c + jl;
+                    const float4 dv = *reinterpret_cast<const float4*>(tb + jl * kEpiLd + 4 * q);
+                    if (MODE == 0) {
+                        // the partial buffer is padded to whole tiles: always in range, 16B aligned
+                        float* out = args.P + (int64_t)z * args.p_stride + (int64_t)j * args.ldp + row0;
+                        *reinterpret_cast<float4*>(out) = dv;
+                    } else if (j < args.w) {
+                        float4 nv;
+                        if (args.overwrite) {
+                            nv = dv;
+                        } else {
+                            nv.x = old[k].x - dv.x;
+                            nv.y = old[k].y - dv.y;
+                            nv.z = old[k].z - dv.z;
+                            nv.w = old[k].w - dv.w;
+                        }
+                        float* cp = args.C + row0 + (int64_t)j * args.ldc;
+                        uint16_t* hp = args.Ch ? reinterpret_cast<uint16_t*>(args.Ch) + row0 + (int64_t)j * args.ldh
+                                               : nullptr;
+                        uint16_t* lp = args.Cl ? reinterpret_cast<uint16_t*>(args.Cl) + row0 + (int64_t)j * args.ldh
+                                               : nullptr;
+                        const float nvv[4] = {nv.x, nv.y, nv.z, nv.w};
+                        ushort4 hb, lb;
+                        uint16_t* hbp = reinterpret_cast<uint16_t*>(&hb);
+                        uint16_t* lbp = reinterpret_cast<uint16_t*>(&lb);
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            hbp[e] = f2h_bits(nvv[e], args.bf16);
+                            lbp[e] = f2h_bits((nvv[e] - h2f_bits(hbp[e], args.bf16)) * 2048.0f, args.bf16);
+                        }
+                        if (row0 + 3 < args.m && args.vec_ok) {
+                            __stcs(reinterpret_cast<float4*>(cp), nv);
+                            if (hp) *reinterpret_cast<ushort4*>(hp) = hb;
+                            if (lp) *reinterpret_cast<ushort4*>(lp) = lb;
+                        } else {
+#pragma unroll
+                            for (int e = 0; e < 4; ++e)
+                                if (row0 + e < args.m) {
+                                    cp[e] = nvv[e];
+                                    if (hp) hp[e] = hbp[e];
+                                    if (lp) lp[e] = lbp[e];
+                                }
+                        }
+                    }
+                }
+                __syncwarp();
+            }
+            if (!waited) {   // this warp had no chunk (EPI_WG > chunks): still consume the phase
+                mbar_wait(&tfull_bar[acc], aphase);
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&tempty_bar[acc]);
+            }
+        }
     }
+
     tc_fence_before();
     __syncthreads();
-    if (warp == 2) tmem_dealloc<kTmemCols>(tmem_base);
+    if (warp == 2) tmem_dealloc<C::kTmemCols>(tmem_base);
 }
 
 // --------------------------------------------------------------------------------------
 // split-K reduction for K1: R12(i,j) = sum_z P[z](i,j) in fixed z order (deterministic),
 // written as fp32 into R (ldr) and rounded to 16 bit (hi, and lo for split mode) into
 // the K2 B-operand image R12h (K-major: column j holds R12(:, j), ld = ldh).
-__global__ void __launch_bounds__(256) proj_reduce_kernel(const float* __restrict__ P, int64_t ldp, int64_t p_stride,
-                                                          int splits, int h, int w, float* __restrict__ R, int64_t ldr,
-                                                          float* __restrict__ Rf, int64_t ldf, uint16_t* __restrict__ Rh,
-                                                          uint16_t* __restrict__ Rl, int64_t ldh, int bf16) {
-    // block (32, 8): 32 consecutive outputs x 8 split lanes; lane ty sums splits ty, ty+8, ...
-    // in order, then the 8 lane sums are added in order (deterministic).
-    __shared__ float part[8][33];
+template <int LANES>
+__global__ void __launch_bounds__(32 * LANES) proj_reduce_kernel(const float* __restrict__ P, int64_t ldp,
+                                                                int64_t p_stride, int splits, int h, int w,
+                                                                float* __restrict__ R, int64_t ldr,
+                                                                float* __restrict__ Rf, int64_t ldf,
+                                                                uint16_t* __restrict__ Rh, uint16_t* __restrict__ Rl,
+                                                                int64_t ldh, int bf16) {
+    // block (32, LANES): 32 consecutive outputs x LANES split lanes; lane ty sums splits
+    // ty, ty+LANES, ... in order, then the lane sums are added in order (deterministic).
+    __shared__ float part[LANES][33];
     const int64_t total = (int64_t)h * w;
     const int64_t e = (int64_t)blockIdx.x * 32 + threadIdx.x;
     const bool valid = e < total;
@@ -277,19 +391,20 @@ __global__ void __launch_bounds__(256) proj_reduce_kernel(const float* __restric
     float s = 0.f;
     if (valid) {
         int z = threadIdx.y;
-        for (; z + 24 < splits; z += 32) {
-            const float a = __ldcg(p + (int64_t)z * p_stride), b = __ldcg(p + (int64_t)(z + 8) * p_stride);
-            const float c = __ldcg(p + (int64_t)(z + 16) * p_stride), d = __ldcg(p + (int64_t)(z + 24) * p_stride);
+        for (; z + 3 * LANES < splits; z += 4 * LANES) {
+            const float a = __ldcg(p + (int64_t)z * p_stride), b = __ldcg(p + (int64_t)(z + LANES) * p_stride);
+            const float c = __ldcg(p + (int64_t)(z + 2 * LANES) * p_stride);
+            const float d = __ldcg(p + (int64_t)(z + 3 * LANES) * p_stride);
             s += a; s += b; s += c; s += d;
         }
-        for (; z < splits; z += 8) s += __ldcg(p + (int64_t)z * p_stride);
+        for (; z < splits; z += LANES) s += __ldcg(p + (int64_t)z * p_stride);
     }
     part[threadIdx.y][threadIdx.x] = s;
     __syncthreads();
     if (threadIdx.y != 0 || !valid) return;
     float t = 0.f;
 #pragma unroll
-    for (int y = 0; y < 8; ++y) t += part[y][threadIdx.x];
+    for (int y = 0; y < LANES; ++y) t += part[y][threadIdx.x];
     if (R) R[i + (int64_t)j * ldr] = t;
     if (Rf) Rf[i + (int64_t)j * ldf] = t;
     if (Rh) {
@@ -316,31 +431,47 @@ __global__ void proj_finish_kernel(const float* __restrict__ Rf, int64_t ldf, in
 }
 
 // ------------------------------------------------------------------ host launchers
-template <int MODE, int BN, int STAGES, bool SPLIT>
-static cudaError_t launch_gemm(dim3 grid, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& al,
+static int g_num_sms = 0;
+static int num_sms() {
+    if (!g_num_sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+        if (g_num_sms <= 0) g_num_sms = 148;
+    }
+    return g_num_sms;
+}
+
+template <int MODE, int BN, int STAGES, bool SPLIT, int EPI_WG>
+static cudaError_t launch_gemm(int units, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& al,
                                const CUtensorMap& bl, const GemmArgs& args, cudaStream_t st) {
-    using L = GemmSmem<BN, STAGES, SPLIT>;
-    auto kern = gemm_tc_kernel<MODE, BN, STAGES, SPLIT>;
+    using C = GemmCfg<BN, STAGES, SPLIT, EPI_WG>;
+    static_assert(C::kTotal <= 227 * 1024, "shared memory budget");
+    auto kern = gemm_tc_kernel<MODE, BN, STAGES, SPLIT, EPI_WG>;
     static bool attr_set = false;
     if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, L::kTotal);
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::kTotal);
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
+    // persistent grid: one CTA per SM (two when the footprint allows), never more than units
+    const int per_sm = (C::kTotal <= 113 * 1024 && C::kTmemCols <= 256) ? 2 : 1;
+    int grid = num_sms() * per_sm;
+    if (grid > units) grid = units;
     ++g_launches;
-    kern<<<grid, kThreads, L::kTotal, st>>>(a, b, al, bl, args);
+    kern<<<grid, C::kThreads, C::kTotal, st>>>(a, b, al, bl, args);
     return cudaGetLastError();
 }
 
 template <int MODE, bool SPLIT>
-static cudaError_t dispatch_bn(int bn, dim3 grid, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& al,
+static cudaError_t dispatch_bn(int bn, int units, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& al,
                                const CUtensorMap& bl, const GemmArgs& args, cudaStream_t st) {
-    // stage counts keep smem <= ~200 KB: (16 KB + BN*128 B) * ops * stages
+    // stage counts keep smem <= 227 KB: stages * (16 KB + BN * 128 B) * ops + epilogue buffers
     switch (bn) {
-        case 32: return launch_gemm<MODE, 32, SPLIT ? 4 : 6, SPLIT>(grid, a, b, al, bl, args, st);
-        case 64: return launch_gemm<MODE, 64, SPLIT ? 4 : 6, SPLIT>(grid, a, b, al, bl, args, st);
-        case 128: return launch_gemm<MODE, 128, SPLIT ? 3 : 5, SPLIT>(grid, a, b, al, bl, args, st);
-        case 256: return launch_gemm<MODE, 256, SPLIT ? 2 : 4, SPLIT>(grid, a, b, al, bl, args, st);
+        case 32: return launch_gemm<MODE, 32, 3, SPLIT, 2>(units, a, b, al, bl, args, st);
+        case 64: return launch_gemm<MODE, 64, SPLIT ? 3 : 4, SPLIT, 2>(units, a, b, al, bl, args, st);
+        case 128: return launch_gemm<MODE, 128, SPLIT ? 2 : 5, SPLIT, 2>(units, a, b, al, bl, args, st);
+        case 256: return launch_gemm<MODE, 256, SPLIT ? 2 : 4, SPLIT, 1>(units, a, b, al, bl, args, st);
         default: return cudaErrorInvalidValue;
     }
 }
@@ -350,21 +481,26 @@ cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int s
                              int64_t ldp, int64_t p_stride, int kb_total, int kb_per_split, int bf16,
                              cudaStream_t st) {
     GemmArgs args{};
+    args.units = tiles_i * tiles_j * splits;
+    args.tiles_i = tiles_i;
+    args.tiles_j = tiles_j;
     args.P = P;
     args.ldp = ldp;
     args.p_stride = p_stride;
     args.kb_total = kb_total;
     args.kb_per_split = kb_per_split;
     args.bf16 = bf16;
-    dim3 grid(tiles_i, tiles_j, splits);
-    return split ? dispatch_bn<0, true>(bn, grid, q1, a2, q1_lo, a2_lo, args, st)
-                 : dispatch_bn<0, false>(bn, grid, q1, a2, q1, a2, args, st);
+    args.vec_ok = 1;
+    return split ? dispatch_bn<0, true>(bn, args.units, q1, a2, q1_lo, a2_lo, args, st)
+                 : dispatch_bn<0, false>(bn, args.units, q1, a2, q1, a2, args, st);
 }
 
 cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, const CUtensorMap& q1_mn,
                                const CUtensorMap& r12, const CUtensorMap& q1_mn_lo, const CUtensorMap& r12_lo,
-                               float* C, int64_t ldc, void* Ch, void* Cl, int64_t ldh, int bf16, cudaStream_t st) {
+                               float* C, int64_t ldc, void* Ch, void* Cl, int64_t ldh, int bf16, cudaStream_t st,
+                               int overwrite) {
     GemmArgs args{};
+    args.overwrite = overwrite;
     args.C = C;
     args.ldc = ldc;
     args.Ch = Ch;
@@ -374,9 +510,13 @@ cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, cons
     args.w = w;
     args.kb_h = (h + kBK - 1) / kBK;
     args.bf16 = bf16;
-    dim3 grid((unsigned)((m + kBM - 1) / kBM), (unsigned)((w + bn - 1) / bn), 1);
-    return split ? dispatch_bn<1, true>(bn, grid, q1_mn, r12, q1_mn_lo, r12_lo, args, st)
-                 : dispatch_bn<1, false>(bn, grid, q1_mn, r12, q1_mn, r12, args, st);
+    args.tiles_i = (int)((m + kBM - 1) / kBM);
+    args.tiles_j = (w + bn - 1) / bn;
+    args.units = args.tiles_i * args.tiles_j;
+    args.vec_ok = ((ldc & 3) == 0) && ((reinterpret_cast<uintptr_t>(C) & 15) == 0) && ((ldh & 3) == 0) &&
+                  ((reinterpret_cast<uintptr_t>(Ch) & 7) == 0) && ((reinterpret_cast<uintptr_t>(Cl) & 7) == 0);
+    return split ? dispatch_bn<1, true>(bn, args.units, q1_mn, r12, q1_mn_lo, r12_lo, args, st)
+                 : dispatch_bn<1, false>(bn, args.units, q1_mn, r12, q1_mn, r12, args, st);
 }
 
 cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, int splits, int h, int w, float* R,
@@ -384,8 +524,13 @@ cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, in
                                cudaStream_t st) {
     const int64_t total = (int64_t)h * w;
     ++g_launches;
-    proj_reduce_kernel<<<(unsigned)((total + 31) / 32), dim3(32, 8), 0, st>>>(P, ldp, p_stride, splits, h, w, R, ldr,
-                                                                              Rf, ldf, Rh, Rl, ldh, bf16);
+    if (splits > 32)
+        proj_reduce_kernel<32><<<(unsigned)((total + 31) / 32), dim3(32, 32), 0, st>>>(P, ldp, p_stride, splits, h, w,
+                                                                                       R, ldr, Rf, ldf, Rh, Rl, ldh,
+                                                                                       bf16);
+    else
+        proj_reduce_kernel<8><<<(unsigned)((total + 31) / 32), dim3(32, 8), 0, st>>>(P, ldp, p_stride, splits, h, w, R,
+                                                                                     ldr, Rf, ldf, Rh, Rl, ldh, bf16);
     return cudaGetLastError();
 }
 

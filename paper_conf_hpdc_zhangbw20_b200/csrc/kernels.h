@@ -52,7 +52,6 @@ cudaError_t launch_panel_stack(const float* Rall, int P, int nc, float* R, int64
 struct CholqrLaunch {
     const float* P;
     int64_t ldp;
-    float* Q1;      // m x 32 workspace (ld m)
     float* Q;
     int64_t ldq;
     uint16_t* Qh;
@@ -61,7 +60,7 @@ struct CholqrLaunch {
     int64_t m;
     int nc;
     double* ws;     // cholqr_ws_doubles(m)
-    int* counter;   // zero-initialised, self-resetting
+    int* counter;   // cholqr_counter_ints(m), zero-initialised, self-resetting
     int* fail;      // set on a failed pivot (guards the MGS fallback)
     float* R;
     int64_t ldr;
@@ -70,6 +69,7 @@ struct CholqrLaunch {
     void* ctx;
 };
 size_t cholqr_ws_doubles(int64_t m);
+size_t cholqr_counter_ints(int64_t m);
 cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st);
 
 // ---- gemm_tc.cu (Alg 1 lines 8-9 on tcgen05)
@@ -79,12 +79,22 @@ cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int s
                              cudaStream_t st);
 cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, const CUtensorMap& q1_mn,
                                const CUtensorMap& r12, const CUtensorMap& q1_mn_lo, const CUtensorMap& r12_lo,
-                               float* C, int64_t ldc, void* Ch, void* Cl, int64_t ldh, int bf16, cudaStream_t st);
+                               float* C, int64_t ldc, void* Ch, void* Cl, int64_t ldh, int bf16, cudaStream_t st,
+                               int overwrite = 0);
 cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, int splits, int h, int w, float* R,
                                int64_t ldr, float* Rf, int64_t ldf, uint16_t* Rh, uint16_t* Rl, int64_t ldh, int bf16,
                                cudaStream_t st);
 cudaError_t launch_proj_finish(const float* Rf, int64_t ldf, int h, int w, float* R, int64_t ldr, uint16_t* Rh,
                                uint16_t* Rl, int64_t ldh, int bf16, cudaStream_t st);
+
+// ---- lowrank.cu
+cudaError_t launch_cast_rows(const float* src, int64_t lds, int64_t rows, int cols, const float* rscale, uint16_t* hi,
+                             uint16_t* lo, int64_t ldd, int bf16, cudaStream_t st);
+cudaError_t launch_cast_rows64(const double* src, int64_t lds, int64_t rows, int cols, const float* rscale,
+                               uint16_t* hi, uint16_t* lo, int64_t ldd, int bf16, cudaStream_t st);
+cudaError_t launch_unscale_rows(float* X, int64_t ldx, int64_t rows, int cols, const float* rscale, cudaStream_t st);
+cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double* W, double* V, double* sig, int* flags,
+                              float* S, float* Ub, float* Vb, cudaStream_t st);
 
 // ---- blas.cu (CGLS vectors, triangular inverse, small products)
 cudaError_t launch_gemv_n(const float* A, int64_t lda, int64_t m, int n, const double* x, double* y, double* work,

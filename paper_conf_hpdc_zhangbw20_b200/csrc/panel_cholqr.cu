@@ -1,18 +1,23 @@
 // panel_cholqr.cu -- CholQR2 leaf panel with an fp64 Gram matrix (north_star: "a
-// bandwidth-bound panel MGS/CholQR kernel"; SURVEY 2.2 A19/8(e) "CholQR2 (fp64 Gram)").
+// bandwidth-bound panel MGS/CholQR kernel"; SURVEY 2.2 A19 / 8(e) "CholQR2 (fp64 Gram)").
 //
-//   G1 = P^T P (fp64)          R1 = chol(G1)     Q1 = P R1^{-1}   (fp32)
-//   G2 = Q1^T Q1 (fp64)        R2 = chol(G2)     Q  = Q1 R2^{-1}  (fp32 + 16-bit shadow)
-//   R  = R2 R1
+//   pass 0:  G1 = P^T P                                   (fp64 accumulation)
+//            -> R1 = chol(G1), R1^{-1}                    (last CTA, one warp)
+//   pass 1:  Q1 = P R1^{-1} (fp32, registers only), G2 = Q1^T Q1
+//            -> R2 = chol(G2), R2^{-1}
+//   pass 2:  Q = (P R1^{-1}) R2^{-1}  -> Q (fp32) + 16-bit shadow;  R = R2 R1
 //
-// Why it replaces the MGS tiles by default on B200: MGS needs 32
-// dependent block-wide reductions per tile plus a tree of stacked-R factorizations, which
-// is latency-bound (~240 us per 65536 x 32 panel measured); CholQR2 is three streaming
-// passes whose only sequential piece is a 32 x 32 Cholesky done redundantly per CTA.
-// With an fp64 Gram, Q1's orthogonality is ~kappa u32 (like MGS) and the second pass
-// brings it to ~u32 while kappa(P) < ~1e7.  If a Cholesky pivot fails the panel sets a
-// device flag and the MGS/TSQR kernels of panel.cu (guarded by that flag) redo the panel
-// from the untouched input, so the result never silently degrades.
+// Q1 is recomputed in pass 2 with the same arithmetic as in pass 1 (bit-identical), so it
+// is never stored: three reads of the panel (L2-resident at these sizes) and one write.
+// Why this is the default B200 leaf: the MGS tiles of Alg 2 need 32
+// dependent block-wide reductions per tile plus a tree of stacked-R factorisations, which
+// is latency-bound on B200 (~240 us per 65536 x 32 panel measured); CholQR2 streams.
+// With an fp64 Gram, Q1's orthogonality is ~kappa u32 and the second pass brings it to
+// ~u32 while kappa(P) < ~1e7.  A failed pivot sets a device flag: the TSQR/MGS kernels of
+// panel.cu (guarded by it) then redo the panel from the untouched input.
+//
+// Reductions are deterministic: CTA partials are summed in fixed order by the last CTA of
+// each group of 16 ("last block" pattern), then by the last group.
 #include <cuda_runtime.h>
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
@@ -27,6 +32,7 @@ constexpr int CQ_LD = CQ_TILE + 1;    // smem column stride (bank-conflict-free 
 constexpr int CQ_THREADS = 256;
 constexpr int CQ_BLK = 36;            // 4x4 blocks in the upper triangle of a 32x32 Gram (8*9/2)
 constexpr int CQ_GROUPS = CQ_THREADS / CQ_BLK;  // 7 row groups of 36 threads
+constexpr int CQ_FAN = 16;            // CTAs per reduction group
 
 __device__ __forceinline__ uint16_t cq_to16(float x, int bf16) {
     if (bf16) {
@@ -41,37 +47,46 @@ __device__ __forceinline__ float cq_from16(uint16_t u, int bf16) {
     return __half2float(*reinterpret_cast<__half*>(&u));
 }
 
+struct CqWs {            // device workspace layout (doubles unless noted)
+    double* part;        // [grid][1024] CTA partial Grams
+    double* gpart;       // [ngroups][1024] group partial Grams
+    double* G;           // [2][1024] reduced Grams (distributed mode reads / writes these)
+    double* R;           // [2][1024] Cholesky factors R1, R2 (fp64, upper, R[i + 32 j])
+    float* Rinv;         // [2][1024] fp32 inverses R1^{-1}, R2^{-1}
+    int* counters;       // [ngroups + 1], zero-initialised, self-resetting
+    int* fail;           // 1 when a Cholesky pivot failed (guards the MGS fallback)
+};
+
 struct CqArgs {
-    const float* P;     // panel input (fp32, ldp)
+    const float* P;      // panel (fp32, ldp); also the in-place output location
     int64_t ldp;
-    float* Q1;          // pass-1 output (workspace, ld = m)
-    float* Q;           // final Q (in place of the panel is allowed), ldq
+    float* Q;            // final Q, ldq (may alias P)
     int64_t ldq;
-    uint16_t* Qh;       // 16-bit shadow (hi) of Q, ldh
-    uint16_t* Ql;       // lo part (split mode) or null
+    uint16_t* Qh;        // 16-bit shadow (hi) of Q, ldh
+    uint16_t* Ql;        // lo part (split mode) or null
     int64_t ldh;
     int64_t m;
     int nc;
-    double* part;       // per-CTA partial Grams [grid][32*32]
-    double* G;          // reduced Gram (32*32, fp64), pass 1 at G, pass 2 at G + 1024
-    double* Rkeep;      // R1 (fp64 32*32) kept for the final product
-    int* counter;       // last-block counter (reset by the last block)
-    int* fail;          // set to 1 when a Cholesky pivot fails (MGS fallback runs)
-    float* R;           // final nc x nc R block (ldr)
+    CqWs ws;
+    float* Rout;         // final nc x nc R block (ldr)
     int64_t ldr;
     int bf16;
-    int distributed;    // 1: the caller allreduces G between passes (no last-block reduce)
+    int distributed;     // 1: stop after the reduced Gram; the host allreduces + factors
 };
 
-// Accumulate the 4x4 Gram block `blk` of the nc-column tile in smem (rows [0, rows)).
-__device__ __forceinline__ void gram_block_accum(const float* tile, int rows, int g, int blk, double (&acc)[4][4]) {
-    // upper-triangular block (bi, bj), bi <= bj, enumerated row-major
-    int bi = 0, rem = blk;
-    while (rem >= 8 - bi) {
-        rem -= 8 - bi;
-        ++bi;
+// ---------------------------------------------------------------- Gram accumulation
+__device__ __forceinline__ void blk_coords(int blk, int& bi, int& bj) {
+    int b = 0, rem = blk;
+    while (rem >= 8 - b) {
+        rem -= 8 - b;
+        ++b;
     }
-    const int bj = bi + rem;
+    bi = b;
+    bj = b + rem;
+}
+
+__device__ __forceinline__ void gram_block_accum(const float* tile, int rows, int g, int bi, int bj,
+                                                 double (&acc)[4][4]) {
     for (int r = g; r < rows; r += CQ_GROUPS) {
         double x[4], y[4];
 #pragma unroll
@@ -86,258 +101,352 @@ __device__ __forceinline__ void gram_block_accum(const float* tile, int rows, in
     }
 }
 
-__device__ __forceinline__ void gram_block_store(double* dst, int blk, const double (&acc)[4][4]) {
-    int bi = 0, rem = blk;
-    while (rem >= 8 - bi) {
-        rem -= 8 - bi;
-        ++bi;
+// ---------------------------------------------------------------- Cholesky + inverse
+// One warp.  G (32x32 fp64, upper triangle valid, nc x nc used, identity-padded).
+// Writes R (fp64 upper, R[i + 32 j]) and Rinv (fp32, Rinv[i + 32 j]); returns false if a
+// pivot is not safely positive (relative to the original diagonal).
+__device__ bool chol_inv_warp(const double* G, int nc, double* Rg, float* Rinvg, double* Rs /*smem 32x33*/) {
+    const int lane = threadIdx.x & 31;
+    double g[32];   // lane i holds row i of the symmetric Gram
+#pragma unroll
+    for (int j = 0; j < 32; ++j) {
+        const int a = min(lane, j), b = max(lane, j);
+        g[j] = (lane < nc && j < nc) ? __ldcg(G + a + 32 * b) : (lane == j ? 1.0 : 0.0);
     }
-    const int bj = bi + rem;
+    double orig = 0.0;
 #pragma unroll
-    for (int u = 0; u < 4; ++u)
+    for (int j = 0; j < 32; ++j)
+        if (j == lane) orig = g[j];
+    bool ok = true;
+    double inv_diag = 1.0;   // lane k keeps 1 / R(k,k)
 #pragma unroll
-        for (int v = 0; v < 4; ++v) dst[(bi * 4 + u) + (bj * 4 + v) * 32] = acc[u][v];
+    for (int k = 0; k < 32; ++k) {
+        const double dkk = __shfl_sync(0xffffffffu, g[k], k);
+        const double okk = __shfl_sync(0xffffffffu, orig, k);
+        const bool good = (dkk > okk * 1e-15) && isfinite(dkk);
+        ok = ok && good;
+        const double irk = good ? rsqrt(dkk) : 1.0;
+        const double rkk = good ? dkk * irk : 1.0;
+        if (lane == k) inv_diag = irk;
+        // row k of the upper factor: R(k, lane); broadcast to the warp through smem
+        const double l = (lane > k) ? g[k] * irk : ((lane == k) ? rkk : 0.0);
+        Rs[k * 33 + lane] = l;
+        __syncwarp();
+#pragma unroll
+        for (int j = k + 1; j < 32; ++j) g[j] = fma(-l, Rs[k * 33 + j], g[j]);
+    }
+    __syncwarp();
+    // Rinv column j (= lane): x = e_j; for k = 31..0: x_k *= 1/R(k,k); x_i -= R(i,k) x_k (i < k)
+    const int j = lane;
+    double x[32];
+#pragma unroll
+    for (int i = 0; i < 32; ++i) x[i] = (i == j) ? 1.0 : 0.0;
+#pragma unroll
+    for (int k = 31; k >= 0; --k) {
+        const double ik = __shfl_sync(0xffffffffu, inv_diag, k);
+        x[k] *= ik;
+#pragma unroll
+        for (int i = 0; i < k; ++i) x[i] = fma(-Rs[i * 33 + k], x[k], x[i]);
+    }
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+        Rinvg[i + 32 * j] = (float)x[i];
+        Rg[i + 32 * j] = (i <= j) ? Rs[i * 33 + j] : 0.0;
+    }
+    return __all_sync(0xffffffffu, ok);
 }
 
-// Sum the per-group partial blocks of this CTA (smem) and write the CTA partial Gram.
-__device__ void cta_gram_flush(double* sred, const double (&acc)[4][4], int blk, int g, double* out) {
-    // sred: [CQ_GROUPS][1024] doubles
-    if (blk < CQ_BLK && g < CQ_GROUPS) gram_block_store(sred + g * 1024, blk, acc);
-    __syncthreads();
+// Sum `n` partial Grams [n][1024] (upper triangle) in fixed order into dst (whole CTA);
+// loads are issued CQ_FAN at a time before the adds so the latency is paid once per chunk.
+__device__ void sum_parts(const double* src, int n, double* dst) {
     for (int e = threadIdx.x; e < 1024; e += blockDim.x) {
+        const int i = e & 31, j = e >> 5;
         double s = 0.0;
-        for (int q = 0; q < CQ_GROUPS; ++q) s += sred[q * 1024 + e];
-        out[e] = s;   // only the upper triangle is meaningful
+        for (int c0 = 0; c0 < n; c0 += CQ_FAN) {
+            double v[CQ_FAN];
+#pragma unroll
+            for (int c = 0; c < CQ_FAN; ++c)
+                v[c] = (i <= j && c0 + c < n) ? __ldcg(src + (int64_t)(c0 + c) * 1024 + e) : 0.0;
+#pragma unroll
+            for (int c = 0; c < CQ_FAN; ++c) s += v[c];
+        }
+        dst[e] = s;
     }
 }
 
-// last CTA sums all CTA partials in fixed order into G (fp64, symmetric fill)
-__device__ bool last_block_reduce(const CqArgs& a, double* Gout) {
-    __shared__ int s_last;
-    __threadfence();
+// R = R2 R1 (fp64 product of upper-triangular factors; positive diagonal) -> a.Rout.
+// R2 is in smem (Rs[i * 33 + j], from chol_inv_warp), R1 in the workspace.
+__device__ void final_r_product(const CqArgs& a, const double* Rs, double* R1s /*smem 32x33*/) {
+    for (int e = threadIdx.x; e < 1024; e += blockDim.x) R1s[(e & 31) * 33 + (e >> 5)] = __ldcg(a.ws.R + e);
+    __syncthreads();
+    for (int e = threadIdx.x; e < a.nc * a.nc; e += blockDim.x) {
+        const int i = e % a.nc, j = e / a.nc;
+        double s = 0.0;
+        for (int k = i; k <= j; ++k) s = fma(Rs[i * 33 + k], R1s[k * 33 + j], s);
+        a.Rout[i + (int64_t)j * a.ldr] = (i <= j) ? (float)s : 0.f;
+    }
+}
+
+// kappa_F(R1) = |R1|_F |R1^{-1}|_F <= 2 nc  ->  one CholQR pass is enough (ws.fail[1] = 1).
+__device__ void single_pass_decision(const CqArgs& a) {
+    __shared__ double red[2][32];
+    double r = 0.0, ri = 0.0;
+    for (int e = threadIdx.x; e < 1024; e += blockDim.x) {
+        const int i = e & 31, j = e >> 5;
+        if (i < a.nc && j < a.nc) {
+            const double x = __ldcg(a.ws.R + e);
+            const double y = (double)__ldcg(a.ws.Rinv + e);
+            r = fma(x, x, r);
+            ri = fma(y, y, ri);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        r += __shfl_xor_sync(0xffffffffu, r, o);
+        ri += __shfl_xor_sync(0xffffffffu, ri, o);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        red[0][threadIdx.x >> 5] = r;
+        red[1][threadIdx.x >> 5] = ri;
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
-        const int old = atomicAdd(a.counter, 1);
-        s_last = (old == (int)gridDim.x - 1);
+        double sr = 0.0, sri = 0.0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) {
+            sr += red[0][w];
+            sri += red[1][w];
+        }
+        a.ws.fail[1] = (sqrt(sr * sri) <= 2.0 * a.nc) ? 1 : 0;
     }
-    __syncthreads();
-    if (!s_last) return false;
+}
+
+// Hierarchical last-block reduction + (single GPU) Cholesky of the reduced Gram.
+__device__ void reduce_and_factor(const CqArgs& a, int pass, double* smem_R, double* smem_R1) {
+    __shared__ int s_last;
+    const int grid = gridDim.x;
+    const int ngroups = (grid + CQ_FAN - 1) / CQ_FAN;
+    const int grp = blockIdx.x / CQ_FAN;
+    const int gsize = min(CQ_FAN, grid - grp * CQ_FAN);
     __threadfence();
-    for (int e = threadIdx.x; e < 1024; e += blockDim.x) {
-        const int i = e & 31, j = e >> 5;
-        double s = 0.0;
-        if (i <= j)
-            for (int c = 0; c < (int)gridDim.x; ++c) s += __ldcg(a.part + (int64_t)c * 1024 + e);
-        Gout[e] = s;
-    }
     __syncthreads();
-    if (threadIdx.x == 0) *a.counter = 0;
-    return true;
-}
-
-// Cholesky G = R^T R (upper R, fp64) of the nc x nc leading block, padded with identity,
-// by warp 0; then Rinv = R^{-1} (fp64).  Returns false (all threads) on a failed pivot.
-__device__ bool chol_inv(const double* Gg, double* Rs /*32x33*/, double* Ri /*32x33*/, int nc) {
+    if (threadIdx.x == 0) s_last = (atomicAdd(&a.ws.counters[grp], 1) == gsize - 1);
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    sum_parts(a.ws.part + (int64_t)grp * CQ_FAN * 1024, gsize, a.ws.gpart + (int64_t)grp * 1024);
+    if (threadIdx.x == 0) a.ws.counters[grp] = 0;
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) s_last = (atomicAdd(&a.ws.counters[ngroups], 1) == ngroups - 1);
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    double* G = a.ws.G + pass * 1024;
+    sum_parts(a.ws.gpart, ngroups, G);
+    if (threadIdx.x == 0) a.ws.counters[ngroups] = 0;
+    __threadfence();
+    __syncthreads();
+    if (a.distributed) return;   // host: allreduce(G) then cq_factor_kernel
     __shared__ int s_ok;
-    const int lane = threadIdx.x & 31;
     if (threadIdx.x < 32) {
-        // load the upper triangle (column j in lane j's view): Rs[i][j] = G(i, j) for i <= j
-        for (int i = 0; i < 32; ++i) {
-            const int j = lane;
-            double v = 0.0;
-            if (i < nc && j < nc) v = (i <= j) ? Gg[i + j * 32] : 0.0;
-            else if (i == j) v = 1.0;
-            Rs[i * 33 + j] = (i <= j) ? v : 0.0;
+        const bool ok = chol_inv_warp(G, a.nc, a.ws.R + pass * 1024, a.ws.Rinv + pass * 1024, smem_R);
+        if (threadIdx.x == 0) {
+            s_ok = ok;
+            if (!ok) *a.ws.fail = 1;
         }
-        __syncwarp();
-        bool ok = true;
-        // right-looking upper Cholesky: for k: R(k,k) = sqrt(G(k,k)); R(k,j) /= R(k,k);
-        // G(i,j) -= R(k,i) R(k,j) for k < i <= j.  Lane j owns column j.
-        for (int k = 0; k < 32; ++k) {
-            const double piv = Rs[k * 33 + k];
-            const double orig = (k < nc) ? Gg[k + k * 32] : 1.0;
-            const bool good = piv > orig * 1e-15 && isfinite(piv);
-            ok = ok && good;
-            const double d = good ? sqrt(piv) : 1.0;
-            __syncwarp();
-            if (lane >= k) Rs[k * 33 + lane] = (lane == k) ? d : Rs[k * 33 + lane] / d;
-            __syncwarp();
-            const double rkj = Rs[k * 33 + lane];
-            for (int i = k + 1; i <= lane; ++i) Rs[i * 33 + lane] -= Rs[k * 33 + i] * rkj;
-            __syncwarp();
-        }
-        // Rinv by column-oriented back substitution: lane j solves R x = e_j
-        for (int i = 0; i < 32; ++i) Ri[i * 33 + lane] = 0.0;
-        __syncwarp();
-        {
-            const int j = lane;
-            double x[32];
-#pragma unroll
-            for (int i = 0; i < 32; ++i) x[i] = (i == j) ? 1.0 : 0.0;
-#pragma unroll
-            for (int k = 31; k >= 0; --k) {
-                if (k <= j) {
-                    x[k] = x[k] / Rs[k * 33 + k];
-#pragma unroll
-                    for (int i = 0; i < k; ++i) x[i] -= Rs[i * 33 + k] * x[k];
-                }
-            }
-#pragma unroll
-            for (int i = 0; i < 32; ++i) Ri[i * 33 + j] = (i <= j) ? x[i] : 0.0;
-        }
-        if (lane == 0) s_ok = ok ? 1 : 0;
     }
     __syncthreads();
-    return s_ok != 0;
+    if (pass == 0 && s_ok) single_pass_decision(a);
+    if (pass == 1 && s_ok) final_r_product(a, smem_R, smem_R1);
 }
 
-// pass 1: CTA partial Grams of P; last block reduces into G (unless distributed).
-__global__ void __launch_bounds__(CQ_THREADS) cq_gram_kernel(CqArgs a) {
-    extern __shared__ double dsm[];
-    float* tile = reinterpret_cast<float*>(dsm + CQ_GROUPS * 1024);
-    double* sred = dsm;
+// ---------------------------------------------------------------- streaming passes
+// PASS 0: partial Gram of P -> (last CTA) R1, R1^{-1}, and the decision whether one
+//         CholQR pass suffices (kappa_F(R1) = |R1|_F |R1^{-1}|_F <= 2 nc: Q1 = P R1^{-1} is
+//         then orthogonal to a few u32, like one MGS pass), stored in ws.fail[1].
+// PASS 1: Q1 = P R1^{-1}; single-pass panels write Q1 as Q (+ shadow) and R = R1;
+//         otherwise partial Gram of Q1 -> (last CTA) R2, R2^{-1}, R = R2 R1.
+// PASS 2: (two-pass panels only) Q = (P R1^{-1}) R2^{-1} (+ shadow).
+//
+// Per 128-row tile, thread t owns rows {t/8 + 32 i} (i < 4) and columns 4 (t%8) .. +3, so
+// every shared-memory load of R^{-1} (one float4) feeds 16 FMAs.
+__device__ __forceinline__ void tile_times_rinv(float* tile, const float* Rinv /*32 x 32, ld 32*/, int tid) {
+    const int cgp = tid & 7, rgp = tid >> 3;
+    float o[4][4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) o[i][c] = 0.f;
+#pragma unroll 8
+    for (int k = 0; k < CQ_NB; ++k) {
+        const float4 rv = *reinterpret_cast<const float4*>(Rinv + k * 32 + 4 * cgp);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const float x = tile[k * CQ_LD + rgp + 32 * i];
+            o[i][0] = fmaf(x, rv.x, o[i][0]);
+            o[i][1] = fmaf(x, rv.y, o[i][1]);
+            o[i][2] = fmaf(x, rv.z, o[i][2]);
+            o[i][3] = fmaf(x, rv.w, o[i][3]);
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) tile[(4 * cgp + c) * CQ_LD + rgp + 32 * i] = o[i][c];
+    __syncthreads();
+}
+
+template <int PASS>
+__global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
+    __shared__ __align__(16) float tile[CQ_NB * CQ_LD + 64];   // also R1 scratch (32 x 33 doubles)
+    __shared__ __align__(16) float Ri[2][32 * 32];
+    __shared__ double sred[2][1024];   // CTA partial-sum scratch (2 row groups at a time); reused
+                                       // as the 32 x 33 Cholesky scratch by the last CTA
     const int tid = threadIdx.x;
-    if (blockIdx.x == 0 && tid == 0) *a.fail = 0;   // the apply passes / MGS fallback read it later
+    if (PASS == 0 && blockIdx.x == 0 && tid == 0) {
+        a.ws.fail[0] = 0;
+        a.ws.fail[1] = 0;
+    }
+    bool single = false;
+    if (PASS > 0) {
+        if (*(volatile int*)a.ws.fail) return;   // the MGS fallback owns this panel
+        single = *(volatile int*)(a.ws.fail + 1) != 0;
+        if (PASS == 2 && single) return;         // finished in pass 1
+        for (int e = tid; e < 1024; e += CQ_THREADS) {
+            Ri[0][e] = a.ws.Rinv[(e & 31) * 32 + (e >> 5)];   // Ri[k][j] = R^{-1}(k, j)
+            if (PASS == 2) Ri[1][e] = a.ws.Rinv[1024 + (e & 31) * 32 + (e >> 5)];
+        }
+        if (PASS == 1 && single && blockIdx.x == 0)
+            for (int e = tid; e < a.nc * a.nc; e += CQ_THREADS) {
+                const int i = e % a.nc, j = e / a.nc;
+                a.Rout[i + (int64_t)j * a.ldr] = (i <= j) ? (float)a.ws.R[i + 32 * j] : 0.f;
+            }
+    }
+    const bool write_q = (PASS == 2) || (PASS == 1 && single);
+    const bool gram = (PASS == 0) || (PASS == 1 && !single);
     const int g = tid / CQ_BLK, blk = tid % CQ_BLK;
+    int bi, bj;
+    blk_coords(blk, bi, bj);
     double acc[4][4] = {};
-    const int64_t rows_per_cta = (a.m + gridDim.x - 1) / gridDim.x;
+    const int64_t rows_per_cta = ((a.m + gridDim.x - 1) / gridDim.x + 3) / 4 * 4;
     const int64_t r0 = (int64_t)blockIdx.x * rows_per_cta;
     const int64_t r1 = min(a.m, r0 + rows_per_cta);
+    // register prefetch of the next tile: thread loads element (r = e % 128, c = e / 128)
+    float pre[16];
+#pragma unroll
+    for (int k = 0; k < 16; ++k) {
+        const int e = tid + k * CQ_THREADS;
+        const int r = e % CQ_TILE, c = e / CQ_TILE;
+        pre[k] = (r0 + r < r1 && c < a.nc) ? a.P[r0 + r + (int64_t)c * a.ldp] : 0.f;
+    }
     for (int64_t base = r0; base < r1; base += CQ_TILE) {
         const int rows = (int)((r1 - base) < CQ_TILE ? (r1 - base) : CQ_TILE);
         __syncthreads();
-        for (int e = tid; e < CQ_TILE * CQ_NB; e += CQ_THREADS) {
+#pragma unroll
+        for (int k = 0; k < 16; ++k) {
+            const int e = tid + k * CQ_THREADS;
+            tile[(e / CQ_TILE) * CQ_LD + (e % CQ_TILE)] = pre[k];
+        }
+        __syncthreads();
+        const int64_t nb = base + CQ_TILE;
+#pragma unroll
+        for (int k = 0; k < 16; ++k) {
+            const int e = tid + k * CQ_THREADS;
             const int r = e % CQ_TILE, c = e / CQ_TILE;
-            tile[c * CQ_LD + r] = (r < rows && c < a.nc) ? a.P[base + r + (int64_t)c * a.ldp] : 0.f;
+            pre[k] = (nb + r < r1 && c < a.nc) ? a.P[nb + r + (int64_t)c * a.ldp] : 0.f;
         }
-        __syncthreads();
-        if (g < CQ_GROUPS) gram_block_accum(tile, rows, g, blk, acc);
-    }
-    __syncthreads();
-    cta_gram_flush(sred, acc, blk, g, a.part + (int64_t)blockIdx.x * 1024);
-    if (!a.distributed) last_block_reduce(a, a.G);
-}
-
-// pass 2 (mode 0): Q1 = P R1^{-1} + partial Grams of Q1 (last block -> G + 1024)
-// pass 3 (mode 1): Q  = Q1 R2^{-1} (+ shadow), R = R2 R1
-template <int MODE>
-__global__ void __launch_bounds__(CQ_THREADS) cq_apply_kernel(CqArgs a) {
-    extern __shared__ double dsm[];
-    double* Rs = dsm;                    // 32 x 33
-    double* Ri = Rs + 32 * 33;           // 32 x 33
-    float* Rif = reinterpret_cast<float*>(Ri + 32 * 33);            // 32 x 33 fp32 R^{-1}
-    double* sred = reinterpret_cast<double*>(Rif + 32 * 34);        // [CQ_GROUPS][1024]
-    float* tile = reinterpret_cast<float*>(sred + CQ_GROUPS * 1024); // 32 x CQ_LD
-    const int tid = threadIdx.x;
-    if (*a.fail) return;   // an earlier pivot failed: the MGS fallback owns this panel
-    const double* Gin = a.G + (MODE == 0 ? 0 : 1024);
-    const bool ok = chol_inv(Gin, Rs, Ri, a.nc);
-    if (!ok) {
-        if (tid == 0) atomicExch(a.fail, 1);
-        return;
-    }
-    for (int e = tid; e < 32 * 32; e += CQ_THREADS) {
-        const int i = e & 31, j = e >> 5;
-        Rif[i * 33 + j] = (float)Ri[i * 33 + j];
-    }
-    if (MODE == 0 && blockIdx.x == 0)
-        for (int e = tid; e < 32 * 32; e += CQ_THREADS) a.Rkeep[e] = Rs[(e & 31) * 33 + (e >> 5)];
-    if (MODE == 1 && blockIdx.x == 0) {
-        // R = R2 R1 (fp64 product of upper-triangular factors, positive diagonal)
-        for (int e = tid; e < a.nc * a.nc; e += CQ_THREADS) {
-            const int i = e % a.nc, j = e / a.nc;
-            double s = 0.0;
-            for (int k = i; k <= j; ++k) s = fma(Rs[i * 33 + k], a.Rkeep[k + j * 32], s);
-            a.R[i + (int64_t)j * a.ldr] = (i <= j) ? (float)s : 0.f;
-        }
-    }
-    __syncthreads();
-    const int g = tid / CQ_BLK, blk = tid % CQ_BLK;
-    double acc[4][4] = {};
-    const float* src = MODE == 0 ? a.P : a.Q1;
-    const int64_t lds = MODE == 0 ? a.ldp : a.m;
-    const int64_t rows_per_cta = (a.m + gridDim.x - 1) / gridDim.x;
-    const int64_t r0 = (int64_t)blockIdx.x * rows_per_cta;
-    const int64_t r1 = min(a.m, r0 + rows_per_cta);
-    const int row = tid & (CQ_TILE - 1), half = tid >> 7;   // 2 threads per row: columns [16 half, 16 half + 16)
-    for (int64_t base = r0; base < r1; base += CQ_TILE) {
-        const int rows = (int)((r1 - base) < CQ_TILE ? (r1 - base) : CQ_TILE);
-        __syncthreads();
-        for (int e = tid; e < CQ_TILE * CQ_NB; e += CQ_THREADS) {
-            const int r = e % CQ_TILE, c = e / CQ_TILE;
-            tile[c * CQ_LD + r] = (r < rows && c < a.nc) ? src[base + r + (int64_t)c * lds] : 0.f;
-        }
-        __syncthreads();
-        float out[16];
+        if (PASS > 0) {
+            tile_times_rinv(tile, Ri[0], tid);                 // tile <- Q1 = P R1^{-1}
+            if (PASS == 2) tile_times_rinv(tile, Ri[1], tid);  // tile <- Q = Q1 R2^{-1}
+            if (write_q) {
 #pragma unroll
-        for (int jj = 0; jj < 16; ++jj) out[jj] = 0.f;
-        if (row < rows) {
-#pragma unroll 4
-            for (int k = 0; k < CQ_NB; ++k) {
-                const float x = tile[k * CQ_LD + row];
-#pragma unroll
-                for (int jj = 0; jj < 16; ++jj) out[jj] = fmaf(x, Rif[k * 33 + half * 16 + jj], out[jj]);
-            }
-        }
-        __syncthreads();
-        if (row < rows) {
-#pragma unroll
-            for (int jj = 0; jj < 16; ++jj) {
-                const int c = half * 16 + jj;
-                if (c < a.nc) {
-                    const int64_t gr = base + row;
-                    if (MODE == 0) {
-                        a.Q1[gr + (int64_t)c * a.m] = out[jj];
-                        tile[c * CQ_LD + row] = out[jj];
-                    } else {
-                        a.Q[gr + (int64_t)c * a.ldq] = out[jj];
+                for (int k = 0; k < 16; ++k) {
+                    const int e = tid + k * CQ_THREADS;
+                    const int r = e % CQ_TILE, c = e / CQ_TILE;
+                    if (r < rows && c < a.nc) {
+                        const float v = tile[c * CQ_LD + r];
+                        const int64_t gr = base + r;
+                        a.Q[gr + (int64_t)c * a.ldq] = v;
                         if (a.Qh) {
-                            const uint16_t hb = cq_to16(out[jj], a.bf16);
+                            const uint16_t hb = cq_to16(v, a.bf16);
                             a.Qh[gr + (int64_t)c * a.ldh] = hb;
-                            if (a.Ql) a.Ql[gr + (int64_t)c * a.ldh] = cq_to16((out[jj] - cq_from16(hb, a.bf16)) * 2048.f,
-                                                                             a.bf16);
+                            if (a.Ql) a.Ql[gr + (int64_t)c * a.ldh] = cq_to16((v - cq_from16(hb, a.bf16)) * 2048.f,
+                                                                               a.bf16);
                         }
                     }
                 }
             }
         }
-        if (MODE == 0) {
-            __syncthreads();
-            if (g < CQ_GROUPS) gram_block_accum(tile, rows, g, blk, acc);
+        if (gram && g < CQ_GROUPS) gram_block_accum(tile, rows, g, bi, bj, acc);
+    }
+    if (!gram) return;
+    // ---- CTA partial Gram: sum the 7 row-group accumulators (2 at a time through smem)
+    double* out = a.ws.part + (int64_t)blockIdx.x * 1024;
+    for (int round = 0; round < 4; ++round) {
+        const int g0 = round * 2;
+        __syncthreads();
+        for (int e = tid; e < 2 * 1024; e += CQ_THREADS) (&sred[0][0])[e] = 0.0;
+        __syncthreads();
+        if (g >= g0 && g < g0 + 2 && g < CQ_GROUPS) {
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+#pragma unroll
+                for (int v = 0; v < 4; ++v) sred[g - g0][(bi * 4 + u) + (bj * 4 + v) * 32] = acc[u][v];
+        }
+        __syncthreads();
+        for (int e = tid; e < 1024; e += CQ_THREADS) {
+            const int i = e & 31, j = e >> 5;
+            double s = (round == 0) ? 0.0 : out[e];
+            s += sred[0][e] + sred[1][e];
+            out[e] = (i <= j) ? s : 0.0;
         }
     }
-    if (MODE == 0) {
-        __syncthreads();
-        cta_gram_flush(sred, acc, blk, g, a.part + (int64_t)blockIdx.x * 1024);
-        if (!a.distributed) last_block_reduce(a, a.G + 1024);
-    }
+    __syncthreads();
+    reduce_and_factor(a, PASS, &sred[0][0], reinterpret_cast<double*>(tile));
 }
 
-// distributed mode: sum the CTA partials (fixed order) into G (before the NCCL allreduce)
-__global__ void cq_sum_parts_kernel(const double* __restrict__ part, int nparts, double* __restrict__ G) {
-    const int e = blockIdx.x * blockDim.x + threadIdx.x;
-    if (e >= 1024) return;
-    double s = 0.0;
-    if ((e & 31) <= (e >> 5))
-        for (int c = 0; c < nparts; ++c) s += part[(int64_t)c * 1024 + e];
-    G[e] = s;
+// distributed mode: after the host allreduce of G (pass `pass`), factor it (one warp)
+__global__ void cq_factor_kernel(CqArgs a, int pass) {
+    __shared__ double Rs[32 * 33];
+    __shared__ double R1s[32 * 33];
+    __shared__ int s_ok;
+    if (pass > 0 && *(volatile int*)a.ws.fail) return;
+    if (threadIdx.x < 32) {
+        const bool ok = chol_inv_warp(a.ws.G + pass * 1024, a.nc, a.ws.R + pass * 1024, a.ws.Rinv + pass * 1024, Rs);
+        if (threadIdx.x == 0) {
+            s_ok = ok;
+            if (!ok) *a.ws.fail = 1;
+        }
+    }
+    __syncthreads();
+    if (pass == 0 && s_ok) single_pass_decision(a);
+    if (pass == 1 && s_ok) final_r_product(a, Rs, R1s);
 }
 
 // ------------------------------------------------------------------ host side
 static int cq_grid(int64_t m) {
-    int64_t g = (m + 511) / 512;   // >= 512 rows per CTA keeps the per-CTA Cholesky amortised
+    int64_t g = (m + 511) / 512;   // >= 512 rows (4 tiles) per CTA
     if (g > 148) g = 148;
     if (g < 1) g = 1;
     return (int)g;
 }
 
-size_t cholqr_ws_doubles(int64_t m) { return (size_t)cq_grid(m) * 1024 + 3 * 1024 + 64; }
+size_t cholqr_ws_doubles(int64_t m) {
+    const int grid = cq_grid(m);
+    const int ngroups = (grid + CQ_FAN - 1) / CQ_FAN;
+    return (size_t)(grid + ngroups) * 1024 + 4 * 1024 + 1024 /*Rinv fp32 x2*/ + 64;
+}
+
+size_t cholqr_counter_ints(int64_t m) {
+    const int grid = cq_grid(m);
+    return (size_t)(grid + CQ_FAN - 1) / CQ_FAN + 2;
+}
 
 cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st) {
     CqArgs a{};
     a.P = L.P;
     a.ldp = L.ldp;
-    a.Q1 = L.Q1;
     a.Q = L.Q;
     a.ldq = L.ldq;
     a.Qh = L.Qh;
@@ -346,45 +455,35 @@ cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st) {
     a.m = L.m;
     a.nc = L.nc;
     const int grid = cq_grid(L.m);
-    a.part = L.ws;
-    a.G = L.ws + (size_t)grid * 1024;
-    a.Rkeep = a.G + 2048;
-    a.counter = L.counter;
-    a.fail = L.fail;
-    a.R = L.R;
+    const int ngroups = (grid + CQ_FAN - 1) / CQ_FAN;
+    a.ws.part = L.ws;
+    a.ws.gpart = a.ws.part + (size_t)grid * 1024;
+    a.ws.G = a.ws.gpart + (size_t)ngroups * 1024;
+    a.ws.R = a.ws.G + 2048;
+    a.ws.Rinv = reinterpret_cast<float*>(a.ws.R + 2048);
+    a.ws.counters = L.counter;
+    a.ws.fail = L.fail;
+    a.Rout = L.R;
     a.ldr = L.ldr;
     a.bf16 = L.bf16;
     a.distributed = L.allreduce_g != nullptr;
-    const size_t smem1 = (size_t)CQ_GROUPS * 1024 * 8 + (size_t)32 * CQ_LD * 4;
-    const size_t smem2 = (size_t)2 * 32 * 33 * 8 + 32 * 34 * 4 + (size_t)CQ_GROUPS * 1024 * 8 + (size_t)32 * CQ_LD * 4;
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(cq_gram_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem1);
-        cudaFuncSetAttribute(cq_apply_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2);
-        cudaFuncSetAttribute(cq_apply_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2);
-        attr = true;
-    }
-    ++g_launches;
-    cq_gram_kernel<<<grid, CQ_THREADS, smem1, st>>>(a);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return e;
-    if (a.distributed) {
+    cudaError_t e;
+    for (int pass = 0; pass < 3; ++pass) {
         ++g_launches;
-        cq_sum_parts_kernel<<<4, 256, 0, st>>>(a.part, grid, a.G);
-        if (L.allreduce_g(a.G, L.ctx) != 0) return cudaErrorUnknown;
+        if (pass == 0) cq_pass_kernel<0><<<grid, CQ_THREADS, 0, st>>>(a);
+        if (pass == 1) cq_pass_kernel<1><<<grid, CQ_THREADS, 0, st>>>(a);
+        if (pass == 2) cq_pass_kernel<2><<<grid, CQ_THREADS, 0, st>>>(a);
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        if (a.distributed && pass < 2) {
+            if (L.allreduce_g(a.ws.G + pass * 1024, L.ctx) != 0) return cudaErrorUnknown;
+            ++g_launches;
+            cq_factor_kernel<<<1, 256, 0, st>>>(a, pass);
+            e = cudaGetLastError();
+            if (e != cudaSuccess) return e;
+        }
     }
-    ++g_launches;
-    cq_apply_kernel<0><<<grid, CQ_THREADS, smem2, st>>>(a);
-    e = cudaGetLastError();
-    if (e != cudaSuccess) return e;
-    if (a.distributed) {
-        ++g_launches;
-        cq_sum_parts_kernel<<<4, 256, 0, st>>>(a.part, grid, a.G + 1024);
-        if (L.allreduce_g(a.G + 1024, L.ctx) != 0) return cudaErrorUnknown;
-    }
-    ++g_launches;
-    cq_apply_kernel<1><<<grid, CQ_THREADS, smem2, st>>>(a);
-    return cudaGetLastError();
+    return cudaSuccess;
 }
 
 }  // namespace rg

@@ -140,7 +140,7 @@ struct rg_handle_s {
     int rank = 0, nranks = 1;
     int64_t last_info = -1;
     // workspace
-    DevBuf cq_q1, cq_ws, cq_flags;                  // CholQR2 panel workspace (flags: counter, fail)
+    DevBuf cq_ws, cq_flags;                         // CholQR2 panel workspace (flags: fail, counters)
     DevBuf qh, ql, P, r12h, r12l, r12f, partial, norm2, scale, status, pws, pcnt, rgather, rstackq;
     DevBuf stageA, stageQ, stageR, stageB, stageX;  // host-pointer staging
     DevBuf cg;                                      // CGLS vectors
@@ -151,7 +151,7 @@ struct rg_handle_s {
     DevBuf aux;                                     // misc (orthogonalize / lowrank)
     int* status_host = nullptr;                     // pinned
     long long last_launches = 0;                    // kernels launched by the last API call
-    std::unique_ptr<Plan> plan;
+    std::vector<std::unique_ptr<Plan>> plans;      // LRU, most recent first
     // profiling
     bool prof = false;
     double prof_ms[PC_N] = {0};
@@ -298,8 +298,22 @@ int make_plan(rg_handle h, Plan& pl) {
             o.tiles_j = (o.w + o.bn - 1) / o.bn;
             o.kb_total = (int)((m + 63) / 64);
             const int tiles = o.tiles_i * o.tiles_j;
-            int splits = std::max(1, (2 * 148 + tiles / 2) / tiles);
-            splits = std::min(splits, std::max(1, o.kb_total / 4));
+            int splits = 1;
+            if (tiles >= 32) {
+                // balance whole waves of 148 persistent CTAs against split-K partial traffic
+                double best = -1.0;
+                for (int s = 1; s <= std::min(32, std::max(1, o.kb_total / 8)); ++s) {
+                    const double units = (double)tiles * s;
+                    const double eff = units / 148.0 / std::ceil(units / 148.0) - 0.01 * s;
+                    if (eff > best + 1e-9) {
+                        best = eff;
+                        splits = s;
+                    }
+                }
+            } else {
+                // small outputs are bandwidth/latency bound: spread the m rows over ~one wave
+                splits = std::max(1, std::min(148 / tiles, o.kb_total / 8));
+            }
             o.kb_per_split = (o.kb_total + splits - 1) / splits;
             o.splits = (o.kb_total + o.kb_per_split - 1) / o.kb_per_split;
             pmax = std::max(pmax, (size_t)o.splits * o.tiles_j * o.bn * o.tiles_i * 128);
@@ -335,8 +349,8 @@ bool ensure_workspace(rg_handle h, int64_t m, int64_t n, int split) {
               h->scale.ensure(n * 4 + 64) && h->status.ensure(64) &&
               h->pws.ensure(rg::panel_ws_floats(m) * 4 + 4096) && h->pcnt.ensure(rg::panel_counters(m) * 4 + 64) &&
               h->rgather.ensure((size_t)64 * 32 * 32 * 4) && h->rstackq.ensure((size_t)64 * 32 * 32 * 4) &&
-              h->cq_q1.ensure((size_t)std::max<int64_t>(m, 8) * 32 * 4) &&
-              h->cq_ws.ensure(rg::cholqr_ws_doubles(m) * 8 + 256) && h->cq_flags.ensure(64);
+              h->cq_ws.ensure(rg::cholqr_ws_doubles(m) * 8 + 256) &&
+              h->cq_flags.ensure((rg::cholqr_counter_ints(m) + 8) * 4);
     return ok;
 }
 
@@ -361,12 +375,14 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     uint16_t* qh = h->qh.as<uint16_t>();
     uint16_t* ql = pl.split ? h->ql.as<uint16_t>() : nullptr;
     int* status = h->status.as<int>();
-    const bool dist = h->nranks > 1 && h->comm;
+    const bool dist = pl.nranks > 1 && h->comm;
     {
         ProfScope _s(h, PC_SCALE, 0, (double)m * n * (pl.split ? 16 : 14));
         RG_CUDA(rg::launch_colnorm(pl.A, pl.lda, m, n, h->partial.as<double>(), h->norm2.as<double>(), st));
-        int rc = nccl_allreduce(h, h->norm2.p, n, ncclFloat64);
-        if (rc) return rc;
+        if (dist) {
+            int rc = nccl_allreduce(h, h->norm2.p, n, ncclFloat64);
+            if (rc) return rc;
+        }
         RG_CUDA(rg::launch_colscale(h->norm2.as<double>(), n, pl.scale, h->scale.as<float>(), status, 0, st));
         RG_CUDA(rg::launch_scale_cast(pl.A, pl.lda, pl.Q, pl.ldq, qh, ql, pl.ldh, m, n, h->scale.as<float>(), pl.bf16,
                                       st));
@@ -389,13 +405,13 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             p.col0 = o.c0;
             p.status = status;
             float* Rdiag = pl.R + o.c0 + (int64_t)o.c0 * pl.ldr;
-            int* cq_fail = h->cq_flags.as<int>() + 1;
+            int* cq_fail = h->cq_flags.as<int>();
+            int* cq_counters = cq_fail + 4;
             if (pl.panel == 0) {
                 // CholQR2 (fp64 Gram); the MGS/TSQR kernels below run only if a pivot failed
                 rg::CholqrLaunch c{};
                 c.P = p.Q;
                 c.ldp = pl.ldq;
-                c.Q1 = h->cq_q1.as<float>();
                 c.Q = p.Q;
                 c.ldq = pl.ldq;
                 c.Qh = p.Qh;
@@ -404,7 +420,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
                 c.m = m;
                 c.nc = o.w;
                 c.ws = h->cq_ws.as<double>();
-                c.counter = h->cq_flags.as<int>();
+                c.counter = cq_counters;
                 c.fail = cq_fail;
                 c.R = Rdiag;
                 c.ldr = pl.ldr;
@@ -496,32 +512,55 @@ int check_status(rg_handle h) {
     return RG_OK;
 }
 
-// run one RGSQR pass (device pointers), with plan caching + CUDA graph replay
+// run one RGSQR pass (device pointers), with an LRU cache of plans + CUDA graph replay.
+// local = true forces the single-GPU path even in row-sharded mode (used for the small
+// replicated factorizations of lowrank_approx).
 int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq, float* R,
-              int64_t ldr, const rg_opts& o, int split) {
+              int64_t ldr, const rg_opts& o, int split, bool local = false) {
     if (!ensure_workspace(h, m, n, split)) return RG_ALLOC;
     const int nb = (o.nb <= 0 || o.nb > 32) ? 32 : o.nb;
-    Plan* pl = h->plan.get();
-    const bool same = pl && pl->m == m && pl->n == n && pl->lda == lda && pl->ldq == ldq && pl->ldr == ldr &&
-                      pl->A == A && pl->Q == Q && pl->R == R && pl->nb == nb && pl->bf16 == o.precision &&
-                      pl->split == split && pl->scale == o.scale && pl->nranks == h->nranks &&
-                      pl->rank == h->rank && pl->panel == o.panel && pl->epoch == g_alloc_epoch;
-    if (!same) {
-        if (pl && pl->exec) cudaGraphExecDestroy(pl->exec);
-        h->plan.reset(new Plan());
-        pl = h->plan.get();
-        pl->m = m; pl->n = n; pl->lda = lda; pl->ldq = ldq; pl->ldr = ldr;
-        pl->A = A; pl->Q = Q; pl->R = R;
-        pl->nb = nb; pl->bf16 = o.precision; pl->split = split; pl->scale = o.scale;
-        pl->nranks = h->nranks; pl->rank = h->rank; pl->panel = o.panel;
-        int rc = make_plan(h, *pl);
+    const int nranks = local ? 1 : h->nranks;
+    Plan* pl = nullptr;
+    for (size_t i = 0; i < h->plans.size(); ++i) {
+        Plan* c = h->plans[i].get();
+        if (c->m == m && c->n == n && c->lda == lda && c->ldq == ldq && c->ldr == ldr && c->A == A && c->Q == Q &&
+            c->R == R && c->nb == nb && c->bf16 == o.precision && c->split == split && c->scale == o.scale &&
+            c->nranks == nranks && c->rank == h->rank && c->panel == o.panel) {
+            if (c->epoch != g_alloc_epoch) {   // a workspace buffer moved: rebuild this plan
+                if (c->exec) cudaGraphExecDestroy(c->exec);
+                h->plans.erase(h->plans.begin() + i);
+                break;
+            }
+            pl = c;
+            std::rotate(h->plans.begin(), h->plans.begin() + i, h->plans.begin() + i + 1);   // most recent first
+            break;
+        }
+    }
+    if (!pl) {
+        std::unique_ptr<Plan> np(new Plan());
+        np->m = m; np->n = n; np->lda = lda; np->ldq = ldq; np->ldr = ldr;
+        np->A = A; np->Q = Q; np->R = R;
+        np->nb = nb; np->bf16 = o.precision; np->split = split; np->scale = o.scale;
+        np->nranks = nranks; np->rank = h->rank; np->panel = o.panel;
+        int rc = make_plan(h, *np);
         if (rc) return rc;
-        if (!h->P.ensure(pl->p_floats * 4 + 4096)) return RG_ALLOC;
-        pl->epoch = g_alloc_epoch;  // P may have moved: the graph is captured below, after this
+        if (!h->P.ensure(np->p_floats * 4 + 4096)) return RG_ALLOC;
+        np->epoch = g_alloc_epoch;
+        // invalidate older plans if P just moved (their graphs captured the old pointer)
+        for (auto& c : h->plans)
+            if (c->epoch != g_alloc_epoch && c->exec) {
+                cudaGraphExecDestroy(c->exec);
+                c->exec = nullptr;
+            }
+        h->plans.insert(h->plans.begin(), std::move(np));
+        while (h->plans.size() > 8) {
+            if (h->plans.back()->exec) cudaGraphExecDestroy(h->plans.back()->exec);
+            h->plans.pop_back();
+        }
+        pl = h->plans.front().get();
     }
     int rc = reset_status(h);
     if (rc) return rc;
-    h->last_launches += 0;
     const bool use_graph = !h->prof && getenv("RGSQR_NO_GRAPH") == nullptr;
     if (!use_graph) {
         rc = enqueue_rgsqr(h, *pl);
@@ -551,8 +590,6 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
     h->last_launches += pl->launches;
     return RG_OK;
 }
-
-
 
 // R <- R2 R (both upper triangular n x n), via a scratch copy
 int trmm_into(rg_handle h, const float* R2, int64_t ld2, float* R, int64_t ldr, int n) {
@@ -703,10 +740,6 @@ int rg_create(rg_handle* out, int device, void* stream) {
 
 int rg_set_stream(rg_handle h, void* stream) {
     if (!h) return -1;
-    if (h->plan && h->plan->exec) {
-        cudaGraphExecDestroy(h->plan->exec);
-        h->plan->exec = nullptr;
-    }
     h->stream = reinterpret_cast<cudaStream_t>(stream);
     return RG_OK;
 }
@@ -715,11 +748,12 @@ int rg_destroy(rg_handle h) {
     if (!h) return -1;
     cudaSetDevice(h->device);
     cudaStreamSynchronize(h->stream);
-    if (h->plan && h->plan->exec) cudaGraphExecDestroy(h->plan->exec);
+    for (auto& p : h->plans)
+        if (p->exec) cudaGraphExecDestroy(p->exec);
     DevBuf* bufs[] = {&h->qh, &h->ql, &h->P, &h->r12h, &h->r12l, &h->r12f, &h->partial, &h->norm2, &h->scale,
                       &h->status, &h->pws, &h->pcnt, &h->rgather, &h->rstackq, &h->stageA, &h->stageQ,
                       &h->stageR, &h->stageB, &h->stageX, &h->cg, &h->aux,
-                      &h->lsQ, &h->lsR, &h->rinv, &h->probeG, &h->probeW, &h->cq_q1, &h->cq_ws,
+                      &h->lsQ, &h->lsR, &h->rinv, &h->probeG, &h->probeW, &h->cq_ws,
                       &h->cq_flags};
     if (h->cgls_exec) cudaGraphExecDestroy(h->cgls_exec);
     for (auto* b : bufs) b->release();
@@ -779,11 +813,9 @@ int rg_comm_init(rg_handle h, const void* id128, int rank, int nranks) {
     h->comm = c;
     h->rank = rank;
     h->nranks = nranks;
-    if (h->plan && h->plan->exec) {
-        cudaGraphExecDestroy(h->plan->exec);
-        h->plan->exec = nullptr;
-    }
-    h->plan.reset();
+    for (auto& p : h->plans)
+        if (p->exec) cudaGraphExecDestroy(p->exec);
+    h->plans.clear();
     return RG_OK;
 }
 

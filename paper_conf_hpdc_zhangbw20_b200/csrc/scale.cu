@@ -96,11 +96,11 @@ __global__ void __launch_bounds__(256) scale_cast_kernel(const float* __restrict
     const int j = blockIdx.y;
     const float s = scale ? scale[j] : 1.0f;
     const float* a = A + (int64_t)j * lda;
-    float* q = Q + (int64_t)j * ldq;
+    float* q = Q ? Q + (int64_t)j * ldq : nullptr;
     uint16_t* qh = Qh ? Qh + (int64_t)j * ldh : nullptr;
     uint16_t* ql = Ql ? Ql + (int64_t)j * ldh : nullptr;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    const bool vec = ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(q)) & 15) == 0 &&
+    const bool vec = ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(q)) & 15) == 0 && q &&
                      (!qh || (reinterpret_cast<uintptr_t>(qh) & 7) == 0) &&
                      (!ql || (reinterpret_cast<uintptr_t>(ql) & 7) == 0);
     if (vec) {
@@ -135,7 +135,7 @@ __global__ void __launch_bounds__(256) scale_cast_kernel(const float* __restrict
     } else {
         for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += stride) {
             const float x = a[i] * s;
-            q[i] = x;
+            if (q) q[i] = x;
             if (qh) {
                 const uint16_t h = s_to16(x, bf16);
                 qh[i] = h;

@@ -1,0 +1,88 @@
+// Standalone timing harness for the CholQR2 panel passes (development tool, not product).
+// nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -I include tools/cq_bench.cu \
+//   paper_conf_hpdc_zhangbw20_b200/csrc/panel_cholqr.cu -o tools/cq_bench
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
+#include <cuda_runtime.h>
+#include "../paper_conf_hpdc_zhangbw20_b200/csrc/panel_cholqr.cu"
+namespace rg { thread_local long long g_launches = 0; }
+int main(int argc, char** argv) {
+    const int64_t m = argc > 1 ? atoll(argv[1]) : 65536;
+    const int nc = 32;
+    std::vector<float> h(m * nc);
+    srand(1);
+    for (auto& x : h) x = (rand() / (float)RAND_MAX) - 0.5f;
+    float *P, *Q, *R; uint16_t* Qh; double* ws; int* flags;
+    cudaMalloc(&P, m * nc * 4); cudaMalloc(&Q, m * nc * 4); cudaMalloc(&R, 32 * 32 * 4);
+    cudaMalloc(&Qh, m * nc * 2);
+    cudaMalloc(&ws, rg::cholqr_ws_doubles(m) * 8); cudaMalloc(&flags, 4096);
+    cudaMemset(flags, 0, 4096);
+    cudaMemcpy(P, h.data(), m * nc * 4, cudaMemcpyHostToDevice);
+    rg::CholqrLaunch L{};
+    L.P = P; L.ldp = m; L.Q = Q; L.ldq = m; L.Qh = Qh; L.ldh = m; L.m = m; L.nc = nc; L.ws = ws;
+    L.fail = flags; L.counter = flags + 4; L.R = R; L.ldr = 32;
+    cudaStream_t st; cudaStreamCreate(&st);
+    for (int i = 0; i < 5; ++i) rg::launch_panel_cholqr(L, st);
+    cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
+    const int iters = 50;
+    cudaEventRecord(a, st);
+    for (int i = 0; i < iters; ++i) rg::launch_panel_cholqr(L, st);
+    cudaEventRecord(b, st);
+    cudaEventSynchronize(b);
+    float ms; cudaEventElapsedTime(&ms, a, b);
+    printf("m=%lld cholqr2 panel: %.2f us per panel (eager launches)\n", (long long)m, ms * 1000 / iters);
+    // graph-captured
+    cudaGraph_t g; cudaGraphExec_t ge;
+    cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
+    for (int i = 0; i < iters; ++i) rg::launch_panel_cholqr(L, st);
+    cudaStreamEndCapture(st, &g);
+    cudaGraphInstantiate(&ge, g, 0);
+    cudaGraphLaunch(ge, st);
+    cudaStreamSynchronize(st);
+    cudaEventRecord(a, st);
+    cudaGraphLaunch(ge, st);
+    cudaEventRecord(b, st);
+    cudaEventSynchronize(b);
+    cudaEventElapsedTime(&ms, a, b);
+    printf("m=%lld cholqr2 panel: %.2f us per panel (graph)\n", (long long)m, ms * 1000 / iters);
+    // per-pass timing (eager, 50 launches each)
+    {
+        rg::CqArgs A{};
+        A.P = P; A.ldp = m; A.Q = Q; A.ldq = m; A.Qh = Qh; A.ldh = m; A.m = m; A.nc = nc;
+        const int grid = rg::cq_grid(m);
+        const int ngroups = (grid + rg::CQ_FAN - 1) / rg::CQ_FAN;
+        A.ws.part = ws; A.ws.gpart = ws + (size_t)grid * 1024; A.ws.G = A.ws.gpart + (size_t)ngroups * 1024;
+        A.ws.R = A.ws.G + 2048; A.ws.Rinv = reinterpret_cast<float*>(A.ws.R + 2048);
+        A.ws.counters = flags + 4; A.ws.fail = flags; A.Rout = R; A.ldr = 32;
+        for (int pass = 0; pass < 3; ++pass) {
+            cudaEventRecord(a, st);
+            for (int i = 0; i < iters; ++i) {
+                if (pass == 0) rg::cq_pass_kernel<0><<<grid, rg::CQ_THREADS, 0, st>>>(A);
+                if (pass == 1) rg::cq_pass_kernel<1><<<grid, rg::CQ_THREADS, 0, st>>>(A);
+                if (pass == 2) rg::cq_pass_kernel<2><<<grid, rg::CQ_THREADS, 0, st>>>(A);
+            }
+            cudaEventRecord(b, st);
+            cudaEventSynchronize(b);
+            cudaEventElapsedTime(&ms, a, b);
+            printf("  pass %d: %.2f us\n", pass, ms * 1000 / iters);
+        }
+        // chol-only kernel timing
+        cudaEventRecord(a, st);
+        for (int i = 0; i < iters; ++i) rg::cq_factor_kernel<<<1, 256, 0, st>>>(A, 0);
+        cudaEventRecord(b, st);
+        cudaEventSynchronize(b);
+        cudaEventElapsedTime(&ms, a, b);
+        printf("  chol_inv (1 CTA): %.2f us\n", ms * 1000 / iters);
+        A.distributed = 1;
+        cudaEventRecord(a, st);
+        for (int i = 0; i < iters; ++i) rg::cq_pass_kernel<0><<<grid, rg::CQ_THREADS, 0, st>>>(A);
+        cudaEventRecord(b, st);
+        cudaEventSynchronize(b);
+        cudaEventElapsedTime(&ms, a, b);
+        printf("  pass 0 without chol (distributed flag): %.2f us\n", ms * 1000 / iters);
+    }
+    int fl; cudaMemcpy(&fl, flags, 4, cudaMemcpyDeviceToHost);
+    printf("fail flag %d, err %s\n", fl, cudaGetErrorString(cudaGetLastError()));
+    return 0;
+}
