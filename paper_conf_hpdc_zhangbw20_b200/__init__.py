@@ -81,9 +81,6 @@ def _lib():
         L.rg_comm_unique_id.argtypes = [vp]
         L.rg_comm_init.argtypes = [vp, vp, i32, i32]
         L.rgsqr_factor.argtypes = [vp, i64, i64, vp, i64, vp, i64, vp, i64, ctypes.POINTER(rg_opts)]
-        for _name in ("lowrank_approx",):
-            if not hasattr(L, _name):  # TEMP during bring-up
-                setattr(L, _name, lambda *a: RG_CUDA_ERROR)
         L.orthogonalize.argtypes = [vp, i64, i64, vp, i64, vp, i64, ctypes.c_double, i32,
                                     ctypes.POINTER(i32), f64p, ctypes.POINTER(rg_opts)]
         L.ls_solve_refined.argtypes = [vp, i64, i64, vp, i64, vp, vp, ctypes.c_double, i32,
@@ -94,8 +91,6 @@ def _lib():
         L.rg_profile_reset.argtypes = [vp]
         L.rg_profile_get.argtypes = [vp, i32, f64p, ctypes.POINTER(i64), f64p, f64p]
         for name in EXPORTS:
-            if not hasattr(getattr(L, name), "restype"):
-                continue
             if getattr(L, name).restype is None and name not in ("rg_opts_default",):
                 getattr(L, name).restype = i32
         L.rg_opts_default.restype = None

@@ -106,6 +106,7 @@ __device__ __forceinline__ void gram_block_accum(const float* tile, int rows, in
 // Writes R (fp64 upper, R[i + 32 j]) and Rinv (fp32, Rinv[i + 32 j]); returns false if a
 // pivot is not safely positive (relative to the original diagonal).
 __device__ bool chol_inv_warp(const double* G, int nc, double* Rg, float* Rinvg, double* Rs /*smem 32x33*/) {
+    __shared__ double dinv[32];
     const int lane = threadIdx.x & 31;
     double g[32];   // lane i holds row i of the symmetric Gram
 #pragma unroll
@@ -118,18 +119,20 @@ __device__ bool chol_inv_warp(const double* G, int nc, double* Rg, float* Rinvg,
     for (int j = 0; j < 32; ++j)
         if (j == lane) orig = g[j];
     bool ok = true;
-    double inv_diag = 1.0;   // lane k keeps 1 / R(k,k)
+    // Right-looking Cholesky; the pivot chain is kept short: lane k+1 forms its own next pivot
+    // g(k+1,k+1) - R(k,k+1)^2 from its private row, and only that value crosses lanes.
+    double dkk = __shfl_sync(0xffffffffu, g[0], 0);
 #pragma unroll
     for (int k = 0; k < 32; ++k) {
-        const double dkk = __shfl_sync(0xffffffffu, g[k], k);
         const double okk = __shfl_sync(0xffffffffu, orig, k);
         const bool good = (dkk > okk * 1e-15) && isfinite(dkk);
         ok = ok && good;
         const double irk = good ? rsqrt(dkk) : 1.0;
         const double rkk = good ? dkk * irk : 1.0;
-        if (lane == k) inv_diag = irk;
-        // row k of the upper factor: R(k, lane); broadcast to the warp through smem
+        if (lane == k) dinv[k] = irk;
+        // l = R(k, lane): row k of the upper factor
         const double l = (lane > k) ? g[k] * irk : ((lane == k) ? rkk : 0.0);
+        if (k + 1 < 32) dkk = __shfl_sync(0xffffffffu, fma(-l, l, g[k + 1]), k + 1);
         Rs[k * 33 + lane] = l;
         __syncwarp();
 #pragma unroll
@@ -143,16 +146,20 @@ __device__ bool chol_inv_warp(const double* G, int nc, double* Rg, float* Rinvg,
     for (int i = 0; i < 32; ++i) x[i] = (i == j) ? 1.0 : 0.0;
 #pragma unroll
     for (int k = 31; k >= 0; --k) {
-        const double ik = __shfl_sync(0xffffffffu, inv_diag, k);
-        x[k] *= ik;
+        x[k] *= dinv[k];
 #pragma unroll
         for (int i = 0; i < k; ++i) x[i] = fma(-Rs[i * 33 + k], x[k], x[i]);
     }
+    // coalesced stores: transpose through smem (Rs is no longer needed after this point)
 #pragma unroll
-    for (int i = 0; i < 32; ++i) {
-        Rinvg[i + 32 * j] = (float)x[i];
-        Rg[i + 32 * j] = (i <= j) ? Rs[i * 33 + j] : 0.0;
-    }
+    for (int i = 0; i < 32; ++i) Rg[i + 32 * j] = (i <= j) ? Rs[i * 33 + j] : 0.0;
+    __syncwarp();
+#pragma unroll
+    for (int i = 0; i < 32; ++i) Rs[j * 33 + i] = x[i];   // Rs[j][i] = Rinv(i, j)
+    __syncwarp();
+#pragma unroll
+    for (int jj = 0; jj < 32; ++jj) Rinvg[lane + 32 * jj] = (float)Rs[jj * 33 + lane];
+    __syncwarp();
     return __all_sync(0xffffffffu, ok);
 }
 
@@ -426,8 +433,8 @@ __global__ void cq_factor_kernel(CqArgs a, int pass) {
 
 // ------------------------------------------------------------------ host side
 static int cq_grid(int64_t m) {
-    int64_t g = (m + 511) / 512;   // >= 512 rows (4 tiles) per CTA
-    if (g > 148) g = 148;
+    int64_t g = (m + 127) / 128;   // one or two 128-row tiles per CTA, two CTAs per SM
+    if (g > 296) g = 296;
     if (g < 1) g = 1;
     return (int)g;
 }

@@ -145,12 +145,15 @@ struct rg_handle_s {
     DevBuf stageA, stageQ, stageR, stageB, stageX;  // host-pointer staging
     DevBuf cg;                                      // CGLS vectors
     DevBuf lsQ, lsR, rinv, probeG, probeW;          // ls_solve_refined / orthogonalize workspace
+    DevBuf lrA16, lrB16, lrB16l, lrY, lrZ, lrQ16, lrQ16l, lrR, lrW, lrV, lrUb, lrVb, lrSig, lrOm, lrScale, lrFlags;
     cudaGraphExec_t cgls_exec = nullptr;            // captured block of CGLS iterations
     const void* cgls_key[4] = {nullptr, nullptr, nullptr, nullptr};
     int64_t cgls_key_mn[3] = {0, 0, 0};
     DevBuf aux;                                     // misc (orthogonalize / lowrank)
     int* status_host = nullptr;                     // pinned
     long long last_launches = 0;                    // kernels launched by the last API call
+    long long call_g0 = 0;                          // rg::g_launches at the start of the call
+    long long replayed = 0;                         // kernels in CUDA-graph replays of this call
     std::vector<std::unique_ptr<Plan>> plans;      // LRU, most recent first
     // profiling
     bool prof = false;
@@ -491,6 +494,13 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     return RG_OK;
 }
 
+void begin_call(rg_handle h) {
+    h->call_g0 = rg::g_launches;
+    h->replayed = 0;
+    h->last_launches = 0;
+}
+void end_call(rg_handle h) { h->last_launches = (rg::g_launches - h->call_g0) + h->replayed; }
+
 int reset_status(rg_handle h) {
     static const int init[4] = {INT_MAX, INT_MAX, 0, 0};
     RG_CUDA(cudaMemcpyAsync(h->status.p, init, sizeof(init), cudaMemcpyHostToDevice, h->stream));
@@ -562,11 +572,7 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
     int rc = reset_status(h);
     if (rc) return rc;
     const bool use_graph = !h->prof && getenv("RGSQR_NO_GRAPH") == nullptr;
-    if (!use_graph) {
-        rc = enqueue_rgsqr(h, *pl);
-        h->last_launches += pl->launches;
-        return rc;
-    }
+    if (!use_graph) return enqueue_rgsqr(h, *pl);
     if (!pl->exec) {
         // capture on the private stream (the user's may be the legacy stream, which cannot
         // capture); the instantiated graph is then launched on the user's stream
@@ -574,7 +580,9 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
         cudaStream_t user = h->stream;
         h->stream = h->capture_stream;
         RG_CUDA(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
+        const long long cap0 = rg::g_launches;
         rc = enqueue_rgsqr(h, *pl);
+        rg::g_launches = cap0;   // captured, not launched: the replay below is counted instead
         cudaError_t ce = cudaStreamEndCapture(h->stream, &g);
         h->stream = user;
         if (rc) {
@@ -587,7 +595,7 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
         RG_CUDA(ie);
     }
     RG_CUDA(cudaGraphLaunch(pl->exec, h->stream));
-    h->last_launches += pl->launches;
+    h->replayed += pl->launches;
     return RG_OK;
 }
 
@@ -669,6 +677,48 @@ int enqueue_cgls_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int 
     return RG_OK;
 }
 
+
+// ------------------------------------------------------------------ general GEMMs (lowrank)
+// C (m x N fp32, ldc) = A (m x K, MN-major 16-bit, lda16) * B (K x N, K-major 16-bit, ldb16);
+// split: A_lo / B_lo images give ~fp32 accuracy (reading #9).
+int gemm_nn(rg_handle h, int64_t m, int N, int K, const uint16_t* Ah, const uint16_t* Al, int64_t lda16,
+            const uint16_t* Bh, const uint16_t* Bl, int64_t ldb16, float* C, int64_t ldc, int bf16) {
+    const int bn = pick_bn(N);
+    CUtensorMap ma, mb, mal, mbl;
+    const bool split = Al && Bl;
+    if (!encode_map(&ma, Ah, m, K, lda16, 64, 64, bf16) || !encode_map(&mb, Bh, K, N, ldb16, 64, bn, bf16) ||
+        !encode_map(&mal, split ? Al : Ah, m, K, lda16, 64, 64, bf16) ||
+        !encode_map(&mbl, split ? Bl : Bh, K, N, ldb16, 64, bn, bf16))
+        return RG_CUDA_ERROR;
+    RG_CUDA(rg::launch_update_gemm(bn, split, m, N, K, ma, mb, mal, mbl, C, ldc, nullptr, nullptr, 0, bf16, h->stream,
+                                   1));
+    return RG_OK;
+}
+
+// O (M x N fp32, ldo) = A^T B with A (K x M, K-major 16-bit, lda16) and B (K x N, lda16
+// layout ldb16): split-K over the K = m rows + deterministic reduction (K1 kernels).
+int gemm_tn(rg_handle h, int64_t K, int M, int N, const uint16_t* Ah, int64_t lda16, const uint16_t* Bh,
+            int64_t ldb16, float* O, int64_t ldo, int bf16) {
+    const int bn = pick_bn(N);
+    CUtensorMap ma, mb;
+    if (!encode_map(&ma, Ah, K, M, lda16, 64, 128, bf16) || !encode_map(&mb, Bh, K, N, ldb16, 64, bn, bf16))
+        return RG_CUDA_ERROR;
+    const int tiles_i = (M + 127) / 128, tiles_j = (N + bn - 1) / bn;
+    const int kb_total = (int)((K + 63) / 64);
+    const int tiles = tiles_i * tiles_j;
+    int splits = tiles >= 148 ? 1 : std::max(1, std::min(148 / tiles, kb_total / 8));
+    const int kps = (kb_total + splits - 1) / splits;
+    splits = (kb_total + kps - 1) / kps;
+    const int64_t ldp = (int64_t)tiles_i * 128;
+    const int64_t pstride = ldp * tiles_j * bn;
+    if (!h->P.ensure((size_t)splits * pstride * 4 + 4096)) return RG_ALLOC;
+    float* P = h->P.as<float>();
+    RG_CUDA(rg::launch_proj_gemm(bn, false, tiles_i, tiles_j, splits, ma, mb, ma, mb, P, ldp, pstride, kb_total, kps,
+                                 bf16, h->stream));
+    RG_CUDA(rg::launch_proj_reduce(P, ldp, pstride, splits, M, N, nullptr, 0, O, ldo, nullptr, nullptr, 0, bf16,
+                                   h->stream));
+    return RG_OK;
+}
 }  // namespace
 
 namespace rg {
@@ -753,7 +803,9 @@ int rg_destroy(rg_handle h) {
     DevBuf* bufs[] = {&h->qh, &h->ql, &h->P, &h->r12h, &h->r12l, &h->r12f, &h->partial, &h->norm2, &h->scale,
                       &h->status, &h->pws, &h->pcnt, &h->rgather, &h->rstackq, &h->stageA, &h->stageQ,
                       &h->stageR, &h->stageB, &h->stageX, &h->cg, &h->aux,
-                      &h->lsQ, &h->lsR, &h->rinv, &h->probeG, &h->probeW, &h->cq_ws,
+                      &h->lsQ, &h->lsR, &h->rinv, &h->probeG, &h->probeW, &h->cq_ws, &h->lrA16, &h->lrB16, &h->lrB16l, &h->lrY,
+                      &h->lrZ, &h->lrQ16, &h->lrQ16l, &h->lrR, &h->lrW, &h->lrV, &h->lrUb, &h->lrVb, &h->lrSig,
+                      &h->lrOm, &h->lrScale, &h->lrFlags,
                       &h->cq_flags};
     if (h->cgls_exec) cudaGraphExecDestroy(h->cgls_exec);
     for (auto* b : bufs) b->release();
@@ -861,7 +913,7 @@ int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_
     if (ldr < n) return -9;
     if (o.precision != 0 && o.precision != 1) return -10;
     cudaSetDevice(h->device);
-    h->last_launches = 0;
+    begin_call(h);
     const bool host = ptr_side(A) == SIDE_HOST;
     if (host && (ptr_side(Q) != SIDE_HOST || ptr_side(R) != SIDE_HOST)) return -6;
     const float* dA = A;
@@ -903,6 +955,7 @@ int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_
         RG_CUDA(cudaMemcpy2DAsync(R, ldr * 4, dR, dldr * 4, n * 4, n, cudaMemcpyDeviceToHost, h->stream));
     }
     if (o.sync || host) rc = check_status(h);
+    end_call(h);
     prof_collect(h);
     return rc;
 }
@@ -920,7 +973,7 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
     if (R && ldr < n) return -7;
     if (max_passes < 1) return -9;
     cudaSetDevice(h->device);
-    h->last_launches = 0;
+    begin_call(h);
     const bool host = ptr_side(A) == SIDE_HOST;
     float* dA = A;
     int64_t dlda = lda;
@@ -967,6 +1020,7 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
     if (host || o.sync) RG_CUDA(cudaStreamSynchronize(h->stream));
     if (passes_out) *passes_out = passes;
     if (orth_est_out) *orth_est_out = est;
+    end_call(h);
     prof_collect(h);
     if (orth_tol > 0 && est > orth_tol) return RG_NOT_CONVERGED;
     return RG_OK;
@@ -986,7 +1040,7 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     if (!(tol >= 0)) return -8;
     if (maxit < 0) return -9;
     cudaSetDevice(h->device);
-    h->last_launches = 0;
+    begin_call(h);
     const bool host = ptr_side(A) == SIDE_HOST;
     const float* dA = A;
     const float* db = b;
@@ -1054,6 +1108,8 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
                 RG_CUDA(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
                 const long long before = rg::g_launches;
                 rc = enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, blk, base);
+                const long long captured = rg::g_launches - before;
+                rg::g_launches = before;
                 h->cgls_key_mn[2] = dlda;
                 cudaError_t ce = cudaStreamEndCapture(h->stream, &g);
                 h->stream = user;
@@ -1067,14 +1123,13 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
                 h->cgls_key[2] = h->rinv.p;
                 h->cgls_key_mn[0] = m_local;
                 h->cgls_key_mn[1] = n;
-                h->cgls_key[3] = (const void*)(intptr_t)(rg::g_launches - before);
+                h->cgls_key[3] = (const void*)(intptr_t)captured;
             }
             RG_CUDA(cudaGraphLaunch(h->cgls_exec, h->stream));
-            h->last_launches += (long long)(intptr_t)h->cgls_key[3];
+            h->replayed += (long long)(intptr_t)h->cgls_key[3];
         } else {
             const long long before = rg::g_launches;
             rc = enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, cnt, base);
-            h->last_launches += rg::g_launches - before;
             if (rc) return rc;
         }
         done_iters += cnt;
@@ -1090,9 +1145,144 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     RG_CUDA(cudaStreamSynchronize(h->stream));
     if (iters_out) *iters_out = (int)hsc[7];
     if (relres_out) *relres_out = hsc[4] > 0 ? hsc[5] / hsc[4] : 0.0;
+    end_call(h);
     prof_collect(h);
     if (!(hsc[6] != 0.0) && maxit > 0 && !(hsc[5] <= tol * hsc[4])) return RG_NOT_CONVERGED;
     return RG_OK;
+}
+
+
+int lowrank_approx(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_t lda, int rank, int oversample,
+                   int power_iters, uint64_t seed, float* U, int64_t ldu, float* S, float* V, int64_t ldv,
+                   const rg_opts* opts) {
+    if (!h) return -1;
+    rg_opts o;
+    if (opts) o = *opts; else rg_opts_default(&o);
+    if (m_local < 1) return -2;
+    if (n < 1 || n > 65535) return -3;
+    if (!A) return -4;
+    if (lda < m_local) return -5;
+    const int l = rank + oversample;
+    if (rank < 1 || oversample < 0 || l > n || (h->nranks <= 1 && l > m_local)) return rank < 1 ? -6 : -7;
+    if (power_iters < 0) return -8;
+    if (!U) return -10;
+    if (ldu < m_local) return -11;
+    if (!S) return -12;
+    if (!V) return -13;
+    if (ldv < n) return -14;
+    cudaSetDevice(h->device);
+    begin_call(h);
+    cudaStream_t st = h->stream;
+    const bool host = ptr_side(A) == SIDE_HOST;
+    const float* dA = A;
+    int64_t dlda = lda;
+    float *dU = U, *dS = S, *dV = V;
+    int64_t dldu = ldu, dldv = ldv;
+    if (host) {
+        if (!h->stageA.ensure((size_t)m_local * n * 4) || !h->stageQ.ensure((size_t)m_local * rank * 4) ||
+            !h->stageR.ensure(((size_t)n * rank + rank) * 4 + 256))
+            return RG_ALLOC;
+        RG_CUDA(cudaMemcpy2DAsync(h->stageA.p, m_local * 4, A, lda * 4, m_local * 4, n, cudaMemcpyHostToDevice, st));
+        dA = h->stageA.as<float>();
+        dlda = m_local;
+        dU = h->stageQ.as<float>();
+        dldu = m_local;
+        dV = h->stageR.as<float>();
+        dldv = n;
+        dS = dV + (size_t)n * rank;
+    }
+    const int bf = o.precision;
+    const int64_t ldm16 = round_up(std::max<int64_t>(m_local, 8), 8);
+    const int64_t ldn16 = round_up(std::max<int64_t>(n, 8), 8);
+    const int64_t ldl16 = round_up(std::max(l, 8), 8);
+    bool ok = h->lrA16.ensure((size_t)ldm16 * n * 2) && h->lrB16.ensure((size_t)ldn16 * l * 2) &&
+              h->lrB16l.ensure((size_t)ldl16 * rank * 2 + 64) && h->lrY.ensure((size_t)m_local * l * 4) &&
+              h->lrZ.ensure((size_t)n * l * 4) && h->lrQ16.ensure((size_t)std::max(ldm16, ldn16) * l * 2) &&
+              h->lrQ16l.ensure((size_t)std::max(ldm16, ldn16) * l * 2) && h->lrR.ensure((size_t)l * l * 4) &&
+              h->lrW.ensure((size_t)l * l * 8) && h->lrV.ensure((size_t)l * l * 8) &&
+              h->lrUb.ensure((size_t)l * l * 4) && h->lrVb.ensure((size_t)l * l * 4) && h->lrSig.ensure(l * 8 + 64) &&
+              h->lrOm.ensure((size_t)n * l * 8) && h->lrScale.ensure(n * 4 + 64) && h->lrFlags.ensure(64) &&
+              h->partial.ensure(rg::colnorm_partial_doubles(m_local, (int)n) * 8 + 64) && h->norm2.ensure(n * 8 + 64) &&
+              h->status.ensure(64);
+    if (!ok) return RG_ALLOC;
+    uint16_t* A16 = h->lrA16.as<uint16_t>();
+    float* sc = h->lrScale.as<float>();
+    float* Y = h->lrY.as<float>();
+    float* Z = h->lrZ.as<float>();
+    float* Rl = h->lrR.as<float>();
+    int rc = reset_status(h);
+    if (rc) return rc;
+    // ---- power-of-two column scaling of A into fp16 range (section 3.5): A16 = fp16(A P)
+    RG_CUDA(rg::launch_colnorm(dA, dlda, m_local, (int)n, h->partial.as<double>(), h->norm2.as<double>(), st));
+    if (h->nranks > 1 && h->comm) {
+        rc = nccl_allreduce(h, h->norm2.p, n, ncclFloat64);
+        if (rc) return rc;
+    }
+    RG_CUDA(rg::launch_colscale(h->norm2.as<double>(), (int)n, 1, sc, h->status.as<int>(), 0, st));
+    RG_CUDA(rg::launch_scale_cast(dA, dlda, nullptr, 0, A16, nullptr, ldm16, m_local, (int)n, sc, bf, st));
+    // ---- sketch: Omega (n x l) ~ N(0,1) (Philox); B16 = fp16(P^{-1} Omega)
+    RG_CUDA(rg::launch_gaussian_philox((int64_t)n * l, seed, h->lrOm.as<double>(), nullptr, st));
+    RG_CUDA(rg::launch_cast_rows64(h->lrOm.as<double>(), n, n, l, sc, h->lrB16.as<uint16_t>(), nullptr, ldn16, bf, st));
+    // Y = A Omega = (A P)(P^{-1} Omega)
+    rc = gemm_nn(h, m_local, l, (int)n, A16, nullptr, ldm16, h->lrB16.as<uint16_t>(), nullptr, ldn16, Y, m_local, bf);
+    if (rc) return rc;
+    rg_opts qo = o;
+    qo.sync = 0;
+    auto project = [&](float* out) -> int {
+        // out (n x l) = A^T Q with Q's fp16 image in the RGSQR workspace (ldh): (A P)^T Q / P
+        int r2 = gemm_tn(h, m_local, (int)n, l, A16, ldm16, h->qh.as<uint16_t>(), round_up(std::max<int64_t>(m_local, 8), 8),
+                         out, n, bf);
+        if (r2) return r2;
+        if (h->nranks > 1 && h->comm) {
+            r2 = nccl_allreduce(h, out, (size_t)n * l, ncclFloat32);
+            if (r2) return r2;
+        }
+        RG_CUDA(rg::launch_unscale_rows(out, n, n, l, sc, st));
+        return RG_OK;
+    };
+    for (int it = 0; it < power_iters; ++it) {
+        rc = run_rgsqr(h, m_local, l, Y, m_local, Y, m_local, Rl, l, qo, 0);          // Q = qr(Y)
+        if (rc) return rc;
+        rc = project(Z);                                                            // Z = A^T Q
+        if (rc) return rc;
+        rc = run_rgsqr(h, n, l, Z, n, Z, n, Rl, l, qo, 0, true);                     // Q_z = qr(Z)
+        if (rc) return rc;
+        RG_CUDA(rg::launch_cast_rows(Z, n, n, l, sc, h->lrB16.as<uint16_t>(), nullptr, ldn16, bf, st));
+        rc = gemm_nn(h, m_local, l, (int)n, A16, nullptr, ldm16, h->lrB16.as<uint16_t>(), nullptr, ldn16, Y, m_local,
+                     bf);                                                           // Y = A Q_z
+        if (rc) return rc;
+    }
+    rc = run_rgsqr(h, m_local, l, Y, m_local, Y, m_local, Rl, l, qo, 0);              // Q = qr(Y)
+    if (rc) return rc;
+    rc = project(Z);                                                                // B^T = A^T Q
+    if (rc) return rc;
+    rc = run_rgsqr(h, n, l, Z, n, Z, n, Rl, l, qo, 0, true);                         // B^T = Q_b R_b
+    if (rc) return rc;
+    // ---- R_b = U_b S V_b^T (one-sided Jacobi, fp64)
+    RG_CUDA(rg::launch_jacobi_svd(Rl, l, l, rank, h->lrW.as<double>(), h->lrV.as<double>(), h->lrSig.as<double>(),
+                                  h->lrFlags.as<int>(), dS, h->lrUb.as<float>(), h->lrVb.as<float>(), st));
+    // ---- U = Q V_b(:, 1:r), V = Q_b U_b(:, 1:r)  (split-precision tensor-core products)
+    uint16_t* q16 = h->lrQ16.as<uint16_t>();
+    uint16_t* q16l = h->lrQ16l.as<uint16_t>();
+    uint16_t* b16 = h->lrB16.as<uint16_t>();
+    uint16_t* b16l = h->lrB16l.as<uint16_t>();
+    RG_CUDA(rg::launch_cast_rows(Y, m_local, m_local, l, nullptr, q16, q16l, ldm16, bf, st));
+    RG_CUDA(rg::launch_cast_rows(h->lrVb.as<float>(), l, l, rank, nullptr, b16, b16l, ldl16, bf, st));
+    rc = gemm_nn(h, m_local, rank, l, q16, q16l, ldm16, b16, b16l, ldl16, dU, dldu, bf);
+    if (rc) return rc;
+    RG_CUDA(rg::launch_cast_rows(Z, n, n, l, nullptr, q16, q16l, ldn16, bf, st));
+    RG_CUDA(rg::launch_cast_rows(h->lrUb.as<float>(), l, l, rank, nullptr, b16, b16l, ldl16, bf, st));
+    rc = gemm_nn(h, n, rank, l, q16, q16l, ldn16, b16, b16l, ldl16, dV, dldv, bf);
+    if (rc) return rc;
+    if (host) {
+        RG_CUDA(cudaMemcpy2DAsync(U, ldu * 4, dU, dldu * 4, m_local * 4, rank, cudaMemcpyDeviceToHost, st));
+        RG_CUDA(cudaMemcpy2DAsync(V, ldv * 4, dV, dldv * 4, n * 4, rank, cudaMemcpyDeviceToHost, st));
+        RG_CUDA(cudaMemcpyAsync(S, dS, rank * 4, cudaMemcpyDeviceToHost, st));
+    }
+    if (o.sync || host) rc = check_status(h);
+    end_call(h);
+    prof_collect(h);
+    return rc;
 }
 
 }  // extern "C"

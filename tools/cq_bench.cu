@@ -7,6 +7,33 @@
 #include <cuda_runtime.h>
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/panel_cholqr.cu"
 namespace rg { thread_local long long g_launches = 0; }
+__global__ void chol_loop_kernel(const double* G, double* Rg, float* Rinvg, int reps, long long* cyc) {
+    __shared__ double Rs[32 * 33];
+    long long t0 = clock64();
+    bool ok = true;
+    for (int r = 0; r < reps; ++r) ok &= rg::chol_inv_warp(G, 32, Rg, Rinvg, Rs);
+    long long t1 = clock64();
+    if (threadIdx.x == 0) { cyc[0] = (t1 - t0) / reps; cyc[1] = ok; }
+}
+__global__ void dfma_latency_kernel(double* out, int n, long long* cyc) {
+    double x = out[threadIdx.x], y = 1.0000001;
+    long long t0 = clock64();
+    for (int i = 0; i < n; ++i) x = fma(x, y, 1e-9);
+    long long t1 = clock64();
+    out[threadIdx.x] = x;
+    if (threadIdx.x == 0) cyc[2] = (t1 - t0) / n;
+    double z = out[threadIdx.x];
+    t0 = clock64();
+    for (int i = 0; i < n; ++i) z = rsqrt(z + 1.0);
+    t1 = clock64();
+    out[threadIdx.x + 32] = z;
+    if (threadIdx.x == 0) cyc[3] = (t1 - t0) / n;
+    t0 = clock64();
+    for (int i = 0; i < n; ++i) z = __shfl_sync(0xffffffffu, z, (threadIdx.x + 1) & 31) + 1.0;
+    t1 = clock64();
+    out[threadIdx.x + 64] = z;
+    if (threadIdx.x == 0) cyc[4] = (t1 - t0) / n;
+}
 int main(int argc, char** argv) {
     const int64_t m = argc > 1 ? atoll(argv[1]) : 65536;
     const int nc = 32;
@@ -81,6 +108,20 @@ int main(int argc, char** argv) {
         cudaEventSynchronize(b);
         cudaEventElapsedTime(&ms, a, b);
         printf("  pass 0 without chol (distributed flag): %.2f us\n", ms * 1000 / iters);
+    }
+    {
+        // Cholesky of an SPD 32x32 (identity + small) in a loop: cycles per call
+        std::vector<double> G(1024, 0.0);
+        for (int i = 0; i < 32; ++i) for (int j = 0; j < 32; ++j) G[i + 32 * j] = (i == j ? 40.0 : 1.0 / (1 + i + j));
+        double *dG, *dR, *dout; float* dRi; long long* cyc;
+        cudaMalloc(&dG, 8192); cudaMalloc(&dR, 8192); cudaMalloc(&dRi, 4096); cudaMalloc(&cyc, 64); cudaMalloc(&dout, 8192);
+        cudaMemcpy(dG, G.data(), 8192, cudaMemcpyHostToDevice);
+        cudaMemset(dout, 0, 8192);
+        chol_loop_kernel<<<1, 32>>>(dG, dR, dRi, 20, cyc);
+        dfma_latency_kernel<<<1, 32>>>(dout, 1000, cyc);
+        long long hc[5]; cudaMemcpy(hc, cyc, 40, cudaMemcpyDeviceToHost);
+        printf("  chol_inv_warp: %lld cycles/call (ok=%lld); DFMA latency %lld cyc; rsqrt(f64) %lld cyc; shfl+DADD %lld cyc\n",
+               hc[0], hc[1], hc[2], hc[3], hc[4]);
     }
     int fl; cudaMemcpy(&fl, flags, 4, cudaMemcpyDeviceToHost);
     printf("fail flag %d, err %s\n", fl, cudaGetErrorString(cudaGetLastError()));
