@@ -153,6 +153,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
+    RG_PDL_ENTRY();   // prologue above overlaps the previous kernel's tail
 
     if (warp == 0) {
         if (elect_one()) {
@@ -379,6 +380,7 @@ __global__ void __launch_bounds__(32 * LANES) proj_reduce_kernel(const float* __
                                                                 float* __restrict__ Rf, int64_t ldf,
                                                                 uint16_t* __restrict__ Rh, uint16_t* __restrict__ Rl,
                                                                 int64_t ldh, int bf16) {
+    RG_PDL_ENTRY();
     // block (32, LANES): 32 consecutive outputs x LANES split lanes; lane ty sums splits
     // ty, ty+LANES, ... in order, then the lane sums are added in order (deterministic).
     __shared__ float part[LANES][33];
@@ -418,6 +420,7 @@ __global__ void __launch_bounds__(32 * LANES) proj_reduce_kernel(const float* __
 __global__ void proj_finish_kernel(const float* __restrict__ Rf, int64_t ldf, int h, int w, float* __restrict__ R,
                                    int64_t ldr, uint16_t* __restrict__ Rh, uint16_t* __restrict__ Rl, int64_t ldh,
                                    int bf16) {
+    RG_PDL_ENTRY();
     const int64_t total = (int64_t)h * w;
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
         const int i = (int)(e % h);
@@ -458,8 +461,7 @@ static cudaError_t launch_gemm(int units, const CUtensorMap& a, const CUtensorMa
     const int per_sm = (C::kTotal <= 113 * 1024 && C::kTmemCols <= 256) ? 2 : 1;
     int grid = num_sms() * per_sm;
     if (grid > units) grid = units;
-    ++g_launches;
-    kern<<<grid, C::kThreads, C::kTotal, st>>>(a, b, al, bl, args);
+    RG_LAUNCH((kern), grid, C::kThreads, C::kTotal, st, a, b, al, bl, args);
     return cudaGetLastError();
 }
 
@@ -523,13 +525,12 @@ cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, in
                                int64_t ldr, float* Rf, int64_t ldf, uint16_t* Rh, uint16_t* Rl, int64_t ldh, int bf16,
                                cudaStream_t st) {
     const int64_t total = (int64_t)h * w;
-    ++g_launches;
     if (splits > 32)
-        proj_reduce_kernel<32><<<(unsigned)((total + 31) / 32), dim3(32, 32), 0, st>>>(P, ldp, p_stride, splits, h, w,
+        RG_LAUNCH((proj_reduce_kernel<32>), (unsigned)((total + 31) / 32), dim3(32, 32), 0, st, P, ldp, p_stride, splits, h, w,
                                                                                        R, ldr, Rf, ldf, Rh, Rl, ldh,
                                                                                        bf16);
     else
-        proj_reduce_kernel<8><<<(unsigned)((total + 31) / 32), dim3(32, 8), 0, st>>>(P, ldp, p_stride, splits, h, w, R,
+        RG_LAUNCH((proj_reduce_kernel<8>), (unsigned)((total + 31) / 32), dim3(32, 8), 0, st, P, ldp, p_stride, splits, h, w, R,
                                                                                      ldr, Rf, ldf, Rh, Rl, ldh, bf16);
     return cudaGetLastError();
 }
@@ -540,8 +541,7 @@ cudaError_t launch_proj_finish(const float* Rf, int64_t ldf, int h, int w, float
     int blocks = (int)((total + 255) / 256);
     if (blocks > 148 * 8) blocks = 148 * 8;
     if (blocks < 1) blocks = 1;
-    ++g_launches;
-    proj_finish_kernel<<<blocks, 256, 0, st>>>(Rf, ldf, h, w, R, ldr, Rh, Rl, ldh, bf16);
+    RG_LAUNCH((proj_finish_kernel), blocks, 256, 0, st, Rf, ldf, h, w, R, ldr, Rh, Rl, ldh, bf16);
     return cudaGetLastError();
 }
 

@@ -6,7 +6,32 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 
+#include <utility>
+
 namespace rg {
+
+// Programmatic dependent launch (PDL): every library kernel is launched with the
+// programmatic-stream-serialisation attribute and starts with RG_PDL_ENTRY(), which lets the
+// next kernel's launch overlap this one's tail and then waits (griddepcontrol.wait) for the
+// previous grid to complete before touching memory.  Opt-in with RGSQR_PDL=1 (measured slower
+// than plain graph edges for this kernel mix; kept for experiments).
+#define RG_PDL_ENTRY()                                           \
+    do {                                                         \
+        asm volatile("griddepcontrol.wait;" ::: "memory");       \
+        asm volatile("griddepcontrol.launch_dependents;" :::);   \
+    } while (0)
+
+bool pdl_enabled();
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                            Args&&... args);
+
+#define RG_LAUNCH(kern, grid, block, smem, st, ...)                                          \
+    do {                                                                                     \
+        cudaError_t _le = ::rg::launch_k(kern, dim3(grid), dim3(block), (size_t)(smem), st, __VA_ARGS__); \
+        if (_le != cudaSuccess) return _le;                                                  \
+    } while (0)
 
 // kernel launches issued by this thread (bench.py "gpu_launches" claim)
 extern thread_local long long g_launches;
@@ -119,4 +144,22 @@ cudaError_t launch_orth_probe_finish(const double* Z, int n, const double* G, do
 cudaError_t launch_trmm_upper(const float* A, int64_t lda, const float* B, int64_t ldb, float* C, int64_t ldc, int n,
                               cudaStream_t st);
 
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                            Args&&... args) {
+    ++g_launches;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl_enabled() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
 }  // namespace rg
+

@@ -40,6 +40,7 @@ template <typename T>
 __global__ void cast_rows_kernel(const T* __restrict__ src, int64_t lds, int64_t rows, int cols,
                                  const float* __restrict__ rscale, uint16_t* __restrict__ hi, uint16_t* __restrict__ lo,
                                  int64_t ldd, int bf16) {
+    RG_PDL_ENTRY();
     const int64_t total = rows * cols;
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
         const int64_t i = e % rows;
@@ -55,6 +56,7 @@ __global__ void cast_rows_kernel(const T* __restrict__ src, int64_t lds, int64_t
 // X(i, :) /= rscale[i] in place (undo a power-of-two row scaling)
 __global__ void unscale_rows_kernel(float* __restrict__ X, int64_t ldx, int64_t rows, int cols,
                                     const float* __restrict__ rscale) {
+    RG_PDL_ENTRY();
     const int64_t total = rows * cols;
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
         const int64_t i = e % rows;
@@ -66,6 +68,7 @@ __global__ void unscale_rows_kernel(float* __restrict__ X, int64_t ldx, int64_t 
 // W (l x l fp64, ld l) = R (upper fp32, ldr), V = I
 __global__ void jacobi_init_kernel(const float* __restrict__ R, int64_t ldr, int l, double* __restrict__ W,
                                    double* __restrict__ V) {
+    RG_PDL_ENTRY();
     const int64_t total = (int64_t)l * l;
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
         const int i = (int)(e % l), j = (int)(e / l);
@@ -99,6 +102,7 @@ __device__ __forceinline__ void rr_pair(int L, int r, int k, int& p, int& q) {
 // flags[0]: rotations above tolerance in the current sweep (int); flags[1]: sweeps done
 __global__ void __launch_bounds__(256) jacobi_sweeps_kernel(double* __restrict__ W, double* __restrict__ V, int l,
                                                             int max_sweeps, double tol, int* flags) {
+    RG_PDL_ENTRY();
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
     const int gwarp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -158,6 +162,7 @@ __global__ void __launch_bounds__(256) jacobi_sweeps_kernel(double* __restrict__
 __global__ void jacobi_extract_kernel(const double* __restrict__ W, const double* __restrict__ V, int l, int r,
                                       float* __restrict__ S, float* __restrict__ Ub, float* __restrict__ Vb,
                                       double* __restrict__ sig) {
+    RG_PDL_ENTRY();
     // one CTA per column j
     const int j = blockIdx.x;
     __shared__ double red[32];
@@ -178,6 +183,7 @@ __global__ void jacobi_extract_kernel(const double* __restrict__ W, const double
 __global__ void jacobi_rank_kernel(const double* __restrict__ W, const double* __restrict__ V, int l, int r,
                                    const double* __restrict__ sig, float* __restrict__ S, float* __restrict__ Ub,
                                    float* __restrict__ Vb) {
+    RG_PDL_ENTRY();
     const int j = blockIdx.x;
     __shared__ int s_rank;
     if (threadIdx.x == 0) {
@@ -205,32 +211,28 @@ __global__ void jacobi_rank_kernel(const double* __restrict__ W, const double* _
 cudaError_t launch_cast_rows(const float* src, int64_t lds, int64_t rows, int cols, const float* rscale, uint16_t* hi,
                              uint16_t* lo, int64_t ldd, int bf16, cudaStream_t st) {
     const int64_t total = rows * cols;
-    ++g_launches;
-    cast_rows_kernel<float><<<(unsigned)std::min<int64_t>((total + 255) / 256, 148 * 16), 256, 0, st>>>(
+    RG_LAUNCH((cast_rows_kernel<float>), (unsigned)std::min<int64_t>((total + 255) / 256, 148 * 16), 256, 0, st, 
         src, lds, rows, cols, rscale, hi, lo, ldd, bf16);
     return cudaGetLastError();
 }
 cudaError_t launch_cast_rows64(const double* src, int64_t lds, int64_t rows, int cols, const float* rscale,
                                uint16_t* hi, uint16_t* lo, int64_t ldd, int bf16, cudaStream_t st) {
     const int64_t total = rows * cols;
-    ++g_launches;
-    cast_rows_kernel<double><<<(unsigned)std::min<int64_t>((total + 255) / 256, 148 * 16), 256, 0, st>>>(
+    RG_LAUNCH((cast_rows_kernel<double>), (unsigned)std::min<int64_t>((total + 255) / 256, 148 * 16), 256, 0, st, 
         src, lds, rows, cols, rscale, hi, lo, ldd, bf16);
     return cudaGetLastError();
 }
 
 cudaError_t launch_unscale_rows(float* X, int64_t ldx, int64_t rows, int cols, const float* rscale, cudaStream_t st) {
     const int64_t total = rows * cols;
-    ++g_launches;
-    unscale_rows_kernel<<<(unsigned)std::min<int64_t>((total + 255) / 256, 148 * 16), 256, 0, st>>>(X, ldx, rows, cols,
+    RG_LAUNCH((unscale_rows_kernel), (unsigned)std::min<int64_t>((total + 255) / 256, 148 * 16), 256, 0, st, X, ldx, rows, cols,
                                                                                                       rscale);
     return cudaGetLastError();
 }
 
 cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double* W, double* V, double* sig, int* flags,
                               float* S, float* Ub, float* Vb, cudaStream_t st) {
-    ++g_launches;
-    jacobi_init_kernel<<<(unsigned)std::min<int64_t>(((int64_t)l * l + 255) / 256, 148 * 8), 256, 0, st>>>(R, ldr, l,
+    RG_LAUNCH((jacobi_init_kernel), (unsigned)std::min<int64_t>(((int64_t)l * l + 255) / 256, 148 * 8), 256, 0, st, R, ldr, l,
                                                                                                              W, V);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
@@ -246,12 +248,10 @@ cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double*
     ++g_launches;
     e = cudaLaunchCooperativeKernel((const void*)jacobi_sweeps_kernel, grid, 256, args, 0, st);
     if (e != cudaSuccess) return e;
-    ++g_launches;
-    jacobi_extract_kernel<<<l, 256, 0, st>>>(W, V, l, r, S, Ub, Vb, sig);
+    RG_LAUNCH((jacobi_extract_kernel), l, 256, 0, st, W, V, l, r, S, Ub, Vb, sig);
     e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    ++g_launches;
-    jacobi_rank_kernel<<<l, 256, 0, st>>>(W, V, l, r, sig, S, Ub, Vb);
+    RG_LAUNCH((jacobi_rank_kernel), l, 256, 0, st, W, V, l, r, sig, S, Ub, Vb);
     return cudaGetLastError();
 }
 

@@ -127,6 +127,7 @@ __device__ __forceinline__ int64_t tile_row0(const PanelArgs& p, int t) {
 }
 
 __global__ void __launch_bounds__(256, 2) panel_tile_kernel(PanelArgs p) {
+    RG_PDL_ENTRY();
     if (p.guard && *p.guard == 0) return;
     __shared__ float qbuf[2 * PT];
     __shared__ float Rs[PNB][33];
@@ -247,6 +248,7 @@ __global__ void __launch_bounds__(256, 2) panel_tile_kernel(PanelArgs p) {
 // Step (4)+(5): Q_tile <- Q_tile * (Qf_1[t] * Qf_2[t/8] * ... * Gq), fp32 + 16-bit shadow.
 // Gq (32x32, ld 32) is the rank's block of the cross-GPU stack factor, or null.
 __global__ void __launch_bounds__(256) panel_apply_kernel(PanelArgs p, const float* __restrict__ Gq) {
+    RG_PDL_ENTRY();
     if (p.guard && *p.guard == 0) return;
     __shared__ float M[PNB][PNB + 1];
     __shared__ float Tm[PNB][PNB + 1];
@@ -316,6 +318,7 @@ __global__ void __launch_bounds__(256) panel_apply_kernel(PanelArgs p, const flo
 __global__ void __launch_bounds__(256) panel_stack_kernel(const float* __restrict__ Rall, int P, int nc, float* R,
                                                           int64_t ldr, float* Qblocks, int* status, int col0,
                                                           const int* guard) {
+    RG_PDL_ENTRY();
     if (guard && *guard == 0) return;
     __shared__ float qbuf[2 * PT];
     __shared__ float Rs[PNB][33];
@@ -416,14 +419,12 @@ cudaError_t launch_panel(const PanelLaunch& pl, cudaStream_t st) {
     p.col0 = pl.col0;
     p.status = pl.status;
     p.guard = pl.guard;
-    ++g_launches;
-    panel_tile_kernel<<<p.ntiles, 256, 0, st>>>(p);
+    RG_LAUNCH((panel_tile_kernel), p.ntiles, 256, 0, st, p);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     if (pl.distributed) return cudaSuccess;  // caller gathers R, then calls launch_panel_apply
     if (p.levels > 0) {
-        ++g_launches;
-        panel_apply_kernel<<<p.ntiles, 256, 0, st>>>(p, nullptr);
+        RG_LAUNCH((panel_apply_kernel), p.ntiles, 256, 0, st, p, nullptr);
         e = cudaGetLastError();
     }
     return e;
@@ -453,15 +454,13 @@ cudaError_t launch_panel_apply(const PanelLaunch& pl, const float* Gq, cudaStrea
     }
     p.bf16 = pl.bf16;
     p.guard = pl.guard;
-    ++g_launches;
-    panel_apply_kernel<<<p.ntiles, 256, 0, st>>>(p, Gq);
+    RG_LAUNCH((panel_apply_kernel), p.ntiles, 256, 0, st, p, Gq);
     return cudaGetLastError();
 }
 
 cudaError_t launch_panel_stack(const float* Rall, int P, int nc, float* R, int64_t ldr, float* Qblocks, int* status,
                                int col0, const int* guard, cudaStream_t st) {
-    ++g_launches;
-    panel_stack_kernel<<<1, 256, 0, st>>>(Rall, P, nc, R, ldr, Qblocks, status, col0, guard);
+    RG_LAUNCH((panel_stack_kernel), 1, 256, 0, st, Rall, P, nc, R, ldr, Qblocks, status, col0, guard);
     return cudaGetLastError();
 }
 

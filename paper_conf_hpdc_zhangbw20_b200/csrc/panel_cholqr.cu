@@ -22,7 +22,14 @@
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
 
+#include <algorithm>
+#include <cstdlib>
+
+#include <cooperative_groups.h>
+
 #include "kernels.h"
+
+namespace cg = cooperative_groups;
 
 namespace rg {
 
@@ -105,6 +112,7 @@ __device__ __forceinline__ void gram_block_accum(const float* tile, int rows, in
 // One warp.  G (32x32 fp64, upper triangle valid, nc x nc used, identity-padded).
 // Writes R (fp64 upper, R[i + 32 j]) and Rinv (fp32, Rinv[i + 32 j]); returns false if a
 // pivot is not safely positive (relative to the original diagonal).
+template <bool kSharedG = false>
 __device__ bool chol_inv_warp(const double* G, int nc, double* Rg, float* Rinvg, double* Rs /*smem 32x33*/) {
     __shared__ double dinv[32];
     const int lane = threadIdx.x & 31;
@@ -112,7 +120,7 @@ __device__ bool chol_inv_warp(const double* G, int nc, double* Rg, float* Rinvg,
 #pragma unroll
     for (int j = 0; j < 32; ++j) {
         const int a = min(lane, j), b = max(lane, j);
-        g[j] = (lane < nc && j < nc) ? __ldcg(G + a + 32 * b) : (lane == j ? 1.0 : 0.0);
+        g[j] = (lane < nc && j < nc) ? (kSharedG ? G[a + 32 * b] : __ldcg(G + a + 32 * b)) : (lane == j ? 1.0 : 0.0);
     }
     double orig = 0.0;
 #pragma unroll
@@ -306,6 +314,7 @@ __device__ __forceinline__ void tile_times_rinv(float* tile, const float* Rinv /
 
 template <int PASS>
 __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
+    RG_PDL_ENTRY();
     __shared__ __align__(16) float tile[CQ_NB * CQ_LD + 64];   // also R1 scratch (32 x 33 doubles)
     __shared__ __align__(16) float Ri[2][32 * 32];
     __shared__ double sred[2][1024];   // CTA partial-sum scratch (2 row groups at a time); reused
@@ -413,8 +422,271 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
     reduce_and_factor(a, PASS, &sred[0][0], reinterpret_cast<double*>(tile));
 }
 
+
+// ---------------------------------------------------------------- fused single-kernel panel
+// Whole CholQR2 panel in one cooperative kernel (m <= CF_MAX_ROWS * gridDim): every CTA keeps
+// its rows of the panel in shared memory for the whole computation, so the panel is read once
+// and written once; the three launches, two "last block" chains and the broadcast of R^{-1}
+// of the streaming version become grid barriers, and every CTA factors the reduced 32 x 32
+// Gram itself (identical arithmetic on identical data -> identical R on every CTA).
+constexpr int CF_THREADS = 256;                  // 255 registers/thread: the Cholesky warp keeps 64 fp64 values
+constexpr int CF_GROUPS = CF_THREADS / CQ_BLK;   // 7 row groups of 36 threads
+constexpr int CF_FAN = 8;                        // CTA partials per first-level group
+constexpr int CF_MAX_ROWS = 1408;                // rows per CTA that fit next to the scratch
+
+struct CfSmem {
+    static size_t bytes(int ld) {
+        return (size_t)32 * ld * 4        // tile (column-major, ld)
+               + 2 * 1024 * 8             // sred
+               + 32 * 33 * 8 * 2          // G (padded) + Cholesky scratch
+               + 2 * 32 * 32 * 4          // R1^{-1}, R2^{-1} (fp32, [k][j])
+               + 1024 * 8                 // R1 (fp64) kept for R = R2 R1
+               + 256;
+    }
+};
+
+// Gram partial of the CTA's tile rows [0, rows) -> out (fp64 upper triangle), fixed order.
+__device__ void cf_gram(const float* tile, int ld, int rows, double* sred, double* out_partial) {
+    const int tid = threadIdx.x;
+    const int g = tid / CQ_BLK, blk = tid % CQ_BLK;
+    int bi = 0, bj = 0;
+    blk_coords(blk, bi, bj);
+    double acc[4][4] = {};
+    if (g < CF_GROUPS) {
+        for (int r = g; r < rows; r += CF_GROUPS) {
+            double x[4], y[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                x[u] = (double)tile[(bi * 4 + u) * ld + r];
+                y[u] = (double)tile[(bj * 4 + u) * ld + r];
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+#pragma unroll
+                for (int v = 0; v < 4; ++v) acc[u][v] = fma(x[u], y[v], acc[u][v]);
+        }
+    }
+    for (int round = 0; round < (CF_GROUPS + 1) / 2; ++round) {
+        const int g0 = round * 2;
+        __syncthreads();
+        for (int e = tid; e < 2 * 1024; e += CF_THREADS) sred[e] = 0.0;
+        __syncthreads();
+        if (g >= g0 && g < g0 + 2 && g < CF_GROUPS) {
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+#pragma unroll
+                for (int v = 0; v < 4; ++v) sred[(g - g0) * 1024 + (bi * 4 + u) + (bj * 4 + v) * 32] = acc[u][v];
+        }
+        __syncthreads();
+        for (int e = tid; e < 1024; e += CF_THREADS) {
+            const int i = e & 31, j = e >> 5;
+            double s = (round == 0) ? 0.0 : out_partial[e];
+            s += sred[e] + sred[1024 + e];
+            out_partial[e] = (i <= j) ? s : 0.0;
+        }
+    }
+    __syncthreads();
+}
+
+// Grid-wide fixed-order reduction of the CTA partials into Gs (smem, fp64, upper) on every CTA.
+__device__ void cf_allreduce_gram(const CqArgs& a, cg::grid_group& grid, double* Gs) {
+    const int ngroups = (gridDim.x + CF_FAN - 1) / CF_FAN;
+    grid.sync();
+    if ((int)blockIdx.x < ngroups) {
+        const int c0 = blockIdx.x * CF_FAN;
+        const int cn = min(CF_FAN, (int)gridDim.x - c0);
+        for (int e = threadIdx.x; e < 1024; e += CF_THREADS) {
+            double v[CF_FAN];
+#pragma unroll
+            for (int c = 0; c < CF_FAN; ++c) v[c] = (c < cn) ? __ldcg(a.ws.part + (int64_t)(c0 + c) * 1024 + e) : 0.0;
+            double sum = 0.0;
+#pragma unroll
+            for (int c = 0; c < CF_FAN; ++c) sum += v[c];
+            a.ws.gpart[(int64_t)blockIdx.x * 1024 + e] = sum;
+        }
+    }
+    grid.sync();
+    for (int e = threadIdx.x; e < 1024; e += CF_THREADS) {
+        double sum = 0.0;
+        for (int g0 = 0; g0 < ngroups; g0 += CF_FAN) {
+            double v[CF_FAN];
+#pragma unroll
+            for (int c = 0; c < CF_FAN; ++c) v[c] = (g0 + c < ngroups) ? __ldcg(a.ws.gpart + (int64_t)(g0 + c) * 1024 + e) : 0.0;
+#pragma unroll
+            for (int c = 0; c < CF_FAN; ++c) sum += v[c];
+        }
+        Gs[e] = sum;
+    }
+    __syncthreads();
+}
+
+// tile (rows x 32, ld) <- tile * Rinv (32 x 32 fp32, [k * 32 + j]), chunks of 4 * CF_THREADS / 8 rows
+__device__ void cf_times_rinv(float* tile, int ld, int rows, const float* Rinv) {
+    constexpr int RG = CF_THREADS / 8;          // row groups x 8 column groups of 4
+    const int tid = threadIdx.x;
+    const int cgp = tid & 7, rgp = tid >> 3;
+    for (int base = 0; base < rows; base += 4 * RG) {
+        float o[4][4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) o[i][c] = 0.f;
+#pragma unroll 8
+        for (int k = 0; k < CQ_NB; ++k) {
+            const float4 rv = *reinterpret_cast<const float4*>(Rinv + k * 32 + 4 * cgp);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int r = base + rgp + RG * i;
+                const float x = (r < rows) ? tile[k * ld + r] : 0.f;
+                o[i][0] = fmaf(x, rv.x, o[i][0]);
+                o[i][1] = fmaf(x, rv.y, o[i][1]);
+                o[i][2] = fmaf(x, rv.z, o[i][2]);
+                o[i][3] = fmaf(x, rv.w, o[i][3]);
+            }
+        }
+        __syncthreads();
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const int r = base + rgp + RG * i;
+            if (r < rows)
+#pragma unroll
+                for (int c = 0; c < 4; ++c) tile[(4 * cgp + c) * ld + r] = o[i][c];
+        }
+        __syncthreads();
+    }
+}
+
+#ifdef RG_CF_TRACE
+__device__ unsigned long long cf_trace[16];
+#define CF_MARK(i)                                                                     \
+    do {                                                                               \
+        if (blockIdx.x == 0 && threadIdx.x == 0) {                                     \
+            unsigned long long t;                                                      \
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));                      \
+            cf_trace[i] = t;                                                           \
+        }                                                                              \
+    } while (0)
+#else
+#define CF_MARK(i) \
+    do {           \
+    } while (0)
+#endif
+
+__global__ void __launch_bounds__(CF_THREADS, 1) cq_fused_kernel(CqArgs a, int ld) {
+    RG_PDL_ENTRY();
+    cg::grid_group grid = cg::this_grid();
+    extern __shared__ __align__(16) uint8_t cf_smem[];
+    float* tile = reinterpret_cast<float*>(cf_smem);
+    double* sred = reinterpret_cast<double*>(cf_smem + (size_t)32 * ld * 4);
+    double* Gs = sred + 2 * 1024;             // 32 x 33 (first 1024 used as G)
+    double* Rs = Gs + 32 * 33;                // Cholesky scratch 32 x 33
+    float* Ri1 = reinterpret_cast<float*>(Rs + 32 * 33);
+    float* Ri2 = Ri1 + 1024;
+    double* R1 = reinterpret_cast<double*>(Ri2 + 1024);
+    __shared__ int s_flag[2];
+    const int tid = threadIdx.x;
+    CF_MARK(0);
+    if (blockIdx.x == 0 && tid == 0) *a.ws.fail = 0;   // set again below only if a pivot fails
+    const int64_t rows_per = (a.m + gridDim.x - 1) / gridDim.x;
+    const int64_t r0 = (int64_t)blockIdx.x * rows_per;
+    const int64_t rem = a.m - r0;
+    const int rows = (int)(rem <= 0 ? 0 : (rem < rows_per ? rem : rows_per));
+    // ---- load the CTA's rows (zero-padded columns beyond nc)
+    for (int e = tid; e < 32 * rows; e += CF_THREADS) {
+        const int r = e % rows, c = e / rows;
+        tile[c * ld + r] = (c < a.nc) ? a.P[r0 + r + (int64_t)c * a.ldp] : 0.f;
+    }
+    __syncthreads();
+    CF_MARK(1);
+    // ---- pass 1: G1 = P^T P -> R1, R1^{-1} on every CTA
+    cf_gram(tile, ld, rows, sred, a.ws.part + (int64_t)blockIdx.x * 1024);
+    CF_MARK(2);
+    cf_allreduce_gram(a, grid, Gs);
+    CF_MARK(3);
+    if (tid < 32) {
+        const bool ok = chol_inv_warp<true>(Gs, a.nc, R1, Ri1, Rs);
+        if (tid == 0) s_flag[0] = ok;
+    }
+    __syncthreads();
+    CF_MARK(4);
+    if (!s_flag[0]) {
+        if (blockIdx.x == 0 && tid == 0) *a.ws.fail = 1;   // the guarded MGS/TSQR kernels take over
+        return;
+    }
+    // kappa_F(R1) <= 2 nc  ->  single CholQR pass (see cq_pass_kernel)
+    if (tid < 32) {
+        double r = 0.0, ri = 0.0;
+        for (int e = tid; e < 1024; e += 32) {
+            const int i = e & 31, j = e >> 5;
+            if (i < a.nc && j < a.nc) {
+                r = fma(R1[e], R1[e], r);
+                const double y = (double)Ri1[e];
+                ri = fma(y, y, ri);
+            }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            r += __shfl_xor_sync(0xffffffffu, r, o);
+            ri += __shfl_xor_sync(0xffffffffu, ri, o);
+        }
+        if (tid == 0) s_flag[1] = (sqrt(r * ri) <= 2.0 * a.nc) ? 1 : 0;
+    }
+    __syncthreads();
+    const bool single = s_flag[1] != 0;
+    // Ri1 is [i + 32 j] (column-major R^{-1}); the product wants [k * 32 + j] = R^{-1}(k, j): transpose
+    for (int e = tid; e < 1024; e += CF_THREADS) Ri2[e] = Ri1[(e >> 5) + 32 * (e & 31)];
+    __syncthreads();
+    cf_times_rinv(tile, ld, rows, Ri2);   // tile <- Q1 = P R1^{-1}
+    CF_MARK(5);
+    if (!single) {
+        // ---- pass 2: G2 = Q1^T Q1 -> R2, R2^{-1}; Q = Q1 R2^{-1}; R = R2 R1
+        cf_gram(tile, ld, rows, sred, a.ws.part + (int64_t)blockIdx.x * 1024);
+        cf_allreduce_gram(a, grid, Gs);
+        if (tid < 32) {   // R2 (fp64, [i + 32 j]) goes to sred, free after the reduction
+            const bool ok = chol_inv_warp<true>(Gs, a.nc, sred, Ri1, Rs);
+            if (tid == 0) s_flag[0] = ok;
+        }
+        __syncthreads();
+        if (!s_flag[0]) {
+            if (blockIdx.x == 0 && tid == 0) *a.ws.fail = 1;
+            return;   // input panel untouched in HBM: the MGS/TSQR fallback redoes it
+        }
+        for (int e = tid; e < 1024; e += CF_THREADS) Ri2[e] = Ri1[(e >> 5) + 32 * (e & 31)];
+        __syncthreads();
+        cf_times_rinv(tile, ld, rows, Ri2);   // tile <- Q
+        if (blockIdx.x == 0) {
+            const double* R2 = reinterpret_cast<const double*>(sred);
+            for (int e = tid; e < a.nc * a.nc; e += CF_THREADS) {
+                const int i = e % a.nc, j = e / a.nc;
+                double s = 0.0;
+                for (int k = i; k <= j; ++k) s = fma(R2[i + 32 * k], R1[k + 32 * j], s);
+                a.Rout[i + (int64_t)j * a.ldr] = (i <= j) ? (float)s : 0.f;
+            }
+        }
+    } else if (blockIdx.x == 0) {
+        for (int e = tid; e < a.nc * a.nc; e += CF_THREADS) {
+            const int i = e % a.nc, j = e / a.nc;
+            a.Rout[i + (int64_t)j * a.ldr] = (i <= j) ? (float)R1[i + 32 * j] : 0.f;
+        }
+    }
+    CF_MARK(6);
+    // ---- write Q (fp32) + 16-bit shadow
+    for (int e = tid; e < a.nc * rows; e += CF_THREADS) {
+        const int r = e % rows, c = e / rows;
+        const float v = tile[c * ld + r];
+        const int64_t gr = r0 + r;
+        a.Q[gr + (int64_t)c * a.ldq] = v;
+        if (a.Qh) {
+            const uint16_t hb = cq_to16(v, a.bf16);
+            a.Qh[gr + (int64_t)c * a.ldh] = hb;
+            if (a.Ql) a.Ql[gr + (int64_t)c * a.ldh] = cq_to16((v - cq_from16(hb, a.bf16)) * 2048.f, a.bf16);
+        }
+    }
+}
+
 // distributed mode: after the host allreduce of G (pass `pass`), factor it (one warp)
 __global__ void cq_factor_kernel(CqArgs a, int pass) {
+    RG_PDL_ENTRY();
     __shared__ double Rs[32 * 33];
     __shared__ double R1s[32 * 33];
     __shared__ int s_ok;
@@ -440,8 +712,8 @@ static int cq_grid(int64_t m) {
 }
 
 size_t cholqr_ws_doubles(int64_t m) {
-    const int grid = cq_grid(m);
-    const int ngroups = (grid + CQ_FAN - 1) / CQ_FAN;
+    const int grid = std::max(cq_grid(m), 160);   // also covers the fused kernel (<= 160 CTAs)
+    const int ngroups = (grid + CQ_FAN - 1) / CQ_FAN + (grid + CF_FAN - 1) / CF_FAN;
     return (size_t)(grid + ngroups) * 1024 + 4 * 1024 + 1024 /*Rinv fp32 x2*/ + 64;
 }
 
@@ -475,17 +747,46 @@ cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st) {
     a.bf16 = L.bf16;
     a.distributed = L.allreduce_g != nullptr;
     cudaError_t e;
-    for (int pass = 0; pass < 3; ++pass) {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    }
+    const int64_t rows_per = (L.m + sms - 1) / sms;
+    if (!a.distributed && rows_per <= CF_MAX_ROWS && getenv("RGSQR_CQ_STREAM") == nullptr) {
+        const int ld = (int)(rows_per | 1);   // odd leading dimension: conflict-free column walks
+        const size_t smem = CfSmem::bytes(ld);
+        static size_t attr = 0;
+        if (smem > attr) {
+            e = cudaFuncSetAttribute(cq_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            if (e != cudaSuccess) return e;
+            attr = smem;
+        }
+        // partial buffers: sms CTA partials + ceil(sms / 8) group partials fit in the workspace
+        a.ws.gpart = a.ws.part + (size_t)sms * 1024;
+        cudaLaunchConfig_t cfg{};
+        cfg.gridDim = dim3(sms);
+        cfg.blockDim = dim3(CF_THREADS);
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = st;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeCooperative;
+        at[0].val.cooperative = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
         ++g_launches;
-        if (pass == 0) cq_pass_kernel<0><<<grid, CQ_THREADS, 0, st>>>(a);
-        if (pass == 1) cq_pass_kernel<1><<<grid, CQ_THREADS, 0, st>>>(a);
-        if (pass == 2) cq_pass_kernel<2><<<grid, CQ_THREADS, 0, st>>>(a);
+        return cudaLaunchKernelEx(&cfg, cq_fused_kernel, a, ld);
+    }
+    for (int pass = 0; pass < 3; ++pass) {
+        if (pass == 0) RG_LAUNCH((cq_pass_kernel<0>), grid, CQ_THREADS, 0, st, a);
+        if (pass == 1) RG_LAUNCH((cq_pass_kernel<1>), grid, CQ_THREADS, 0, st, a);
+        if (pass == 2) RG_LAUNCH((cq_pass_kernel<2>), grid, CQ_THREADS, 0, st, a);
         e = cudaGetLastError();
         if (e != cudaSuccess) return e;
         if (a.distributed && pass < 2) {
             if (L.allreduce_g(a.ws.G + pass * 1024, L.ctx) != 0) return cudaErrorUnknown;
-            ++g_launches;
-            cq_factor_kernel<<<1, 256, 0, st>>>(a, pass);
+            RG_LAUNCH((cq_factor_kernel), 1, 256, 0, st, a, pass);
             e = cudaGetLastError();
             if (e != cudaSuccess) return e;
         }

@@ -723,6 +723,10 @@ int gemm_tn(rg_handle h, int64_t K, int M, int N, const uint16_t* Ah, int64_t ld
 
 namespace rg {
 thread_local long long g_launches = 0;
+bool pdl_enabled() {   // opt-in: measured slower than plain graph edges for this kernel mix
+    static const bool on = getenv("RGSQR_PDL") != nullptr;
+    return on;
+}
 }
 
 // ====================================================================== C-ABI

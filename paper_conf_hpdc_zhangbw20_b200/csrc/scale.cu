@@ -32,6 +32,7 @@ __device__ __forceinline__ float s_from16(uint16_t u, int bf16) {
 // partial[y * n + j] = sum_{i in chunk y} A(i, j)^2   (fp64 accumulation)
 __global__ void __launch_bounds__(256) colnorm_partial_kernel(const float* __restrict__ A, int64_t lda, int64_t m,
                                                               int n, double* __restrict__ partial) {
+    RG_PDL_ENTRY();
     const int j = blockIdx.x;
     const int64_t i0 = (int64_t)blockIdx.y * kNormChunk;
     const int64_t i1 = min(m, i0 + kNormChunk);
@@ -63,6 +64,7 @@ __global__ void __launch_bounds__(256) colnorm_partial_kernel(const float* __res
 
 // norm2[j] = sum_y partial (fixed order, deterministic).
 __global__ void colnorm_sum_kernel(const double* __restrict__ partial, int chunks, int n, double* __restrict__ norm2) {
+    RG_PDL_ENTRY();
     const int j = blockIdx.x * blockDim.x + threadIdx.x;
     if (j >= n) return;
     double s = 0.0;
@@ -74,6 +76,7 @@ __global__ void colnorm_sum_kernel(const double* __restrict__ partial, int chunk
 // is off; status[1] <- min column with a non-finite norm, status[0] <- min zero column.
 __global__ void colscale_kernel(const double* __restrict__ norm2, int n, int do_scale, float* __restrict__ scale,
                                 int* status, int col0) {
+    RG_PDL_ENTRY();
     const int j = blockIdx.x * blockDim.x + threadIdx.x;
     if (j >= n) return;
     const double s = norm2[j];
@@ -93,6 +96,7 @@ __global__ void __launch_bounds__(256) scale_cast_kernel(const float* __restrict
                                                          int64_t ldq, uint16_t* __restrict__ Qh,
                                                          uint16_t* __restrict__ Ql, int64_t ldh, int64_t m, int n,
                                                          const float* __restrict__ scale, int bf16) {
+    RG_PDL_ENTRY();
     const int j = blockIdx.y;
     const float s = scale ? scale[j] : 1.0f;
     const float* a = A + (int64_t)j * lda;
@@ -147,6 +151,7 @@ __global__ void __launch_bounds__(256) scale_cast_kernel(const float* __restrict
 
 // R(:, j) <- R(:, j) / scale[j] (exact: powers of two); strictly-lower part zeroed.
 __global__ void unscale_r_kernel(float* R, int64_t ldr, int n, const float* __restrict__ scale) {
+    RG_PDL_ENTRY();
     const int64_t total = (int64_t)n * n;
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
         const int i = (int)(e % n), j = (int)(e / n);
@@ -159,19 +164,16 @@ cudaError_t launch_colnorm(const float* A, int64_t lda, int64_t m, int n, double
                            cudaStream_t st) {
     const int chunks = (int)((m + kNormChunk - 1) / kNormChunk);
     dim3 grid(n, chunks);
-    ++g_launches;
-    colnorm_partial_kernel<<<grid, 256, 0, st>>>(A, lda, m, n, partial);
+    RG_LAUNCH((colnorm_partial_kernel), grid, 256, 0, st, A, lda, m, n, partial);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    ++g_launches;
-    colnorm_sum_kernel<<<(n + 127) / 128, 128, 0, st>>>(partial, chunks, n, norm2);
+    RG_LAUNCH((colnorm_sum_kernel), (n + 127) / 128, 128, 0, st, partial, chunks, n, norm2);
     return cudaGetLastError();
 }
 
 cudaError_t launch_colscale(const double* norm2, int n, int do_scale, float* scale, int* status, int col0,
                             cudaStream_t st) {
-    ++g_launches;
-    colscale_kernel<<<(n + 127) / 128, 128, 0, st>>>(norm2, n, do_scale, scale, status, col0);
+    RG_LAUNCH((colscale_kernel), (n + 127) / 128, 128, 0, st, norm2, n, do_scale, scale, status, col0);
     return cudaGetLastError();
 }
 
@@ -187,8 +189,7 @@ cudaError_t launch_scale_cast(const float* A, int64_t lda, float* Q, int64_t ldq
     int bx = (int)(per_col < target ? per_col : target);
     if (bx < 1) bx = 1;
     dim3 grid(bx, n);
-    ++g_launches;
-    scale_cast_kernel<<<grid, 256, 0, st>>>(A, lda, Q, ldq, Qh, Ql, ldh, m, n, scale, bf16);
+    RG_LAUNCH((scale_cast_kernel), grid, 256, 0, st, A, lda, Q, ldq, Qh, Ql, ldh, m, n, scale, bf16);
     return cudaGetLastError();
 }
 
@@ -196,8 +197,7 @@ cudaError_t launch_unscale_r(float* R, int64_t ldr, int n, const float* scale, c
     const int64_t total = (int64_t)n * n;
     int blocks = (int)((total + 255) / 256);
     if (blocks > 148 * 8) blocks = 148 * 8;
-    ++g_launches;
-    unscale_r_kernel<<<blocks, 256, 0, st>>>(R, ldr, n, scale);
+    RG_LAUNCH((unscale_r_kernel), blocks, 256, 0, st, R, ldr, n, scale);
     return cudaGetLastError();
 }
 

@@ -154,6 +154,17 @@ def test_rgsqr_breakdown_status(rg):
     assert e.value.status == rg.RG_NONFINITE and e.value.info == 5
 
 
+def test_rgsqr_after_breakdown_is_clean(rg):
+    """A failed panel (CholQR pivot) must not leak its fallback flag into later calls."""
+    A = synth.gaussian(512, 40, seed=11).astype(np.float32)
+    A[:, 3] = 0.0
+    with pytest.raises(rg.RGError):
+        _run(rg, A)
+    B = synth.svd_matrix(4096, 96, "geometric", 1e2, seed=12).astype(np.float32)
+    Q, R = _run(rg, B)
+    _check_qr(B, Q, R, kappa=1e2, orth_scale=1.0)
+
+
 def test_rgsqr_invalid_arguments(rg):
     import ctypes
     h = rg.default_handle()

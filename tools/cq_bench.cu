@@ -5,8 +5,10 @@
 #include <cstdlib>
 #include <vector>
 #include <cuda_runtime.h>
+#define RG_CF_TRACE 1
+#include "../paper_conf_hpdc_zhangbw20_b200/csrc/kernels.h"
+namespace rg { thread_local long long g_launches = 0; bool pdl_enabled() { return getenv("RGSQR_NO_PDL") == nullptr; } }
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/panel_cholqr.cu"
-namespace rg { thread_local long long g_launches = 0; }
 __global__ void chol_loop_kernel(const double* G, double* Rg, float* Rinvg, int reps, long long* cyc) {
     __shared__ double Rs[32 * 33];
     long long t0 = clock64();
@@ -122,6 +124,15 @@ int main(int argc, char** argv) {
         long long hc[5]; cudaMemcpy(hc, cyc, 40, cudaMemcpyDeviceToHost);
         printf("  chol_inv_warp: %lld cycles/call (ok=%lld); DFMA latency %lld cyc; rsqrt(f64) %lld cyc; shfl+DADD %lld cyc\n",
                hc[0], hc[1], hc[2], hc[3], hc[4]);
+    }
+    {
+        unsigned long long tr[16];
+        rg::launch_panel_cholqr(L, st);
+        cudaStreamSynchronize(st);
+        cudaMemcpyFromSymbol(tr, rg::cf_trace, sizeof(tr));
+        printf("  fused trace (us from start): load %.2f gram %.2f reduce %.2f chol %.2f apply %.2f pre-write %.2f\n",
+               (tr[1] - tr[0]) / 1e3, (tr[2] - tr[0]) / 1e3, (tr[3] - tr[0]) / 1e3, (tr[4] - tr[0]) / 1e3,
+               (tr[5] - tr[0]) / 1e3, (tr[6] - tr[0]) / 1e3);
     }
     int fl; cudaMemcpy(&fl, flags, 4, cudaMemcpyDeviceToHost);
     printf("fail flag %d, err %s\n", fl, cudaGetErrorString(cudaGetLastError()));
