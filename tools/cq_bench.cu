@@ -3,17 +3,31 @@
 //   paper_conf_hpdc_zhangbw20_b200/csrc/panel_cholqr.cu -o tools/cq_bench
 #include <cstdio>
 #include <cstdlib>
+#include <cmath>
+#include <algorithm>
 #include <vector>
 #include <cuda_runtime.h>
 #define RG_CF_TRACE 1
+// #define RG_CHOL_TRACE 1
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/kernels.h"
 namespace rg { thread_local long long g_launches = 0; bool pdl_enabled() { return getenv("RGSQR_NO_PDL") == nullptr; } }
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/panel_cholqr.cu"
-__global__ void chol_loop_kernel(const double* G, double* Rg, float* Rinvg, int reps, long long* cyc) {
-    __shared__ double Rs[32 * 33];
+template <int NT>
+__global__ void chol_nt_kernel(const double* G, double* Rg, float* Rinvg, int reps, long long* cyc) {
+    __shared__ __align__(16) double Rs[32 * 34], Ys[32 * 34], Gs[1024];
+    for (int e = threadIdx.x; e < 1024; e += NT) Gs[e] = G[e];
+    __syncthreads();
     long long t0 = clock64();
     bool ok = true;
-    for (int r = 0; r < reps; ++r) ok &= rg::chol_inv_warp(G, 32, Rg, Rinvg, Rs);
+    for (int r = 0; r < reps; ++r) ok &= rg::chol_inv_cta<NT, true>(Gs, 32, Rs, Ys, Rg, Rinvg, false);
+    long long t1 = clock64();
+    if (threadIdx.x == 0) { cyc[0] = (t1 - t0) / reps; cyc[1] = ok; }
+}
+__global__ void chol_loop_kernel(const double* G, double* Rg, float* Rinvg, int reps, long long* cyc) {
+    __shared__ __align__(16) double Rs[32 * 34], Ys[32 * 34];
+    long long t0 = clock64();
+    bool ok = true;
+    for (int r = 0; r < reps; ++r) ok &= rg::chol_inv_cta<256, false>(G, 32, Rs, Ys, Rg, Rinvg, false);
     long long t1 = clock64();
     if (threadIdx.x == 0) { cyc[0] = (t1 - t0) / reps; cyc[1] = ok; }
 }
@@ -45,8 +59,8 @@ int main(int argc, char** argv) {
     float *P, *Q, *R; uint16_t* Qh; double* ws; int* flags;
     cudaMalloc(&P, m * nc * 4); cudaMalloc(&Q, m * nc * 4); cudaMalloc(&R, 32 * 32 * 4);
     cudaMalloc(&Qh, m * nc * 2);
-    cudaMalloc(&ws, rg::cholqr_ws_doubles(m) * 8); cudaMalloc(&flags, 4096);
-    cudaMemset(flags, 0, 4096);
+    cudaMalloc(&ws, rg::cholqr_ws_doubles(m) * 8); cudaMalloc(&flags, 16384);
+    cudaMemset(flags, 0, 16384);
     cudaMemcpy(P, h.data(), m * nc * 4, cudaMemcpyHostToDevice);
     rg::CholqrLaunch L{};
     L.P = P; L.ldp = m; L.Q = Q; L.ldq = m; L.Qh = Qh; L.ldh = m; L.m = m; L.nc = nc; L.ws = ws;
@@ -119,10 +133,45 @@ int main(int argc, char** argv) {
         cudaMalloc(&dG, 8192); cudaMalloc(&dR, 8192); cudaMalloc(&dRi, 4096); cudaMalloc(&cyc, 64); cudaMalloc(&dout, 8192);
         cudaMemcpy(dG, G.data(), 8192, cudaMemcpyHostToDevice);
         cudaMemset(dout, 0, 8192);
-        chol_loop_kernel<<<1, 32>>>(dG, dR, dRi, 20, cyc);
+        chol_loop_kernel<<<1, 256>>>(dG, dR, dRi, 20, cyc);
         dfma_latency_kernel<<<1, 32>>>(dout, 1000, cyc);
         long long hc[5]; cudaMemcpy(hc, cyc, 40, cudaMemcpyDeviceToHost);
-        printf("  chol_inv_warp: %lld cycles/call (ok=%lld); DFMA latency %lld cyc; rsqrt(f64) %lld cyc; shfl+DADD %lld cyc\n",
+        {   // check R^T R = G and R Rinv = I
+            std::vector<double> R(1024); std::vector<float> Ri(1024);
+            cudaMemcpy(R.data(), dR, 8192, cudaMemcpyDeviceToHost); cudaMemcpy(Ri.data(), dRi, 4096, cudaMemcpyDeviceToHost);
+            double e1 = 0, e2 = 0;
+            for (int i = 0; i < 32; ++i) for (int j = 0; j < 32; ++j) {
+                double s = 0, t = 0;
+                for (int k = 0; k < 32; ++k) { s += R[k + 32 * i] * R[k + 32 * j]; t += R[i + 32 * k] * Ri[k + 32 * j]; }
+                e1 = fmax(e1, fabs(s - G[std::min(i, j) + 32 * std::max(i, j)]));
+                e2 = fmax(e2, fabs(t - (i == j)));
+            }
+            printf("  chol check: |R^T R - G| %.2e  |R Rinv - I| %.2e\n", e1, e2);
+        }
+#ifdef RG_CHOL_TRACE
+        {
+            long long tr[40]; cudaMemcpyFromSymbol(tr, rg::chol_trace, sizeof(tr));
+            printf("  chol step cycles:");
+            for (int k = 0; k < 8; ++k) printf(" [p1 %lld bar %lld p2 %lld bar %lld]", tr[10 + k] - tr[k], tr[20 + k] - tr[10 + k], tr[30 + k] - tr[20 + k], tr[k + 1] - tr[30 + k]);
+            printf("\n");
+        }
+#endif
+        {
+            long long h2[2];
+            chol_nt_kernel<32><<<1, 32>>>(dG, dR, dRi, 20, cyc); cudaMemcpy(h2, cyc, 16, cudaMemcpyDeviceToHost);
+            printf("  NT=32: %lld cyc;", h2[0]);
+            chol_nt_kernel<64><<<1, 64>>>(dG, dR, dRi, 20, cyc); cudaMemcpy(h2, cyc, 16, cudaMemcpyDeviceToHost);
+            printf(" NT=64: %lld cyc;", h2[0]);
+            chol_nt_kernel<128><<<1, 128>>>(dG, dR, dRi, 20, cyc); cudaMemcpy(h2, cyc, 16, cudaMemcpyDeviceToHost);
+            printf(" NT=128: %lld cyc;", h2[0]);
+            chol_nt_kernel<256><<<1, 256>>>(dG, dR, dRi, getenv("CHOL_REPS") ? atoi(getenv("CHOL_REPS")) : 20, cyc); cudaMemcpy(h2, cyc, 16, cudaMemcpyDeviceToHost);
+            printf(" NT=256: %lld cyc;", h2[0]);
+            chol_nt_kernel<512><<<1, 512>>>(dG, dR, dRi, 20, cyc); cudaMemcpy(h2, cyc, 16, cudaMemcpyDeviceToHost);
+            printf(" NT=512: %lld cyc;", h2[0]);
+            chol_nt_kernel<1024><<<1, 1024>>>(dG, dR, dRi, 20, cyc); cudaMemcpy(h2, cyc, 16, cudaMemcpyDeviceToHost);
+            printf(" NT=1024: %lld cyc\n", h2[0]);
+        }
+        printf("  chol_inv_cta: %lld cycles/call (ok=%lld); DFMA latency %lld cyc; rsqrt(f64) %lld cyc; shfl+DADD %lld cyc\n",
                hc[0], hc[1], hc[2], hc[3], hc[4]);
     }
     {
@@ -133,6 +182,16 @@ int main(int argc, char** argv) {
         printf("  fused trace (us from start): load %.2f gram %.2f reduce %.2f chol %.2f apply %.2f pre-write %.2f\n",
                (tr[1] - tr[0]) / 1e3, (tr[2] - tr[0]) / 1e3, (tr[3] - tr[0]) / 1e3, (tr[4] - tr[0]) / 1e3,
                (tr[5] - tr[0]) / 1e3, (tr[6] - tr[0]) / 1e3);
+        {
+            static unsigned long long ct[4][160];
+            cudaMemcpyFromSymbol(ct, rg::cf_cta, sizeof(ct));
+            for (int k = 0; k < 4; ++k) {
+                unsigned long long mn = ~0ull, mx = 0;
+                for (int b = 0; b < 148; ++b) { if (!ct[k][b]) continue; mn = std::min(mn, ct[k][b]); mx = std::max(mx, ct[k][b]); }
+                printf("  cta mark %d: min %.2f max %.2f us (rel. to CTA0 start)\n", k, ((double)mn - tr[0]) / 1e3, ((double)mx - tr[0]) / 1e3);
+            }
+        }
+        printf("  marks: 0=spin exit 1=group-sum done (last arrivers only) 2=gram done 3=arrived; flag set at %.2f\n", (tr[8] - tr[0]) / 1e3);
     }
     int fl; cudaMemcpy(&fl, flags, 4, cudaMemcpyDeviceToHost);
     printf("fail flag %d, err %s\n", fl, cudaGetErrorString(cudaGetLastError()));
