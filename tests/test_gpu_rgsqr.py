@@ -68,6 +68,36 @@ def test_rgsqr_ill_conditioned_backward_error(rg, kappa):
     assert np.all(np.diag(R) > 0)
 
 
+@pytest.mark.parametrize("kappa", [10.0, 1e5])
+@pytest.mark.parametrize("n", [32, 96])
+def test_rgsqr_streaming_cholqr_panel(rg, monkeypatch, kappa, n):
+    """The three-launch streaming CholQR2 panel (used when a panel's rows do not fit in the
+    fused kernel's shared memory) forced on a small case; kappa = 1e5 makes the panels take
+    the second CholQR pass, whose R = R2 R1 product reads R2 back from the elimination scratch."""
+    monkeypatch.setenv("RGSQR_CQ_STREAM", "1")
+    h = rg.Handle(0)
+    A = synth.svd_matrix(3000, n, "geometric", kappa, seed=31).astype(np.float32)
+    Q, R = rg.rgsqr_factor(_dev(A), handle=h)
+    torch.cuda.synchronize()
+    Q = Q.cpu().numpy().astype(np.float64)
+    R = R.cpu().numpy().astype(np.float64)
+    A64 = A.astype(np.float64)
+    be = oracle.backward_error(A64, Q, R)
+    assert be < (1e-6 if n == 32 else 5e-3)
+    Qo, Ro, _ = oracle.householder(A64)
+    # forward error of R ~ kappa * backward error (as in _check_qr)
+    assert np.linalg.norm(R - Ro) / np.linalg.norm(Ro) <= max(10 * kappa * be, 1e-5)
+    if n == 32:
+        assert oracle.orthogonality(Q) < 1e-5
+
+
+def test_rgsqr_tall_panel_streaming_path(rg):
+    """m = 200000: more rows per CTA than the fused panel holds -> streaming passes by design."""
+    A = synth.gaussian(200000, 40, seed=41).astype(np.float32)
+    Q, R = _run(rg, A)
+    _check_qr(A, Q, R, kappa=np.linalg.cond(A))
+
+
 def test_rgsqr_config1(rg):
     """BASELINE config 1: 1024 x 64, cond ~ 10 (geometric spectrum), vs the fp64 oracle."""
     A = synth.svd_matrix(1024, 64, "geometric", 10.0, seed=synth.SEED_BASE + 0).astype(np.float32)
