@@ -62,7 +62,7 @@ class ClockSampler:
     def __enter__(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "25"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.thread = threading.Thread(target=self._read, daemon=True)
             self.thread.start()
@@ -150,7 +150,7 @@ def run_reference(args, ws, rank):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-ls", action="store_true")
@@ -240,6 +240,13 @@ def main():
         roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / pk["hbm_gbs"], "peak_src": f"{pk['src']} copy bandwidth"}
     roof["traffic"] = None
+    tpath = os.path.join(ROOT, "profiles", "r01_ncu_traffic.json")
+    if os.path.exists(tpath):
+        with open(tpath) as f:
+            tr = json.load(f).get(dom)
+        if tr:
+            roof["traffic"] = tr["dram_read_bytes"] + tr["dram_write_bytes"]
+            roof["traffic_src"] = f"{tr['source']}; algorithmic bytes per launch {d['bytes'] / max(d['launches'], 1):.0f}"
     roof["share_of_step"] = d["ms"] / 2 / step_ms_prof if step_ms_prof > 0 else None
     roof["launches_per_step"] = d["launches"] / 2
     breakdown = {c: {"ms_per_step": p["ms"] / 2, "launches_per_step": p["launches"] / 2,

@@ -393,7 +393,8 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     }
     for (auto& o : pl.ops) {
         if (o.kind == Op::PANEL) {
-            ProfScope _s(h, PC_PANEL, 2.0 * m * o.w * o.w, (double)m * o.w * (pl.split ? 16 : 14));
+            // algorithmic bytes: read the panel (fp32), write Q (fp32) + 16-bit shadow (+ lo shadow)
+            ProfScope _s(h, PC_PANEL, 2.0 * m * o.w * o.w, (double)m * o.w * (pl.split ? 12 : 10));
             rg::PanelLaunch p{};
             p.Q = pl.Q + (int64_t)o.c0 * pl.ldq;
             p.ldq = pl.ldq;
