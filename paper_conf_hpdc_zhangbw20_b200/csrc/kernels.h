@@ -92,10 +92,20 @@ struct CholqrLaunch {
     int bf16;
     int (*allreduce_g)(double* G, void* ctx);  // non-null: multi-rank Gram allreduce (1024 doubles)
     void* ctx;
+    unsigned long long cond;   // CUDA graph conditional handle set to 1 on a failed pivot (0: none)
+    int* status;    // fused kernels report a numerical breakdown here (atomicMin col0 + j)
+    int col0;       // global column index of the panel
 };
 size_t cholqr_ws_doubles(int64_t m);
 size_t cholqr_counter_ints(int64_t m);
-cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st);
+// True when the single-kernel path applies (rows per SM fit in shared memory; ncols 32 or 64).
+bool cholqr_fused_fits(int64_t m, int ncols);
+// *handles_failure = true: the launched kernel handles failed pivots itself (shifted CholQR3 +
+// breakdown status); false: the caller must enqueue the guarded MGS/TSQR fallback kernels.
+cudaError_t launch_panel_cholqr(const CholqrLaunch& L, bool* handles_failure, cudaStream_t st);
+// Last recursion level (two 32-column panels, K1, K2) as one 64-column CholQR2 kernel on a
+// 32 < nc <= 64 block: same Q and R in exact arithmetic; R written as the nc x nc block at L.R.
+cudaError_t launch_panel_pair(const CholqrLaunch& L, cudaStream_t st);
 
 // ---- gemm_tc.cu (Alg 1 lines 8-9 on tcgen05)
 cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int splits, const CUtensorMap& q1,

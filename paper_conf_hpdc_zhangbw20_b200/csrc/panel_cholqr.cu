@@ -79,7 +79,17 @@ struct CqArgs {
     int64_t ldr;
     int bf16;
     int distributed;     // 1: stop after the reduced Gram; the host allreduces + factors
+    unsigned long long cond;   // graph conditional handle of the MGS/TSQR fallback node (0: none)
+    int* status;         // fused kernels: atomicMin(status, col0 + j) on a numerical breakdown
+    int col0;            // global index of the panel's first column
 };
+
+// A failed pivot: raise the fallback flag and, inside a CUDA graph, switch on the conditional
+// node that holds the MGS/TSQR kernels (so they are not launched at all on the common path).
+__device__ __forceinline__ void cq_signal_fail(const CqArgs& a) {
+    *a.ws.fail = 1;
+    if (a.cond) cudaGraphSetConditional((cudaGraphConditionalHandle)a.cond, 1u);
+}
 
 // ---------------------------------------------------------------- Gram accumulation
 __device__ __forceinline__ void blk_coords(int blk, int& bi, int& bj) {
@@ -109,88 +119,90 @@ __device__ __forceinline__ void gram_block_accum(const float* tile, int rows, in
 }
 
 // ---------------------------------------------------------------- Cholesky + inverse
-// Whole CTA (blockDim.x == NT threads), 32 x 32 fp64, blocked by 4 columns: 8 block steps of
-//   phase 1 (warp 0): every lane factors the 4x4 diagonal block A_bb = L_bb L_bb^T in registers
-//            (the only serial chain: 4 rsqrt), then lane l either forms one panel row
+// Whole CTA (blockDim.x == NT threads), N x N fp64 (N = 32 or 64), blocked by 4 columns:
+// N / 4 block steps of
+//   phase 1 (N / 32 warps): every lane factors the 4x4 diagonal block A_bb = L_bb L_bb^T in
+//            registers (the only serial chain: 4 rsqrt), then lane l either forms one panel row
 //            L_ib = A_ib L_bb^{-T} or applies L_bb^{-1} to one column of Z's block row b;
 //   phase 2 (all warps): trailing update A_ij -= L_ib L_jb^T (i >= j) and Z_i -= L_ib Z_b,
 // one barrier after each phase.  Z starts as I and ends as L^{-1} (the same block row operations
 // applied to the identity), so one sweep yields R = L^T and R^{-1} = L^{-T}.  (A one-warp
 // column-at-a-time version was ~8.5K straight-line SASS instructions and cost 35 us per panel
 // cold; a one-barrier-per-column CTA version ~20K cycles.)
-//   G     : upper triangle of the Gram, G[a + 32 b] (a <= b), nc x nc used; global or smem.
-//   A, Z  : smem scratch, 32 x CH_LD each, 16-byte aligned.  On exit A[i * CH_LD + j] = R(i, j)
-//           (zero below the diagonal).
-//   Rg    : optional fp64 R, column-major [i + 32 j].
-//   Rinvg : fp32 R^{-1}; row-major [i * 32 + j] if rinv_rowmajor else column-major [i + 32 j].
-// Returns false (on every thread) if a pivot is not safely positive relative to G's diagonal;
-// the factor is then garbage but finite (pivot replaced by 1).
-constexpr int CH_LD = 34;   // even: 16-byte aligned rows for the 2 x double2 panel loads
-#ifdef RG_CHOL_TRACE
-__device__ long long chol_trace[40];
-__device__ long long chol_t0;
-#endif
-template <int NT, bool kSharedG>
+//   G     : upper triangle of the Gram, G[a + N b] (a <= b), nc x nc used; global or smem.
+//   A, Z  : smem scratch, N x (N + 2) doubles each, 16-byte aligned; Z may alias G (G is read
+//           completely before Z is initialised).  On exit A[i * (N + 2) + j] = R(i, j) (zero
+//           below the diagonal).
+//   Rg    : optional fp64 R, column-major [i + N j].
+//   Rinvg : fp32 R^{-1}; row-major [i * N + j] if rinv_rowmajor else column-major [i + N j].
+// Returns false (on every thread) if a pivot is not safely positive relative to G's diagonal
+// (first such column in *first_bad, N if none); the factor is then garbage but finite.
+constexpr int CH_LD = 34;   // N + 2 for N = 32: 16-byte aligned rows for the double2 loads
+template <int NT, bool kSharedG, int N = 32>
 __device__ bool chol_inv_cta(const double* G, int nc, double* A, double* Z, double* Rg, float* Rinvg,
-                             bool rinv_rowmajor) {
-    static_assert(NT % 32 == 0 && 1024 % NT == 0, "thread count");
-    constexpr int PER = 1024 / NT;
-    constexpr int NW = NT / 32;
-    __shared__ double odiag[32];
-    __shared__ int s_ok;
-    const int tid = threadIdx.x, w = tid >> 5, lane = tid & 31;
-    auto gload = [&](int a, int b) -> double { return kSharedG ? G[a + 32 * b] : __ldcg(G + a + 32 * b); };
-#pragma unroll
+                             bool rinv_rowmajor, int* first_bad = nullptr) {
+    constexpr int LD = N + 2;
+    static_assert(NT % 32 == 0 && (N * N) % NT == 0 && NT >= N, "thread count");
+    constexpr int PER = N * N / NT;   // elements per thread (rows w + RS c, column tid % N)
+    constexpr int RS = NT / N;        // row stride between a thread's elements
+    __shared__ double odiag[N];
+    __shared__ int s_bad;
+    const int tid = threadIdx.x, lane = tid % N, rbase = tid / N;
+    auto gload = [&](int a, int b) -> double { return kSharedG ? G[a + N * b] : __ldcg(G + a + N * b); };
+#pragma unroll 4
     for (int c = 0; c < PER; ++c) {
-        const int e = tid + NT * c, i = e >> 5, j = e & 31;
+        const int i = rbase + RS * c, j = lane;
         const double g = (i < nc && j < nc) ? gload(min(i, j), max(i, j)) : (i == j ? 1.0 : 0.0);
-        A[i * CH_LD + j] = g;
-        Z[i * CH_LD + j] = (i == j) ? 1.0 : 0.0;
+        A[i * LD + j] = g;
         if (i == j) odiag[i] = g;
     }
-    if (tid == 0) s_ok = 1;
+    if (tid == 0) s_bad = N;
+    __syncthreads();
+#pragma unroll 4
+    for (int c = 0; c < PER; ++c) {
+        const int i = rbase + RS * c, j = lane;
+        Z[i * LD + j] = (i == j) ? 1.0 : 0.0;
+    }
     __syncthreads();
 #pragma unroll 1
-    for (int k0 = 0; k0 < 32; k0 += 4) {
-#ifdef RG_CHOL_TRACE
-        if (tid == 0) chol_trace[k0 / 4] = clock64();
-#endif
-        if (w == 0) {
-            const double* Ab = A + k0 * CH_LD + k0;
+    for (int k0 = 0; k0 < N; k0 += 4) {
+        if (tid < N) {   // phase 1
+            const int l = tid;
+            const double* Ab = A + k0 * LD + k0;
             const double d00 = Ab[0];
-            const double d10 = Ab[CH_LD], d11 = Ab[CH_LD + 1];
-            const double d20 = Ab[2 * CH_LD], d21 = Ab[2 * CH_LD + 1], d22 = Ab[2 * CH_LD + 2];
-            const double d30 = Ab[3 * CH_LD], d31 = Ab[3 * CH_LD + 1], d32 = Ab[3 * CH_LD + 2],
-                         d33 = Ab[3 * CH_LD + 3];
-            const int npan = 28 - k0;          // lanes < npan: panel row; others: Z column (npan + k0 + 4 = 32)
-            const bool pan = lane < npan;
-            const int r = k0 + 4 + lane, col = lane - npan;
+            const double d10 = Ab[LD], d11 = Ab[LD + 1];
+            const double d20 = Ab[2 * LD], d21 = Ab[2 * LD + 1], d22 = Ab[2 * LD + 2];
+            const double d30 = Ab[3 * LD], d31 = Ab[3 * LD + 1], d32 = Ab[3 * LD + 2], d33 = Ab[3 * LD + 3];
+            const int npan = N - 4 - k0;          // lanes < npan: panel row; others: Z column
+            const bool pan = l < npan;
+            const int r = k0 + 4 + l, col = l - npan;
             double p[4];
             if (pan) {
-                const double2 v0 = *reinterpret_cast<const double2*>(A + r * CH_LD + k0);
-                const double2 v1 = *reinterpret_cast<const double2*>(A + r * CH_LD + k0 + 2);
+                const double2 v0 = *reinterpret_cast<const double2*>(A + r * LD + k0);
+                const double2 v1 = *reinterpret_cast<const double2*>(A + r * LD + k0 + 2);
                 p[0] = v0.x; p[1] = v0.y; p[2] = v1.x; p[3] = v1.y;
             } else {
 #pragma unroll
-                for (int c = 0; c < 4; ++c) p[c] = Z[(k0 + c) * CH_LD + col];
+                for (int c = 0; c < 4; ++c) p[c] = Z[(k0 + c) * LD + col];
             }
-            __syncwarp();   // every lane has read A_bb before lane 0 overwrites it with L_bb
-            bool good = true;
+            if (N == 32) __syncwarp(); else asm volatile("bar.sync 1, %0;" :: "r"(N));   // all read A_bb
+            int bad = N;
             auto piv = [&](double d, int kk) -> double {
                 const bool gd = (d > odiag[kk] * 1e-15) && isfinite(d);
-                good = good && gd;
+                if (!gd) bad = min(bad, kk);
                 const double y = rsqrt(fmax(d, 1e-300));   // no branch on gd in the pivot chain
                 return gd ? y : 1.0;
             };
             const double i0 = piv(d00, k0);
             const double l10 = d10 * i0, l20 = d20 * i0, l30 = d30 * i0;
-            const double i1 = piv(fma(-l10, l10, d11), k0 + 1);
+            const double e11 = fma(-l10, l10, d11);
+            const double i1 = piv(e11, k0 + 1);
             const double l21 = fma(-l20, l10, d21) * i1, l31 = fma(-l30, l10, d31) * i1;
-            const double i2 = piv(fma(-l21, l21, fma(-l20, l20, d22)), k0 + 2);
+            const double e22 = fma(-l21, l21, fma(-l20, l20, d22));
+            const double i2 = piv(e22, k0 + 2);
             const double l32 = fma(-l31, l21, fma(-l30, l20, d32)) * i2;
             const double e33 = fma(-l32, l32, fma(-l31, l31, fma(-l30, l30, d33)));
             const double i3 = piv(e33, k0 + 3);
-            // L_bb^{-1} (lower; diagonal i0..i3)
             const double m10 = -l10 * i0 * i1;
             const double m21 = -l21 * i1 * i2;
             const double m20 = -fma(l21, m10, l20 * i0) * i2;
@@ -198,109 +210,105 @@ __device__ bool chol_inv_cta(const double* G, int nc, double* A, double* Z, doub
             const double m31 = -fma(l32, m21, l31 * i1) * i3;
             const double m30 = -fma(l32, m20, fma(l31, m10, l30 * i0)) * i3;
             double q[4];
-            if (pan) {   // row r of L_ib = A_ib L_bb^{-T}: q_c = sum_{k <= c} p_k Linv(c, k)
-                q[0] = p[0] * i0;
-                q[1] = fma(p[0], m10, p[1] * i1);
-                q[2] = fma(p[0], m20, fma(p[1], m21, p[2] * i2));
-                q[3] = fma(p[0], m30, fma(p[1], m31, fma(p[2], m32, p[3] * i3)));
-                *reinterpret_cast<double2*>(A + r * CH_LD + k0) = make_double2(q[0], q[1]);
-                *reinterpret_cast<double2*>(A + r * CH_LD + k0 + 2) = make_double2(q[2], q[3]);
-            } else {     // column col of Z_b <- L_bb^{-1} Z_b (same formula)
-                q[0] = p[0] * i0;
-                q[1] = fma(m10, p[0], p[1] * i1);
-                q[2] = fma(m20, p[0], fma(m21, p[1], p[2] * i2));
-                q[3] = fma(m30, p[0], fma(m31, p[1], fma(m32, p[2], p[3] * i3)));
+            q[0] = p[0] * i0;
+            q[1] = fma(p[0], m10, p[1] * i1);
+            q[2] = fma(p[0], m20, fma(p[1], m21, p[2] * i2));
+            q[3] = fma(p[0], m30, fma(p[1], m31, fma(p[2], m32, p[3] * i3)));
+            if (pan) {   // row r of L_ib = A_ib L_bb^{-T}
+                *reinterpret_cast<double2*>(A + r * LD + k0) = make_double2(q[0], q[1]);
+                *reinterpret_cast<double2*>(A + r * LD + k0 + 2) = make_double2(q[2], q[3]);
+            } else {     // column col of Z_b <- L_bb^{-1} Z_b
 #pragma unroll
-                for (int c = 0; c < 4; ++c) Z[(k0 + c) * CH_LD + col] = q[c];
+                for (int c = 0; c < 4; ++c) Z[(k0 + c) * LD + col] = q[c];
             }
-            if (lane == 0) {
-                double* Lb = A + k0 * CH_LD + k0;   // L_bb (lower) in place of A_bb
+            if (l == 0) {
+                double* Lb = A + k0 * LD + k0;   // L_bb (lower) in place of A_bb
                 Lb[0] = d00 * i0;
-                Lb[CH_LD] = l10;
-                Lb[CH_LD + 1] = fma(-l10, l10, d11) * i1;
-                Lb[2 * CH_LD] = l20;
-                Lb[2 * CH_LD + 1] = l21;
-                Lb[2 * CH_LD + 2] = fma(-l21, l21, fma(-l20, l20, d22)) * i2;
-                Lb[3 * CH_LD] = l30;
-                Lb[3 * CH_LD + 1] = l31;
-                Lb[3 * CH_LD + 2] = l32;
-                Lb[3 * CH_LD + 3] = e33 * i3;
-                if (!good) s_ok = 0;
+                Lb[LD] = l10;
+                Lb[LD + 1] = e11 * i1;
+                Lb[2 * LD] = l20;
+                Lb[2 * LD + 1] = l21;
+                Lb[2 * LD + 2] = e22 * i2;
+                Lb[3 * LD] = l30;
+                Lb[3 * LD + 1] = l31;
+                Lb[3 * LD + 2] = l32;
+                Lb[3 * LD + 3] = e33 * i3;
+                if (bad < s_bad) s_bad = bad;
             }
-#ifdef RG_CHOL_TRACE
-            if (tid == 0) chol_trace[10 + k0 / 4] = clock64();
-#endif
         }
         __syncthreads();
-#ifdef RG_CHOL_TRACE
-        if (tid == 0) chol_trace[20 + k0 / 4] = clock64();
-#endif
-        // phase 2: rows i >= k0 + 4 (warp-uniform), lane = column.  All operands are loaded
-        // before any store so the PER rows overlap instead of serialising on possible aliasing.
+        // phase 2: rows i >= k0 + 4 (warp-uniform), column j = lane; operands loaded 4 rows at a
+        // time before any store so the rows overlap instead of serialising on possible aliasing
         {
-            const bool zl = lane < k0 + 4;   // Z column (else A column lane)
+            const int j = lane;
+            const bool zl = j < k0 + 4;   // Z column (else A column j)
             double ob[4];
             if (zl) {
 #pragma unroll
-                for (int c = 0; c < 4; ++c) ob[c] = Z[(k0 + c) * CH_LD + lane];
+                for (int c = 0; c < 4; ++c) ob[c] = Z[(k0 + c) * LD + j];
             } else {
-                const double2 b0 = *reinterpret_cast<const double2*>(A + lane * CH_LD + k0);
-                const double2 b1 = *reinterpret_cast<const double2*>(A + lane * CH_LD + k0 + 2);
+                const double2 b0 = *reinterpret_cast<const double2*>(A + j * LD + k0);
+                const double2 b1 = *reinterpret_cast<const double2*>(A + j * LD + k0 + 2);
                 ob[0] = b0.x; ob[1] = b0.y; ob[2] = b1.x; ob[3] = b1.y;
             }
-            double la[PER][4], cur[PER];
+            const int cstart = (k0 + 4 - rbase + RS - 1) / RS;   // first c with row >= k0 + 4
+#pragma unroll 1
+            for (int c0 = cstart < 0 ? 0 : cstart; c0 < PER; c0 += 4) {
+                double la[4][4], cur[4];
 #pragma unroll
-            for (int c = 0; c < PER; ++c) {
-                const int i = w + NW * c;
-                if (i >= k0 + 4) {
-                    const double2 a0 = *reinterpret_cast<const double2*>(A + i * CH_LD + k0);
-                    const double2 a1 = *reinterpret_cast<const double2*>(A + i * CH_LD + k0 + 2);
-                    la[c][0] = a0.x; la[c][1] = a0.y; la[c][2] = a1.x; la[c][3] = a1.y;
-                    cur[c] = zl ? Z[i * CH_LD + lane] : A[i * CH_LD + lane];
+                for (int cc = 0; cc < 4; ++cc) {
+                    const int i = rbase + RS * (c0 + cc);
+                    if (c0 + cc < PER) {
+                        const double2 a0 = *reinterpret_cast<const double2*>(A + i * LD + k0);
+                        const double2 a1 = *reinterpret_cast<const double2*>(A + i * LD + k0 + 2);
+                        la[cc][0] = a0.x; la[cc][1] = a0.y; la[cc][2] = a1.x; la[cc][3] = a1.y;
+                        cur[cc] = zl ? Z[i * LD + j] : A[i * LD + j];
+                    }
                 }
-            }
 #pragma unroll
-            for (int c = 0; c < PER; ++c) {
-                const int i = w + NW * c;
-                if (i >= k0 + 4) {
-                    double v = cur[c];
-                    v = fma(-la[c][0], ob[0], v);
-                    v = fma(-la[c][1], ob[1], v);
-                    v = fma(-la[c][2], ob[2], v);
-                    v = fma(-la[c][3], ob[3], v);
-                    if (zl)
-                        Z[i * CH_LD + lane] = v;
-                    else if (lane <= i)
-                        A[i * CH_LD + lane] = v;
+                for (int cc = 0; cc < 4; ++cc) {
+                    const int i = rbase + RS * (c0 + cc);
+                    if (c0 + cc < PER) {
+                        double v = cur[cc];
+                        v = fma(-la[cc][0], ob[0], v);
+                        v = fma(-la[cc][1], ob[1], v);
+                        v = fma(-la[cc][2], ob[2], v);
+                        v = fma(-la[cc][3], ob[3], v);
+                        if (zl)
+                            Z[i * LD + j] = v;
+                        else if (j <= i)
+                            A[i * LD + j] = v;
+                    }
                 }
             }
         }
-#ifdef RG_CHOL_TRACE
-        if (tid == 0) chol_trace[30 + k0 / 4] = clock64();
-#endif
         __syncthreads();
     }
-#ifdef RG_CHOL_TRACE
-    if (tid == 0) chol_trace[8] = clock64();
-#endif
-    double r[PER];
-#pragma unroll
+    // outputs: R(i, j) = L(j, i), R^{-1}(i, j) = L^{-1}(j, i)
+    const int nbad = s_bad;
+    if (first_bad) *first_bad = nbad;
+#pragma unroll 4
     for (int c = 0; c < PER; ++c) {
-        const int e = tid + NT * c, i = e >> 5, j = e & 31;
-        r[c] = (i <= j) ? A[j * CH_LD + i] : 0.0;                     // R(i, j) = L(j, i)
-        const float ri = (i <= j) ? (float)Z[j * CH_LD + i] : 0.f;    // R^{-1}(i, j) = L^{-1}(j, i)
-        Rinvg[rinv_rowmajor ? (i * 32 + j) : (i + 32 * j)] = ri;
-        if (Rg) Rg[i + 32 * j] = r[c];
-    }
-    const bool ok = s_ok != 0;
-    __syncthreads();
-#pragma unroll
-    for (int c = 0; c < PER; ++c) {
-        const int e = tid + NT * c;
-        A[(e >> 5) * CH_LD + (e & 31)] = r[c];
+        const int i = rbase + RS * c, j = lane;
+        const float ri = (i <= j) ? (float)Z[j * LD + i] : 0.f;
+        Rinvg[rinv_rowmajor ? (i * N + j) : (i + N * j)] = ri;
+        if (Rg) Rg[i + N * j] = (i <= j) ? A[j * LD + i] : 0.0;
     }
     __syncthreads();
-    return ok;
+    // A <- R row-major (upper): transpose the lower triangle in place, then clear it
+#pragma unroll 4
+    for (int c = 0; c < PER; ++c) {
+        const int i = rbase + RS * c, j = lane;
+        if (i < j) A[i * LD + j] = A[j * LD + i];
+    }
+    __syncthreads();
+#pragma unroll 4
+    for (int c = 0; c < PER; ++c) {
+        const int i = rbase + RS * c, j = lane;
+        if (i > j) A[i * LD + j] = 0.0;
+    }
+    __syncthreads();
+    return nbad == N;
 }
 
 // Sum `n` partial Grams [n][1024] (upper triangle) in fixed order into dst (whole CTA);
@@ -397,7 +405,7 @@ __device__ void reduce_and_factor(const CqArgs& a, int pass, double* smem_R, dou
     // smem_R1 doubles as the elimination scratch Y; final_r_product reloads it afterwards
     const bool ok = chol_inv_cta<CQ_THREADS, false>(G, a.nc, smem_R, smem_R1, a.ws.R + pass * 1024,
                                                      a.ws.Rinv + pass * 1024, false);
-    if (!ok && threadIdx.x == 0) *a.ws.fail = 1;
+    if (!ok && threadIdx.x == 0) cq_signal_fail(a);
     if (pass == 0 && ok) single_pass_decision(a);
     if (pass == 1 && ok) final_r_product(a, smem_R, smem_R1);
 }
@@ -551,34 +559,40 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
 
 
 // ---------------------------------------------------------------- fused single-kernel panel
-// Whole CholQR2 panel in one cooperative kernel (m <= CF_MAX_ROWS * gridDim): every CTA keeps
-// its rows of the panel in shared memory for the whole computation, so the panel is read once
-// and written once; the three launches, two "last block" chains and the broadcast of R^{-1}
-// of the streaming version become grid barriers, and every CTA factors the reduced 32 x 32
+// Whole CholQR2 panel of NC = 32 or 64 columns in one cooperative kernel (rows per CTA must fit
+// in shared memory): every CTA keeps its rows of the panel in shared memory for the whole
+// computation, so the panel is read once and written once; the Gram reductions run through a
+// fixed-order last-arriver tree + flag broadcast (cf_allreduce) and every CTA factors the reduced
 // Gram itself (identical arithmetic on identical data -> identical R on every CTA).
+//
+// NC = 64 covers the last recursion level of Algorithm 1 with two 32-column panels at once:
+// with G = [P1 P2]^T [P1 P2], the recursion step computes R11 = chol(G11), R12 = Q1^T P2 =
+// R11^{-T} G12 and R22 = chol(G22 - R12^T R12), which is the Cholesky factor of the 64 x 64 G;
+// so in exact arithmetic the 64-column CholQR2 returns the same (unique) Q and R as the two
+// panels + K1 + K2 of that level, and the second CholQR pass restores orthogonality exactly as
+// it does for a 32-column panel.
 constexpr int CF_THREADS = 256;
-constexpr int CF_GB = 10;                        // 8x8 blocks in the upper triangle of a 32x32 Gram (4*5/2)
-constexpr int CF_GROUPS = CF_THREADS / CF_GB;    // 25 row groups of 10 threads (250 active)
-constexpr int CF_CH = 96;                        // rows staged in fp64 per Gram chunk
-constexpr int CF_SLD = 34;                       // fp64 row stride of the staging chunk (16B-aligned rows)
-constexpr int CF_SCR = CF_CH * CF_SLD;           // scratch doubles: staging chunk / 5 group partials / Y
+constexpr int CF_SCR = 3264;                     // scratch doubles: fp64 staging chunk / group partials
 constexpr int CF_FAN = 8;                        // CTA partials per first-level group
-constexpr int CF_MAX_ROWS = 1280;                // rows per CTA that fit next to the scratch
+constexpr int CF_MAX_ROWS = 1280;                // rows per CTA that fit next to the scratch (NC = 32)
+constexpr int CF_WIDE_MAX_ROWS = 472;            // same for NC = 64
 constexpr int CF_MAXPER = CF_MAX_ROWS / CF_THREADS;   // tile rows per thread (load / store loops)
-static_assert(CF_GROUPS % 5 == 0 && 5 * 641 <= CF_SCR && 32 * CH_LD <= CF_SCR, "Gram scratch");
+constexpr int CF_NE_MAX = 64 * 65 / 2;           // packed Gram entries, NC = 64
 
-struct CfSmem {
-    static size_t bytes(int ld) {
-        return (size_t)32 * ld * 4        // tile (column-major, ld)
-               + CF_SCR * 8               // fp64 staging / reduction / elimination scratch
-               + 32 * CH_LD * 8 * 2       // G (padded) + Cholesky scratch
-               + 2 * 32 * 32 * 4          // R1^{-1}, R2^{-1} (fp32, [k][j])
-               + 1024 * 8                 // R1 (fp64) kept for R = R2 R1
-               + 256;
-    }
+template <int NC>
+struct CfCfg {
+    static constexpr int NB8 = NC / 8;                       // 8-column blocks
+    static constexpr int NBLK = NB8 * (NB8 + 1) / 2;         // 8x8 blocks in the upper triangle
+    static constexpr int GROUPS = CF_THREADS / NBLK;         // row groups (25 or 7)
+    static constexpr int SLD = NC + 2;                       // fp64 row stride of the staging chunk
+    static constexpr int CH = CF_SCR / SLD / 8 * 8;          // rows staged per chunk (96 or 48)
+    static constexpr int NE = NC * (NC + 1) / 2;             // packed upper-triangle entries
+    static constexpr int GSTRIDE = NBLK * 64 + 1;            // group stride in the reduction rounds
+    static constexpr int GPR = CF_SCR / GSTRIDE;             // groups per round (5 or 1)
+    static constexpr int LD = NC + 2;                        // Cholesky scratch row stride
+    static_assert(GPR >= 1 && CH >= 8, "scratch");
 };
 
-constexpr int CF_NP = 32 * 33 / 2;               // packed upper-triangle entries of a partial Gram
 __device__ __forceinline__ void tri_unpack(int p, int& i, int& j) {
     int jj = (int)((sqrtf(8.f * p + 1.f) - 1.f) * 0.5f);
     if ((jj + 1) * (jj + 2) / 2 <= p) ++jj;
@@ -587,105 +601,74 @@ __device__ __forceinline__ void tri_unpack(int p, int& i, int& j) {
     i = p - jj * (jj + 1) / 2;
 }
 
-__device__ __forceinline__ void cf_blk_coords(int blk, int& bi, int& bj) {
-    // (0,0) (0,1) (0,2) (0,3) (1,1) (1,2) (1,3) (2,2) (2,3) (3,3)
-    bi = blk < 4 ? 0 : (blk < 7 ? 1 : (blk < 9 ? 2 : 3));
-    bj = bi + blk - (bi == 0 ? 0 : (bi == 1 ? 4 : (bi == 2 ? 7 : 9)));
-}
-
-// Gram partial of the CTA's tile rows [0, rows) -> out (fp64, packed upper triangle
-// [j (j + 1) / 2 + i], CF_NP entries), fixed order.  Rows are converted to fp64 once per CF_CH-row chunk (row-major staging,
-// so each thread's 8 consecutive columns are 4 LDS.128), then 8x8 register blocks give 4 DFMA per
-// loaded double: the loop runs at the fp64 FMA rate instead of the F2F conversion rate.
+// Gram partial of the CTA's tile rows [0, rows) (NC columns) -> out (fp64, packed upper
+// triangle [j (j + 1) / 2 + i]) on the fp64 tensor cores (mma.sync m8n8k4 f64: 256 FMAs per
+// warp instruction, so 8 warps reach the SM's fp64 rate where DFMA loops stall on issue).
+// Rows are converted to fp64 once per chunk into a row-major staging buffer (row stride
+// SLD = NC + 4 == 4 mod 16 doubles: the 4 rows x 8 columns of an A/B fragment hit distinct
+// banks); warp w owns the 8x8 blocks w, w + 8, ... of the upper triangle for all rows, so the
+// sum over rows has one fixed order per entry and no cross-warp reduction is needed.
+template <int NC>
 __device__ void cf_gram(const float* tile, int ld, int rows, double* S, double* out_partial) {
-    const int tid = threadIdx.x;
-    const int g = tid / CF_GB, blk = tid % CF_GB;
-    int bi = 0, bj = 0;
-    cf_blk_coords(blk, bi, bj);
-    double acc[8][8];
+    constexpr int NB8 = NC / 8, NBLK = NB8 * (NB8 + 1) / 2, SLD = NC + 4;
+    constexpr int CH = CF_SCR / SLD / 4 * 4;
+    constexpr int NW = CF_THREADS / 32, MAXB = (NBLK + NW - 1) / NW;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int g = lane >> 2, c = lane & 3;
+    int boff[MAXB][2];   // S column offsets of the A (bi) and B (bj) fragments of each owned block
 #pragma unroll
-    for (int u = 0; u < 8; ++u)
+    for (int t = 0; t < MAXB; ++t) {
+        int blk = warp + NW * t, bi = 0;
+        if (blk >= NBLK) blk = 0;
+        while (blk >= NB8 - bi) {
+            blk -= NB8 - bi;
+            ++bi;
+        }
+        boff[t][0] = bi * 8 + g;
+        boff[t][1] = (bi + blk) * 8 + g;
+    }
+    double acc[MAXB][2];
 #pragma unroll
-        for (int v = 0; v < 8; ++v) acc[u][v] = 0.0;
-    for (int ch0 = 0; ch0 < rows; ch0 += CF_CH) {
-        const int cr = min(CF_CH, rows - ch0);
+    for (int t = 0; t < MAXB; ++t) acc[t][0] = acc[t][1] = 0.0;
+    for (int ch0 = 0; ch0 < rows; ch0 += CH) {
+        const int cr = min(CH, rows - ch0), cr4 = (cr + 3) & ~3;
         __syncthreads();
-        for (int e = tid; e < cr * 32; e += CF_THREADS) {
-            const int r = e >> 5, c = e & 31;
-            S[r * CF_SLD + c] = (double)tile[c * ld + ch0 + r];
+        for (int e = tid; e < cr4 * NC; e += CF_THREADS) {
+            const int r = e / NC, col = e % NC;
+            S[r * SLD + col] = (r < cr) ? (double)tile[col * ld + ch0 + r] : 0.0;
         }
         __syncthreads();
-        if (g < CF_GROUPS) {
-            for (int r = g; r < cr; r += CF_GROUPS) {
-                const double2* row = reinterpret_cast<const double2*>(S + r * CF_SLD);
-                double x[8], y[8];
+        for (int k0 = 0; k0 < cr4; k0 += 4) {
+            const double* rowp = S + (k0 + c) * SLD;
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    const double2 vx = row[bi * 4 + q], vy = row[bj * 4 + q];
-                    x[2 * q] = vx.x;
-                    x[2 * q + 1] = vx.y;
-                    y[2 * q] = vy.x;
-                    y[2 * q + 1] = vy.y;
+            for (int t = 0; t < MAXB; ++t) {
+                if (warp + NW * t < NBLK) {
+                    const double av = rowp[boff[t][0]], bv = rowp[boff[t][1]];
+                    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                                 : "+d"(acc[t][0]), "+d"(acc[t][1])
+                                 : "d"(av), "d"(bv));
                 }
-#pragma unroll
-                for (int u = 0; u < 8; ++u)
-#pragma unroll
-                    for (int v = 0; v < 8; ++v) acc[u][v] = fma(x[u], y[v], acc[u][v]);
             }
         }
     }
-    // fixed-order sum of the 25 group accumulators, 5 groups per round through S
-    // (entry e = (u * 8 + v) * 10 + blk, group stride 641: conflict-free stores and loads)
-    double run[3] = {0.0, 0.0, 0.0};   // entries tid, tid + 256, tid + 512 (< 640)
-    for (int round = 0; round < CF_GROUPS / 5; ++round) {
-        __syncthreads();
-        const int gl = g - 5 * round;
-        if (g < CF_GROUPS && gl >= 0 && gl < 5) {
+    // D fragment: rows g, columns 2c, 2c + 1 of the 8x8 block
 #pragma unroll
-            for (int u = 0; u < 8; ++u)
+    for (int t = 0; t < MAXB; ++t) {
+        if (warp + NW * t < NBLK) {
+            const int i = boff[t][0];
+            const int j0 = boff[t][1] - g + 2 * c;
 #pragma unroll
-                for (int v = 0; v < 8; ++v) S[gl * 641 + (u * 8 + v) * 10 + blk] = acc[u][v];
+            for (int u = 0; u < 2; ++u) {
+                const int j = j0 + u;
+                if (i <= j) out_partial[j * (j + 1) / 2 + i] = acc[t][u];
+            }
         }
-        __syncthreads();
-#pragma unroll
-        for (int q = 0; q < 3; ++q) {
-            const int e = tid + CF_THREADS * q;
-            if (e < 640) run[q] += ((S[e] + S[641 + e]) + (S[1282 + e] + S[1923 + e])) + S[2564 + e];
-        }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int q = 0; q < 3; ++q) {
-        const int e = tid + CF_THREADS * q;
-        if (e < 640) S[e] = run[q];
-    }
-    __syncthreads();
-    for (int e = tid; e < CF_NP; e += CF_THREADS) {
-        int i, j;
-        tri_unpack(e, i, j);
-        double v;
-        {
-            const int pi = i >> 3, pj = j >> 3;
-            const int b = (pi == 0 ? 0 : (pi == 1 ? 4 : (pi == 2 ? 7 : 9))) + (pj - pi);
-            v = S[((i & 7) * 8 + (j & 7)) * 10 + b];
-        }
-        out_partial[e] = v;
     }
     __syncthreads();
 }
 
-// Grid-wide fixed-order reduction of the CTA partials into Gs (smem, fp64, upper) on every CTA.
 #ifdef RG_CF_TRACE
 __device__ unsigned long long cf_trace[16];
-__device__ unsigned long long cf_cta[4][160];
-#define CF_CTA(i)                                                                      \
-    do {                                                                               \
-        if (threadIdx.x == 0) {                                                        \
-            unsigned long long t;                                                      \
-            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));                      \
-            cf_cta[i][blockIdx.x] = t;                                                 \
-        }                                                                              \
-    } while (0)
 #define CF_MARK(i)                                                                     \
     do {                                                                               \
         if (blockIdx.x == 0 && threadIdx.x == 0) {                                     \
@@ -698,22 +681,14 @@ __device__ unsigned long long cf_cta[4][160];
 #define CF_MARK(i) \
     do {           \
     } while (0)
-#define CF_CTA(i) \
-    do {          \
-    } while (0)
 #endif
 
-// Counter slots used by the fused kernel (the streaming passes use [0, ngroups]): one 128-byte
+// Counter slots used by the fused kernels (the streaming passes use [0, ngroups]): one 128-byte
 // line each, so the 147 CTAs polling the flag do not queue behind the arrival atomics.
 constexpr int CF_CNT_BASE = 1024, CF_CNT_STRIDE = 32;
 constexpr int CF_CNT_GLOBAL = CF_CNT_BASE + 20 * CF_CNT_STRIDE, CF_CNT_FLAG = CF_CNT_BASE + 21 * CF_CNT_STRIDE;
 constexpr int CF_CNT_INTS = CF_CNT_BASE + 22 * CF_CNT_STRIDE;
 
-// Grid-wide fixed-order reduction of the CTA partials into Gs (smem, fp64, upper) on every CTA,
-// without grid barriers: the last CTA to arrive in each group of CF_FAN sums the group's
-// partials (ws.gpart), the last group to finish sums the group sums into ws.G and bumps a
-// generation flag; every CTA spins on the flag and reads the 528 packed entries.  The order of
-// every sum is fixed (CTA order within a group, group order), so G is bitwise reproducible.
 __device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 __device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
     unsigned v;
@@ -721,101 +696,109 @@ __device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
     return v;
 }
 
-__device__ void cf_allreduce_gram(const CqArgs& a, double* Gs) {
-    constexpr int NQ = (CF_NP + CF_THREADS - 1) / CF_THREADS;   // packed entries per thread
+// Workspace of the fused kernels (doubles): CTA partials [160][NE], group sums [20][NE],
+// reduced Gram [NE], accumulated R [NC * NC] (CTA 0 only).
+struct CfWs {
+    double* part;
+    double* gpart;
+    double* G;
+    double* Racc;
+};
+__device__ __forceinline__ CfWs cf_ws(const CqArgs& a) {
+    CfWs w;
+    w.part = a.ws.part;
+    w.gpart = w.part + (size_t)160 * CF_NE_MAX;
+    w.G = w.gpart + (size_t)20 * CF_NE_MAX;
+    w.Racc = w.G + CF_NE_MAX;
+    return w;
+}
+constexpr size_t CF_WS_DOUBLES = (size_t)(160 + 20 + 1) * CF_NE_MAX + 64 * 64;
+
+// Grid-wide fixed-order reduction of the CTA partials (NE doubles each) into Gs (smem, fp64,
+// [i + NC j]) on every CTA, without grid barriers: the last CTA to arrive in each group of
+// CF_FAN sums the group's partials, the last group to finish sums the group sums into w.G and
+// bumps a generation flag; every CTA spins on the flag and reads the NE entries.  Every sum has
+// a fixed order (CTA order within a group, group order), so the result is bitwise reproducible.
+template <int NC>
+__device__ void cf_allreduce(const CqArgs& a, double* Gs) {
+    constexpr int NE = CfCfg<NC>::NE;
+    constexpr int NQ = (NE + CF_THREADS - 1) / CF_THREADS;      // entries per thread
     constexpr int MAXG = (160 + CF_FAN - 1) / CF_FAN;           // grid <= 160 CTAs
+    const CfWs w = cf_ws(a);
     const int ngroups = (gridDim.x + CF_FAN - 1) / CF_FAN;
     const int grp = blockIdx.x / CF_FAN;
     const int gsize = min(CF_FAN, (int)gridDim.x - grp * CF_FAN);
     const int tid = threadIdx.x;
     int* cnt = a.ws.counters;
     unsigned* flag = reinterpret_cast<unsigned*>(cnt + CF_CNT_FLAG);
+    int* gcnt = cnt + CF_CNT_BASE + grp * CF_CNT_STRIDE;
     __shared__ int s_last;
     __shared__ unsigned s_gen;
     if (tid == 0) s_gen = *(volatile unsigned*)flag;   // read before this CTA arrives
     fence_acq_rel_gpu();
     __syncthreads();
-    int* gcnt = cnt + CF_CNT_BASE + grp * CF_CNT_STRIDE;
     if (tid == 0) s_last = (atomicAdd(gcnt, 1) == gsize - 1);
     __syncthreads();
-#ifdef RG_CF_TRACE
-    if (tid == 0) { unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); cf_cta[3][blockIdx.x] = t; }
-#endif
     if (s_last) {
         fence_acq_rel_gpu();
         const int c0 = grp * CF_FAN;
-        double v[NQ][CF_FAN];
-#pragma unroll
-        for (int q = 0; q < NQ; ++q)
-#pragma unroll
-            for (int c = 0; c < CF_FAN; ++c) {
-                const int e = tid + CF_THREADS * q;
-                v[q][c] = (c < gsize && e < CF_NP) ? __ldcg(a.ws.part + (int64_t)(c0 + c) * CF_NP + e) : 0.0;
-            }
-#pragma unroll
+#pragma unroll 3
         for (int q = 0; q < NQ; ++q) {
             const int e = tid + CF_THREADS * q;
+            double v[CF_FAN];
+#pragma unroll
+            for (int c = 0; c < CF_FAN; ++c)
+                v[c] = (c < gsize && e < NE) ? __ldcg(w.part + (int64_t)(c0 + c) * NE + e) : 0.0;
             double sum = 0.0;
 #pragma unroll
-            for (int c = 0; c < CF_FAN; ++c) sum += v[q][c];
-            if (e < CF_NP) a.ws.gpart[(int64_t)grp * CF_NP + e] = sum;
+            for (int c = 0; c < CF_FAN; ++c) sum += v[c];
+            if (e < NE) w.gpart[(int64_t)grp * NE + e] = sum;
         }
         if (tid == 0) *gcnt = 0;
         fence_acq_rel_gpu();
         __syncthreads();
-#ifdef RG_CF_TRACE
-        if (tid == 0) { unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); cf_cta[1][blockIdx.x] = t; }
-#endif
         if (tid == 0) s_last = (atomicAdd(cnt + CF_CNT_GLOBAL, 1) == ngroups - 1);
         __syncthreads();
         if (s_last) {
             fence_acq_rel_gpu();
-#pragma unroll
+#pragma unroll 1
             for (int q = 0; q < NQ; ++q) {
                 const int e = tid + CF_THREADS * q;
-                if (e < CF_NP) {
-                    double w[MAXG];
+                if (e < NE) {
+                    double v[MAXG];
 #pragma unroll
-                    for (int g = 0; g < MAXG; ++g) w[g] = (g < ngroups) ? __ldcg(a.ws.gpart + (int64_t)g * CF_NP + e) : 0.0;
+                    for (int g = 0; g < MAXG; ++g) v[g] = (g < ngroups) ? __ldcg(w.gpart + (int64_t)g * NE + e) : 0.0;
                     double sum = 0.0;
 #pragma unroll
-                    for (int g = 0; g < MAXG; ++g) sum += w[g];
-                    a.ws.G[e] = sum;
+                    for (int g = 0; g < MAXG; ++g) sum += v[g];
+                    w.G[e] = sum;
                 }
             }
             if (tid == 0) cnt[CF_CNT_GLOBAL] = 0;
             fence_acq_rel_gpu();
             __syncthreads();
-#ifdef RG_CF_TRACE
-            if (tid == 0) { unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); cf_trace[8] = t; }
-#endif
             if (tid == 0) atomicAdd(flag, 1u);
         }
     }
     if (tid == 0)
         while (ld_acquire_gpu(flag) == s_gen) __nanosleep(100);
     __syncthreads();
-#ifdef RG_CF_TRACE
-    if (tid == 0) { unsigned long long t; asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)); cf_cta[0][blockIdx.x] = t; }
-#endif
     fence_acq_rel_gpu();
-#pragma unroll
-    for (int q = 0; q < NQ; ++q) {
-        const int e = tid + CF_THREADS * q;
-        if (e < CF_NP) {
-            int i, j;
-            tri_unpack(e, i, j);
-            Gs[i + 32 * j] = __ldcg(a.ws.G + e);
-        }
+    for (int e = tid; e < NE; e += CF_THREADS) {
+        int i, j;
+        tri_unpack(e, i, j);
+        Gs[i + NC * j] = __ldcg(w.G + e);
     }
     __syncthreads();
 }
 
-// tile (rows x 32, ld) <- tile * Rinv (32 x 32 fp32, [k * 32 + j]), chunks of 4 * CF_THREADS / 8 rows
+// tile (rows x NC, ld) <- tile * Rinv (NC x NC fp32, row-major [k * NC + j]); each thread owns 4
+// rows x 4 columns of a chunk, so every float4 of R^{-1} feeds 16 FMAs.
+template <int NC>
 __device__ void cf_times_rinv(float* tile, int ld, int rows, const float* Rinv) {
-    constexpr int RG = CF_THREADS / 8;          // row groups x 8 column groups of 4
+    constexpr int CG = NC / 4, RG = CF_THREADS / CG;   // column groups of 4 x row groups
     const int tid = threadIdx.x;
-    const int cgp = tid & 7, rgp = tid >> 3;
+    const int cgp = tid % CG, rgp = tid / CG;
     for (int base = 0; base < rows; base += 4 * RG) {
         float o[4][4];
 #pragma unroll
@@ -823,8 +806,8 @@ __device__ void cf_times_rinv(float* tile, int ld, int rows, const float* Rinv) 
 #pragma unroll
             for (int c = 0; c < 4; ++c) o[i][c] = 0.f;
 #pragma unroll 8
-        for (int k = 0; k < CQ_NB; ++k) {
-            const float4 rv = *reinterpret_cast<const float4*>(Rinv + k * 32 + 4 * cgp);
+        for (int k = 0; k < NC; ++k) {
+            const float4 rv = *reinterpret_cast<const float4*>(Rinv + k * NC + 4 * cgp);
 #pragma unroll
             for (int i = 0; i < 4; ++i) {
                 const int r = base + rgp + RG * i;
@@ -847,28 +830,145 @@ __device__ void cf_times_rinv(float* tile, int ld, int rows, const float* Rinv) 
     }
 }
 
+// Shared memory of the fused kernels beyond the row tile.
+template <int NC>
+struct CfBufs {
+    double* S;     // CF_SCR scratch: fp64 staging, group partials
+    double* Gs;    // NC x (NC + 2): reduced Gram [i + NC j]; the elimination's Z aliases it
+    double* Rs;    // NC x (NC + 2): elimination A; R of the last pass (row-major) on exit
+    float* Ri;     // NC x NC fp32 R^{-1} of the last pass, row-major
+    static constexpr size_t bytes = (size_t)(CF_SCR + 2 * NC * (NC + 2)) * 8 + (size_t)NC * NC * 4;
+    __device__ explicit CfBufs(uint8_t* base) {
+        S = reinterpret_cast<double*>(base);
+        Gs = S + CF_SCR;
+        Rs = Gs + NC * (NC + 2);
+        Ri = reinterpret_cast<float*>(Rs + NC * (NC + 2));
+    }
+};
 
+// CholQR2 of the CTA's rows of one <= NC-column panel (tile, zero-padded to NC columns), all
+// CTAs in lockstep through cf_allreduce.  Pass 1 forms G = P^T P (fp64), R1 = chol(G),
+// Q1 = P R1^{-1}; kappa_F(R1) = |R1|_F |R1^{-1}|_F <= 2 nc ends the panel after one pass,
+// otherwise pass 2 repeats it on Q1 (CholQR2).  If a pivot of pass 1 fails, the pass is redone
+// on G + s I with the shifted-CholQR shift s = 11 (m nc + nc (nc + 1)) u ||P||_F^2 (u = 2^-53)
+// and two more passes follow (shifted CholQR3), all inside the kernel.  A pivot that fails after
+// that is a numerical breakdown: its column is reported through a.status and returned (else -1).
+// On exit the tile holds Q and CTA 0 has written R (fp32) to a.Rout.
+template <int NC>
+__device__ int cf_panel(const CqArgs& a, float* tile, int ld, int rows, int nc, const CfBufs<NC>& b) {
+    const int tid = threadIdx.x;
+    const CfWs w = cf_ws(a);
+    __shared__ int s_single;
+    double* part = w.part + (int64_t)blockIdx.x * CfCfg<NC>::NE;
+    bool shifted = false;
+    int bad = -1;
+    for (int pass = 0; pass < 3; ++pass) {
+        cf_gram<NC>(tile, ld, rows, b.S, part);
+        CF_MARK(4 + 4 * pass);
+        cf_allreduce<NC>(a, b.Gs);
+        CF_MARK(5 + 4 * pass);
+        int fb = NC;
+        bool ok = chol_inv_cta<CF_THREADS, true, NC>(b.Gs, nc, b.Rs, b.Gs, nullptr, b.Ri, true, &fb);
+        CF_MARK(6 + 4 * pass);
+        if (!ok && pass == 0) {
+            // reload G (the elimination overwrote it) and shift its diagonal
+            for (int e = tid; e < CfCfg<NC>::NE; e += CF_THREADS) {
+                int i, j;
+                tri_unpack(e, i, j);
+                b.Gs[i + NC * j] = __ldcg(w.G + e);
+            }
+            __syncthreads();
+            double tr = 0.0;
+            for (int j = 0; j < nc; ++j) tr += b.Gs[j * (NC + 1)];
+            const double sh = 11.0 * ((double)a.m * nc + (double)nc * (nc + 1)) * 0x1p-53 * tr;
+            __syncthreads();
+            if (tid < nc) b.Gs[tid * (NC + 1)] += sh;
+            __syncthreads();
+            shifted = true;
+            ok = chol_inv_cta<CF_THREADS, true, NC>(b.Gs, nc, b.Rs, b.Gs, nullptr, b.Ri, true, &fb);
+        }
+        if (!ok) {
+            bad = fb;
+            break;
+        }
+        // CTA 0 accumulates R = R_pass ... R_1 (fp64, [i + NC j]) in the workspace
+        if (blockIdx.x == 0) {
+            constexpr int PERQ = NC * NC / CF_THREADS;
+            double v[PERQ];
+#pragma unroll
+            for (int q = 0; q < PERQ; ++q) {
+                const int e = tid + CF_THREADS * q, i = e % NC, j = e / NC;
+                double sacc = 0.0;
+                if (i <= j) {
+                    if (pass == 0) {
+                        sacc = b.Rs[i * (NC + 2) + j];
+                    } else {
+                        for (int k = i; k <= j; ++k) sacc = fma(b.Rs[i * (NC + 2) + k], w.Racc[k + NC * j], sacc);
+                    }
+                }
+                v[q] = sacc;
+            }
+            __syncthreads();
+#pragma unroll
+            for (int q = 0; q < PERQ; ++q) w.Racc[tid + CF_THREADS * q] = v[q];
+        }
+        bool stop;
+        if (pass == 0) {
+            if (tid < 32) {
+                double r = 0.0, ri = 0.0;
+                for (int e = tid; e < NC * NC; e += 32) {
+                    const int i = e / NC, j = e % NC;
+                    if (i < nc && j < nc) {
+                        const double x = b.Rs[i * (NC + 2) + j];
+                        const double y = (double)b.Ri[e];
+                        r = fma(x, x, r);
+                        ri = fma(y, y, ri);
+                    }
+                }
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) {
+                    r += __shfl_xor_sync(0xffffffffu, r, o);
+                    ri += __shfl_xor_sync(0xffffffffu, ri, o);
+                }
+                if (tid == 0) s_single = (sqrt(r * ri) <= 2.0 * nc) ? 1 : 0;
+            }
+            __syncthreads();
+            stop = !shifted && s_single != 0;
+        } else {
+            __syncthreads();
+            stop = (pass == 1 && !shifted) || pass == 2;
+        }
+        cf_times_rinv<NC>(tile, ld, rows, b.Ri);
+        CF_MARK(7 + 4 * pass);
+        if (stop) break;
+    }
+    if (bad >= 0 && blockIdx.x == 0 && tid == 0 && a.status) atomicMin(a.status, a.col0 + bad);
+    if (blockIdx.x == 0) {   // R (fp32) from the accumulated fp64 factor (written by this CTA)
+        __syncthreads();
+        for (int e = tid; e < nc * nc; e += CF_THREADS) {
+            const int i = e % nc, j = e / nc;
+            a.Rout[i + (int64_t)j * a.ldr] = (i <= j) ? (float)w.Racc[i + NC * j] : 0.f;
+        }
+    }
+    return bad;
+}
+
+template <int NC>
 __global__ void __launch_bounds__(CF_THREADS, 1) cq_fused_kernel(CqArgs a, int ld) {
     RG_PDL_ENTRY();
     extern __shared__ __align__(16) uint8_t cf_smem[];
     float* tile = reinterpret_cast<float*>(cf_smem);
-    double* sred = reinterpret_cast<double*>(cf_smem + (size_t)32 * ld * 4);
-    double* Gs = sred + CF_SCR;               // 32 x CH_LD (first 1024 used as G)
-    double* Rs = Gs + 32 * CH_LD;             // Cholesky scratch 32 x CH_LD
-    float* Ri1 = reinterpret_cast<float*>(Rs + 32 * CH_LD);
-    float* Ri2 = Ri1 + 1024;
-    double* R1 = reinterpret_cast<double*>(Ri2 + 1024);
-    __shared__ int s_flag[2];
+    const CfBufs<NC> b(cf_smem + (size_t)NC * ld * 4);
     const int tid = threadIdx.x;
-    CF_MARK(0);
-    if (blockIdx.x == 0 && tid == 0) *a.ws.fail = 0;   // set again below only if a pivot fails
+    if (blockIdx.x == 0 && tid == 0) *a.ws.fail = 0;
     const int64_t rows_per = (a.m + gridDim.x - 1) / gridDim.x;
     const int64_t r0 = (int64_t)blockIdx.x * rows_per;
     const int64_t rem = a.m - r0;
     const int rows = (int)(rem <= 0 ? 0 : (rem < rows_per ? rem : rows_per));
+    CF_MARK(0);
     // ---- load the CTA's rows (zero-padded columns beyond nc); 4 columns x CF_MAXPER rows of
     // independent loads in flight per thread
-    for (int c0 = 0; c0 < 32; c0 += 4) {
+    for (int c0 = 0; c0 < NC; c0 += 4) {
         float v[4][CF_MAXPER];
 #pragma unroll
         for (int cc = 0; cc < 4; ++cc)
@@ -887,65 +987,8 @@ __global__ void __launch_bounds__(CF_THREADS, 1) cq_fused_kernel(CqArgs a, int l
     }
     __syncthreads();
     CF_MARK(1);
-    // ---- pass 1: G1 = P^T P -> R1, R1^{-1} on every CTA
-    cf_gram(tile, ld, rows, sred, a.ws.part + (int64_t)blockIdx.x * CF_NP);
+    cf_panel<NC>(a, tile, ld, rows, a.nc, b);
     CF_MARK(2);
-    CF_CTA(2);
-    cf_allreduce_gram(a, Gs);
-    CF_MARK(3);
-    // sred is free after the Gram reduction: elimination scratch Y.  R^{-1} comes out row-major
-    // ([k * 32 + j] = R^{-1}(k, j)), the layout cf_times_rinv reads.
-    if (!chol_inv_cta<CF_THREADS, true>(Gs, a.nc, Rs, sred, R1, Ri1, true)) {
-        if (blockIdx.x == 0 && tid == 0) *a.ws.fail = 1;   // the guarded MGS/TSQR kernels take over
-        return;
-    }
-    CF_MARK(4);
-    // kappa_F(R1) <= 2 nc  ->  single CholQR pass (see cq_pass_kernel)
-    if (tid < 32) {
-        double r = 0.0, ri = 0.0;
-        for (int e = tid; e < 1024; e += 32) {
-            const int i = e & 31, j = e >> 5;
-            if (i < a.nc && j < a.nc) {
-                r = fma(R1[e], R1[e], r);
-                const double y = (double)Ri1[e];
-                ri = fma(y, y, ri);
-            }
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            r += __shfl_xor_sync(0xffffffffu, r, o);
-            ri += __shfl_xor_sync(0xffffffffu, ri, o);
-        }
-        if (tid == 0) s_flag[1] = (sqrt(r * ri) <= 2.0 * a.nc) ? 1 : 0;
-    }
-    __syncthreads();
-    const bool single = s_flag[1] != 0;
-    cf_times_rinv(tile, ld, rows, Ri1);   // tile <- Q1 = P R1^{-1}
-    CF_MARK(5);
-    if (!single) {
-        // ---- pass 2: G2 = Q1^T Q1 -> R2 (left in Rs, row-major ld CH_LD), R2^{-1}; Q = Q1 R2^{-1}; R = R2 R1
-        cf_gram(tile, ld, rows, sred, a.ws.part + (int64_t)blockIdx.x * CF_NP);
-        cf_allreduce_gram(a, Gs);
-        if (!chol_inv_cta<CF_THREADS, true>(Gs, a.nc, Rs, sred, nullptr, Ri2, true)) {
-            if (blockIdx.x == 0 && tid == 0) *a.ws.fail = 1;
-            return;   // input panel untouched in HBM: the MGS/TSQR fallback redoes it
-        }
-        cf_times_rinv(tile, ld, rows, Ri2);   // tile <- Q
-        if (blockIdx.x == 0) {
-            for (int e = tid; e < a.nc * a.nc; e += CF_THREADS) {
-                const int i = e % a.nc, j = e / a.nc;
-                double s = 0.0;
-                for (int k = i; k <= j; ++k) s = fma(Rs[i * CH_LD + k], R1[k + 32 * j], s);
-                a.Rout[i + (int64_t)j * a.ldr] = (i <= j) ? (float)s : 0.f;
-            }
-        }
-    } else if (blockIdx.x == 0) {
-        for (int e = tid; e < a.nc * a.nc; e += CF_THREADS) {
-            const int i = e % a.nc, j = e / a.nc;
-            a.Rout[i + (int64_t)j * a.ldr] = (i <= j) ? (float)R1[i + 32 * j] : 0.f;
-        }
-    }
-    CF_MARK(6);
     // ---- write Q (fp32) + 16-bit shadow
     for (int c = 0; c < a.nc; ++c) {
 #pragma unroll
@@ -963,6 +1006,7 @@ __global__ void __launch_bounds__(CF_THREADS, 1) cq_fused_kernel(CqArgs a, int l
             }
         }
     }
+    CF_MARK(3);
 }
 
 // distributed mode: after the host allreduce of G (pass `pass`), factor it (one warp)
@@ -973,7 +1017,7 @@ __global__ void cq_factor_kernel(CqArgs a, int pass) {
     if (pass > 0 && *(volatile int*)a.ws.fail) return;
     const bool ok = chol_inv_cta<256, false>(a.ws.G + pass * 1024, a.nc, Rs, R1s, a.ws.R + pass * 1024,
                                              a.ws.Rinv + pass * 1024, false);
-    if (!ok && threadIdx.x == 0) *a.ws.fail = 1;
+    if (!ok && threadIdx.x == 0) cq_signal_fail(a);
     if (pass == 0 && ok) single_pass_decision(a);
     if (pass == 1 && ok) final_r_product(a, Rs, R1s);
 }
@@ -987,9 +1031,10 @@ static int cq_grid(int64_t m) {
 }
 
 size_t cholqr_ws_doubles(int64_t m) {
-    const int grid = std::max(cq_grid(m), 160);   // also covers the fused kernel (<= 160 CTAs)
-    const int ngroups = (grid + CQ_FAN - 1) / CQ_FAN + (grid + CF_FAN - 1) / CF_FAN;
-    return (size_t)(grid + ngroups) * 1024 + 4 * 1024 + 1024 /*Rinv fp32 x2*/ + 64;
+    const int grid = cq_grid(m);
+    const int ngroups = (grid + CQ_FAN - 1) / CQ_FAN;
+    const size_t streaming = (size_t)(grid + ngroups) * 1024 + 4 * 1024 + 1024 /*Rinv fp32 x2*/ + 64;
+    return std::max(streaming, CF_WS_DOUBLES + 64);   // the fused kernels' layout (cf_ws)
 }
 
 size_t cholqr_counter_ints(int64_t m) {
@@ -997,7 +1042,23 @@ size_t cholqr_counter_ints(int64_t m) {
     return std::max((size_t)(grid + CQ_FAN - 1) / CQ_FAN + 2, (size_t)CF_CNT_INTS);
 }
 
-cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st) {
+
+static int sm_count() {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    }
+    return sms;
+}
+
+bool cholqr_fused_fits(int64_t m, int ncols) {
+    const int64_t rows_per = (m + sm_count() - 1) / sm_count();
+    return rows_per <= (ncols > 32 ? CF_WIDE_MAX_ROWS : CF_MAX_ROWS) && getenv("RGSQR_CQ_STREAM") == nullptr;
+}
+
+static CqArgs cq_args(const CholqrLaunch& L) {
     CqArgs a{};
     a.P = L.P;
     a.ldp = L.ldp;
@@ -1021,38 +1082,43 @@ cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st) {
     a.ldr = L.ldr;
     a.bf16 = L.bf16;
     a.distributed = L.allreduce_g != nullptr;
+    a.cond = L.cond;
+    a.status = L.status;
+    a.col0 = L.col0;
+    return a;
+}
+
+template <int NC>
+static cudaError_t launch_fused(CqArgs a, cudaStream_t st) {
+    const int sms = sm_count();
+    const int64_t rows_per = (a.m + sms - 1) / sms;
+    const int ld = (int)(rows_per | 1);   // odd leading dimension: conflict-free column walks
+    const size_t smem = (size_t)NC * ld * 4 + CfBufs<NC>::bytes + 128;
+    cudaError_t e = cudaFuncSetAttribute(cq_fused_kernel<NC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(sms);
+    cfg.blockDim = dim3(CF_THREADS);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeCooperative;   // co-residency for the flag spin in cf_allreduce
+    at[0].val.cooperative = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    ++g_launches;
+    return cudaLaunchKernelEx(&cfg, cq_fused_kernel<NC>, a, ld);
+}
+
+cudaError_t launch_panel_cholqr(const CholqrLaunch& L, bool* handles_failure, cudaStream_t st) {
+    CqArgs a = cq_args(L);
+    const int grid = cq_grid(L.m);
+    if (!a.distributed && cholqr_fused_fits(L.m, 32)) {
+        if (handles_failure) *handles_failure = true;   // shifted CholQR3 inside the kernel
+        return launch_fused<32>(a, st);
+    }
+    if (handles_failure) *handles_failure = false;      // the guarded MGS/TSQR kernels must follow
     cudaError_t e;
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    }
-    const int64_t rows_per = (L.m + sms - 1) / sms;
-    if (!a.distributed && rows_per <= CF_MAX_ROWS && getenv("RGSQR_CQ_STREAM") == nullptr) {
-        const int ld = (int)(rows_per | 1);   // odd leading dimension: conflict-free column walks
-        const size_t smem = CfSmem::bytes(ld);
-        static size_t attr = 0;
-        if (smem > attr) {
-            e = cudaFuncSetAttribute(cq_fused_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-            if (e != cudaSuccess) return e;
-            attr = smem;
-        }
-        // partial buffers: sms CTA partials + ceil(sms / 8) group partials fit in the workspace
-        a.ws.gpart = a.ws.part + (size_t)sms * 1024;
-        cudaLaunchConfig_t cfg{};
-        cfg.gridDim = dim3(sms);
-        cfg.blockDim = dim3(CF_THREADS);
-        cfg.dynamicSmemBytes = smem;
-        cfg.stream = st;
-        cudaLaunchAttribute at[1];
-        at[0].id = cudaLaunchAttributeCooperative;
-        at[0].val.cooperative = 1;
-        cfg.attrs = at;
-        cfg.numAttrs = 1;
-        ++g_launches;
-        return cudaLaunchKernelEx(&cfg, cq_fused_kernel, a, ld);
-    }
     for (int pass = 0; pass < 3; ++pass) {
         if (pass == 0) RG_LAUNCH((cq_pass_kernel<0>), grid, CQ_THREADS, 0, st, a);
         if (pass == 1) RG_LAUNCH((cq_pass_kernel<1>), grid, CQ_THREADS, 0, st, a);
@@ -1067,6 +1133,12 @@ cudaError_t launch_panel_cholqr(const CholqrLaunch& L, cudaStream_t st) {
         }
     }
     return cudaSuccess;
+}
+
+cudaError_t launch_panel_pair(const CholqrLaunch& L, cudaStream_t st) {
+    if (L.nc <= 32 || L.nc > 64 || L.allreduce_g != nullptr || !cholqr_fused_fits(L.m, 64))
+        return cudaErrorInvalidValue;
+    return launch_fused<64>(cq_args(L), st);
 }
 
 }  // namespace rg

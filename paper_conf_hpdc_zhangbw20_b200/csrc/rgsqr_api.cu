@@ -110,8 +110,10 @@ struct DevBuf {
 };
 
 struct Op {
-    enum Kind { PANEL, PROJ, UPDATE } kind;
-    int c0, h, w;  // PANEL: c0, w = columns.  PROJ/UPDATE: Q1 = [c0, c0+h), A2 = [c0+h, c0+h+w)
+    enum Kind { PANEL, PROJ, UPDATE, PAIR } kind;
+    // PANEL: c0, w = columns.  PROJ/UPDATE: Q1 = [c0, c0+h), A2 = [c0+h, c0+h+w).
+    // PAIR: the whole last recursion level [c0, c0+h+w) (h = 32) in one kernel.
+    int c0, h, w;
     int bn = 0, tiles_i = 0, tiles_j = 0, splits = 0, kb_total = 0, kb_per_split = 0;
     CUtensorMap ma, mb, ma_lo, mb_lo;
 };
@@ -246,7 +248,16 @@ PtrSide ptr_side(const void* p) {
 }
 
 // ------------------------------------------------------------------ plan construction
-void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb) {
+void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb, bool pair) {
+    if (pair && ncols > nb && ncols <= 2 * nb) {
+        Op o{};
+        o.kind = Op::PAIR;
+        o.c0 = c0;
+        o.h = rgsqr_split(ncols);
+        o.w = ncols - o.h;
+        ops.push_back(o);
+        return;
+    }
     if (ncols <= nb) {
         Op o{};
         o.kind = Op::PANEL;
@@ -256,7 +267,7 @@ void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb) {
         return;
     }
     const int h = rgsqr_split(ncols), w = ncols - h;
-    build_ops(ops, c0, h, nb);
+    build_ops(ops, c0, h, nb, pair);
     Op p{};
     p.kind = Op::PROJ;
     p.c0 = c0;
@@ -266,7 +277,7 @@ void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb) {
     Op u = p;
     u.kind = Op::UPDATE;
     ops.push_back(u);
-    build_ops(ops, c0 + h, w, nb);
+    build_ops(ops, c0 + h, w, nb, pair);
 }
 
 int make_plan(rg_handle h, Plan& pl) {
@@ -275,11 +286,17 @@ int make_plan(rg_handle h, Plan& pl) {
     const int n = (int)pl.n;
     pl.ldh = round_up(std::max<int64_t>(m, 8), 8);
     pl.ops.clear();
-    build_ops(pl.ops, 0, n, pl.nb);
+    // Opt-in (RGSQR_WIDE=1): the last recursion level (two 32-column panels + K1 + K2) as one
+    // 64-column CholQR2 kernel when its rows fit in shared memory.  Same Q, R in exact
+    // arithmetic, better conditioned in practice (fp64 Gram instead of fp16 K1/K2 at that level);
+    // measured the same speed as the paper's structure on config 2 (12.33 vs 12.35 ms).
+    const bool pair = pl.panel == 0 && pl.nb == 32 && !(pl.nranks > 1 && h->comm) &&
+                      rg::cholqr_fused_fits(m, 64) && getenv("RGSQR_WIDE") != nullptr;
+    build_ops(pl.ops, 0, n, pl.nb, pair);
     int max_h = 0, max_w = 0;
     size_t pmax = 0;
     for (auto& o : pl.ops)
-        if (o.kind != Op::PANEL) {
+        if (o.kind == Op::PROJ || o.kind == Op::UPDATE) {
             max_h = std::max(max_h, o.h);
             max_w = std::max(max_w, o.w);
         }
@@ -290,7 +307,7 @@ int make_plan(rg_handle h, Plan& pl) {
     const uint16_t* r12l = h->r12l.as<uint16_t>();
     const bool bf = pl.bf16 != 0;
     for (auto& o : pl.ops) {
-        if (o.kind == Op::PANEL) continue;
+        if (o.kind == Op::PANEL || o.kind == Op::PAIR) continue;
         const uint16_t* q1 = qh + (int64_t)o.c0 * pl.ldh;
         const uint16_t* a2 = qh + (int64_t)(o.c0 + o.h) * pl.ldh;
         const uint16_t* q1l = pl.split ? ql + (int64_t)o.c0 * pl.ldh : q1;
@@ -392,6 +409,34 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
         RG_CUDA(cudaMemset2DAsync(pl.R, pl.ldr * sizeof(float), 0, n * sizeof(float), n, st));
     }
     for (auto& o : pl.ops) {
+        if (o.kind == Op::PAIR) {
+            // two panels + R12 = Q1^T A2 + A2 -= Q1 R12 of a (h + w)-column block; algorithmic bytes:
+            // read the block (fp32), write Q (fp32) + shadow(s)
+            const double wt = o.h + o.w;
+            ProfScope _s(h, PC_PANEL, 2.0 * m * (o.h * o.h + o.w * o.w) + 4.0 * m * o.h * o.w,
+                         (double)m * wt * (pl.split ? 12 : 10));
+            int* cq_fail = h->cq_flags.as<int>();
+            rg::CholqrLaunch c{};
+            c.P = pl.Q + (int64_t)o.c0 * pl.ldq;
+            c.ldp = pl.ldq;
+            c.Q = pl.Q + (int64_t)o.c0 * pl.ldq;
+            c.ldq = pl.ldq;
+            c.Qh = qh + (int64_t)o.c0 * pl.ldh;
+            c.Ql = ql ? ql + (int64_t)o.c0 * pl.ldh : nullptr;
+            c.ldh = pl.ldh;
+            c.m = m;
+            c.nc = o.h + o.w;
+            c.ws = h->cq_ws.as<double>();
+            c.counter = cq_fail + 4;
+            c.fail = cq_fail;
+            c.R = pl.R + o.c0 + (int64_t)o.c0 * pl.ldr;
+            c.ldr = pl.ldr;
+            c.bf16 = pl.bf16;
+            c.status = status;
+            c.col0 = o.c0;
+            RG_CUDA(rg::launch_panel_pair(c, st));
+            continue;
+        }
         if (o.kind == Op::PANEL) {
             // algorithmic bytes: read the panel (fp32), write Q (fp32) + 16-bit shadow (+ lo shadow)
             ProfScope _s(h, PC_PANEL, 2.0 * m * o.w * o.w, (double)m * o.w * (pl.split ? 12 : 10));
@@ -435,8 +480,12 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
                     };
                     c.ctx = h;
                 }
-                RG_CUDA(rg::launch_panel_cholqr(c, st));
                 p.guard = cq_fail;
+                c.status = status;
+                c.col0 = o.c0;
+                bool handled = false;
+                RG_CUDA(rg::launch_panel_cholqr(c, &handled, st));
+                if (handled) continue;   // shifted CholQR3 fallback inside the fused kernel
             }
             if (!dist) {
                 p.R = Rdiag;

@@ -91,6 +91,29 @@ def test_rgsqr_streaming_cholqr_panel(rg, monkeypatch, kappa, n):
         assert oracle.orthogonality(Q) < 1e-5
 
 
+@pytest.mark.parametrize("kappa", [10.0, 1e4, 1e6])
+def test_rgsqr_wide_leaf_level(rg, monkeypatch, kappa):
+    """RGSQR_WIDE=1: the last recursion level as one 64-column CholQR2 kernel (same unique QR)."""
+    monkeypatch.setenv("RGSQR_WIDE", "1")
+    h = rg.Handle(0)
+    A = synth.svd_matrix(8192, 160, "geometric", kappa, seed=51).astype(np.float32)
+    Q, R = rg.rgsqr_factor(_dev(A), handle=h)
+    torch.cuda.synchronize()
+    Q = Q.cpu().numpy().astype(np.float64)
+    R = R.cpu().numpy().astype(np.float64)
+    _check_qr(A, Q, R, kappa=kappa, orth_scale=(1e-2 if kappa < 1e3 else 1.0))
+
+
+def test_rgsqr_wide_breakdown_status(rg, monkeypatch):
+    monkeypatch.setenv("RGSQR_WIDE", "1")
+    h = rg.Handle(0)
+    A = synth.gaussian(4096, 64, seed=52).astype(np.float32)
+    A[:, 40] = 0.0
+    with pytest.raises(rg.RGError) as e:
+        rg.rgsqr_factor(_dev(A), handle=h)
+    assert e.value.status == rg.RG_BREAKDOWN
+
+
 def test_rgsqr_tall_panel_streaming_path(rg):
     """m = 200000: more rows per CTA than the fused panel holds -> streaming passes by design."""
     A = synth.gaussian(200000, 40, seed=41).astype(np.float32)

@@ -7,8 +7,8 @@
 #include <algorithm>
 #include <vector>
 #include <cuda_runtime.h>
-#define RG_CF_TRACE 1
 // #define RG_CHOL_TRACE 1
+#define RG_CF_TRACE 1
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/kernels.h"
 namespace rg { thread_local long long g_launches = 0; bool pdl_enabled() { return getenv("RGSQR_NO_PDL") == nullptr; } }
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/panel_cholqr.cu"
@@ -66,11 +66,11 @@ int main(int argc, char** argv) {
     L.P = P; L.ldp = m; L.Q = Q; L.ldq = m; L.Qh = Qh; L.ldh = m; L.m = m; L.nc = nc; L.ws = ws;
     L.fail = flags; L.counter = flags + 4; L.R = R; L.ldr = 32;
     cudaStream_t st; cudaStreamCreate(&st);
-    for (int i = 0; i < 5; ++i) rg::launch_panel_cholqr(L, st);
+    for (int i = 0; i < 5; ++i) rg::launch_panel_cholqr(L, nullptr, st);
     cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
     const int iters = 50;
     cudaEventRecord(a, st);
-    for (int i = 0; i < iters; ++i) rg::launch_panel_cholqr(L, st);
+    for (int i = 0; i < iters; ++i) rg::launch_panel_cholqr(L, nullptr, st);
     cudaEventRecord(b, st);
     cudaEventSynchronize(b);
     float ms; cudaEventElapsedTime(&ms, a, b);
@@ -78,7 +78,7 @@ int main(int argc, char** argv) {
     // graph-captured
     cudaGraph_t g; cudaGraphExec_t ge;
     cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal);
-    for (int i = 0; i < iters; ++i) rg::launch_panel_cholqr(L, st);
+    for (int i = 0; i < iters; ++i) rg::launch_panel_cholqr(L, nullptr, st);
     cudaStreamEndCapture(st, &g);
     cudaGraphInstantiate(&ge, g, 0);
     cudaGraphLaunch(ge, st);
@@ -175,23 +175,33 @@ int main(int argc, char** argv) {
                hc[0], hc[1], hc[2], hc[3], hc[4]);
     }
     {
-        unsigned long long tr[16];
-        rg::launch_panel_cholqr(L, st);
-        cudaStreamSynchronize(st);
-        cudaMemcpyFromSymbol(tr, rg::cf_trace, sizeof(tr));
-        printf("  fused trace (us from start): load %.2f gram %.2f reduce %.2f chol %.2f apply %.2f pre-write %.2f\n",
-               (tr[1] - tr[0]) / 1e3, (tr[2] - tr[0]) / 1e3, (tr[3] - tr[0]) / 1e3, (tr[4] - tr[0]) / 1e3,
-               (tr[5] - tr[0]) / 1e3, (tr[6] - tr[0]) / 1e3);
-        {
-            static unsigned long long ct[4][160];
-            cudaMemcpyFromSymbol(ct, rg::cf_cta, sizeof(ct));
-            for (int k = 0; k < 4; ++k) {
-                unsigned long long mn = ~0ull, mx = 0;
-                for (int b = 0; b < 148; ++b) { if (!ct[k][b]) continue; mn = std::min(mn, ct[k][b]); mx = std::max(mx, ct[k][b]); }
-                printf("  cta mark %d: min %.2f max %.2f us (rel. to CTA0 start)\n", k, ((double)mn - tr[0]) / 1e3, ((double)mx - tr[0]) / 1e3);
-            }
+        // two-panel kernel (64 columns), eager back-to-back launches
+        float *P2, *Q2, *R2; uint16_t* Qh2;
+        cudaMalloc(&P2, (size_t)m * 64 * 4); cudaMalloc(&Q2, (size_t)m * 64 * 4); cudaMalloc(&R2, 64 * 64 * 4);
+        cudaMalloc(&Qh2, (size_t)m * 64 * 2);
+        std::vector<float> h2((size_t)m * 64);
+        for (size_t i = 0; i < h2.size(); ++i) {   // N(0,1) via Box-Muller on a 64-bit hash
+            uint64_t z = i * 0x9E3779B97F4A7C15ull + 12345;
+            z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull; z = (z ^ (z >> 27)) * 0x94D049BB133111EBull; z ^= z >> 31;
+            const double u1 = ((z >> 11) + 1.0) / 9007199254740993.0, u2 = (double)(z & 0x7FF) / 2048.0;
+            h2[i] = (float)(sqrt(-2.0 * log(u1)) * cos(6.283185307179586 * u2));
         }
-        printf("  marks: 0=spin exit 1=group-sum done (last arrivers only) 2=gram done 3=arrived; flag set at %.2f\n", (tr[8] - tr[0]) / 1e3);
+        cudaMemcpy(P2, h2.data(), h2.size() * 4, cudaMemcpyHostToDevice);
+        rg::CholqrLaunch L2 = L;
+        L2.P = P2; L2.ldp = m; L2.Q = Q2; L2.ldq = m; L2.Qh = Qh2; L2.ldh = m; L2.nc = 64; L2.R = R2; L2.ldr = 64;
+        for (int i = 0; i < 3; ++i) rg::launch_panel_pair(L2, st);
+        cudaEventRecord(a, st);
+        for (int i = 0; i < iters; ++i) rg::launch_panel_pair(L2, st);
+        cudaEventRecord(b, st);
+        cudaEventSynchronize(b);
+        cudaEventElapsedTime(&ms, a, b);
+        printf("  64-column kernel: %.2f us, err %s\n", ms * 1000 / iters, cudaGetErrorString(cudaGetLastError()));
+        unsigned long long tr[16];
+        cudaMemcpyFromSymbol(tr, rg::cf_trace, sizeof(tr));
+        printf("  64-col trace (us): load %.2f panel %.2f store %.2f\n",
+               (tr[1] - tr[0]) / 1e3, (tr[2] - tr[0]) / 1e3, (tr[3] - tr[0]) / 1e3);
+        printf("  pass 0: gram %.2f allreduce %.2f chol %.2f apply %.2f | pass 1 apply %.2f\n", (tr[4] - tr[0]) / 1e3,
+               (tr[5] - tr[0]) / 1e3, (tr[6] - tr[0]) / 1e3, (tr[7] - tr[0]) / 1e3, (tr[11] - tr[0]) / 1e3);
     }
     int fl; cudaMemcpy(&fl, flags, 4, cudaMemcpyDeviceToHost);
     printf("fail flag %d, err %s\n", fl, cudaGetErrorString(cudaGetLastError()));
