@@ -249,6 +249,33 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
         const int q = lane & 7;       // row quad within the warp's 32 rows
         const int jsub = lane >> 3;   // column within a group of 4
         int cnt = 0;
+        constexpr int kChunks = BN / 32;
+        const bool rmw = (MODE == 1) && !args.overwrite;
+        // K2: the fp32 C values of a chunk are loaded one chunk ahead (the next tile's first
+        // chunk during the current tile's last), so each epilogue warp keeps two chunks of
+        // HBM reads in flight instead of paying a full memory latency per chunk.
+        auto load_old = [&](int t0x, int t1x, int chx, float4 (&o)[8]) {
+            const int64_t r0x = (int64_t)t0x + ew * 32 + 4 * q;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                const int j = t1x + chx * 32 + k * 4 + jsub;
+                const float* cp = args.C + r0x + (int64_t)j * args.ldc;
+                if (j < args.w && r0x + 3 < args.m && args.vec_ok) {
+                    o[k] = __ldcs(reinterpret_cast<const float4*>(cp));
+                } else {
+                    o[k].x = (j < args.w && r0x + 0 < args.m) ? cp[0] : 0.f;
+                    o[k].y = (j < args.w && r0x + 1 < args.m) ? cp[1] : 0.f;
+                    o[k].z = (j < args.w && r0x + 2 < args.m) ? cp[2] : 0.f;
+                    o[k].w = (j < args.w && r0x + 3 < args.m) ? cp[3] : 0.f;
+                }
+            }
+        };
+        float4 old[8], nxt[8];
+        if (rmw && blockIdx.x < args.units && wg < kChunks) {
+            int t0, tj, z, kb0, kb1;
+            unit_coords<MODE>(args, blockIdx.x, t0, tj, z, kb0, kb1);
+            load_old(t0, tj * BN, wg, old);
+        }
         for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
             int t0, tj, z, kb0, kb1;
             unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
@@ -256,25 +283,16 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
             const int acc = cnt % C::kAcc;
             const uint32_t aphase = (uint32_t)(cnt / C::kAcc) & 1u;
             const int64_t row0 = (int64_t)t0 + ew * 32 + 4 * q;   // first of this lane's 4 rows
-            constexpr int kChunks = BN / 32;
             bool waited = false;
             for (int ch = wg; ch < kChunks; ch += EPI_WG) {
                 const int c = ch * 32;
-                // ---- K2: prefetch the fp32 C values of this chunk before touching TMEM
-                float4 old[8];
-                if (MODE == 1 && !args.overwrite) {
-#pragma unroll
-                    for (int k = 0; k < 8; ++k) {
-                        const int j = t1 + c + k * 4 + jsub;
-                        const float* cp = args.C + row0 + (int64_t)j * args.ldc;
-                        if (j < args.w && row0 + 3 < args.m && args.vec_ok) {
-                            old[k] = __ldcs(reinterpret_cast<const float4*>(cp));
-                        } else {
-                            old[k].x = (j < args.w && row0 + 0 < args.m) ? cp[0] : 0.f;
-                            old[k].y = (j < args.w && row0 + 1 < args.m) ? cp[1] : 0.f;
-                            old[k].z = (j < args.w && row0 + 2 < args.m) ? cp[2] : 0.f;
-                            old[k].w = (j < args.w && row0 + 3 < args.m) ? cp[3] : 0.f;
-                        }
+                if (rmw) {
+                    if (ch + EPI_WG < kChunks) {
+                        load_old(t0, t1, ch + EPI_WG, nxt);
+                    } else if (u + (int)gridDim.x < args.units) {
+                        int t0n, tjn, zn, kb0n, kb1n;
+                        unit_coords<MODE>(args, u + gridDim.x, t0n, tjn, zn, kb0n, kb1n);
+                        load_old(t0n, tjn * BN, wg, nxt);
                     }
                 }
                 if (!waited) {
@@ -354,6 +372,10 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
                     }
                 }
                 __syncwarp();
+                if (rmw) {
+#pragma unroll
+                    for (int k = 0; k < 8; ++k) old[k] = nxt[k];
+                }
             }
             if (!waited) {   // this warp had no chunk (EPI_WG > chunks): still consume the phase
                 mbar_wait(&tfull_bar[acc], aphase);
@@ -416,6 +438,70 @@ __global__ void __launch_bounds__(32 * LANES) proj_reduce_kernel(const float* __
     }
 }
 
+// Same reduction for large outputs: persistent grid-stride blocks, each unit = 128 consecutive
+// rows i (4 per lane, float4 loads; the partial buffers are padded to whole 128-row tiles) of
+// one column j, LANES split lanes.  The one-output-per-thread kernel above spends most of its
+// time scheduling ~10^5 tiny blocks at the top recursion levels.
+template <int LANES>
+__global__ void __launch_bounds__(32 * LANES) proj_reduce4_kernel(const float* __restrict__ P, int64_t ldp,
+                                                                 int64_t p_stride, int splits, int h, int w,
+                                                                 float* __restrict__ R, int64_t ldr,
+                                                                 float* __restrict__ Rf, int64_t ldf,
+                                                                 uint16_t* __restrict__ Rh, uint16_t* __restrict__ Rl,
+                                                                 int64_t ldh, int bf16) {
+    RG_PDL_ENTRY();
+    __shared__ float4 part[LANES][33];
+    const int nic = (h + 127) / 128;
+    const int units = nic * w;
+    const int tx = threadIdx.x, ty = threadIdx.y;
+    for (int u = blockIdx.x; u < units; u += gridDim.x) {
+        const int ic = u % nic, j = u / nic;
+        const int i0 = ic * 128 + 4 * tx;
+        const float* p = P + (int64_t)j * ldp + i0;
+        float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+        int z = ty;
+        for (; z + 3 * LANES < splits; z += 4 * LANES) {
+            const float4 a = __ldcg(reinterpret_cast<const float4*>(p + (int64_t)z * p_stride));
+            const float4 b = __ldcg(reinterpret_cast<const float4*>(p + (int64_t)(z + LANES) * p_stride));
+            const float4 c = __ldcg(reinterpret_cast<const float4*>(p + (int64_t)(z + 2 * LANES) * p_stride));
+            const float4 d = __ldcg(reinterpret_cast<const float4*>(p + (int64_t)(z + 3 * LANES) * p_stride));
+            s.x += a.x; s.y += a.y; s.z += a.z; s.w += a.w;
+            s.x += b.x; s.y += b.y; s.z += b.z; s.w += b.w;
+            s.x += c.x; s.y += c.y; s.z += c.z; s.w += c.w;
+            s.x += d.x; s.y += d.y; s.z += d.z; s.w += d.w;
+        }
+        for (; z < splits; z += LANES) {
+            const float4 a = __ldcg(reinterpret_cast<const float4*>(p + (int64_t)z * p_stride));
+            s.x += a.x; s.y += a.y; s.z += a.z; s.w += a.w;
+        }
+        part[ty][tx] = s;
+        __syncthreads();
+        if (ty == 0) {
+            float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+            for (int y = 0; y < LANES; ++y) {
+                const float4 v = part[y][tx];
+                t.x += v.x; t.y += v.y; t.z += v.z; t.w += v.w;
+            }
+            const float tv[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                const int i = i0 + e;
+                if (i < h) {
+                    if (R) R[i + (int64_t)j * ldr] = tv[e];
+                    if (Rf) Rf[i + (int64_t)j * ldf] = tv[e];
+                    if (Rh) {
+                        const uint16_t hb = f2h_bits(tv[e], bf16);
+                        Rh[i + (int64_t)j * ldh] = hb;
+                        if (Rl) Rl[i + (int64_t)j * ldh] = f2h_bits((tv[e] - h2f_bits(hb, bf16)) * 2048.0f, bf16);
+                    }
+                }
+            }
+        }
+        __syncthreads();
+    }
+}
+
 // After a cross-rank allreduce of Rf: write R and the 16-bit images.
 __global__ void proj_finish_kernel(const float* __restrict__ Rf, int64_t ldf, int h, int w, float* __restrict__ R,
                                    int64_t ldr, uint16_t* __restrict__ Rh, uint16_t* __restrict__ Rl, int64_t ldh,
@@ -473,7 +559,12 @@ static cudaError_t dispatch_bn(int bn, int units, const CUtensorMap& a, const CU
         case 32: return launch_gemm<MODE, 32, 3, SPLIT, 2>(units, a, b, al, bl, args, st);
         case 64: return launch_gemm<MODE, 64, SPLIT ? 3 : 4, SPLIT, 2>(units, a, b, al, bl, args, st);
         case 128: return launch_gemm<MODE, 128, SPLIT ? 2 : 5, SPLIT, 2>(units, a, b, al, bl, args, st);
-        case 256: return launch_gemm<MODE, 256, SPLIT ? 2 : 4, SPLIT, 1>(units, a, b, al, bl, args, st);
+        case 256:
+            // K2 at wide levels is bound by the fp32 read-modify-write of A2: 8 epilogue warps
+            // (3 stages to fit) double the HBM traffic in flight; K1 keeps 4 stages
+            if constexpr (MODE == 1 && !SPLIT) return launch_gemm<MODE, 256, 3, SPLIT, 2>(units, a, b, al, bl, args, st);
+            else
+            return launch_gemm<MODE, 256, SPLIT ? 2 : 4, SPLIT, 1>(units, a, b, al, bl, args, st);
         default: return cudaErrorInvalidValue;
     }
 }
@@ -525,7 +616,12 @@ cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, in
                                int64_t ldr, float* Rf, int64_t ldf, uint16_t* Rh, uint16_t* Rl, int64_t ldh, int bf16,
                                cudaStream_t st) {
     const int64_t total = (int64_t)h * w;
-    if (splits > 32)
+    if (total >= 65536 && (ldp & 3) == 0 && (p_stride & 3) == 0 && (reinterpret_cast<uintptr_t>(P) & 15) == 0) {
+        const int64_t units = (int64_t)((h + 127) / 128) * w;
+        const int grid = (int)std::min<int64_t>(units, (int64_t)num_sms() * 8);
+        RG_LAUNCH((proj_reduce4_kernel<8>), grid, dim3(32, 8), 0, st, P, ldp, p_stride, splits, h, w, R, ldr, Rf, ldf,
+                  Rh, Rl, ldh, bf16);
+    } else if (splits > 32)
         RG_LAUNCH((proj_reduce_kernel<32>), (unsigned)((total + 31) / 32), dim3(32, 32), 0, st, P, ldp, p_stride, splits, h, w,
                                                                                        R, ldr, Rf, ldf, Rh, Rl, ldh,
                                                                                        bf16);
