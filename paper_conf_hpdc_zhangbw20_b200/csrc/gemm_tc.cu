@@ -251,6 +251,9 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
         int cnt = 0;
         constexpr int kChunks = BN / 32;
         const bool rmw = (MODE == 1) && !args.overwrite;
+        // measured: the one-chunk-ahead prefetch pays off at BN = 256 (4-8 chunks per tile) and
+        // costs a little at the narrow levels, which keep the per-chunk load
+        constexpr bool kAhead = (BN >= 256);
         // K2: the fp32 C values of a chunk are loaded one chunk ahead (the next tile's first
         // chunk during the current tile's last), so each epilogue warp keeps two chunks of
         // HBM reads in flight instead of paying a full memory latency per chunk.
@@ -271,7 +274,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
             }
         };
         float4 old[8], nxt[8];
-        if (rmw && blockIdx.x < args.units && wg < kChunks) {
+        if (kAhead && rmw && blockIdx.x < args.units && wg < kChunks) {
             int t0, tj, z, kb0, kb1;
             unit_coords<MODE>(args, blockIdx.x, t0, tj, z, kb0, kb1);
             load_old(t0, tj * BN, wg, old);
@@ -286,7 +289,8 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
             bool waited = false;
             for (int ch = wg; ch < kChunks; ch += EPI_WG) {
                 const int c = ch * 32;
-                if (rmw) {
+                if (!kAhead && rmw) load_old(t0, t1, ch, old);
+                if (kAhead && rmw) {
                     if (ch + EPI_WG < kChunks) {
                         load_old(t0, t1, ch + EPI_WG, nxt);
                     } else if (u + (int)gridDim.x < args.units) {
@@ -372,7 +376,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
                     }
                 }
                 __syncwarp();
-                if (rmw) {
+                if (kAhead && rmw) {
 #pragma unroll
                     for (int k = 0; k < 8; ++k) old[k] = nxt[k];
                 }

@@ -95,6 +95,12 @@ struct CholqrLaunch {
     unsigned long long cond;   // CUDA graph conditional handle set to 1 on a failed pivot (0: none)
     int* status;    // fused kernels report a numerical breakdown here (atomicMin col0 + j)
     int col0;       // global column index of the panel
+    // fused single-panel kernel only: first apply Algorithm 1 line 9, P <- P - Q1 R12 (uh <= 64)
+    const float* uq = nullptr;   // Q1, fp32 m x uh (ld uq_ld)
+    int64_t uq_ld = 0;
+    const float* ur = nullptr;   // R12, fp32 uh x nc (ld ur_ld)
+    int64_t ur_ld = 0;
+    int uh = 0;
 };
 size_t cholqr_ws_doubles(int64_t m);
 size_t cholqr_counter_ints(int64_t m);

@@ -82,6 +82,12 @@ struct CqArgs {
     unsigned long long cond;   // graph conditional handle of the MGS/TSQR fallback node (0: none)
     int* status;         // fused kernels: atomicMin(status, col0 + j) on a numerical breakdown
     int col0;            // global index of the panel's first column
+    // fused kernels: Algorithm 1 line 9 for this panel first, P <- P - Q1 R12 (uh > 0)
+    const float* uq;     // Q1 (fp32, m x uh, ld uq_ld)
+    int64_t uq_ld;
+    const float* ur;     // R12 (fp32, uh x nc, ld ur_ld)
+    int64_t ur_ld;
+    int uh;
 };
 
 // A failed pivot: raise the fallback flag and, inside a CUDA graph, switch on the conditional
@@ -572,25 +578,15 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
 // panels + K1 + K2 of that level, and the second CholQR pass restores orthogonality exactly as
 // it does for a 32-column panel.
 constexpr int CF_THREADS = 256;
-constexpr int CF_SCR = 3264;                     // scratch doubles: fp64 staging chunk / group partials
 constexpr int CF_FAN = 8;                        // CTA partials per first-level group
 constexpr int CF_MAX_ROWS = 1280;                // rows per CTA that fit next to the scratch (NC = 32)
-constexpr int CF_WIDE_MAX_ROWS = 472;            // same for NC = 64
+constexpr int CF_WIDE_MAX_ROWS = 560;            // same for NC = 64
 constexpr int CF_MAXPER = CF_MAX_ROWS / CF_THREADS;   // tile rows per thread (load / store loops)
 constexpr int CF_NE_MAX = 64 * 65 / 2;           // packed Gram entries, NC = 64
 
 template <int NC>
 struct CfCfg {
-    static constexpr int NB8 = NC / 8;                       // 8-column blocks
-    static constexpr int NBLK = NB8 * (NB8 + 1) / 2;         // 8x8 blocks in the upper triangle
-    static constexpr int GROUPS = CF_THREADS / NBLK;         // row groups (25 or 7)
-    static constexpr int SLD = NC + 2;                       // fp64 row stride of the staging chunk
-    static constexpr int CH = CF_SCR / SLD / 8 * 8;          // rows staged per chunk (96 or 48)
     static constexpr int NE = NC * (NC + 1) / 2;             // packed upper-triangle entries
-    static constexpr int GSTRIDE = NBLK * 64 + 1;            // group stride in the reduction rounds
-    static constexpr int GPR = CF_SCR / GSTRIDE;             // groups per round (5 or 1)
-    static constexpr int LD = NC + 2;                        // Cholesky scratch row stride
-    static_assert(GPR >= 1 && CH >= 8, "scratch");
 };
 
 __device__ __forceinline__ void tri_unpack(int p, int& i, int& j) {
@@ -603,66 +599,97 @@ __device__ __forceinline__ void tri_unpack(int p, int& i, int& j) {
 
 // Gram partial of the CTA's tile rows [0, rows) (NC columns) -> out (fp64, packed upper
 // triangle [j (j + 1) / 2 + i]) on the fp64 tensor cores (mma.sync m8n8k4 f64: 256 FMAs per
-// warp instruction, so 8 warps reach the SM's fp64 rate where DFMA loops stall on issue).
-// Rows are converted to fp64 once per chunk into a row-major staging buffer (row stride
-// SLD = NC + 4 == 4 mod 16 doubles: the 4 rows x 8 columns of an A/B fragment hit distinct
-// banks); warp w owns the 8x8 blocks w, w + 8, ... of the upper triangle for all rows, so the
-// sum over rows has one fixed order per entry and no cross-warp reduction is needed.
+// warp instruction).  Rows are converted to fp64 once per chunk into a row-major staging
+// buffer (row stride SLD = NC + 4 == 4 mod 16 doubles: the 4 rows x 8 columns of a fragment hit
+// distinct banks).  Warp w takes the 4-row k-steps w, w + 8, ... and keeps one accumulator per
+// 8x8 block of the upper triangle, so its DMMAs are independent and the NB8 fragments it loads
+// per k-step are reused by every block (A and B of a Gram are the same rows).  The eight warp
+// partials are then added in warp order through the scratch (fixed order: deterministic).
 template <int NC>
-__device__ void cf_gram(const float* tile, int ld, int rows, double* S, double* out_partial) {
+__device__ void cf_gram(const float* tile, int ld, int rows, double* S, int s_cap, double* out_partial) {
     constexpr int NB8 = NC / 8, NBLK = NB8 * (NB8 + 1) / 2, SLD = NC + 4;
-    constexpr int CH = CF_SCR / SLD / 4 * 4;
-    constexpr int NW = CF_THREADS / 32, MAXB = (NBLK + NW - 1) / NW;
+    constexpr int NW = CF_THREADS / 32;
+    const int CH = s_cap / SLD / 32 * 32;                 // rows per chunk, whole k-step rounds
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int g = lane >> 2, c = lane & 3;
-    int boff[MAXB][2];   // S column offsets of the A (bi) and B (bj) fragments of each owned block
+    double acc[NBLK][2];
 #pragma unroll
-    for (int t = 0; t < MAXB; ++t) {
-        int blk = warp + NW * t, bi = 0;
-        if (blk >= NBLK) blk = 0;
-        while (blk >= NB8 - bi) {
-            blk -= NB8 - bi;
-            ++bi;
-        }
-        boff[t][0] = bi * 8 + g;
-        boff[t][1] = (bi + blk) * 8 + g;
-    }
-    double acc[MAXB][2];
-#pragma unroll
-    for (int t = 0; t < MAXB; ++t) acc[t][0] = acc[t][1] = 0.0;
+    for (int t = 0; t < NBLK; ++t) acc[t][0] = acc[t][1] = 0.0;
     for (int ch0 = 0; ch0 < rows; ch0 += CH) {
         const int cr = min(CH, rows - ch0), cr4 = (cr + 3) & ~3;
         __syncthreads();
-        for (int e = tid; e < cr4 * NC; e += CF_THREADS) {
-            const int r = e / NC, col = e % NC;
-            S[r * SLD + col] = (r < cr) ? (double)tile[col * ld + ch0 + r] : 0.0;
+        // fp32 -> fp64 staging, 8 conversions in flight per thread
+        for (int e0 = 0; e0 < cr4 * NC; e0 += 8 * CF_THREADS) {
+            float x[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                const int e = e0 + tid + u * CF_THREADS, r = e / NC, col = e % NC;
+                x[u] = (r < cr) ? tile[col * ld + ch0 + r] : 0.f;
+            }
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                const int e = e0 + tid + u * CF_THREADS, r = e / NC, col = e % NC;
+                if (e < cr4 * NC) S[r * SLD + col] = (double)x[u];
+            }
         }
         __syncthreads();
-        for (int k0 = 0; k0 < cr4; k0 += 4) {
-            const double* rowp = S + (k0 + c) * SLD;
+        for (int k0 = 4 * warp; k0 < cr4; k0 += 4 * NW) {
+            const double* rowp = S + (k0 + c) * SLD + g;
+            double f[NB8];
 #pragma unroll
-            for (int t = 0; t < MAXB; ++t) {
-                if (warp + NW * t < NBLK) {
-                    const double av = rowp[boff[t][0]], bv = rowp[boff[t][1]];
+            for (int bi = 0; bi < NB8; ++bi) f[bi] = rowp[bi * 8];
+            int t = 0;
+#pragma unroll
+            for (int bi = 0; bi < NB8; ++bi)
+#pragma unroll
+                for (int bj = bi; bj < NB8; ++bj, ++t)
                     asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
                                  : "+d"(acc[t][0]), "+d"(acc[t][1])
-                                 : "d"(av), "d"(bv));
-                }
-            }
+                                 : "d"(f[bi]), "d"(f[bj]));
         }
     }
-    // D fragment: rows g, columns 2c, 2c + 1 of the 8x8 block
+    // warp partials -> S in rounds of WPR warps, summed in warp order by all threads; entry
+    // e = (t * 2 + u) * 32 + lane (block t, element u of this lane's D fragment)
+    constexpr int NENT = NBLK * 64;
+    const int WPR = s_cap / NENT < NW ? s_cap / NENT : NW;
+    constexpr int NQ = (NENT + CF_THREADS - 1) / CF_THREADS;
+    double run[NQ];
 #pragma unroll
-    for (int t = 0; t < MAXB; ++t) {
-        if (warp + NW * t < NBLK) {
-            const int i = boff[t][0];
-            const int j0 = boff[t][1] - g + 2 * c;
+    for (int q = 0; q < NQ; ++q) run[q] = 0.0;
+    for (int w0 = 0; w0 < NW; w0 += WPR) {
+        __syncthreads();
+        if (warp >= w0 && warp < w0 + WPR) {
+            double* dst = S + (warp - w0) * NENT + lane;
 #pragma unroll
-            for (int u = 0; u < 2; ++u) {
-                const int j = j0 + u;
-                if (i <= j) out_partial[j * (j + 1) / 2 + i] = acc[t][u];
+            for (int t = 0; t < NBLK; ++t) {
+                dst[(t * 2 + 0) * 32] = acc[t][0];
+                dst[(t * 2 + 1) * 32] = acc[t][1];
             }
         }
+        __syncthreads();
+        const int nw = min(WPR, NW - w0);
+#pragma unroll
+        for (int q = 0; q < NQ; ++q) {
+            const int e = tid + CF_THREADS * q;
+            if (e < NENT)
+                for (int k = 0; k < nw; ++k) run[q] += S[k * NENT + e];
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < NQ; ++q) {
+        const int e = tid + CF_THREADS * q;
+        if (e < NENT) S[e] = run[q];
+    }
+    __syncthreads();
+    // D fragment of block (bi, bj): lane holds rows g, columns 2c, 2c + 1
+    for (int e = tid; e < CfCfg<NC>::NE; e += CF_THREADS) {
+        int i, j;
+        tri_unpack(e, i, j);
+        const int bi = i >> 3, bj = j >> 3;
+        const int t = bi * NB8 - bi * (bi - 1) / 2 + (bj - bi);
+        const int ln = (i & 7) * 4 + ((j & 7) >> 1), u = j & 1;
+        out_partial[e] = S[(t * 2 + u) * 32 + ln];
     }
     __syncthreads();
 }
@@ -830,19 +857,23 @@ __device__ void cf_times_rinv(float* tile, int ld, int rows, const float* Rinv) 
     }
 }
 
-// Shared memory of the fused kernels beyond the row tile.
+// Shared memory of the fused kernels beyond the row tile: Gs, then Rs, Ri and all remaining
+// shared memory, which the Gram staging S reuses (S is dead between the Gram of a pass and the
+// elimination of the next; Rs / Ri are dead between the R^{-1} product and the next Gram).
 template <int NC>
 struct CfBufs {
-    double* S;     // CF_SCR scratch: fp64 staging, group partials
     double* Gs;    // NC x (NC + 2): reduced Gram [i + NC j]; the elimination's Z aliases it
     double* Rs;    // NC x (NC + 2): elimination A; R of the last pass (row-major) on exit
     float* Ri;     // NC x NC fp32 R^{-1} of the last pass, row-major
-    static constexpr size_t bytes = (size_t)(CF_SCR + 2 * NC * (NC + 2)) * 8 + (size_t)NC * NC * 4;
-    __device__ explicit CfBufs(uint8_t* base) {
-        S = reinterpret_cast<double*>(base);
-        Gs = S + CF_SCR;
+    double* S;     // fp64 staging / warp partials of the Gram (aliases Rs, Ri, ...)
+    int s_cap;     // doubles available at S
+    static constexpr size_t fixed_bytes = (size_t)(2 * NC * (NC + 2)) * 8 + (size_t)NC * NC * 4;
+    __device__ CfBufs(uint8_t* base, int cap) {
+        Gs = reinterpret_cast<double*>(base);
         Rs = Gs + NC * (NC + 2);
         Ri = reinterpret_cast<float*>(Rs + NC * (NC + 2));
+        S = Rs;
+        s_cap = cap;
     }
 };
 
@@ -863,7 +894,7 @@ __device__ int cf_panel(const CqArgs& a, float* tile, int ld, int rows, int nc, 
     bool shifted = false;
     int bad = -1;
     for (int pass = 0; pass < 3; ++pass) {
-        cf_gram<NC>(tile, ld, rows, b.S, part);
+        cf_gram<NC>(tile, ld, rows, b.S, b.s_cap, part);
         CF_MARK(4 + 4 * pass);
         cf_allreduce<NC>(a, b.Gs);
         CF_MARK(5 + 4 * pass);
@@ -953,12 +984,81 @@ __device__ int cf_panel(const CqArgs& a, float* tile, int ld, int rows, int nc, 
     return bad;
 }
 
+// P <- P - Q1 R12 on the CTA's rows (Algorithm 1 line 9 for the panel that follows an update):
+// the leaf-level K2 folded into the panel's load instead of a separate read-modify-write pass
+// over the panel.  fp32 Q1 and R12 (the values the tensor-core K2 rounds to 16 bit), fp32 FMAs.
+// R12 is staged in S as [k * NC + j]; Q1 in chunks of 128 rows as [k * 132 + r].
 template <int NC>
-__global__ void __launch_bounds__(CF_THREADS, 1) cq_fused_kernel(CqArgs a, int ld) {
+__device__ void cf_pre_update(const CqArgs& a, float* tile, int ld, int rows, int64_t r0, double* Sd, int s_cap) {
+    constexpr int CG = NC / 4, RG = CF_THREADS / CG;
+    const int tid = threadIdx.x, cgp = tid % CG, rgp = tid / CG;
+    const int uh = a.uh;
+    float* Rf = reinterpret_cast<float*>(Sd);
+    float* Qc = Rf + 64 * NC;
+    // all of the CTA's Q1 rows at once when they fit (one round of loads), else 128-row chunks
+    const int cap_rows = (int)(((int64_t)s_cap * 2 - 64 * NC) / (uh > 0 ? uh : 1)) - 4;
+    const int chunk = rows <= cap_rows ? ((rows + 3) & ~3) : 4 * RG;
+    const int qld = chunk + 4;
+    for (int e = tid; e < uh * NC; e += CF_THREADS) {
+        const int k = e / NC, j = e % NC;
+        Rf[e] = (j < a.nc) ? a.ur[k + (int64_t)j * a.ur_ld] : 0.f;
+    }
+    for (int base = 0; base < rows; base += chunk) {
+        const int cr = min(chunk, rows - base);
+        __syncthreads();
+        for (int e0 = 0; e0 < uh * cr; e0 += 8 * CF_THREADS) {
+            float x[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                const int e = e0 + tid + u * CF_THREADS, k = e / cr, r = e % cr;
+                x[u] = (e < uh * cr) ? a.uq[r0 + base + r + (int64_t)k * a.uq_ld] : 0.f;
+            }
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                const int e = e0 + tid + u * CF_THREADS, k = e / cr, r = e % cr;
+                if (e < uh * cr) Qc[k * qld + r] = x[u];
+            }
+        }
+        __syncthreads();
+        for (int sb = 0; sb < cr; sb += 4 * RG) {
+            float o[4][4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int r = sb + rgp + RG * i;
+#pragma unroll
+                for (int c = 0; c < 4; ++c) o[i][c] = (r < cr) ? tile[(4 * cgp + c) * ld + base + r] : 0.f;
+            }
+#pragma unroll 8
+            for (int k = 0; k < uh; ++k) {
+                const float4 rv = *reinterpret_cast<const float4*>(Rf + k * NC + 4 * cgp);
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const int r = sb + rgp + RG * i;
+                    const float x = (r < cr) ? Qc[k * qld + r] : 0.f;
+                    o[i][0] = fmaf(-x, rv.x, o[i][0]);
+                    o[i][1] = fmaf(-x, rv.y, o[i][1]);
+                    o[i][2] = fmaf(-x, rv.z, o[i][2]);
+                    o[i][3] = fmaf(-x, rv.w, o[i][3]);
+                }
+            }
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int r = sb + rgp + RG * i;
+                if (r < cr)
+#pragma unroll
+                    for (int c = 0; c < 4; ++c) tile[(4 * cgp + c) * ld + base + r] = o[i][c];
+            }
+        }
+    }
+    __syncthreads();
+}
+
+template <int NC>
+__global__ void __launch_bounds__(CF_THREADS, 1) cq_fused_kernel(CqArgs a, int ld, int s_cap) {
     RG_PDL_ENTRY();
     extern __shared__ __align__(16) uint8_t cf_smem[];
     float* tile = reinterpret_cast<float*>(cf_smem);
-    const CfBufs<NC> b(cf_smem + (size_t)NC * ld * 4);
+    const CfBufs<NC> b(cf_smem + (((size_t)NC * ld * 4 + 15) & ~(size_t)15), s_cap);
     const int tid = threadIdx.x;
     if (blockIdx.x == 0 && tid == 0) *a.ws.fail = 0;
     const int64_t rows_per = (a.m + gridDim.x - 1) / gridDim.x;
@@ -986,6 +1086,7 @@ __global__ void __launch_bounds__(CF_THREADS, 1) cq_fused_kernel(CqArgs a, int l
             }
     }
     __syncthreads();
+    if (a.uh > 0) cf_pre_update<NC>(a, tile, ld, rows, r0, b.S, b.s_cap);
     CF_MARK(1);
     cf_panel<NC>(a, tile, ld, rows, a.nc, b);
     CF_MARK(2);
@@ -1085,6 +1186,11 @@ static CqArgs cq_args(const CholqrLaunch& L) {
     a.cond = L.cond;
     a.status = L.status;
     a.col0 = L.col0;
+    a.uq = L.uq;
+    a.uq_ld = L.uq_ld;
+    a.ur = L.ur;
+    a.ur_ld = L.ur_ld;
+    a.uh = L.uh;
     return a;
 }
 
@@ -1093,7 +1199,19 @@ static cudaError_t launch_fused(CqArgs a, cudaStream_t st) {
     const int sms = sm_count();
     const int64_t rows_per = (a.m + sms - 1) / sms;
     const int ld = (int)(rows_per | 1);   // odd leading dimension: conflict-free column walks
-    const size_t smem = (size_t)NC * ld * 4 + CfBufs<NC>::bytes + 128;
+    // all of shared memory: the tile, Gs, and the rest for Rs / Ri / Gram staging
+    static int smem_max = 0;
+    if (!smem_max) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+        smem_max -= 2048;   // static shared memory of the kernel + slack
+    }
+    const size_t tile_bytes = (((size_t)NC * ld * 4 + 15) & ~(size_t)15);
+    const size_t gs_bytes = (size_t)NC * (NC + 2) * 8;
+    if (tile_bytes + CfBufs<NC>::fixed_bytes > (size_t)smem_max) return cudaErrorInvalidValue;
+    const int s_cap = (int)(((size_t)smem_max - tile_bytes - gs_bytes) / 8);
+    const size_t smem = (size_t)smem_max;
     cudaError_t e = cudaFuncSetAttribute(cq_fused_kernel<NC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
@@ -1107,12 +1225,13 @@ static cudaError_t launch_fused(CqArgs a, cudaStream_t st) {
     cfg.attrs = at;
     cfg.numAttrs = 1;
     ++g_launches;
-    return cudaLaunchKernelEx(&cfg, cq_fused_kernel<NC>, a, ld);
+    return cudaLaunchKernelEx(&cfg, cq_fused_kernel<NC>, a, ld, s_cap);
 }
 
 cudaError_t launch_panel_cholqr(const CholqrLaunch& L, bool* handles_failure, cudaStream_t st) {
     CqArgs a = cq_args(L);
     const int grid = cq_grid(L.m);
+    if (L.uh > 0 && (a.distributed || !cholqr_fused_fits(L.m, 32) || L.uh > 64)) return cudaErrorInvalidValue;
     if (!a.distributed && cholqr_fused_fits(L.m, 32)) {
         if (handles_failure) *handles_failure = true;   // shifted CholQR3 inside the kernel
         return launch_fused<32>(a, st);

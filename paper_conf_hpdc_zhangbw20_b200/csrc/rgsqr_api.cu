@@ -408,7 +408,15 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
                                       st));
         RG_CUDA(cudaMemset2DAsync(pl.R, pl.ldr * sizeof(float), 0, n * sizeof(float), n, st));
     }
-    for (auto& o : pl.ops) {
+    const Op* pending_update = nullptr;   // leaf-level K2 folded into the next panel's load
+    for (size_t oi = 0; oi < pl.ops.size(); ++oi) {
+        const Op& o = pl.ops[oi];
+        if (o.kind == Op::UPDATE && !dist && pl.panel == 0 && o.h <= 64 && oi + 1 < pl.ops.size() &&
+            pl.ops[oi + 1].kind == Op::PANEL && pl.ops[oi + 1].c0 == o.c0 + o.h && pl.ops[oi + 1].w == o.w &&
+            rg::cholqr_fused_fits(m, 32) && getenv("RGSQR_NO_FOLD") == nullptr) {
+            pending_update = &o;
+            continue;
+        }
         if (o.kind == Op::PAIR) {
             // two panels + R12 = Q1^T A2 + A2 -= Q1 R12 of a (h + w)-column block; algorithmic bytes:
             // read the block (fp32), write Q (fp32) + shadow(s)
@@ -483,6 +491,15 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
                 p.guard = cq_fail;
                 c.status = status;
                 c.col0 = o.c0;
+                if (pending_update) {
+                    const Op& u = *pending_update;
+                    c.uq = pl.Q + (int64_t)u.c0 * pl.ldq;
+                    c.uq_ld = pl.ldq;
+                    c.ur = pl.R + u.c0 + (int64_t)(u.c0 + u.h) * pl.ldr;
+                    c.ur_ld = pl.ldr;
+                    c.uh = u.h;
+                    pending_update = nullptr;
+                }
                 bool handled = false;
                 RG_CUDA(rg::launch_panel_cholqr(c, &handled, st));
                 if (handled) continue;   // shifted CholQR3 fallback inside the fused kernel

@@ -45,7 +45,10 @@ def _check_qr(A32, Q, R, kappa=10.0, orth_scale=1e-2):
     assert orth <= orth_scale * np.sqrt(n), orth
     Qo, Ro, _ = oracle.householder(A)
     dr = np.linalg.norm(R - Ro) / np.linalg.norm(Ro)
-    assert dr <= max(10 * kappa * be, 1e-5), (dr, be)
+    # first-order perturbation of the unique R: kappa(A) times (backward error + loss of
+    # orthogonality); the 16-bit K1 rounding shows up in orth, not in be, when the update that
+    # follows it is done in fp32 (leaf-level K2 folded into the panel)
+    assert dr <= max(10 * kappa * (be + orth / np.sqrt(n)), 1e-5), (dr, be, orth)
     return be, orth, dr
 
 

@@ -175,6 +175,15 @@ int main(int argc, char** argv) {
                hc[0], hc[1], hc[2], hc[3], hc[4]);
     }
     {
+        unsigned long long tr[16];
+        rg::launch_panel_cholqr(L, nullptr, st);
+        cudaStreamSynchronize(st);
+        cudaMemcpyFromSymbol(tr, rg::cf_trace, sizeof(tr));
+        printf("  32-col trace (us): load %.2f gram %.2f allreduce %.2f chol %.2f apply %.2f panel %.2f store %.2f\n",
+               (tr[1] - tr[0]) / 1e3, (tr[4] - tr[0]) / 1e3, (tr[5] - tr[0]) / 1e3, (tr[6] - tr[0]) / 1e3,
+               (tr[7] - tr[0]) / 1e3, (tr[2] - tr[0]) / 1e3, (tr[3] - tr[0]) / 1e3);
+    }
+    {
         // two-panel kernel (64 columns), eager back-to-back launches
         float *P2, *Q2, *R2; uint16_t* Qh2;
         cudaMalloc(&P2, (size_t)m * 64 * 4); cudaMalloc(&Q2, (size_t)m * 64 * 4); cudaMalloc(&R2, 64 * 64 * 4);
