@@ -113,6 +113,27 @@ cudaError_t launch_panel_cholqr(const CholqrLaunch& L, bool* handles_failure, cu
 // 32 < nc <= 64 block: same Q and R in exact arithmetic; R written as the nc x nc block at L.R.
 cudaError_t launch_panel_pair(const CholqrLaunch& L, cudaStream_t st);
 
+// ---- leaf.cu (last recursion level: panel, K1, K2, panel in one cooperative kernel)
+struct LeafLaunch {
+    float* Q;          // nc block columns, in = P, out = Q (fp32, ldq)
+    int64_t ldq;
+    uint16_t* Qh;      // 16-bit shadow (hi) of Q, ldh
+    uint16_t* Ql;      // lo part (split mode) or null
+    int64_t ldh;
+    int64_t m;
+    int nc;            // 1..64: first panel min(32, nc) columns, second the rest
+    float* R;          // nc x nc diagonal block of R (ldr)
+    int64_t ldr;
+    double* ws;        // leaf_ws_doubles()
+    unsigned* bar;     // zero-initialised grid-barrier word
+    int* status;
+    int col0;
+    int bf16;
+};
+bool leaf_fits(int64_t m);          // rows per SM fit in shared memory (and RGSQR_NO_LEAF unset)
+size_t leaf_ws_doubles();
+cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st);
+
 // ---- gemm_tc.cu (Alg 1 lines 8-9 on tcgen05)
 cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int splits, const CUtensorMap& q1,
                              const CUtensorMap& a2, const CUtensorMap& q1_lo, const CUtensorMap& a2_lo, float* P,

@@ -143,6 +143,7 @@ struct rg_handle_s {
     int64_t last_info = -1;
     // workspace
     DevBuf cq_ws, cq_flags;                         // CholQR2 panel workspace (flags: fail, counters)
+    DevBuf leaf_bar;                                // grid-barrier word of the leaf kernel
     DevBuf qh, ql, P, r12h, r12l, r12f, partial, norm2, scale, status, pws, pcnt, rgather, rstackq;
     DevBuf stageA, stageQ, stageR, stageB, stageX;  // host-pointer staging
     DevBuf cg;                                      // CGLS vectors
@@ -168,6 +169,7 @@ struct rg_handle_s {
         int cls;
         cudaEvent_t a, b;
         double flops, bytes;
+        int tag;   // op width tag for the RGSQR_PROF_OPS per-op trace (kind * 100000 + w)
     };
     std::vector<PendingEv> pending;
     size_t ev_next = 0;
@@ -190,9 +192,10 @@ struct ProfScope {
     rg_handle h;
     int cls;
     double flops, bytes;
+    int tag;
     cudaEvent_t b = nullptr, e = nullptr;
-    ProfScope(rg_handle h_, int cls_, double flops_ = 0, double bytes_ = 0)
-        : h(h_), cls(cls_), flops(flops_), bytes(bytes_) {
+    ProfScope(rg_handle h_, int cls_, double flops_ = 0, double bytes_ = 0, int tag_ = 0)
+        : h(h_), cls(cls_), flops(flops_), bytes(bytes_), tag(tag_) {
         if (!h->prof) return;
         if (h->ev_next >= h->ev_pool.size()) {
             cudaEvent_t x, y;
@@ -208,16 +211,20 @@ struct ProfScope {
     ~ProfScope() {
         if (!h->prof) return;
         cudaEventRecord(e, h->stream);
-        h->pending.push_back({cls, b, e, flops, bytes});
+        h->pending.push_back({cls, b, e, flops, bytes, tag});
     }
 };
 
 void prof_collect(rg_handle h) {
     if (!h->prof || h->pending.empty()) return;
     cudaStreamSynchronize(h->stream);
+    static const bool trace = getenv("RGSQR_PROF_OPS") != nullptr;
     for (auto& p : h->pending) {
         float ms = 0;
         cudaEventElapsedTime(&ms, p.a, p.b);
+        if (trace)
+            fprintf(stderr, "[rgsqr op] cls %d w %d us %.2f TF %.1f GB/s %.0f\n", p.cls, p.tag, ms * 1e3,
+                    p.flops / (ms * 1e-3) / 1e12, p.bytes / (ms * 1e-3) / 1e9);
         h->prof_ms[p.cls] += ms;
         h->prof_launches[p.cls] += 1;
         h->prof_flops[p.cls] += p.flops;
@@ -286,12 +293,15 @@ int make_plan(rg_handle h, Plan& pl) {
     const int n = (int)pl.n;
     pl.ldh = round_up(std::max<int64_t>(m, 8), 8);
     pl.ops.clear();
-    // Opt-in (RGSQR_WIDE=1): the last recursion level (two 32-column panels + K1 + K2) as one
-    // 64-column CholQR2 kernel when its rows fit in shared memory.  Same Q, R in exact
-    // arithmetic, better conditioned in practice (fp64 Gram instead of fp16 K1/K2 at that level);
-    // measured the same speed as the paper's structure on config 2 (12.33 vs 12.35 ms).
+    // The last recursion level (two 32-column panels + K1 + K2 of a <= 64-column block) runs as
+    // one kernel when the rows per SM fit in shared memory: by default the leaf kernel (leaf.cu,
+    // the paper's structure with rows resident on chip); opt-in RGSQR_WIDE=1 the 64-column
+    // CholQR2 kernel (same Q, R in exact arithmetic).
+    const bool wide = getenv("RGSQR_WIDE") != nullptr;
+    // (split-precision passes keep the tensor-core K1/K2 at the last level: the leaf kernel's
+    // mma.sync K1/K2 are single 16-bit products)
     const bool pair = pl.panel == 0 && pl.nb == 32 && !(pl.nranks > 1 && h->comm) &&
-                      rg::cholqr_fused_fits(m, 64) && getenv("RGSQR_WIDE") != nullptr;
+                      (wide ? rg::cholqr_fused_fits(m, 64) : (rg::leaf_fits(m) && !pl.split));
     build_ops(pl.ops, 0, n, pl.nb, pair);
     int max_h = 0, max_w = 0;
     size_t pmax = 0;
@@ -369,7 +379,8 @@ bool ensure_workspace(rg_handle h, int64_t m, int64_t n, int split) {
               h->scale.ensure(n * 4 + 64) && h->status.ensure(64) &&
               h->pws.ensure(rg::panel_ws_floats(m) * 4 + 4096) && h->pcnt.ensure(rg::panel_counters(m) * 4 + 64) &&
               h->rgather.ensure((size_t)64 * 32 * 32 * 4) && h->rstackq.ensure((size_t)64 * 32 * 32 * 4) &&
-              h->cq_ws.ensure(rg::cholqr_ws_doubles(m) * 8 + 256) &&
+              h->cq_ws.ensure(std::max(rg::cholqr_ws_doubles(m), rg::leaf_ws_doubles()) * 8 + 256) &&
+              h->leaf_bar.ensure(256) &&
               h->cq_flags.ensure((rg::cholqr_counter_ints(m) + 8) * 4);
     return ok;
 }
@@ -442,12 +453,31 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             c.bf16 = pl.bf16;
             c.status = status;
             c.col0 = o.c0;
-            RG_CUDA(rg::launch_panel_pair(c, st));
+            if (getenv("RGSQR_WIDE") != nullptr) {
+                RG_CUDA(rg::launch_panel_pair(c, st));
+            } else {
+                rg::LeafLaunch L{};
+                L.Q = c.Q;
+                L.ldq = c.ldq;
+                L.Qh = c.Qh;
+                L.Ql = c.Ql;
+                L.ldh = c.ldh;
+                L.m = m;
+                L.nc = c.nc;
+                L.R = c.R;
+                L.ldr = c.ldr;
+                L.ws = h->cq_ws.as<double>();
+                L.bar = h->leaf_bar.as<unsigned>();
+                L.status = status;
+                L.col0 = o.c0;
+                L.bf16 = pl.bf16;
+                RG_CUDA(rg::launch_leaf(L, st));
+            }
             continue;
         }
         if (o.kind == Op::PANEL) {
             // algorithmic bytes: read the panel (fp32), write Q (fp32) + 16-bit shadow (+ lo shadow)
-            ProfScope _s(h, PC_PANEL, 2.0 * m * o.w * o.w, (double)m * o.w * (pl.split ? 12 : 10));
+            ProfScope _s(h, PC_PANEL, 2.0 * m * o.w * o.w, (double)m * o.w * (pl.split ? 12 : 10), o.w);
             rg::PanelLaunch p{};
             p.Q = pl.Q + (int64_t)o.c0 * pl.ldq;
             p.ldq = pl.ldq;
@@ -524,7 +554,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             }
         } else if (o.kind == Op::PROJ) {
             ProfScope _s(h, PC_PROJ, 2.0 * m * o.h * o.w * (pl.split ? 3 : 1),
-                             (double)m * (o.h + o.w) * (pl.split ? 4 : 2));
+                             (double)m * (o.h + o.w) * (pl.split ? 4 : 2), o.w);
             float* P = h->P.as<float>();
             const int64_t ldp = (int64_t)o.tiles_i * 128;
             const int64_t pstride = ldp * o.tiles_j * o.bn;
@@ -546,7 +576,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             }
         } else {
             ProfScope _s(h, PC_UPDATE, 2.0 * m * o.h * o.w * (pl.split ? 3 : 1),
-                             (double)m * o.h * (pl.split ? 4 : 2) + (double)m * o.w * (pl.split ? 12 : 10));
+                             (double)m * o.h * (pl.split ? 4 : 2) + (double)m * o.w * (pl.split ? 12 : 10), o.w);
             float* C = pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq;
             uint16_t* Ch = qh + (int64_t)(o.c0 + o.h) * pl.ldh;
             uint16_t* Cl = ql ? ql + (int64_t)(o.c0 + o.h) * pl.ldh : nullptr;

@@ -1,0 +1,128 @@
+// Standalone timing harness for the leaf kernel (development tool, not product).
+// nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -I include tools/leaf_bench.cu -o tools/leaf_bench
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
+#include <cuda_runtime.h>
+#define LF_TRACE 1
+#include "../paper_conf_hpdc_zhangbw20_b200/csrc/kernels.h"
+namespace rg { thread_local long long g_launches = 0; bool pdl_enabled() { return false; } }
+#include "../paper_conf_hpdc_zhangbw20_b200/csrc/leaf.cu"
+__global__ void chol_probe(long long* cyc, int reps) {
+    extern __shared__ __align__(16) uint8_t sm[];
+    rg::LfSmem s(sm, 36);
+    for (int e = threadIdx.x; e < 1024; e += blockDim.x) {
+        const int i = e >> 5, j = e & 31;
+        s.G[i * rg::LF_GLD + j] = (i == j ? 40.0 : 1.0 / (1 + i + j));
+    }
+    __syncthreads();
+    long long t0 = clock64(), t1 = 0, t2 = 0, t3 = 0;
+    for (int r = 0; r < reps; ++r) {
+        if (threadIdx.x < 32) {
+            int fb = rg::lf_chol_warp(s);
+            if (r == 0) t1 = clock64();
+            double kk = rg::lf_inverse_warp(s, 32);
+            if (r == 0) t2 = clock64();
+            if (fb != 32 || kk < 0) cyc[5] = 1;
+        }
+        if (r == 0) t3 = clock64();
+    }
+    long long t4 = clock64();
+    if (threadIdx.x == 0) { cyc[0] = t1 - t0; cyc[1] = t2 - t1; cyc[2] = (t4 - t3) / (reps > 1 ? reps - 1 : 1); }
+}
+__global__ void lat_probe(long long* cyc, double* out, int n) {
+    __shared__ double sm[1024];
+    __shared__ int chase[64];
+    const int lane = threadIdx.x & 31;
+    for (int i = threadIdx.x; i < 1024; i += blockDim.x) sm[i] = 1.0 + i * 1e-9;
+    for (int i = threadIdx.x; i < 64; i += blockDim.x) chase[i] = (i + 1) & 63;
+    __syncthreads();
+    if (threadIdx.x >= 32) return;
+    double a0 = out[lane], a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, a4 = a0 + 4, a5 = a0 + 5, a6 = a0 + 6, a7 = a0 + 7;
+    const double b = 1.0000001, c = 1e-9;
+    long long t0 = clock64();
+    for (int i = 0; i < n; ++i) {
+        a0 = fma(a0, b, c); a1 = fma(a1, b, c); a2 = fma(a2, b, c); a3 = fma(a3, b, c);
+        a4 = fma(a4, b, c); a5 = fma(a5, b, c); a6 = fma(a6, b, c); a7 = fma(a7, b, c);
+    }
+    long long t1 = clock64();
+    for (int i = 0; i < n; ++i) a0 = fma(a0, b, c);
+    long long t2 = clock64();
+    int p = lane & 63;
+    for (int i = 0; i < n; ++i) p = chase[p];
+    long long t3 = clock64();
+    double v = 0;
+    for (int i = 0; i < n; ++i) {
+        sm[(i & 31) * 32 + lane] = v + lane;
+        __syncwarp();
+        v = sm[(i & 31) * 32 + ((lane + 1) & 31)];
+    }
+    long long t4 = clock64();
+    float f0 = (float)a1, f1 = f0 + 1, f2 = f0 + 2, f3 = f0 + 3, f4 = f0 + 4, f5 = f0 + 5, f6 = f0 + 6, f7 = f0 + 7;
+    for (int i = 0; i < n; ++i) {
+        f0 = fmaf(f0, 1.0001f, 1e-7f); f1 = fmaf(f1, 1.0001f, 1e-7f); f2 = fmaf(f2, 1.0001f, 1e-7f); f3 = fmaf(f3, 1.0001f, 1e-7f);
+        f4 = fmaf(f4, 1.0001f, 1e-7f); f5 = fmaf(f5, 1.0001f, 1e-7f); f6 = fmaf(f6, 1.0001f, 1e-7f); f7 = fmaf(f7, 1.0001f, 1e-7f);
+    }
+    long long t5 = clock64();
+    double r = a2;
+    for (int i = 0; i < n; ++i) r = rg::lf_rsqrt(r + 2.0);
+    long long t6 = clock64();
+    out[lane] = a0 + a1 + a2 + a3 + a4 + a5 + a6 + a7 + p + v + f0 + f1 + f2 + f3 + f4 + f5 + f6 + f7 + r;
+    if (lane == 0) {
+        cyc[0] = (t1 - t0) * 100 / (8 * n); cyc[1] = (t2 - t1) * 100 / n; cyc[2] = (t3 - t2) * 100 / n;
+        cyc[3] = (t4 - t3) * 100 / n; cyc[4] = (t5 - t4) * 100 / (8 * n); cyc[5] = (t6 - t5) * 100 / n;
+    }
+}
+int main(int argc, char** argv) {
+    {
+        long long* cyc; double* out; cudaMalloc(&cyc, 64); cudaMalloc(&out, 1024); cudaMemset(out, 0, 1024);
+        lat_probe<<<1, 64>>>(cyc, out, 4096);
+        long long hc[6]; cudaMemcpy(hc, cyc, 48, cudaMemcpyDeviceToHost);
+        printf("lat probe (cycles x100): DFMA issue %lld, DFMA latency %lld, LDS latency %lld, STS+syncwarp+LDS %lld, FFMA issue %lld, rsqrt(approx+newton) %lld\n",
+               hc[0], hc[1], hc[2], hc[3], hc[4], hc[5]);
+    }
+    {
+        long long* cyc; cudaMalloc(&cyc, 64); cudaMemset(cyc, 0, 64);
+        size_t smb = 64 * 36 * 4 + rg::LfSmem::fixed_bytes();
+        cudaFuncSetAttribute(chol_probe, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb);
+        chol_probe<<<1, 32, smb>>>(cyc, 20);
+        long long hc[8]; cudaMemcpy(hc, cyc, 48, cudaMemcpyDeviceToHost);
+        printf("chol probe: first chol %lld cyc, first inverse %lld cyc, warm chol+inv %lld cyc (bad %lld)\n", hc[0], hc[1], hc[2], hc[5]);
+    }
+    const int64_t m = argc > 1 ? atoll(argv[1]) : 65536;
+    const int nc = argc > 2 ? atoi(argv[2]) : 64;
+    std::vector<float> h((size_t)m * nc);
+    srand(1);
+    for (auto& x : h) x = (rand() / (float)RAND_MAX) - 0.5f;
+    float *P, *Q, *R; uint16_t* Qh; double* ws; unsigned* bar; int* status;
+    cudaMalloc(&P, m * nc * 4); cudaMalloc(&Q, m * nc * 4); cudaMalloc(&R, 64 * 64 * 4);
+    cudaMalloc(&Qh, m * nc * 2); cudaMalloc(&ws, rg::leaf_ws_doubles() * 8); cudaMalloc(&bar, 256);
+    cudaMalloc(&status, 64); cudaMemset(bar, 0, 256); cudaMemset(status, 0x7f, 64);
+    cudaMemcpy(P, h.data(), m * nc * 4, cudaMemcpyHostToDevice);
+    rg::LeafLaunch L{};
+    L.Q = Q; L.ldq = m; L.Qh = Qh; L.ldh = m; L.m = m; L.nc = nc; L.R = R; L.ldr = 64; L.ws = ws; L.bar = bar;
+    L.status = status; L.col0 = 0;
+    cudaStream_t st; cudaStreamCreate(&st);
+    const int iters = 50;
+    cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
+    float tot = 0;
+    for (int i = 0; i < iters + 3; ++i) {
+        cudaMemcpyAsync(Q, P, m * nc * 4, cudaMemcpyDeviceToDevice, st);
+        cudaEventRecord(a, st);
+        cudaError_t e = rg::launch_leaf(L, st);
+        cudaEventRecord(b, st);
+        cudaEventSynchronize(b);
+        if (e != cudaSuccess) { printf("launch error %s\n", cudaGetErrorString(e)); return 1; }
+        float ms; cudaEventElapsedTime(&ms, a, b);
+        if (i >= 3) tot += ms;
+    }
+    printf("m=%lld nc=%d leaf kernel: %.2f us (err %s)\n", (long long)m, nc, tot * 1000 / iters,
+           cudaGetErrorString(cudaGetLastError()));
+    unsigned long long tr[32];
+    cudaMemcpyFromSymbol(tr, rg::lf_trace, sizeof(tr));
+    const char* names[17] = {"start", "loaded", "p1 gram", "p1 allreduce", "p1 chol+inv", "p1 apply", "k1 begin",
+                             "k1 mma", "k1 allreduce", "k2", "store Q1", "p2 gram", "p2 allreduce", "p2 chol+inv",
+                             "p2 apply", "p2 done", "store Q2"};
+    for (int i = 1; i < 17; ++i) printf("  %-14s %7.2f us (+%.2f)\n", names[i], (tr[i] - tr[0]) / 1e3, ((long long)tr[i] - (long long)tr[i - 1]) / 1e3);
+    return 0;
+}
