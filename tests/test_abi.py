@@ -60,7 +60,13 @@ def test_library_is_sm100a(rg):
     assert "UTCHMMA" in sass          # tcgen05.mma
     assert "UTMALDG" in sass          # TMA tensor loads
     assert "LDTM" in sass             # tcgen05.ld (TMEM -> registers)
-    assert " HMMA" not in sass        # no legacy mma.sync tensor path
+    # the recursive-update GEMMs (K1/K2 of every level above the leaf) are tcgen05 only; the only
+    # mma.sync (HMMA) users are the leaf kernel's in-shared-memory 32-column K1/K2 (leaf.cu)
+    funcs = sass.split("Function : ")
+    hmma = sorted({f.split()[0] for f in funcs[1:] if " HMMA" in f})
+    assert all("leaf_kernel" in name for name in hmma), hmma
+    gemm = [f for f in funcs[1:] if "gemm_tc_kernel" in f.split()[0]]
+    assert gemm and all(" HMMA" not in f for f in gemm)
 
 
 def test_opts_defaults_and_status_strings(rg):
