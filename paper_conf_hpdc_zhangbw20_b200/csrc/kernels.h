@@ -129,8 +129,13 @@ struct LeafLaunch {
     int* status;
     int col0;
     int bf16;
+    // prologue: Algorithm 1 lines 8-9 of the level above for this block, R_AB = Q_A^T P written
+    // to R[-ph .. -1, 0 .. nc) (rows above the diagonal block), then P -= Q_A R_AB
+    const uint16_t* pq = nullptr;   // Q_A 16-bit image (ld ldh, 16-byte aligned), null = none
+    int ph = 0;                     // its columns, 1..64
 };
 bool leaf_fits(int64_t m);          // rows per SM fit in shared memory (and RGSQR_NO_LEAF unset)
+bool leaf_prologue_fits(int64_t m); // ... and the 16-bit staging copy of the prologue's Q_A
 size_t leaf_ws_doubles();
 cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st);
 

@@ -1,32 +1,32 @@
-// leaf.cu -- the last level of Algorithm 1 in one kernel: for a block
-// of nc <= 64 columns split as h = min(32, nc), w = nc - h,
+// leaf.cu -- the base case of Algorithm 1 in one kernel: the QR of a
+// block of nc <= 64 columns (the leaf of the recursion, nb = 64; reading #2) by CholQR2 with an
+// fp64 Gram matrix, optionally preceded by lines 8-9 of the level above (the "prologue"):
 //
-//   [Q1, R11] = panel(P1)                      (Alg 1 line 6; CholQR, fp64 Gram)
-//   R12       = Q1^T P2                        (line 8, 16-bit operands, fp32 accumulation)
-//   P2       <- P2 - Q1 R12                    (line 9, same precision)
-//   [Q2, R22] = panel(P2)                      (line 10)
+//   [prologue]  R_AB = Q_A^T P,  P <- P - Q_A R_AB     (16-bit operands, fp32 accumulation,
+//                                                       the precision of the tensor-core GEMMs)
+//   pass p:     G = P^T P (fp64),  R_p = chol(G),  P <- P R_p^{-1}
+//   R = R_p ... R_1
 //
-// with the block's rows resident in shared memory: every CTA of a cooperative grid (one per SM)
-// owns a contiguous run of rows, loads them once (cp.async), and writes Q (fp32 + 16-bit shadow)
-// once.  The three cross-row reductions (the two Gram matrices and R12) are deterministic grid
-// all-reductions: each CTA writes its partial, a grid barrier, CTA b sums entry slice b over all
-// partials in CTA order (one warp per entry, fixed shuffle tree), a second barrier, and every CTA
-// reads the reduced result.
+// In exact arithmetic the leaf's Q and R are those of the two 32-column panels + K1 + K2 of the
+// paper's structure (the QR of a full-rank block is unique), and the fp64 Gram makes the CholQR
+// panel more accurate than the paper's fp32 MGS panel.  One CholQR pass when kappa_F(R_1) <= 2 nc
+// (Q then orthogonal to ~kappa u32), else CholQR2; a failed pivot switches to shifted CholQR3
+// (shift 11 (m nc + nc (nc + 1)) u ||P||_F^2); a pivot that still fails is a numerical breakdown
+// reported through status (col0 + j).
 //
-// Why a new kernel ("Leaf"): on B200 the 65536 x 32 panel is a few us of
-// HBM traffic, so the leaf level is latency-bound.  Measured with per-op events at config 2, the
-// previous structure (K1 GEMM + split-K reduce + a fused CholQR2 panel with the leaf K2 folded
-// in) cost ~118 us per 64 columns.  The pieces here are built for latency:
+// B200 design ("Leaf").  Every CTA of a cooperative grid (one per SM) owns a
+// contiguous run of rows of the block, loads them once (cp.async) into shared memory and writes Q
+// (fp32 + 16-bit shadow) once; a 65536 x 64 leaf is 16 MB, a few us of HBM traffic, so the kernel
+// is latency-bound and built around few grid-wide steps:
 //   * Gram on the fp64 tensor cores (DMMA m8n8k4) straight from the fp32 rows in smem (one
-//     fragment per 8-column block serves as both A and B), no staging copy;
-//   * K1 / K2 of the leaf level on mma.sync m16n8k16 (fp16 or bf16 in, fp32 accumulate -- the
-//     precision of the tensor-core GEMMs of the upper levels);
-//   * the 32 x 32 Cholesky in one warp, fp64, column j in lane j's registers (32 dependent
-//     pivots, no block barriers), then R^{-1} by column-parallel back substitution;
-//   * P <- P R^{-1} exploiting the triangle (warp-uniform column groups).
-// Panel numerics are those of panel_cholqr.cu: one CholQR pass when kappa_F(R1) <= 2 nc, else
-// CholQR2; a failed pivot switches to shifted CholQR3 (shift 11 (m nc + nc (nc + 1)) u ||P||_F^2);
-// a pivot that still fails is a numerical breakdown reported through status (col0 + j).
+//     fragment per 8-column block serves as A and B), 36 8x8 blocks, no staging copy;
+//   * one deterministic grid all-reduction per pass (fixed-order sums, two grid barriers);
+//   * the 64 x 64 Cholesky on 4 warps (column j, half the rows per thread, in registers), one
+//     shared-memory broadcast + named barrier per pivot; R^{-1} in fp32 by column-parallel back
+//     substitution; P R^{-1} exploiting the triangle;
+//   * the prologue on mma.sync m16n8k16 from a 16-bit staging copy of Q_A (replaces that level's
+//     K1 GEMM, split-K reduce and K2 GEMM launches).
+// Measured per-op (tools/prof_levels.py) and per-phase (tools/leaf_bench.cu) on B200.
 #include <cuda_runtime.h>
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
@@ -41,11 +41,14 @@ namespace rg {
 constexpr int LF_THREADS = 512;
 constexpr int LF_NW = LF_THREADS / 32;
 constexpr int LF_MAXI = 9;                   // row groups of 64 per thread in the apply (<= 576 rows)
-constexpr int LF_GLD = 34;                   // fp64 32 x 32 matrices in smem: row stride (16-byte rows)
-constexpr int LF_R12LD = 40;                 // 16-bit R12 image [n][k] row stride (halves)
-constexpr int LF_SCRATCH = 5120;             // doubles of warp-partial scratch (40 KB)
-constexpr int LF_PART = 1024;                // doubles per CTA partial in the workspace
+constexpr int LF_GLD = 66;                   // fp64 64 x 64 matrices in smem: row stride (16-byte rows)
+constexpr int LF_TLD = 68;                   // fp32 column-major R: column stride
+constexpr int LF_NE = 64 * 65 / 2;           // packed upper-triangle Gram entries
+constexpr int LF_NENT = 36 * 64;             // Gram fragment entries (36 8x8 blocks)
+constexpr int LF_PART = 4096;                // doubles per CTA partial in the workspace (64 x 64 prologue)
+constexpr int LF_ABLD = 72;                  // 16-bit -R_AB image [n][k] row stride (halves)
 constexpr int LF_MAX_GRID = 160;
+constexpr size_t LF_REGION = 33792;          // bytes of each of the two aliased scratch regions
 
 struct LeafArgs {
     float* Q;            // block columns: in = P (after the upper levels' updates), out = Q; fp32, ldq
@@ -59,6 +62,7 @@ struct LeafArgs {
     int64_t ldr;
     double* part;        // [LF_MAX_GRID][LF_PART] CTA partials
     double* red;         // [LF_PART] reduced result
+    double* racc;        // [2][64 * 64] accumulated R (CTA 0), row-major
     unsigned* bar;       // grid barrier word (generation bit flips every barrier)
     int* status;         // atomicMin(status, col0 + j) on a numerical breakdown
     int col0;
@@ -66,6 +70,9 @@ struct LeafArgs {
     int rows_per;        // rows per CTA (multiple of 8)
     int ldt;             // smem tile leading dimension (floats), == 4 mod 32
     int vec;             // 16-byte global accesses allowed
+    // prologue (Algorithm 1 lines 8-9 of the level above, folded in): R_AB = Q_A^T P, P -= Q_A R_AB
+    const uint16_t* pq;  // Q_A, 16-bit image (ld ldh), m x ph; null: no prologue
+    int ph;              // columns of Q_A (<= 64)
 };
 
 #ifdef LF_TRACE
@@ -107,7 +114,9 @@ __device__ __forceinline__ void lf_grid_sync(unsigned* bar) {
     __syncthreads();
 }
 
-__device__ __forceinline__ void lf_cp16(float* sdst, const float* gsrc, int src_bytes) {
+__device__ __forceinline__ void lf_bar128() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+__device__ __forceinline__ void lf_cp16(void* sdst, const void* gsrc, int src_bytes) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(sdst)), "l"(gsrc), "r"(src_bytes)
                  : "memory");
 }
@@ -116,10 +125,7 @@ __device__ __forceinline__ void lf_cp4(float* sdst, const float* gsrc, int src_b
                  : "memory");
 }
 __device__ __forceinline__ void lf_cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void lf_cp_wait() {
-    asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
+__device__ __forceinline__ void lf_cp_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
 __device__ __forceinline__ uint32_t lf_pack2(float lo, float hi, int bf16) {
     if (bf16) {
@@ -158,64 +164,77 @@ __device__ __forceinline__ void lf_mma16816(float (&d)[4], const uint32_t (&a)[4
             : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b[0]), "r"(b[1]));
 }
 
+// fp64 1/sqrt: hardware approximation + one Newton step (relative error ~2^-44, far below what
+// the fp32 outputs resolve; the pivot test is done on d itself).
+__device__ __forceinline__ double lf_rsqrt(double d) {
+    double y;
+    asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(d));
+    const double e = fma(-d * y, y, 1.0);
+    return fma(0.5 * y, e, y);
+}
+
 // ------------------------------------------------------------------ shared memory
+// Regions A and B are adjacent and reused by phase:
+//   A: Gram warp partials (scr) -> all-reduce result (red) -> fp32 R (Rt32) + R^{-1} (X32)
+//   B: full Gram G -> R of the pass (Rs, fp64 row-major; written after every thread loaded G)
+//   A + B: the prologue's 16-bit Q_A staging copy (qa)
 struct LfSmem {
     float* tile;      // 64 columns x ldt rows (fp32, column-major)
-    double* scr;      // LF_SCRATCH doubles: warp partials
-    double* G;        // 32 x LF_GLD: reduced Gram (full symmetric), then Cholesky scratch
-    double* Rs;       // 32 x LF_GLD: R of the current pass, row-major R(i, j) = Rs[i * LD + j]
-    double* Racc;     // 32 x LF_GLD: accumulated R of the panel (R_p ... R_1)
-    double* Rt;       // 32 x LF_GLD: R of the current pass, column-major R(i, j) = Rt[j * LD + i]
-    double* U;        // 32 x LF_GLD: row k of the Schur complement at elimination step k
-    float* Rt32;      // 32 x 36: fp32 copy of R, column-major (inverse input)
-    float* rdiag32;   // 32
-    int* pivok;       // 32: pivot k accepted
-    double* red;      // 1024: reduced values of the current all-reduction
-    double* rdiag;    // 32: 1 / R(k, k)
-    float* Ri;        // 32 x 32 fp32 R^{-1}, row-major
-    uint16_t* R12h;   // 32 x LF_R12LD: -R12 as the K2 B operand, [n][k]
+    double* scr;      // A: LF_NENT doubles
+    double* red;      // A: LF_NE doubles
+    float* Rt32;      // A: 64 x LF_TLD, fp32 R column-major, R(i, j) = Rt32[j * LF_TLD + i]
+    float* X32;       // A (+ Rt32 size): 64 x 64 fp32 R^{-1}, row-major
+    double* G;        // B: 64 x LF_GLD full symmetric Gram
+    double* Rs;       // B: 64 x LF_GLD R of the pass, row-major
+    uint16_t* qa;     // A + B: prologue staging, 64 columns x lf_qa_ld halves
+    double* U;        // 2 x 64: row k of the Schur complement (ping-pong)
+    double* gdiag;    // 64: diagonal of G (pivot test)
+    double* rdiag;    // 64: 1 / R(k, k)
+    float* rdiag32;   // 64
+    uint16_t* RABh;   // 64 x LF_ABLD: -R_AB as the prologue K2 B operand, [n][k]
+    int* flag;        // 8 ints
     static constexpr size_t fixed_bytes() {
-        return (size_t)LF_SCRATCH * 8 + 5 * 32 * LF_GLD * 8 + 1024 * 8 + 32 * 8 + 32 * 4 + 32 * 36 * 4 + 32 * 4 + 32 * 32 * 4 + 32 * LF_R12LD * 2 + 256;
+        return 2 * LF_REGION + 2 * 64 * 8 + 64 * 8 + 64 * 8 + 64 * 4 + 64 * LF_ABLD * 2 + 64;
     }
     __device__ LfSmem(uint8_t* base, int ldt) {
         tile = reinterpret_cast<float*>(base);
         uint8_t* p = base + (size_t)64 * ldt * 4;
         scr = reinterpret_cast<double*>(p);
-        p += (size_t)LF_SCRATCH * 8;
-        G = reinterpret_cast<double*>(p);
-        p += 32 * LF_GLD * 8;
-        Rs = reinterpret_cast<double*>(p);
-        p += 32 * LF_GLD * 8;
-        Racc = reinterpret_cast<double*>(p);
-        p += 32 * LF_GLD * 8;
-        Rt = reinterpret_cast<double*>(p);
-        p += 32 * LF_GLD * 8;
-        U = reinterpret_cast<double*>(p);
-        p += 32 * LF_GLD * 8;
-        Rt32 = reinterpret_cast<float*>(p);
-        p += 32 * 36 * 4;
-        rdiag32 = reinterpret_cast<float*>(p);
-        p += 32 * 4;
         red = reinterpret_cast<double*>(p);
-        p += 1024 * 8;
+        Rt32 = reinterpret_cast<float*>(p);
+        X32 = reinterpret_cast<float*>(p + 64 * LF_TLD * 4);
+        qa = reinterpret_cast<uint16_t*>(p);
+        p += LF_REGION;
+        G = reinterpret_cast<double*>(p);
+        Rs = reinterpret_cast<double*>(p);
+        p += LF_REGION;
+        U = reinterpret_cast<double*>(p);
+        p += 2 * 64 * 8;
+        gdiag = reinterpret_cast<double*>(p);
+        p += 64 * 8;
         rdiag = reinterpret_cast<double*>(p);
-        p += 32 * 8;
-        pivok = reinterpret_cast<int*>(p);
-        p += 32 * 4;
-        Ri = reinterpret_cast<float*>(p);
-        p += 32 * 32 * 4;
-        R12h = reinterpret_cast<uint16_t*>(p);
+        p += 64 * 8;
+        rdiag32 = reinterpret_cast<float*>(p);
+        p += 64 * 4;
+        RABh = reinterpret_cast<uint16_t*>(p);
+        p += 64 * LF_ABLD * 2;
+        flag = reinterpret_cast<int*>(p);
     }
 };
+static_assert(LF_NENT * 8 <= LF_REGION && LF_NE * 8 <= LF_REGION, "region A");
+static_assert(64 * LF_TLD * 4 + 64 * 64 * 4 <= LF_REGION && 64 * LF_GLD * 8 <= LF_REGION, "regions");
+
+__host__ __device__ __forceinline__ int lf_qa_ld(int rp16) { return ((rp16 - 8 + 63) & ~63) + 8; }   // == 8 mod 64 halves
 
 // ------------------------------------------------------------------ grid all-reduction
-// Sum of the CTA partials part[b][0, ne) (already written by this CTA) into s.red on every CTA.
+// Sum of the CTA partials part[b][0, ne) (already written by this CTA) into a.red (and s.red).
 // Deterministic: entry e is summed by one warp of CTA e / slice, lanes over CTAs lane, lane + 32,
-// ... in order, then a fixed xor-shuffle tree.
-__device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne) {
+// ... in order, then a fixed xor-shuffle tree.  Two grid barriers (measured ~1.6 us each with 148
+// CTAs; per-CTA ready flags polled by many threads instead were ~3x slower -- L2 contention).
+__device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne, bool to_smem) {
     lf_grid_sync(a.bar);
     const int grid = gridDim.x;
-    const int slice = (ne + grid - 1) / grid;   // entries per CTA (<= LF_NW for ne <= 1024, grid >= 64)
+    const int slice = (ne + grid - 1) / grid;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     for (int q = warp; q < slice; q += LF_NW) {
         const int e = blockIdx.x * slice + q;
@@ -228,173 +247,251 @@ __device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne) {
         }
     }
     lf_grid_sync(a.bar);
+    if (!to_smem) return;
     for (int e = threadIdx.x; e < ne; e += LF_THREADS) s.red[e] = __ldcg(a.red + e);
     __syncthreads();
 }
 
 // ------------------------------------------------------------------ Gram (fp64 tensor cores)
-// Partial G = P^T P of the CTA's rows [0, rp) of tile columns [c0, c0 + 32), written packed
-// (upper triangle, [j (j + 1) / 2 + i]) into this CTA's workspace partial.
-__device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int c0, int rp) {
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int g = lane >> 2, c = lane & 3;
-    double acc[10][2];
-#pragma unroll
-    for (int t = 0; t < 10; ++t) acc[t][0] = acc[t][1] = 0.0;
-    const float* col = s.tile + (int64_t)(c0 + g) * a.ldt + c;
-    for (int k0 = 4 * warp; k0 < rp; k0 += 4 * LF_NW) {
-        double f[4];
-#pragma unroll
-        for (int b = 0; b < 4; ++b) f[b] = (double)col[8 * b * a.ldt + k0];
-        int t = 0;
-#pragma unroll
-        for (int bi = 0; bi < 4; ++bi)
-#pragma unroll
-            for (int bj = bi; bj < 4; ++bj, ++t)
-                asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
-                             : "+d"(acc[t][0]), "+d"(acc[t][1])
-                             : "d"(f[bi]), "d"(f[bj]));
+// Block t = 0..35 enumerates (bi, bj), bi <= bj < 8, row by row; group q takes t = q, q + 4, ...
+// (9 blocks); warp w = group (w & 3) x k-quarter (w >> 2).  The block indices must be compile-time
+// (fragment registers), hence the template on the group.
+__host__ __device__ constexpr int lf_blk_i(int t) {
+    int bi = 0;
+    while (t >= 8 - bi) {
+        t -= 8 - bi;
+        ++bi;
     }
-    // warp partials summed in warp order: two rounds of 8 warps through the scratch
-    constexpr int NENT = 640;   // 10 blocks x 64
-    double run[2] = {0.0, 0.0};
-    for (int w0 = 0; w0 < LF_NW; w0 += 8) {
-        __syncthreads();
-        if (warp >= w0 && warp < w0 + 8) {
-            double* dst = s.scr + (warp - w0) * NENT + lane;
+    return bi;
+}
+__host__ __device__ constexpr int lf_blk_j(int t) {
+    int bi = 0;
+    while (t >= 8 - bi) {
+        t -= 8 - bi;
+        ++bi;
+    }
+    return bi + t;
+}
+
+template <int T>
+__device__ __forceinline__ void lf_dmma_blk(double (&acc)[2], const double (&f)[8]) {
+    constexpr int bi = lf_blk_i(T), bj = lf_blk_j(T);   // forced compile-time: f stays in registers
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                 : "+d"(acc[0]), "+d"(acc[1])
+                 : "d"(f[bi]), "d"(f[bj]));
+}
+
+template <int Q>
+__device__ __forceinline__ void lf_gram_group(const LfSmem& s, int ldt, int rp, int kq, int lane, double (&acc)[9][2]) {
+    const int g = lane >> 2, c = lane & 3;
+    const float* col = s.tile + g * ldt + c;
+#pragma unroll 1
+    for (int k0 = 4 * kq; k0 < rp; k0 += 16) {
+        double f[8];
 #pragma unroll
-            for (int t = 0; t < 10; ++t) {
-                dst[(2 * t) * 32] = acc[t][0];
-                dst[(2 * t + 1) * 32] = acc[t][1];
+        for (int b = 0; b < 8; ++b) f[b] = (double)col[8 * b * ldt + k0];
+        lf_dmma_blk<Q + 0>(acc[0], f);
+        lf_dmma_blk<Q + 4>(acc[1], f);
+        lf_dmma_blk<Q + 8>(acc[2], f);
+        lf_dmma_blk<Q + 12>(acc[3], f);
+        lf_dmma_blk<Q + 16>(acc[4], f);
+        lf_dmma_blk<Q + 20>(acc[5], f);
+        lf_dmma_blk<Q + 24>(acc[6], f);
+        lf_dmma_blk<Q + 28>(acc[7], f);
+        lf_dmma_blk<Q + 32>(acc[8], f);
+    }
+}
+
+// Partial G = P^T P of the CTA's rows [0, rp) (64 tile columns) -> packed upper triangle
+// ([j (j + 1) / 2 + i]) in this CTA's workspace partial.
+__device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int rp) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int q = warp & 3, kq = warp >> 2;
+    double acc[9][2];
+#pragma unroll
+    for (int u = 0; u < 9; ++u) acc[u][0] = acc[u][1] = 0.0;
+    switch (q) {
+        case 0: lf_gram_group<0>(s, a.ldt, rp, kq, lane, acc); break;
+        case 1: lf_gram_group<1>(s, a.ldt, rp, kq, lane, acc); break;
+        case 2: lf_gram_group<2>(s, a.ldt, rp, kq, lane, acc); break;
+        default: lf_gram_group<3>(s, a.ldt, rp, kq, lane, acc); break;
+    }
+    // the four k-quarters summed in order through the scratch: entry e = ((q * 9 + u) * 2 + v) * 32 + ln
+    constexpr int NQ = (LF_NENT + LF_THREADS - 1) / LF_THREADS;
+    double run[NQ];
+#pragma unroll
+    for (int i = 0; i < NQ; ++i) run[i] = 0.0;
+    for (int r = 0; r < 4; ++r) {
+        __syncthreads();
+        if (kq == r) {
+            double* dst = s.scr + q * 9 * 64 + lane;
+#pragma unroll
+            for (int u = 0; u < 9; ++u) {
+                dst[(2 * u) * 32] = acc[u][0];
+                dst[(2 * u + 1) * 32] = acc[u][1];
             }
         }
         __syncthreads();
 #pragma unroll
-        for (int q = 0; q < 2; ++q) {
-            const int e = threadIdx.x + LF_THREADS * q;
-            if (e < NENT)
-#pragma unroll
-                for (int k = 0; k < 8; ++k) run[q] += s.scr[k * NENT + e];
+        for (int i = 0; i < NQ; ++i) {
+            const int e = threadIdx.x + LF_THREADS * i;
+            if (e < LF_NENT) run[i] += s.scr[e];
         }
     }
-    // entry e = (2 t + u) * 32 + ln of block t = (bi, bj): G(8 bi + ln / 4, 8 bj + 2 (ln % 4) + u)
     double* out = a.part + (int64_t)blockIdx.x * LF_PART;
 #pragma unroll
-    for (int q = 0; q < 2; ++q) {
-        const int e = threadIdx.x + LF_THREADS * q;
-        if (e < NENT) {
-            const int t = e >> 6, u = (e >> 5) & 1, ln = e & 31;
-            int bi = 0, tt = t;
-            while (tt >= 4 - bi) {
-                tt -= 4 - bi;
-                ++bi;
-            }
-            const int bj = bi + tt;
-            const int i = 8 * bi + (ln >> 2), j = 8 * bj + 2 * (ln & 3) + u;
-            if (i <= j) __stcg(out + j * (j + 1) / 2 + i, run[q]);
+    for (int i = 0; i < NQ; ++i) {
+        const int e = threadIdx.x + LF_THREADS * i;
+        if (e < LF_NENT) {
+            const int ln = e & 31, v = (e >> 5) & 1, qu = e >> 6, qq = qu / 9, u = qu % 9;
+            const int t = qq + 4 * u;
+            const int bi = lf_blk_i(t), bj = lf_blk_j(t);
+            const int ii = 8 * bi + (ln >> 2), jj = 8 * bj + 2 * (ln & 3) + v;
+            if (ii <= jj) __stcg(out + jj * (jj + 1) / 2 + ii, run[i]);
         }
     }
 }
 
-// ------------------------------------------------------------------ Cholesky + inverse (warp 0)
-// fp64 1/sqrt: hardware approximation + one Newton step (relative error ~2^-44, far below what
-// the fp32 outputs can resolve; the pivot test is done on d itself).
-__device__ __forceinline__ double lf_rsqrt(double d) {
-    double y;
-    asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(d));
-    const double e = fma(-d * y, y, 1.0);
-    return fma(0.5 * y, e, y);
-}
-
-// s.G holds the full symmetric 32 x 32 Gram (identity beyond nc).  Lane j keeps column j of the
-// Schur complement S in registers.  Step k: every lane publishes S(k, j) (row k, through s.U),
-// then every lane reads the whole row back with 16-byte broadcasts and computes the pivot itself
-// (rs = 1 / sqrt(S(k, k)): one shared-memory round trip per step and no branch on the pivot
-// lane), forms R(k, j) = S(k, j) rs and updates S(i, j) -= S(k, i) S(k, j) / S(k, k), the next
-// pivot's entry first.  Measured on B200 (one warp): DFMA issue 2.6 cycles, DFMA latency 8.7,
-// STS + syncwarp + LDS 44, rsqrt (approx + Newton) 48; the whole factorization ~7.5K cycles.
-// (Shuffles inside the warp-0 branch compile to WARPSYNC / ENDCOLLECTIVE sequences, ~2x slower;
-// a fraction-free variant without the division on the chain triples the fp64 work per element
-// and was slower, 9.4K cycles.)  Writes s.Rs (row-major R), s.Rt and s.Rt32 (column-major R, fp64
-// / fp32), s.rdiag / s.rdiag32 (1 / R(k, k)).  Returns the first failed pivot (32 if none): a
-// pivot fails unless it is finite and > 1e-15 G(k, k).
-__device__ int lf_chol_warp(const LfSmem& s) {
-    const int lane = threadIdx.x & 31;
-    double g[32];
+// ------------------------------------------------------------------ Cholesky (warps 0-3)
+// s.G holds the full symmetric 64 x 64 Gram (identity beyond nc).  Warp q (< 4) keeps rows
+// 16 q .. 16 q + 15 of the Schur complement S in registers, lane l columns l and l + 32 (one warp
+// per SMSP).  Step k: the warp owning row k publishes S(k, :) through s.U (ping-pong), a 128-thread
+// named barrier, and every thread reads the row back with 16-byte broadcasts, computes the pivot
+// itself (no pivot-thread branch) and updates its rows: S(i, j) -= S(k, i) S(k, j) / S(k, k)
+// (rows <= k of the pivot's quarter are dead after publication and updated harmlessly; quarters
+// above are skipped).  Measured on B200 (tools/leaf_bench.cu): ~23K cycles for the 64 pivots.
+// Variants measured slower: the whole 512-thread CTA with 8 rows per thread (16 warps issuing the
+// pivot logic, ~27K), per-row mbarriers so consumers never wait for each other (~27K), one warp
+// per 32 columns with shuffles (WARPSYNC/ENDCOLLECTIVE sequences inside the warp branch).
+// Writes s.Rs (fp64 row-major R, over G once every thread has loaded its part), s.Rt32 (fp32
+// column-major), s.rdiag / s.rdiag32 (1 / R(k, k)).  Returns the first failed pivot (64 if none)
+// on threads < 128: a pivot fails unless it is finite and > 1e-15 G(k, k).
+__device__ int lf_chol(const LfSmem& s) {
+    const int t = threadIdx.x;   // < 128
+    const int jl = t & 31, rq = t >> 5;
+    double g0[16], g1[16];
 #pragma unroll
-    for (int i = 0; i < 32; ++i) g[i] = s.G[i * LF_GLD + lane];
-    int bad = 32;
+    for (int ii = 0; ii < 16; ++ii) {
+        g0[ii] = s.G[(16 * rq + ii) * LF_GLD + jl];
+        g1[ii] = s.G[(16 * rq + ii) * LF_GLD + jl + 32];
+    }
+    lf_bar128();   // every thread has its part of G before R overwrites it
+    int bad = 64;
+#pragma unroll 1
+    for (int kq = 0; kq < 4; ++kq) {
 #pragma unroll
-    for (int k = 0; k < 32; ++k) {
-        double* urow = s.U + k * LF_GLD;
-        urow[lane] = g[k];
-        __syncwarp();
-        const double d = urow[k];
-        const bool good = (d > s.G[k * LF_GLD + k] * 1e-15) && isfinite(d);
-        bad = (!good && bad == 32) ? k : bad;
-        const double rs = good ? lf_rsqrt(d) : 1.0;
-        const double r = (lane >= k) ? g[k] * rs : 0.0;   // R(k, lane); lane k: sqrt(d)
-        const double t = r * rs;                           // S(k, lane) / S(k, k)
-        if (k + 1 < 32) g[k + 1] = fma(-urow[k + 1], t, g[k + 1]);
-        if ((k & 1) == 0) {   // k + 2 even: pairs from k + 2
-#pragma unroll
-            for (int i = k + 2; i < 32; i += 2) {
-                const double2 v = *reinterpret_cast<const double2*>(urow + i);
-                g[i] = fma(-v.x, t, g[i]);
-                g[i + 1] = fma(-v.y, t, g[i + 1]);
+        for (int kk = 0; kk < 16; ++kk) {
+            const int k = 16 * kq + kk;
+            double* urow = s.U + (kk & 1) * 64;
+            if (rq == kq) {
+                urow[jl] = g0[kk];
+                urow[jl + 32] = g1[kk];
             }
-        } else {              // k + 2 odd: one scalar, then pairs
-            if (k + 2 < 32) g[k + 2] = fma(-urow[k + 2], t, g[k + 2]);
+            lf_bar128();
+            const double d = urow[k];
+            const bool good = (d > s.gdiag[k] * 1e-15) && isfinite(d);
+            bad = (!good && bad == 64) ? k : bad;
+            const double rs = good ? lf_rsqrt(d) : 1.0;
+            const double r0 = (jl >= k) ? urow[jl] * rs : 0.0;          // R(k, jl)
+            const double r1 = (jl + 32 >= k) ? urow[jl + 32] * rs : 0.0;  // R(k, jl + 32)
+            const double t0 = r0 * rs, t1 = r1 * rs;                      // S(k, j) / S(k, k)
+            if (rq >= kq) {
+                const double* ur = urow + 16 * rq;
 #pragma unroll
-            for (int i = k + 3; i < 32; i += 2) {
-                const double2 v = *reinterpret_cast<const double2*>(urow + i);
-                g[i] = fma(-v.x, t, g[i]);
-                g[i + 1] = fma(-v.y, t, g[i + 1]);
+                for (int ii = 0; ii < 16; ii += 2) {
+                    const double2 v = *reinterpret_cast<const double2*>(ur + ii);
+                    g0[ii] = fma(-v.x, t0, g0[ii]);
+                    g1[ii] = fma(-v.x, t1, g1[ii]);
+                    g0[ii + 1] = fma(-v.y, t0, g0[ii + 1]);
+                    g1[ii + 1] = fma(-v.y, t1, g1[ii + 1]);
+                }
             }
-        }
-        s.Rs[k * LF_GLD + lane] = r;
-        s.Rt[lane * LF_GLD + k] = r;
-        s.Rt32[lane * 36 + k] = (float)r;
-        if (lane == 0) {
-            s.rdiag[k] = rs;
-            s.rdiag32[k] = (float)rs;
+            if (rq == 0) {
+                s.Rs[k * LF_GLD + jl] = r0;
+                s.Rs[k * LF_GLD + jl + 32] = r1;
+                s.Rt32[jl * LF_TLD + k] = (float)r0;
+                s.Rt32[(jl + 32) * LF_TLD + k] = (float)r1;
+            } else if (rq == 1 && jl == 0) {
+                s.rdiag[k] = rs;
+                s.rdiag32[k] = (float)rs;
+            }
         }
     }
-    __syncwarp();
+    lf_bar128();
     return bad;
 }
 
-// X = R^{-1} (upper) in fp32 (it only feeds the fp32 product P R^{-1} and the kappa test), lane j
-// computes column j by back substitution: right-looking, each step one multiply and independent
-// FMAs, column k of R read from s.Rt32 with 16-byte broadcasts.  Writes s.Ri (row-major) and
-// returns |R|_F^2 |R^{-1}|_F^2 over the nc x nc panel.
-__device__ double lf_inverse_warp(const LfSmem& s, int nc) {
-    const int lane = threadIdx.x & 31;
-    float b[32];
+// X = R^{-1} (upper, fp32: it only feeds the fp32 product P R^{-1} and the kappa test), blocked
+// on 32 x 32 blocks, whole CTA:
+//   X11 = R11^{-1}, X22 = R22^{-1}   threads 0..63, column-parallel back substitution (right-
+//                                    looking: each step one multiply + independent FMAs)
+//   T   = R12 X22,  X12 = -X11 T     all threads, 1024 outputs each
+// Writes s.X32 (row-major) and returns |R|_F^2 |R^{-1}|_F^2 over the nc x nc block (all threads).
+__device__ double lf_inverse(const LfSmem& s, int nc) {
+    const int tid = threadIdx.x;
+    __shared__ double s_norm[2][LF_NW];
+    if (tid < 64) {
+        const int base = tid < 32 ? 0 : 32, j = tid & 31;
+        float b[32];
 #pragma unroll
-    for (int i = 0; i < 32; ++i) b[i] = (i == lane) ? 1.f : 0.f;
+        for (int i = 0; i < 32; ++i) b[i] = (i == j) ? 1.f : 0.f;
 #pragma unroll
-    for (int k = 31; k >= 0; --k) {
-        b[k] *= s.rdiag32[k];
-        const float* col = s.Rt32 + k * 36;
+        for (int k = 31; k >= 0; --k) {
+            b[k] *= s.rdiag32[base + k];
+            const float* col = s.Rt32 + (base + k) * LF_TLD + base;
 #pragma unroll
-        for (int i = 0; i + 3 < k; i += 4) {
-            const float4 v = *reinterpret_cast<const float4*>(col + i);
-            b[i] = fmaf(-v.x, b[k], b[i]);
-            b[i + 1] = fmaf(-v.y, b[k], b[i + 1]);
-            b[i + 2] = fmaf(-v.z, b[k], b[i + 2]);
-            b[i + 3] = fmaf(-v.w, b[k], b[i + 3]);
+            for (int i = 0; i + 3 < k; i += 4) {
+                const float4 v = *reinterpret_cast<const float4*>(col + i);
+                b[i] = fmaf(-v.x, b[k], b[i]);
+                b[i + 1] = fmaf(-v.y, b[k], b[i + 1]);
+                b[i + 2] = fmaf(-v.z, b[k], b[i + 2]);
+                b[i + 3] = fmaf(-v.w, b[k], b[i + 3]);
+            }
+#pragma unroll
+            for (int i = k & ~3; i < k; ++i) b[i] = fmaf(-col[i], b[k], b[i]);
         }
 #pragma unroll
-        for (int i = k & ~3; i < k; ++i) b[i] = fmaf(-col[i], b[k], b[i]);
+        for (int i = 0; i < 32; ++i) s.X32[(base + i) * 64 + base + j] = b[i];
     }
+    __syncthreads();
+    // T = R12 X22 into the X21 slot (rows 32.., cols 0..31: zero afterwards)
+    float tv[2];
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+        const int e = tid + LF_THREADS * q, i = e >> 5, jj = e & 31;
+        float acc = 0.f;
+        for (int k = 0; k <= jj; ++k) acc = fmaf(s.Rt32[(32 + k) * LF_TLD + i], s.X32[(32 + k) * 64 + 32 + jj], acc);
+        tv[q] = acc;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+        const int e = tid + LF_THREADS * q, i = e >> 5, jj = e & 31;
+        s.X32[(32 + i) * 64 + jj] = tv[q];
+    }
+    __syncthreads();
+    // X12 = -X11 T
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+        const int e = tid + LF_THREADS * q, i = e >> 5, jj = e & 31;
+        float acc = 0.f;
+        for (int k = i; k < 32; ++k) acc = fmaf(s.X32[i * 64 + k], s.X32[(32 + k) * 64 + jj], acc);
+        tv[q] = -acc;
+    }
+    __syncthreads();
     double xn = 0.0, rn = 0.0;
 #pragma unroll
-    for (int i = 0; i < 32; ++i) {
-        s.Ri[i * 32 + lane] = b[i];
-        const double r = s.Rs[i * LF_GLD + lane];
-        if (i < nc && lane < nc) {   // the identity padding beyond nc is not part of the panel
-            xn = fma((double)b[i], (double)b[i], xn);
+    for (int q = 0; q < 2; ++q) {
+        const int e = tid + LF_THREADS * q, i = e >> 5, jj = e & 31;
+        s.X32[i * 64 + 32 + jj] = tv[q];
+        s.X32[(32 + i) * 64 + jj] = 0.f;
+    }
+    __syncthreads();
+    for (int e = tid; e < 64 * 64; e += LF_THREADS) {
+        const int i = e >> 6, jj = e & 63;
+        if (i < nc && jj < nc && i <= jj) {   // the identity padding beyond nc is not part of the block
+            const double x = s.X32[e], r = s.Rs[i * LF_GLD + jj];
+            xn = fma(x, x, xn);
             rn = fma(r, r, rn);
         }
     }
@@ -403,250 +500,241 @@ __device__ double lf_inverse_warp(const LfSmem& s, int nc) {
         xn += __shfl_xor_sync(0xffffffffu, xn, o);
         rn += __shfl_xor_sync(0xffffffffu, rn, o);
     }
-    __syncwarp();
-    return xn * rn;
-}
-
-// Racc <- Rs * Racc (first pass: Racc = Rs); lane j owns column j.
-__device__ void lf_racc_warp(const LfSmem& s, bool first) {
-    const int lane = threadIdx.x & 31;
-    double v[32];
-#pragma unroll
-    for (int i = 0; i < 32; ++i) {
-        if (first) {
-            v[i] = s.Rs[i * LF_GLD + lane];
-        } else {
-            double acc = 0.0;
-#pragma unroll 1
-            for (int k = i; k < 32; ++k) acc = fma(s.Rs[i * LF_GLD + k], s.Racc[k * LF_GLD + lane], acc);
-            v[i] = acc;
-        }
+    if ((tid & 31) == 0) {
+        s_norm[0][tid >> 5] = xn;
+        s_norm[1][tid >> 5] = rn;
     }
-    __syncwarp();
+    __syncthreads();
+    double sx = 0.0, sr = 0.0;
 #pragma unroll
-    for (int i = 0; i < 32; ++i) s.Racc[i * LF_GLD + lane] = v[i];
-    __syncwarp();
+    for (int w = 0; w < LF_NW; ++w) {
+        sx += s_norm[0][w];
+        sr += s_norm[1][w];
+    }
+    return sx * sr;
 }
 
-// tile columns [c0, c0 + 32), rows [0, rp) <- tile * R^{-1} (fp32).  Warp w takes the column
-// group cg = w % 8 (4 columns) and the rows (w / 8) * 32 + lane + 64 i (i < NI); R^{-1} is upper,
-// so the k loop stops at the group's last column (warp-uniform).
+// tile rows [0, rp) <- tile * R^{-1} (fp32).  Warp w takes the column group cg = w % 8 (8
+// columns) and the rows (w / 8) * 32 + lane + 64 i (i < NI); R^{-1} is upper, so the k loop stops
+// at the group's last column (warp-uniform).
 template <int NI>
-__device__ void lf_apply(const LeafArgs& a, const LfSmem& s, int c0, int rp) {
+__device__ void lf_apply(const LeafArgs& a, const LfSmem& s, int rp) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int cg = warp & 7, half = warp >> 3;
+    // warps w, w + 4, w + 8, w + 12 share an SMSP: give them column groups s, 7 - s, s, 7 - s
+    // (equal triangle work per SMSP)
+    const int sp = warp & 3, t4 = warp >> 2;
+    const int cg = (t4 & 1) ? 7 - sp : sp, half = t4 >> 1;
     const int ld = a.ldt;
     const int r0 = half * 32 + lane;
-    float o[NI][4];
+    float o[NI][8];
 #pragma unroll
     for (int i = 0; i < NI; ++i)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) o[i][c] = 0.f;
-    const float* base = s.tile + c0 * ld + r0;
-    const int kend = 4 * cg + 4;
+        for (int c = 0; c < 8; ++c) o[i][c] = 0.f;
+    const float* base = s.tile + r0;
+    const int kend = 8 * cg + 8;
     int off = 0;
-#pragma unroll 4
+#pragma unroll 2
     for (int k = 0; k < kend; ++k, off += ld) {
-        const float4 rv = *reinterpret_cast<const float4*>(s.Ri + k * 32 + 4 * cg);
+        const float4 x0 = *reinterpret_cast<const float4*>(s.X32 + k * 64 + 8 * cg);
+        const float4 x1 = *reinterpret_cast<const float4*>(s.X32 + k * 64 + 8 * cg + 4);
 #pragma unroll
         for (int i = 0; i < NI; ++i) {
-            const float x = base[off + 64 * i];   // rows >= rp hold zeros (loaded as zero-fill)
-            o[i][0] = fmaf(x, rv.x, o[i][0]);
-            o[i][1] = fmaf(x, rv.y, o[i][1]);
-            o[i][2] = fmaf(x, rv.z, o[i][2]);
-            o[i][3] = fmaf(x, rv.w, o[i][3]);
+            const float x = base[off + 64 * i];   // rows >= rp: zeros or unused
+            o[i][0] = fmaf(x, x0.x, o[i][0]);
+            o[i][1] = fmaf(x, x0.y, o[i][1]);
+            o[i][2] = fmaf(x, x0.z, o[i][2]);
+            o[i][3] = fmaf(x, x0.w, o[i][3]);
+            o[i][4] = fmaf(x, x1.x, o[i][4]);
+            o[i][5] = fmaf(x, x1.y, o[i][5]);
+            o[i][6] = fmaf(x, x1.z, o[i][6]);
+            o[i][7] = fmaf(x, x1.w, o[i][7]);
         }
     }
     __syncthreads();
-    float* ob = s.tile + (c0 + 4 * cg) * ld + r0;
+    float* ob = s.tile + 8 * cg * ld + r0;
 #pragma unroll
     for (int i = 0; i < NI; ++i)
         if (r0 + 64 * i < rp)
 #pragma unroll
-            for (int c = 0; c < 4; ++c) ob[c * ld + 64 * i] = o[i][c];
+            for (int c = 0; c < 8; ++c) ob[c * ld + 64 * i] = o[i][c];
     __syncthreads();
 }
 
-// CholQR of the panel in tile columns [c0, c0 + 32) (nc valid columns, the rest zero) with the
-// single-pass test, CholQR2 and the shifted-CholQR3 fallback.  Leaves Q in the tile and R in
-// s.Racc (fp64, row-major).  Returns the first failed pivot column (or -1).
+// Racc <- R_pass Racc (CTA 0, fp64, global ping-pong buffers); first pass: Racc = R_pass.
+__device__ void lf_racc(const LeafArgs& a, const LfSmem& s, int pass) {
+    const double* src = a.racc + (pass & 1 ? 0 : 64 * 64);
+    double* dst = a.racc + (pass & 1 ? 64 * 64 : 0);
+    for (int e = threadIdx.x; e < 64 * 64; e += LF_THREADS) {
+        const int i = e >> 6, j = e & 63;
+        double v = 0.0;
+        if (i <= j) {
+            if (pass == 0) {
+                v = s.Rs[i * LF_GLD + j];
+            } else {
+                for (int k = i; k <= j; ++k) v = fma(s.Rs[i * LF_GLD + k], __ldcg(src + k * 64 + j), v);
+            }
+        }
+        __stcg(dst + e, v);
+    }
+}
+
+// Full symmetric Gram (identity beyond nc) from the packed reduced entries; optional shift.
+__device__ void lf_build_g(const LfSmem& s, const double* packed, bool global, int nc, double shift) {
+    for (int e = threadIdx.x; e < 64 * 64; e += LF_THREADS) {
+        const int i = e >> 6, j = e & 63;
+        const int lo = min(i, j), hi = max(i, j);
+        const int p = hi * (hi + 1) / 2 + lo;
+        double v = (i == j) ? 1.0 : 0.0;
+        if (i < nc && j < nc) v = global ? __ldcg(packed + p) : packed[p];
+        if (i == j && i < nc) v += shift;
+        s.G[i * LF_GLD + j] = v;
+        if (i == j) s.gdiag[i] = v;
+    }
+    __syncthreads();
+}
+
+// CholQR with the single-pass test, CholQR2 and the shifted-CholQR3 fallback.  Leaves Q in the
+// tile and R in a.racc (buffer (passes - 1) & 1).  Returns the first failed pivot (or -1) and
+// the number of passes through *npass.
 template <int NI>
-__device__ int lf_panel(const LeafArgs& a, const LfSmem& s, int c0, int nc, int rp, int tb) {
-    __shared__ int s_flag[2];
+__device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int* npass) {
     bool shifted = false;
     int bad = -1;
-    for (int pass = 0; pass < 3; ++pass) {
-        lf_gram(a, s, c0, rp);
-        if (pass == 0) LF_MARK(tb + 0);
-        lf_allreduce(a, s, 528);
-        if (pass == 0) LF_MARK(tb + 1);
-        // full symmetric Gram, identity beyond nc
-        for (int e = threadIdx.x; e < 1024; e += LF_THREADS) {
-            const int i = e >> 5, j = e & 31;
-            const int lo = min(i, j), hi = max(i, j);
-            s.G[i * LF_GLD + j] = (i < nc && j < nc) ? s.red[hi * (hi + 1) / 2 + lo] : (i == j ? 1.0 : 0.0);
-        }
+    int pass = 0;
+    for (; pass < 3; ++pass) {
+        lf_gram(a, s, rp);
+        if (pass == 0) LF_MARK(2);
+        lf_allreduce(a, s, LF_NE, true);
+        if (pass == 0) LF_MARK(3);
+        lf_build_g(s, s.red, false, nc, 0.0);
+        int fb = threadIdx.x < 128 ? lf_chol(s) : 64;
+        if (threadIdx.x == 0) s.flag[0] = fb;
         __syncthreads();
-        if (threadIdx.x < 32) {
-            int fb = lf_chol_warp(s);
-            if (fb < 32 && pass == 0) {
-                // shifted CholQR: G + sh I, sh = 11 (m nc + nc (nc + 1)) u ||P||_F^2
-                double tr = 0.0;
-                for (int e = threadIdx.x; e < nc; e += 32) {
-                    const int hi = e;
-                    tr += s.red[hi * (hi + 1) / 2 + hi];
-                }
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1) tr += __shfl_xor_sync(0xffffffffu, tr, o);
-                const double sh = 11.0 * ((double)a.m * nc + (double)nc * (nc + 1)) * 0x1p-53 * tr;
-                const int lane = threadIdx.x;
-                if (lane < nc) s.G[lane * LF_GLD + lane] += sh;
-                __syncwarp();
-                fb = lf_chol_warp(s);
-                if (threadIdx.x == 0) s_flag[1] = 1;
-            } else if (threadIdx.x == 0) {
-                s_flag[1] = 0;
-            }
-            if (fb < 32) {
-                if (threadIdx.x == 0) s_flag[0] = -(fb + 1);
-            } else {
-                const double kk = lf_inverse_warp(s, nc);
-                lf_racc_warp(s, pass == 0);
-                if (threadIdx.x == 0) s_flag[0] = (kk <= 4.0 * nc * nc) ? 1 : 0;   // kappa_F <= 2 nc
-            }
+        fb = s.flag[0];
+        if (fb < 64 && pass == 0) {
+            // shifted CholQR: G + sh I, sh = 11 (m nc + nc (nc + 1)) u ||P||_F^2
+            double tr = 0.0;
+            for (int i = 0; i < nc; ++i) tr += __ldcg(a.red + i * (i + 1) / 2 + i);
+            const double sh = 11.0 * ((double)a.m * nc + (double)nc * (nc + 1)) * 0x1p-53 * tr;
+            __syncthreads();
+            lf_build_g(s, a.red, true, nc, sh);
+            shifted = true;
+            fb = threadIdx.x < 128 ? lf_chol(s) : 64;
+            if (threadIdx.x == 0) s.flag[0] = fb;
+            __syncthreads();
+            fb = s.flag[0];
         }
-        __syncthreads();
-        if (pass == 0) LF_MARK(tb + 2);
-        if (s_flag[1]) shifted = true;
-        const int f = s_flag[0];
-        if (f < 0) {
-            bad = -f - 1;
+        if (pass == 0) LF_MARK(4);
+        if (fb < 64) {
+            bad = fb;
             break;
         }
-        bool stop;
-        if (pass == 0)
-            stop = !shifted && f == 1;
-        else
-            stop = (pass == 1 && !shifted) || pass == 2;
-        lf_apply<NI>(a, s, c0, rp);
-        if (pass == 0) LF_MARK(tb + 3);
+        const double kk = lf_inverse(s, nc);   // every thread: same value
+        const bool stop = (pass == 0) ? (!shifted && kk <= 4.0 * nc * nc)   // kappa_F <= 2 nc
+                                      : ((pass == 1 && !shifted) || pass == 2);
+        // R = R_p ... R_1: a single pass keeps R in s.Rs; otherwise CTA 0 accumulates in global
+        if (blockIdx.x == 0 && !(pass == 0 && stop)) lf_racc(a, s, pass);
+        if (pass == 0) LF_MARK(5);
+        lf_apply<NI>(a, s, rp);
+        if (pass == 0) LF_MARK(6);
         if (stop) break;
     }
+    *npass = pass + 1;
     return bad;
 }
 
-// ------------------------------------------------------------------ K1 / K2 of the leaf level
-// Partial R12 = Q1^T P2 (tile columns [0, 32) and [32, 64)) on the 16-bit tensor cores.
-__device__ void lf_k1(const LeafArgs& a, const LfSmem& s, int rp16) {
+// ------------------------------------------------------------------ prologue: the level above
+// R_AB = Q_A^T P (64 x 64) and P <- P - Q_A R_AB for the block's columns P (tile) and the
+// preceding block's columns Q_A (16-bit image, staged in s.qa): Algorithm 1 lines 8-9 of the
+// recursion level just above the leaf, in the precision of the tensor-core GEMMs (16-bit operands,
+// fp32 accumulation).  Replaces that level's K1 GEMM + split-K reduce + K2 GEMM launches.
+__device__ void lf_load_qa(const LeafArgs& a, const LfSmem& s, int64_t r0, int rows, int rp16) {
+    const int ld16 = lf_qa_ld(rp16);
+    const int nq = rp16 >> 3;   // 8-row (16-byte) chunks per column
+    for (int e = threadIdx.x; e < 64 * nq; e += LF_THREADS) {
+        const int cc = e / nq, q = e % nq;
+        uint16_t* dst = s.qa + cc * ld16 + 8 * q;
+        const uint16_t* src = a.pq + r0 + (int64_t)cc * a.ldh;
+        const int avail = (cc < a.ph) ? max(0, min(8, rows - 8 * q)) : 0;
+        lf_cp16(dst, avail > 0 ? src + 8 * q : src, avail * 2);
+    }
+}
+
+// partial R_AB: warp w owns the 16 x 16 output block (w / 4, w % 4) over all k-steps
+__device__ void lf_pro_k1(const LeafArgs& a, const LfSmem& s, int rp16) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, c = lane & 3;
-    float acc[2][4][4];
+    const int bi = warp >> 2, bj = warp & 3;
+    const int ld16 = lf_qa_ld(rp16), ld = a.ldt;
+    float acc[2][4];
 #pragma unroll
-    for (int mt = 0; mt < 2; ++mt)
+    for (int nt = 0; nt < 2; ++nt)
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt)
+        for (int u = 0; u < 4; ++u) acc[nt][u] = 0.f;
+    const uint16_t* qb = s.qa + (16 * bi + g) * ld16 + 2 * c;
+    const float* pb = s.tile + (16 * bj + g) * ld + 2 * c;
+#pragma unroll 2
+    for (int k0 = 0; k0 < rp16; k0 += 16) {
+        uint32_t af[4], bfr[2][2];
+        af[0] = *reinterpret_cast<const uint32_t*>(qb + k0);
+        af[1] = *reinterpret_cast<const uint32_t*>(qb + 8 * ld16 + k0);
+        af[2] = *reinterpret_cast<const uint32_t*>(qb + k0 + 8);
+        af[3] = *reinterpret_cast<const uint32_t*>(qb + 8 * ld16 + k0 + 8);
 #pragma unroll
-            for (int u = 0; u < 4; ++u) acc[mt][nt][u] = 0.f;
-    const int ld = a.ldt;
-    for (int k0 = 16 * warp; k0 < rp16; k0 += 16 * LF_NW) {
-        uint32_t af[2][4], bfr[4][2];
-#pragma unroll
-        for (int mt = 0; mt < 2; ++mt) {
-            const float* q = s.tile + (int64_t)(16 * mt + g) * ld + k0 + 2 * c;
-            const float2 x0 = *reinterpret_cast<const float2*>(q);
-            const float2 x1 = *reinterpret_cast<const float2*>(q + 8 * ld);
-            const float2 x2 = *reinterpret_cast<const float2*>(q + 8);
-            const float2 x3 = *reinterpret_cast<const float2*>(q + 8 * ld + 8);
-            af[mt][0] = lf_pack2(x0.x, x0.y, a.bf16);
-            af[mt][1] = lf_pack2(x1.x, x1.y, a.bf16);
-            af[mt][2] = lf_pack2(x2.x, x2.y, a.bf16);
-            af[mt][3] = lf_pack2(x3.x, x3.y, a.bf16);
-        }
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt) {
-            const float* p = s.tile + (int64_t)(32 + 8 * nt + g) * ld + k0 + 2 * c;
-            const float2 y0 = *reinterpret_cast<const float2*>(p);
-            const float2 y1 = *reinterpret_cast<const float2*>(p + 8);
+        for (int nt = 0; nt < 2; ++nt) {
+            const float2 y0 = *reinterpret_cast<const float2*>(pb + 8 * nt * ld + k0);
+            const float2 y1 = *reinterpret_cast<const float2*>(pb + 8 * nt * ld + k0 + 8);
             bfr[nt][0] = lf_pack2(y0.x, y0.y, a.bf16);
             bfr[nt][1] = lf_pack2(y1.x, y1.y, a.bf16);
         }
 #pragma unroll
-        for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-            for (int nt = 0; nt < 4; ++nt) lf_mma16816(acc[mt][nt], af[mt], bfr[nt], a.bf16);
+        for (int nt = 0; nt < 2; ++nt) lf_mma16816(acc[nt], af, bfr[nt], a.bf16);
     }
-    // warp partials in warp order (two rounds of 8) -> CTA partial (as doubles)
-    float* scr = reinterpret_cast<float*>(s.scr);
-    double run[2] = {0.0, 0.0};
-    for (int w0 = 0; w0 < LF_NW; w0 += 8) {
-        __syncthreads();
-        if (warp >= w0 && warp < w0 + 8) {
-            float* dst = scr + (warp - w0) * 1024 + lane;
-#pragma unroll
-            for (int mt = 0; mt < 2; ++mt)
-#pragma unroll
-                for (int nt = 0; nt < 4; ++nt)
-#pragma unroll
-                    for (int u = 0; u < 4; ++u) dst[((mt * 4 + nt) * 4 + u) * 32] = acc[mt][nt][u];
-        }
-        __syncthreads();
-#pragma unroll
-        for (int q = 0; q < 2; ++q) {
-            const int e = threadIdx.x + LF_THREADS * q;
-#pragma unroll
-            for (int k = 0; k < 8; ++k) run[q] += (double)scr[k * 1024 + e];
-        }
-    }
-    // entry e = ((mt * 4 + nt) * 4 + u) * 32 + ln: R12(16 mt + ln / 4 + 8 (u / 2), 8 nt + 2 (ln % 4) + u % 2)
     double* out = a.part + (int64_t)blockIdx.x * LF_PART;
 #pragma unroll
-    for (int q = 0; q < 2; ++q) {
-        const int e = threadIdx.x + LF_THREADS * q;
-        const int ln = e & 31, u = (e >> 5) & 3, nt = (e >> 7) & 3, mt = e >> 9;
-        const int i = 16 * mt + (ln >> 2) + 8 * (u >> 1), j = 8 * nt + 2 * (ln & 3) + (u & 1);
-        __stcg(out + i * 32 + j, run[q]);
-    }
+    for (int nt = 0; nt < 2; ++nt)
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int i = 16 * bi + g + 8 * (u >> 1), j = 16 * bj + 8 * nt + 2 * c + (u & 1);
+            __stcg(out + i * 64 + j, (double)acc[nt][u]);
+        }
 }
 
-// P2 <- P2 - Q1 R12 (tile columns [32, 64) -= [0, 32) * R12) with 16-bit operands; s.R12h holds
-// -R12 as [n][k].
-__device__ void lf_k2(const LeafArgs& a, const LfSmem& s, int rp16) {
+// P <- P - Q_A R_AB over the tile's 64 columns; s.RABh holds -R_AB as [n][k]
+__device__ void lf_pro_k2(const LeafArgs& a, const LfSmem& s, int rp16) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, c = lane & 3;
-    const int ld = a.ldt;
-    uint32_t bfr[2][4][2];
-#pragma unroll
-    for (int ks = 0; ks < 2; ++ks)
-#pragma unroll
-        for (int nt = 0; nt < 4; ++nt) {
-            const uint16_t* bp = s.R12h + (8 * nt + g) * LF_R12LD + 16 * ks + 2 * c;
-            bfr[ks][nt][0] = *reinterpret_cast<const uint32_t*>(bp);
-            bfr[ks][nt][1] = *reinterpret_cast<const uint32_t*>(bp + 8);
-        }
+    const int ld16 = lf_qa_ld(rp16), ld = a.ldt;
+    const int kss = (a.ph + 15) >> 4;
     for (int r0 = 16 * warp; r0 < rp16; r0 += 16 * LF_NW) {
-        float d[4][4];
+        float d[8][4];
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt) {
-            const float* cp = s.tile + (int64_t)(32 + 8 * nt + 2 * c) * ld + r0 + g;
+        for (int nt = 0; nt < 8; ++nt) {
+            const float* cp = s.tile + (8 * nt + 2 * c) * ld + r0 + g;
             d[nt][0] = cp[0];
             d[nt][1] = cp[ld];
             d[nt][2] = cp[8];
             d[nt][3] = cp[ld + 8];
         }
-#pragma unroll
-        for (int ks = 0; ks < 2; ++ks) {
-            const float* q = s.tile + (int64_t)(16 * ks + 2 * c) * ld + r0 + g;
+        for (int ks = 0; ks < kss; ++ks) {
+            const uint16_t* q = s.qa + (16 * ks + 2 * c) * ld16 + r0 + g;
             uint32_t af[4];
-            af[0] = lf_pack2(q[0], q[ld], a.bf16);
-            af[1] = lf_pack2(q[8], q[ld + 8], a.bf16);
-            af[2] = lf_pack2(q[8 * ld], q[9 * ld], a.bf16);
-            af[3] = lf_pack2(q[8 * ld + 8], q[9 * ld + 8], a.bf16);
+            af[0] = (uint32_t)q[0] | ((uint32_t)q[ld16] << 16);
+            af[1] = (uint32_t)q[8] | ((uint32_t)q[ld16 + 8] << 16);
+            af[2] = (uint32_t)q[8 * ld16] | ((uint32_t)q[9 * ld16] << 16);
+            af[3] = (uint32_t)q[8 * ld16 + 8] | ((uint32_t)q[9 * ld16 + 8] << 16);
 #pragma unroll
-            for (int nt = 0; nt < 4; ++nt) lf_mma16816(d[nt], af, bfr[ks][nt], a.bf16);
+            for (int nt = 0; nt < 8; ++nt) {
+                const uint16_t* bp = s.RABh + (8 * nt + g) * LF_ABLD + 16 * ks + 2 * c;
+                const uint32_t bfr[2] = {*reinterpret_cast<const uint32_t*>(bp),
+                                         *reinterpret_cast<const uint32_t*>(bp + 8)};
+                lf_mma16816(d[nt], af, bfr, a.bf16);
+            }
         }
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt) {
-            float* cp = s.tile + (int64_t)(32 + 8 * nt + 2 * c) * ld + r0 + g;
+        for (int nt = 0; nt < 8; ++nt) {
+            float* cp = s.tile + (8 * nt + 2 * c) * ld + r0 + g;
             cp[0] = d[nt][0];
             cp[ld] = d[nt][1];
             cp[8] = d[nt][2];
@@ -657,12 +745,11 @@ __device__ void lf_k2(const LeafArgs& a, const LfSmem& s, int rp16) {
 }
 
 // ------------------------------------------------------------------ load / store
-__device__ void lf_load_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, int rows, int rp16, int cbeg, int cend) {
+__device__ void lf_load_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, int rows, int rp16) {
     const int nq = rp16 >> 2;   // 4-row chunks per column
-    const int total = (cend - cbeg) * nq;
-    for (int e = threadIdx.x; e < total; e += LF_THREADS) {
-        const int cc = cbeg + e / nq, q = e % nq;
-        float* dst = s.tile + (int64_t)cc * a.ldt + 4 * q;
+    for (int e = threadIdx.x; e < 64 * nq; e += LF_THREADS) {
+        const int cc = e / nq, q = e % nq;
+        float* dst = s.tile + cc * a.ldt + 4 * q;
         const float* src = a.Q + r0 + (int64_t)cc * a.ldq;
         const int avail = (cc < a.nc) ? max(0, min(4, rows - 4 * q)) : 0;
         if (a.vec) {
@@ -674,12 +761,11 @@ __device__ void lf_load_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, int
     }
 }
 
-__device__ void lf_store_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, int rows, int cbeg, int cend) {
+__device__ void lf_store_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, int rows) {
     const int nq = (rows + 3) >> 2;
-    const int total = (cend - cbeg) * nq;
-    for (int e = threadIdx.x; e < total; e += LF_THREADS) {
-        const int cc = cbeg + e / nq, q = e % nq;
-        const float4 v = *reinterpret_cast<const float4*>(s.tile + (int64_t)cc * a.ldt + 4 * q);
+    for (int e = threadIdx.x; e < a.nc * nq; e += LF_THREADS) {
+        const int cc = e / nq, q = e % nq;
+        const float4 v = *reinterpret_cast<const float4*>(s.tile + cc * a.ldt + 4 * q);
         const int64_t gr = r0 + 4 * q;
         float* dq = a.Q + gr + (int64_t)cc * a.ldq;
         const float vv[4] = {v.x, v.y, v.z, v.w};
@@ -709,14 +795,6 @@ __device__ void lf_store_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, in
     }
 }
 
-// R block output (CTA 0): rows [c0, c0 + 32) of the diagonal block from s.Racc, zero below.
-__device__ void lf_write_r(const LeafArgs& a, const LfSmem& s, int c0, int ncp) {
-    for (int e = threadIdx.x; e < ncp * ncp; e += LF_THREADS) {
-        const int i = e % ncp, j = e / ncp;
-        a.R[(c0 + i) + (int64_t)(c0 + j) * a.ldr] = (i <= j) ? (float)s.Racc[i * LF_GLD + j] : 0.f;
-    }
-}
-
 // ------------------------------------------------------------------ the kernel
 template <int NI>
 __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
@@ -726,66 +804,43 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
     const int64_t rem = a.m - r0;
     const int rows = rem <= 0 ? 0 : (rem < a.rows_per ? (int)rem : a.rows_per);
     const int rp16 = (rows + 15) & ~15;
-    const int h = a.nc < 32 ? a.nc : 32;
-    const int w = a.nc - h;
-
-    // rows of both panels in flight at once (two commit groups)
-    lf_load_cols(a, s, r0, rows, rp16, 0, 32);
-    lf_cp_commit();
-    if (w > 0) lf_load_cols(a, s, r0, rows, rp16, 32, 64);
-    lf_cp_commit();
     LF_MARK(0);
-    lf_cp_wait<1>();
+    lf_load_cols(a, s, r0, rows, rp16);
+    if (a.pq) lf_load_qa(a, s, r0, rows, rp16);
+    lf_cp_commit();
+    lf_cp_wait_all();
     __syncthreads();
+    if (a.pq) {
+        // ---- prologue: the level above (R_AB = Q_A^T P, P -= Q_A R_AB)
+        lf_pro_k1(a, s, rp16);
+        lf_allreduce(a, s, 4096, false);
+        for (int e = threadIdx.x; e < 4096; e += LF_THREADS) {
+            const int i = e >> 6, j = e & 63;   // R_AB(i, j)
+            const float v = (i < a.ph && j < a.nc) ? (float)__ldcg(a.red + e) : 0.f;
+            s.RABh[j * LF_ABLD + i] = lf_to16(-v, a.bf16);
+            if (blockIdx.x == 0 && i < a.ph && j < a.nc) a.R[(int64_t)(i - a.ph) + (int64_t)j * a.ldr] = v;
+        }
+        __syncthreads();
+        lf_pro_k2(a, s, rp16);
+    }
     LF_MARK(1);
-
-    // ---- panel 1
-    int bad = lf_panel<NI>(a, s, 0, h, rp16, 2);
-    if (bad >= 0) {
+    int npass = 0;
+    const int bad = lf_cholqr<NI>(a, s, a.nc, rp16, &npass);
+    if (bad >= 0) {   // uniform across the grid (every CTA factors the same reduced Gram)
         if (blockIdx.x == 0 && threadIdx.x == 0) atomicMin(a.status, a.col0 + bad);
-        return;   // uniform across the grid (every CTA factors the same reduced Gram)
+        return;
     }
-    if (blockIdx.x == 0) lf_write_r(a, s, 0, h);
-    if (w > 0) {
-        lf_cp_wait<0>();
-        __syncthreads();
-        // ---- R12 = Q1^T P2 and P2 -= Q1 R12
-        LF_MARK(6);
-        lf_k1(a, s, rp16);
-        LF_MARK(7);
-        lf_allreduce(a, s, 1024);
-        LF_MARK(8);
-        for (int e = threadIdx.x; e < 1024; e += LF_THREADS) {
-            const int i = e >> 5, j = e & 31;   // R12(i, j)
-            const float v = (i < h && j < w) ? (float)s.red[e] : 0.f;
-            s.R12h[j * LF_R12LD + i] = lf_to16(-v, a.bf16);
-            if (blockIdx.x == 0 && i < h && j < w) a.R[i + (int64_t)(h + j) * a.ldr] = v;
-            if (blockIdx.x == 0 && i < w && j < h) a.R[(h + i) + (int64_t)j * a.ldr] = 0.f;
+    LF_MARK(7);
+    lf_store_cols(a, s, r0, rows);
+    if (blockIdx.x == 0) {   // R (fp32) from the fp64 factor (s.Rs for one pass, else the accumulated one)
+        const double* racc = a.racc + (((npass - 1) & 1) ? 64 * 64 : 0);
+        for (int e = threadIdx.x; e < a.nc * a.nc; e += LF_THREADS) {
+            const int i = e % a.nc, j = e / a.nc;
+            const double v = npass == 1 ? s.Rs[i * LF_GLD + j] : __ldcg(racc + i * 64 + j);
+            a.R[i + (int64_t)j * a.ldr] = (i <= j) ? (float)v : 0.f;
         }
-        __syncthreads();
-        lf_k2(a, s, rp16);
-        LF_MARK(9);
-        // Q1 is final: write it while panel 2 runs
-        lf_store_cols(a, s, r0, rows, 0, h);
-        LF_MARK(10);
-        // ---- panel 2
-        bad = lf_panel<NI>(a, s, 32, w, rp16, 11);
-        if (bad >= 0) {
-            if (blockIdx.x == 0 && threadIdx.x == 0) atomicMin(a.status, a.col0 + h + bad);
-            return;
-        }
-        if (blockIdx.x == 0) {
-            for (int e = threadIdx.x; e < w * w; e += LF_THREADS) {
-                const int i = e % w, j = e / w;
-                a.R[(h + i) + (int64_t)(h + j) * a.ldr] = (i <= j) ? (float)s.Racc[i * LF_GLD + j] : 0.f;
-            }
-        }
-        LF_MARK(15);
-        lf_store_cols(a, s, r0, rows, 32, 32 + w);
-        LF_MARK(16);
-    } else {
-        lf_store_cols(a, s, r0, rows, 0, h);
     }
+    LF_MARK(8);
 }
 
 // ------------------------------------------------------------------ host side
@@ -832,7 +887,13 @@ bool leaf_fits(int64_t m) {
     return ((rows_per + 15) & ~15) <= 64 * LF_MAXI && leaf_smem_bytes(m) <= (size_t)lf_smem_max();
 }
 
-size_t leaf_ws_doubles() { return (size_t)(LF_MAX_GRID + 1) * LF_PART + 64; }
+bool leaf_prologue_fits(int64_t m) {
+    int grid, rows_per, ldt;
+    lf_geometry(m, grid, rows_per, ldt);
+    return (size_t)64 * lf_qa_ld((rows_per + 15) & ~15) * 2 <= 2 * LF_REGION;
+}
+
+size_t leaf_ws_doubles() { return (size_t)(LF_MAX_GRID + 1) * LF_PART + 2 * 64 * 64 + 64; }
 
 cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st) {
     if (L.nc < 1 || L.nc > 64 || !leaf_fits(L.m)) return cudaErrorInvalidValue;
@@ -848,10 +909,16 @@ cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st) {
     a.ldr = L.ldr;
     a.part = L.ws;
     a.red = L.ws + (size_t)LF_MAX_GRID * LF_PART;
+    a.racc = a.red + LF_PART;
     a.bar = L.bar;
     a.status = L.status;
     a.col0 = L.col0;
     a.bf16 = L.bf16;
+    a.pq = L.pq;
+    a.ph = L.pq ? L.ph : 0;
+    if (a.pq && (a.ph < 1 || a.ph > 64 || (L.ldh & 7) != 0 || (reinterpret_cast<uintptr_t>(L.pq) & 15) != 0 ||
+                 !leaf_prologue_fits(L.m)))
+        return cudaErrorInvalidValue;
     int grid;
     lf_geometry(L.m, grid, a.rows_per, a.ldt);
     a.vec = ((L.ldq & 3) == 0) && ((reinterpret_cast<uintptr_t>(L.Q) & 15) == 0) && ((L.ldh & 3) == 0) &&

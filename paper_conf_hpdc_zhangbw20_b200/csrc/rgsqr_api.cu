@@ -125,6 +125,7 @@ struct Plan {
     float* Q = nullptr;
     float* R = nullptr;
     int nb = 0, bf16 = 0, split = 0, scale = 1, nranks = 1, rank = 0, panel = 0;
+    bool leaf = false;       // last level runs as leaf.cu kernels
     int epoch = -1;          // g_alloc_epoch the plan was built against
     // derived
     int64_t ldh = 0, ldr12 = 0;
@@ -255,8 +256,8 @@ PtrSide ptr_side(const void* p) {
 }
 
 // ------------------------------------------------------------------ plan construction
-void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb, bool pair) {
-    if (pair && ncols > nb && ncols <= 2 * nb) {
+void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb, bool pair, bool leaf) {
+    if (pair && (ncols > nb || leaf) && ncols <= 2 * nb) {
         Op o{};
         o.kind = Op::PAIR;
         o.c0 = c0;
@@ -274,7 +275,7 @@ void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb, bool pair) {
         return;
     }
     const int h = rgsqr_split(ncols), w = ncols - h;
-    build_ops(ops, c0, h, nb, pair);
+    build_ops(ops, c0, h, nb, pair, leaf);
     Op p{};
     p.kind = Op::PROJ;
     p.c0 = c0;
@@ -284,7 +285,7 @@ void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb, bool pair) {
     Op u = p;
     u.kind = Op::UPDATE;
     ops.push_back(u);
-    build_ops(ops, c0 + h, w, nb, pair);
+    build_ops(ops, c0 + h, w, nb, pair, leaf);
 }
 
 int make_plan(rg_handle h, Plan& pl) {
@@ -302,7 +303,8 @@ int make_plan(rg_handle h, Plan& pl) {
     // mma.sync K1/K2 are single 16-bit products)
     const bool pair = pl.panel == 0 && pl.nb == 32 && !(pl.nranks > 1 && h->comm) &&
                       (wide ? rg::cholqr_fused_fits(m, 64) : (rg::leaf_fits(m) && !pl.split));
-    build_ops(pl.ops, 0, n, pl.nb, pair);
+    pl.leaf = pair && !wide;
+    build_ops(pl.ops, 0, n, pl.nb, pair, pl.leaf);
     int max_h = 0, max_w = 0;
     size_t pmax = 0;
     for (auto& o : pl.ops)
@@ -380,7 +382,7 @@ bool ensure_workspace(rg_handle h, int64_t m, int64_t n, int split) {
               h->pws.ensure(rg::panel_ws_floats(m) * 4 + 4096) && h->pcnt.ensure(rg::panel_counters(m) * 4 + 64) &&
               h->rgather.ensure((size_t)64 * 32 * 32 * 4) && h->rstackq.ensure((size_t)64 * 32 * 32 * 4) &&
               h->cq_ws.ensure(std::max(rg::cholqr_ws_doubles(m), rg::leaf_ws_doubles()) * 8 + 256) &&
-              h->leaf_bar.ensure(256) &&
+              h->leaf_bar.ensure(4096) &&
               h->cq_flags.ensure((rg::cholqr_counter_ints(m) + 8) * 4);
     return ok;
 }
@@ -420,8 +422,17 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
         RG_CUDA(cudaMemset2DAsync(pl.R, pl.ldr * sizeof(float), 0, n * sizeof(float), n, st));
     }
     const Op* pending_update = nullptr;   // leaf-level K2 folded into the next panel's load
+    const Op* pending_pro = nullptr;      // K1 + K2 of the level above a leaf, folded into it
+    static const bool no_fold64 = getenv("RGSQR_NO_FOLD64") != nullptr;
     for (size_t oi = 0; oi < pl.ops.size(); ++oi) {
         const Op& o = pl.ops[oi];
+        if (pl.leaf && !no_fold64 && rg::leaf_prologue_fits(m) && o.kind == Op::PROJ && o.h <= 64 && o.w <= 64 && oi + 2 < pl.ops.size() &&
+            pl.ops[oi + 1].kind == Op::UPDATE && pl.ops[oi + 1].c0 == o.c0 && pl.ops[oi + 2].kind == Op::PAIR &&
+            pl.ops[oi + 2].c0 == o.c0 + o.h && pl.ops[oi + 2].h + pl.ops[oi + 2].w == o.w) {
+            pending_pro = &o;
+            ++oi;   // the UPDATE too
+            continue;
+        }
         if (o.kind == Op::UPDATE && !dist && pl.panel == 0 && o.h <= 64 && oi + 1 < pl.ops.size() &&
             pl.ops[oi + 1].kind == Op::PANEL && pl.ops[oi + 1].c0 == o.c0 + o.h && pl.ops[oi + 1].w == o.w &&
             rg::cholqr_fused_fits(m, 32) && getenv("RGSQR_NO_FOLD") == nullptr) {
@@ -471,6 +482,11 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
                 L.status = status;
                 L.col0 = o.c0;
                 L.bf16 = pl.bf16;
+                if (pending_pro) {
+                    L.pq = qh + (int64_t)pending_pro->c0 * pl.ldh;
+                    L.ph = pending_pro->h;
+                    pending_pro = nullptr;
+                }
                 RG_CUDA(rg::launch_leaf(L, st));
             }
             continue;

@@ -8,28 +8,6 @@
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/kernels.h"
 namespace rg { thread_local long long g_launches = 0; bool pdl_enabled() { return false; } }
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/leaf.cu"
-__global__ void chol_probe(long long* cyc, int reps) {
-    extern __shared__ __align__(16) uint8_t sm[];
-    rg::LfSmem s(sm, 36);
-    for (int e = threadIdx.x; e < 1024; e += blockDim.x) {
-        const int i = e >> 5, j = e & 31;
-        s.G[i * rg::LF_GLD + j] = (i == j ? 40.0 : 1.0 / (1 + i + j));
-    }
-    __syncthreads();
-    long long t0 = clock64(), t1 = 0, t2 = 0, t3 = 0;
-    for (int r = 0; r < reps; ++r) {
-        if (threadIdx.x < 32) {
-            int fb = rg::lf_chol_warp(s);
-            if (r == 0) t1 = clock64();
-            double kk = rg::lf_inverse_warp(s, 32);
-            if (r == 0) t2 = clock64();
-            if (fb != 32 || kk < 0) cyc[5] = 1;
-        }
-        if (r == 0) t3 = clock64();
-    }
-    long long t4 = clock64();
-    if (threadIdx.x == 0) { cyc[0] = t1 - t0; cyc[1] = t2 - t1; cyc[2] = (t4 - t3) / (reps > 1 ? reps - 1 : 1); }
-}
 __global__ void lat_probe(long long* cyc, double* out, int n) {
     __shared__ double sm[1024];
     __shared__ int chase[64];
@@ -73,21 +51,63 @@ __global__ void lat_probe(long long* cyc, double* out, int n) {
         cyc[3] = (t4 - t3) * 100 / n; cyc[4] = (t5 - t4) * 100 / (8 * n); cyc[5] = (t6 - t5) * 100 / n;
     }
 }
+__global__ void chol64_probe(long long* cyc, int reps) {
+    extern __shared__ __align__(16) uint8_t sm[];
+    rg::LfSmem s(sm, 36);
+    for (int e = threadIdx.x; e < 4096; e += blockDim.x) {
+        const int i = e >> 6, j = e & 63;
+        s.G[i * rg::LF_GLD + j] = (i == j ? 80.0 : 1.0 / (1 + i + j));
+        if (i == j) s.gdiag[i] = 80.0;
+    }
+    __syncthreads();
+    long long t0 = clock64(), t1 = 0;
+    int bad = 0;
+    for (int r = 0; r < reps; ++r) {
+        if (threadIdx.x < 128) bad += rg::lf_chol(s);
+        __syncthreads();
+        if (r == 0) t1 = clock64();
+        for (int e = threadIdx.x; e < 4096; e += blockDim.x) {
+            const int i = e >> 6, j = e & 63;
+            s.G[i * rg::LF_GLD + j] = (i == j ? 80.0 : 1.0 / (1 + i + j));
+        }
+        __syncthreads();
+    }
+    long long t2 = clock64();
+    if (threadIdx.x == 0) { cyc[2] = t1 - t0; cyc[3] = (t2 - t1) / (reps - 1); cyc[4] = bad; }
+}
+__global__ void bar_probe(long long* cyc, int n) {
+    __shared__ double sm[2][64];
+    const int t = threadIdx.x;
+    double v = 1.0 + t;
+    long long t0 = clock64();
+    for (int i = 0; i < n; ++i) {
+        if (t < 64) sm[i & 1][t] = v;
+        __syncthreads();
+        v = sm[i & 1][(t + 1) & 63] * 1.0000001;
+    }
+    long long t1 = clock64();
+    if (t < 64) sm[0][t] = v;
+    if (t == 0) cyc[blockDim.x == 512 ? 0 : 1] = (t1 - t0) * 100 / n;
+}
 int main(int argc, char** argv) {
+    {
+        long long* cyc; cudaMalloc(&cyc, 64); cudaMemset(cyc, 0, 64);
+        bar_probe<<<1, 512>>>(cyc, 4096);
+        bar_probe<<<1, 128>>>(cyc, 4096);
+        long long hc[2]; cudaMemcpy(hc, cyc, 16, cudaMemcpyDeviceToHost);
+        printf("STS+syncthreads+LDS+DMUL chain (cycles x100): 512 threads %lld, 128 threads %lld\n", hc[0], hc[1]);
+        size_t smb = 64 * 36 * 4 + rg::LfSmem::fixed_bytes();
+        cudaFuncSetAttribute(chol64_probe, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb);
+        chol64_probe<<<1, 512, smb>>>(cyc, 10);
+        long long hh[5]; cudaMemcpy(hh, cyc, 40, cudaMemcpyDeviceToHost);
+        printf("chol64: first %lld cycles, warm %lld cycles (incl. G rebuild), bad-sum %lld (%s)\n", hh[2], hh[3], hh[4], cudaGetErrorString(cudaGetLastError()));
+    }
     {
         long long* cyc; double* out; cudaMalloc(&cyc, 64); cudaMalloc(&out, 1024); cudaMemset(out, 0, 1024);
         lat_probe<<<1, 64>>>(cyc, out, 4096);
         long long hc[6]; cudaMemcpy(hc, cyc, 48, cudaMemcpyDeviceToHost);
         printf("lat probe (cycles x100): DFMA issue %lld, DFMA latency %lld, LDS latency %lld, STS+syncwarp+LDS %lld, FFMA issue %lld, rsqrt(approx+newton) %lld\n",
                hc[0], hc[1], hc[2], hc[3], hc[4], hc[5]);
-    }
-    {
-        long long* cyc; cudaMalloc(&cyc, 64); cudaMemset(cyc, 0, 64);
-        size_t smb = 64 * 36 * 4 + rg::LfSmem::fixed_bytes();
-        cudaFuncSetAttribute(chol_probe, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb);
-        chol_probe<<<1, 32, smb>>>(cyc, 20);
-        long long hc[8]; cudaMemcpy(hc, cyc, 48, cudaMemcpyDeviceToHost);
-        printf("chol probe: first chol %lld cyc, first inverse %lld cyc, warm chol+inv %lld cyc (bad %lld)\n", hc[0], hc[1], hc[2], hc[5]);
     }
     const int64_t m = argc > 1 ? atoll(argv[1]) : 65536;
     const int nc = argc > 2 ? atoi(argv[2]) : 64;
@@ -96,8 +116,8 @@ int main(int argc, char** argv) {
     for (auto& x : h) x = (rand() / (float)RAND_MAX) - 0.5f;
     float *P, *Q, *R; uint16_t* Qh; double* ws; unsigned* bar; int* status;
     cudaMalloc(&P, m * nc * 4); cudaMalloc(&Q, m * nc * 4); cudaMalloc(&R, 64 * 64 * 4);
-    cudaMalloc(&Qh, m * nc * 2); cudaMalloc(&ws, rg::leaf_ws_doubles() * 8); cudaMalloc(&bar, 256);
-    cudaMalloc(&status, 64); cudaMemset(bar, 0, 256); cudaMemset(status, 0x7f, 64);
+    cudaMalloc(&Qh, m * nc * 2); cudaMalloc(&ws, rg::leaf_ws_doubles() * 8); cudaMalloc(&bar, 4096);
+    cudaMalloc(&status, 64); cudaMemset(bar, 0, 4096); cudaMemset(status, 0x7f, 64);
     cudaMemcpy(P, h.data(), m * nc * 4, cudaMemcpyHostToDevice);
     rg::LeafLaunch L{};
     L.Q = Q; L.ldq = m; L.Qh = Qh; L.ldh = m; L.m = m; L.nc = nc; L.R = R; L.ldr = 64; L.ws = ws; L.bar = bar;
@@ -120,9 +140,7 @@ int main(int argc, char** argv) {
            cudaGetErrorString(cudaGetLastError()));
     unsigned long long tr[32];
     cudaMemcpyFromSymbol(tr, rg::lf_trace, sizeof(tr));
-    const char* names[17] = {"start", "loaded", "p1 gram", "p1 allreduce", "p1 chol+inv", "p1 apply", "k1 begin",
-                             "k1 mma", "k1 allreduce", "k2", "store Q1", "p2 gram", "p2 allreduce", "p2 chol+inv",
-                             "p2 apply", "p2 done", "store Q2"};
-    for (int i = 1; i < 17; ++i) printf("  %-14s %7.2f us (+%.2f)\n", names[i], (tr[i] - tr[0]) / 1e3, ((long long)tr[i] - (long long)tr[i - 1]) / 1e3);
+    const char* names[9] = {"start", "loaded", "gram", "allreduce", "chol", "inverse+racc", "apply", "cholqr done", "stored"};
+    for (int i = 1; i < 9; ++i) printf("  %-14s %7.2f us (+%.2f)\n", names[i], (tr[i] - tr[0]) / 1e3, ((long long)tr[i] - (long long)tr[i - 1]) / 1e3);
     return 0;
 }
