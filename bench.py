@@ -237,7 +237,9 @@ def main():
                 "peak_src": f"{pk['src']} bf16 sustained (fp16 same rate)"}
     else:
         achieved = d["bytes"] / (d["ms"] * 1e-3) / 1e9
-        roof = {"kernel": dom, "bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
+        label = {"panel": "leaf (64-column CholQR2 panel + folded level above; latency-bound)",
+                 "scale": "column scaling (colnorm + scale/cast)"}.get(dom, dom)
+        roof = {"kernel": label, "bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / pk["hbm_gbs"], "peak_src": f"{pk['src']} copy bandwidth"}
     roof["traffic"] = None
     tpath = os.path.join(ROOT, "profiles", "r01_ncu_traffic.json")

@@ -77,6 +77,7 @@ struct LeafArgs {
 
 #ifdef LF_TRACE
 __device__ unsigned long long lf_trace[32];
+__device__ long long lf_clk[2];
 #define LF_MARK(i)                                                                     \
     do {                                                                               \
         if (blockIdx.x == 0 && threadIdx.x == 0) {                                     \
@@ -805,6 +806,9 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
     const int rows = rem <= 0 ? 0 : (rem < a.rows_per ? (int)rem : a.rows_per);
     const int rp16 = (rows + 15) & ~15;
     LF_MARK(0);
+#ifdef LF_TRACE
+    if (blockIdx.x == 0 && threadIdx.x == 0) lf_clk[0] = clock64();
+#endif
     lf_load_cols(a, s, r0, rows, rp16);
     if (a.pq) lf_load_qa(a, s, r0, rows, rp16);
     lf_cp_commit();
@@ -812,8 +816,11 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
     __syncthreads();
     if (a.pq) {
         // ---- prologue: the level above (R_AB = Q_A^T P, P -= Q_A R_AB)
+        LF_MARK(10);
         lf_pro_k1(a, s, rp16);
+        LF_MARK(11);
         lf_allreduce(a, s, 4096, false);
+        LF_MARK(12);
         for (int e = threadIdx.x; e < 4096; e += LF_THREADS) {
             const int i = e >> 6, j = e & 63;   // R_AB(i, j)
             const float v = (i < a.ph && j < a.nc) ? (float)__ldcg(a.red + e) : 0.f;
@@ -821,6 +828,7 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
             if (blockIdx.x == 0 && i < a.ph && j < a.nc) a.R[(int64_t)(i - a.ph) + (int64_t)j * a.ldr] = v;
         }
         __syncthreads();
+        LF_MARK(13);
         lf_pro_k2(a, s, rp16);
     }
     LF_MARK(1);
@@ -841,6 +849,9 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
         }
     }
     LF_MARK(8);
+#ifdef LF_TRACE
+    if (blockIdx.x == 0 && threadIdx.x == 0) lf_clk[1] = clock64();
+#endif
 }
 
 // ------------------------------------------------------------------ host side

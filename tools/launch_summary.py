@@ -19,6 +19,8 @@ def short(name):
 
 
 def klass(n):
+    if "leaf_kernel" in n:
+        return "leaf (64-col CholQR2 panel + folded K1/K2 of w=64)"
     if "gemm_tc_kernel" in n:
         return "gemm (K1 proj / K2 update, tcgen05)"
     if "proj_reduce" in n or "proj_finish" in n:

@@ -122,6 +122,16 @@ int main(int argc, char** argv) {
     rg::LeafLaunch L{};
     L.Q = Q; L.ldq = m; L.Qh = Qh; L.ldh = m; L.m = m; L.nc = nc; L.R = R; L.ldr = 64; L.ws = ws; L.bar = bar;
     L.status = status; L.col0 = 0;
+    uint16_t* qa16 = nullptr;
+    if (argc > 3 && atoi(argv[3])) {   // prologue with a random 64-column 16-bit Q_A
+        std::vector<uint16_t> hq((size_t)m * 64);
+        for (size_t i = 0; i < hq.size(); ++i) hq[i] = 0x2000 + (uint16_t)(rand() & 0x3ff);   // small positive halves
+        cudaMalloc(&qa16, hq.size() * 2);
+        cudaMemcpy(qa16, hq.data(), hq.size() * 2, cudaMemcpyHostToDevice);
+        L.pq = qa16; L.ph = 64;
+        cudaMalloc(&R, 128 * 64 * 4);
+        L.R = R + 64; L.ldr = 128;
+    }
     cudaStream_t st; cudaStreamCreate(&st);
     const int iters = 50;
     cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
@@ -141,6 +151,11 @@ int main(int argc, char** argv) {
     unsigned long long tr[32];
     cudaMemcpyFromSymbol(tr, rg::lf_trace, sizeof(tr));
     const char* names[9] = {"start", "loaded", "gram", "allreduce", "chol", "inverse+racc", "apply", "cholqr done", "stored"};
+    long long ck[2];
+    cudaMemcpyFromSymbol(ck, rg::lf_clk, sizeof(ck));
+    printf("  SM clock during the kernel: %.0f MHz\n", (ck[1] - ck[0]) / ((tr[8] - tr[0]) * 1e-3));
+    if (L.pq) printf("  prologue: qa load %.2f, k1 %.2f, allreduce %.2f, R_AB %.2f, k2 %.2f us\n", (tr[10] - tr[0]) / 1e3,
+                     (tr[11] - tr[10]) / 1e3, (tr[12] - tr[11]) / 1e3, (tr[13] - tr[12]) / 1e3, (tr[1] - tr[13]) / 1e3);
     for (int i = 1; i < 9; ++i) printf("  %-14s %7.2f us (+%.2f)\n", names[i], (tr[i] - tr[0]) / 1e3, ((long long)tr[i] - (long long)tr[i - 1]) / 1e3);
     return 0;
 }
