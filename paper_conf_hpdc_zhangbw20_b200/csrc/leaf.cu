@@ -354,16 +354,29 @@ __device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int rp) {
 }
 
 // ------------------------------------------------------------------ Cholesky (warps 0-3)
+// fp64 1/d: hardware approximation + two Newton steps (full precision for the Schur updates).
+__device__ __forceinline__ double lf_rcp(double d) {
+    double y;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(d));
+    double e = fma(-d, y, 1.0);
+    y = fma(y, e, y);
+    e = fma(-d, y, 1.0);
+    return fma(y, e, y);
+}
+
 // s.G holds the full symmetric 64 x 64 Gram (identity beyond nc).  Warp q (< 4) keeps rows
 // 16 q .. 16 q + 15 of the Schur complement S in registers, lane l columns l and l + 32 (one warp
-// per SMSP).  Step k: the warp owning row k publishes S(k, :) through s.U (ping-pong), a 128-thread
-// named barrier, and every thread reads the row back with 16-byte broadcasts, computes the pivot
-// itself (no pivot-thread branch) and updates its rows: S(i, j) -= S(k, i) S(k, j) / S(k, k)
-// (rows <= k of the pivot's quarter are dead after publication and updated harmlessly; quarters
-// above are skipped).  Measured on B200 (tools/leaf_bench.cu): ~23K cycles for the 64 pivots.
-// Variants measured slower: the whole 512-thread CTA with 8 rows per thread (16 warps issuing the
-// pivot logic, ~27K), per-row mbarriers so consumers never wait for each other (~27K), one warp
-// per 32 columns with shuffles (WARPSYNC/ENDCOLLECTIVE sequences inside the warp branch).
+// per SMSP).  Step k: the warp owning row k writes S(k, :) (unnormalised) into s.Rs row k, a
+// 128-thread named barrier, and every thread reads the row back with 16-byte broadcasts, forms
+// t_j = S(k, j) / S(k, k) itself (no pivot-thread branch) and updates its rows,
+// S(i, j) -= S(k, i) t_j (rows <= k of the pivot's quarter are dead after publication and updated
+// harmlessly; quarters above, and the columns < 32 once k >= 32, are skipped).  The chain per
+// pivot is barrier + LDS + 1/d + DMUL + DFMA; the square roots, the pivot test and the row
+// normalisation R(k, :) = S(k, :) / sqrt(S(k, k)) are done for all rows after the elimination.
+// Measured on B200 (tools/leaf_bench.cu).  Variants measured slower: the whole 512-thread CTA with
+// 8 rows per thread (16 warps issuing the pivot logic), per-row mbarriers so consumers never wait
+// for each other, one warp per 32 columns with shuffles (WARPSYNC/ENDCOLLECTIVE sequences inside
+// the warp branch), a fraction-free update (3x the fp64 work).
 // Writes s.Rs (fp64 row-major R, over G once every thread has loaded its part), s.Rt32 (fp32
 // column-major), s.rdiag / s.rdiag32 (1 / R(k, k)).  Returns the first failed pivot (64 if none)
 // on threads < 128: a pivot fails unless it is finite and > 1e-15 G(k, k).
@@ -376,50 +389,64 @@ __device__ int lf_chol(const LfSmem& s) {
         g0[ii] = s.G[(16 * rq + ii) * LF_GLD + jl];
         g1[ii] = s.G[(16 * rq + ii) * LF_GLD + jl + 32];
     }
-    lf_bar128();   // every thread has its part of G before R overwrites it
-    int bad = 64;
+    lf_bar128();   // every thread has its part of G before the rows overwrite it
 #pragma unroll 1
     for (int kq = 0; kq < 4; ++kq) {
 #pragma unroll
         for (int kk = 0; kk < 16; ++kk) {
             const int k = 16 * kq + kk;
-            double* urow = s.U + (kk & 1) * 64;
+            double* row = s.Rs + k * LF_GLD;
             if (rq == kq) {
-                urow[jl] = g0[kk];
-                urow[jl + 32] = g1[kk];
+                row[jl] = g0[kk];
+                row[jl + 32] = g1[kk];
             }
             lf_bar128();
-            const double d = urow[k];
-            const bool good = (d > s.gdiag[k] * 1e-15) && isfinite(d);
-            bad = (!good && bad == 64) ? k : bad;
-            const double rs = good ? lf_rsqrt(d) : 1.0;
-            const double r0 = (jl >= k) ? urow[jl] * rs : 0.0;          // R(k, jl)
-            const double r1 = (jl + 32 >= k) ? urow[jl + 32] * rs : 0.0;  // R(k, jl + 32)
-            const double t0 = r0 * rs, t1 = r1 * rs;                      // S(k, j) / S(k, k)
+            const double rd = lf_rcp(row[k]);
+            const double t1 = (jl + 32 >= k) ? row[jl + 32] * rd : 0.0;
             if (rq >= kq) {
-                const double* ur = urow + 16 * rq;
+                const double* ur = row + 16 * rq;
+                if (kq < 2) {
+                    const double t0 = (jl >= k) ? row[jl] * rd : 0.0;
 #pragma unroll
-                for (int ii = 0; ii < 16; ii += 2) {
-                    const double2 v = *reinterpret_cast<const double2*>(ur + ii);
-                    g0[ii] = fma(-v.x, t0, g0[ii]);
-                    g1[ii] = fma(-v.x, t1, g1[ii]);
-                    g0[ii + 1] = fma(-v.y, t0, g0[ii + 1]);
-                    g1[ii + 1] = fma(-v.y, t1, g1[ii + 1]);
+                    for (int ii = 0; ii < 16; ii += 2) {
+                        const double2 v = *reinterpret_cast<const double2*>(ur + ii);
+                        g1[ii] = fma(-v.x, t1, g1[ii]);
+                        g1[ii + 1] = fma(-v.y, t1, g1[ii + 1]);
+                        g0[ii] = fma(-v.x, t0, g0[ii]);
+                        g0[ii + 1] = fma(-v.y, t0, g0[ii + 1]);
+                    }
+                } else {   // columns < 32 are finished
+#pragma unroll
+                    for (int ii = 0; ii < 16; ii += 2) {
+                        const double2 v = *reinterpret_cast<const double2*>(ur + ii);
+                        g1[ii] = fma(-v.x, t1, g1[ii]);
+                        g1[ii + 1] = fma(-v.y, t1, g1[ii + 1]);
+                    }
                 }
-            }
-            if (rq == 0) {
-                s.Rs[k * LF_GLD + jl] = r0;
-                s.Rs[k * LF_GLD + jl + 32] = r1;
-                s.Rt32[jl * LF_TLD + k] = (float)r0;
-                s.Rt32[(jl + 32) * LF_TLD + k] = (float)r1;
-            } else if (rq == 1 && jl == 0) {
-                s.rdiag[k] = rs;
-                s.rdiag32[k] = (float)rs;
             }
         }
     }
     lf_bar128();
-    return bad;
+    // pivots -> 1 / R(k, k) and the pivot test; then R(k, j) = S(k, j) / sqrt(S(k, k)), j >= k
+    __shared__ int s_bad[2];
+    if (t < 64) {
+        const double d = s.Rs[t * LF_GLD + t];
+        const bool good = (d > s.gdiag[t] * 1e-15) && isfinite(d);
+        const double rs = good ? lf_rsqrt(d) : 1.0;
+        s.rdiag[t] = rs;
+        s.rdiag32[t] = (float)rs;
+        const unsigned badm = __ballot_sync(0xffffffffu, !good);
+        if (jl == 0) s_bad[t >> 5] = badm ? (__ffs(badm) - 1 + 32 * (t >> 5)) : 64;
+    }
+    lf_bar128();
+    for (int e = t; e < 64 * 64; e += 128) {
+        const int i = e >> 6, j = e & 63;
+        const double r = (j >= i) ? s.Rs[i * LF_GLD + j] * s.rdiag[i] : 0.0;
+        s.Rs[i * LF_GLD + j] = r;
+        s.Rt32[j * LF_TLD + i] = (float)r;
+    }
+    lf_bar128();
+    return min(s_bad[0], s_bad[1]);
 }
 
 // X = R^{-1} (upper, fp32: it only feeds the fp32 product P R^{-1} and the kappa test), blocked
@@ -632,7 +659,7 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
             break;
         }
         const double kk = lf_inverse(s, nc);   // every thread: same value
-        const bool stop = (pass == 0) ? (!shifted && kk <= 4.0 * nc * nc)   // kappa_F <= 2 nc
+        const bool stop = (pass == 0) ? (!shifted && kk <= 4.0 * nc * nc)
                                       : ((pass == 1 && !shifted) || pass == 2);
         // R = R_p ... R_1: a single pass keeps R in s.Rs; otherwise CTA 0 accumulates in global
         if (blockIdx.x == 0 && !(pass == 0 && stop)) lf_racc(a, s, pass);
