@@ -164,12 +164,15 @@ cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double*
                               float* S, float* Ub, float* Vb, cudaStream_t st);
 
 // ---- blas.cu (CGLS vectors, triangular inverse, small products)
+// y = A x (fp32 A, fp64 x, y); with sq: also sq[sq_idx] = |y|^2 via sq_part (>= 1184 doubles)
 cudaError_t launch_gemv_n(const float* A, int64_t lda, int64_t m, int n, const double* x, double* y, double* work,
-                          const double* done, cudaStream_t st);
+                          const double* done, cudaStream_t st, double* sq = nullptr, int sq_idx = 0,
+                          double* sq_part = nullptr);
 size_t gemv_n_work_doubles(int64_t m, int n);
 cudaError_t launch_gemv_t(const float* A, int64_t lda, int64_t m, int n, const double* r, double* s, double* work,
                           const double* done, cudaStream_t st);
 size_t gemv_t_work_doubles(int64_t m, int n);
+// Rinv: 2 n^2 doubles -- R^{-1} column-major, then its row-major copy (read by launch_trmv(.., 0, ..))
 cudaError_t launch_trinv_upper(const float* R, int64_t ldr, int n, double* Rinv, cudaStream_t st);
 cudaError_t launch_trmv(const double* Rinv, int n, const double* x, double* y, int transpose, const double* done,
                         cudaStream_t st);

@@ -772,12 +772,13 @@ int enqueue_cgls_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int 
     double* r = sv + n;
     double* q = r + m;
     double* work = q + m;
+    double* sqp = work + std::max(rg::gemv_n_work_doubles(m, n), rg::gemv_t_work_doubles(m, n));
     const double* done = sc + 6;
     for (int k = 0; k < iters; ++k) {
         ProfScope _s(h, PC_CGLS, 4.0 * m * n, 8.0 * m * n);
         RG_CUDA(rg::launch_trmv(Rinv, n, p, t, 0, done, st));                 // t = R \ p
-        RG_CUDA(rg::launch_gemv_n(A, lda, m, n, t, q, work, done, st));         // line 11: q = A t
-        RG_CUDA(rg::launch_sqnorm(q, m, sc, 1, st));                           // line 12: delta
+        // line 11: q = A t; line 12: delta = |q|^2 (partials from the split sums, fixed order)
+        RG_CUDA(rg::launch_gemv_n(A, lda, m, n, t, q, work, done, st, sc, 1, sqp));
         int rc = nccl_allreduce(h, sc + 1, 1, ncclFloat64);
         if (rc) return rc;
         RG_CUDA(rg::launch_cgls_xr(x, t, r, q, m, n, sc, st));                 // lines 13-15
@@ -1181,11 +1182,11 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     rc = check_status(h);
     if (rc) return rc;
     // ---- explicit R^{-1} (fp64)
-    if (!h->rinv.ensure((size_t)n * n * 8 + 64)) return RG_ALLOC;
+    if (!h->rinv.ensure((size_t)2 * n * n * 8 + 64)) return RG_ALLOC;   // Rinv + its row-major copy
     RG_CUDA(rg::launch_trinv_upper(Rw, n, (int)n, h->rinv.as<double>(), h->stream));
     // ---- CGLS state: sc[16] | x p s t sv (n each) | r q (m each) | gemv work
     const size_t work = std::max(rg::gemv_n_work_doubles(m_local, (int)n), rg::gemv_t_work_doubles(m_local, (int)n));
-    if (!h->cg.ensure((16 + 5 * (size_t)n + 2 * (size_t)m_local + work) * 8 + 256)) return RG_ALLOC;
+    if (!h->cg.ensure((16 + 5 * (size_t)n + 2 * (size_t)m_local + work + 2048) * 8 + 256)) return RG_ALLOC;
     double* base = h->cg.as<double>();
     double* sc = base;
     double* xd = sc + 16;
