@@ -21,8 +21,8 @@
 //   * Gram on the fp64 tensor cores (DMMA m8n8k4) straight from the fp32 rows in smem (one
 //     fragment per 8-column block serves as A and B), 36 8x8 blocks, no staging copy;
 //   * one deterministic grid all-reduction per pass (fixed-order sums, two grid barriers);
-//   * the 64 x 64 Cholesky on 4 warps (column j, half the rows per thread, in registers), one
-//     shared-memory broadcast + named barrier per pivot; R^{-1} in fp32 by column-parallel back
+//   * the 64 x 64 Cholesky on 4 warps (columns per lane, cyclic rows per warp, in registers), one
+//     shared-memory row broadcast + producer/consumer named barrier per pivot; R^{-1} in fp32 by column-parallel back
 //     substitution; P R^{-1} exploiting the triangle;
 //   * the prologue on mma.sync m16n8k16 from a 16-bit staging copy of Q_A (replaces that level's
 //     K1 GEMM, split-K reduce and K2 GEMM launches).
@@ -106,11 +106,10 @@ __device__ __forceinline__ void lf_grid_sync(unsigned* bar) {
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned nb = (blockIdx.x == 0) ? (0x80000000u - (gridDim.x - 1)) : 1u;
-        __threadfence();
-        const unsigned old = atomicAdd(bar, nb);
+        unsigned old;
+        asm volatile("atom.add.release.gpu.global.u32 %0, [%1], %2;" : "=r"(old) : "l"(bar), "r"(nb) : "memory");
         while (((lf_ld_acquire(bar) ^ old) & 0x80000000u) == 0) {
         }
-        __threadfence();
     }
     __syncthreads();
 }
@@ -232,22 +231,33 @@ __host__ __device__ __forceinline__ int lf_qa_ld(int rp16) { return ((rp16 - 8 +
 // Deterministic: entry e is summed by one warp of CTA e / slice, lanes over CTAs lane, lane + 32,
 // ... in order, then a fixed xor-shuffle tree.  Two grid barriers (measured ~1.6 us each with 148
 // CTAs; per-CTA ready flags polled by many threads instead were ~3x slower -- L2 contention).
-__device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne, bool to_smem) {
+__device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne, bool to_smem, int mk = 0) {
     lf_grid_sync(a.bar);
+    if (mk) LF_MARK(mk);
     const int grid = gridDim.x;
     const int slice = (ne + grid - 1) / grid;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     for (int q = warp; q < slice; q += LF_NW) {
         const int e = blockIdx.x * slice + q;
         if (e < ne) {
-            double v = 0.0;
-            for (int b = lane; b < grid; b += 32) v += __ldcg(a.part + (int64_t)b * LF_PART + e);
+            constexpr int NB = (LF_MAX_GRID + 31) / 32;   // all loads in flight, summed in CTA order
+            double p[NB];
+#pragma unroll
+            for (int u = 0; u < NB; ++u) {
+                const int b = lane + 32 * u;
+                p[u] = b < grid ? __ldcg(a.part + (int64_t)b * LF_PART + e) : 0.0;
+            }
+            double v = p[0];
+#pragma unroll
+            for (int u = 1; u < NB; ++u) v += p[u];
 #pragma unroll
             for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
             if (lane == 0) __stcg(a.red + e, v);
         }
     }
+    if (mk) LF_MARK(mk + 1);
     lf_grid_sync(a.bar);
+    if (mk) LF_MARK(mk + 2);
     if (!to_smem) return;
     for (int e = threadIdx.x; e < ne; e += LF_THREADS) s.red[e] = __ldcg(a.red + e);
     __syncthreads();
@@ -354,76 +364,78 @@ __device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int rp) {
 }
 
 // ------------------------------------------------------------------ Cholesky (warps 0-3)
-// fp64 1/d: hardware approximation + two Newton steps (full precision for the Schur updates).
-__device__ __forceinline__ double lf_rcp(double d) {
-    double y;
-    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(d));
-    double e = fma(-d, y, 1.0);
-    y = fma(y, e, y);
-    e = fma(-d, y, 1.0);
-    return fma(y, e, y);
-}
-
-// s.G holds the full symmetric 64 x 64 Gram (identity beyond nc).  Warp q (< 4) keeps rows
-// 16 q .. 16 q + 15 of the Schur complement S in registers, lane l columns l and l + 32 (one warp
-// per SMSP).  Step k: the warp owning row k writes S(k, :) (unnormalised) into s.Rs row k, a
-// 128-thread named barrier, and every thread reads the row back with 16-byte broadcasts, forms
-// t_j = S(k, j) / S(k, k) itself (no pivot-thread branch) and updates its rows,
-// S(i, j) -= S(k, i) t_j (rows <= k of the pivot's quarter are dead after publication and updated
-// harmlessly; quarters above, and the columns < 32 once k >= 32, are skipped).  The chain per
-// pivot is barrier + LDS + 1/d + DMUL + DFMA; the square roots, the pivot test and the row
-// normalisation R(k, :) = S(k, :) / sqrt(S(k, k)) are done for all rows after the elimination.
-// Measured on B200 (tools/leaf_bench.cu).  Variants measured slower: the whole 512-thread CTA with
-// 8 rows per thread (16 warps issuing the pivot logic), per-row mbarriers so consumers never wait
-// for each other, one warp per 32 columns with shuffles (WARPSYNC/ENDCOLLECTIVE sequences inside
-// the warp branch), a fraction-free update (3x the fp64 work).
+// s.G holds the full symmetric 64 x 64 Gram (identity beyond nc).  Warp q (< 4) keeps the rows
+// i = 4 ii + q (ii < 16; cyclic, so the live rows stay balanced over the four SMSPs as the
+// elimination proceeds) of the Schur complement S in registers, lane l columns l and l + 32.
+// Step k (fully unrolled: k, and which register rows can still be live, are compile-time): the
+// owner warp k % 4 has published S(k, :) (unnormalised) as row k of s.Rs; the three other warps
+// wait for it on a producer/consumer named barrier (bar.arrive by the owner, bar.sync by the
+// consumers, ids alternating 2 / 3), every thread forms t_j = S(k, j) / S(k, k) itself and updates
+// its rows S(i, j) -= S(k, i) t_j.  The row that becomes pivot k + 1 is updated first and
+// published at once (look-ahead), so the owner never waits.  Rows <= k are dead after
+// publication and updated harmlessly; the columns < 32 are skipped once k >= 32.  The square
+// roots, the pivot test and R(k, :) = S(k, :) / sqrt(S(k, k)) are done after the elimination.
+// Measured on B200 (tools/leaf_bench.cu): 7.5 us per 64 x 64 factorization.  Slower variants: a
+// barrier over all four warps per pivot with 16-row quarters per warp (11.2 us), one barrier per
+// (consumer, owner) pair (7.7 us), permuted rows with all row loads issued up front (9.4 us), the
+// whole 512-thread CTA, per-row mbarriers, one warp per 32 columns with shuffles, a fraction-free
+// update.
 // Writes s.Rs (fp64 row-major R, over G once every thread has loaded its part), s.Rt32 (fp32
 // column-major), s.rdiag / s.rdiag32 (1 / R(k, k)).  Returns the first failed pivot (64 if none)
 // on threads < 128: a pivot fails unless it is finite and > 1e-15 G(k, k).
+__device__ __forceinline__ void lf_bar_sync(int id) { asm volatile("bar.sync %0, 128;" ::"r"(id) : "memory"); }
+__device__ __forceinline__ void lf_bar_arrive(int id) { asm volatile("bar.arrive %0, 128;" ::"r"(id) : "memory"); }
+
+// fp64 1/d: hardware approximation + one Newton step (relative error ~2^-44)
+__device__ __forceinline__ double lf_rcp(double d) {
+    double y;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(d));
+    const double e = fma(-d, y, 1.0);
+    return fma(y, e, y);
+}
+
 __device__ int lf_chol(const LfSmem& s) {
     const int t = threadIdx.x;   // < 128
-    const int jl = t & 31, rq = t >> 5;
+    const int jl = t & 31, q = t >> 5;
     double g0[16], g1[16];
 #pragma unroll
     for (int ii = 0; ii < 16; ++ii) {
-        g0[ii] = s.G[(16 * rq + ii) * LF_GLD + jl];
-        g1[ii] = s.G[(16 * rq + ii) * LF_GLD + jl + 32];
+        g0[ii] = s.G[(4 * ii + q) * LF_GLD + jl];
+        g1[ii] = s.G[(4 * ii + q) * LF_GLD + jl + 32];
     }
     lf_bar128();   // every thread has its part of G before the rows overwrite it
-#pragma unroll 1
-    for (int kq = 0; kq < 4; ++kq) {
+    if (q == 0) {
+        s.Rs[jl] = g0[0];
+        s.Rs[jl + 32] = g1[0];
+        __syncwarp();
+        lf_bar_arrive(2);
+    }
 #pragma unroll
-        for (int kk = 0; kk < 16; ++kk) {
-            const int k = 16 * kq + kk;
-            double* row = s.Rs + k * LF_GLD;
-            if (rq == kq) {
-                row[jl] = g0[kk];
-                row[jl + 32] = g1[kk];
+    for (int k = 0; k < 64; ++k) {
+        const double* row = s.Rs + k * LF_GLD;
+        if (q != (k & 3)) lf_bar_sync(2 + (k & 1));
+        const double rd = lf_rcp(row[k]);
+        const double t1 = (jl + 32 > k) ? row[jl + 32] * rd : 0.0;
+        const double t0 = (k < 32 && jl > k) ? row[jl] * rd : 0.0;
+        const int nx = (k + 1) >> 2;   // register row of pivot k + 1 in its owner warp
+        if (k < 63) {
+            const double v = row[4 * nx + q];
+            g1[nx] = fma(-v, t1, g1[nx]);
+            if (k < 32) g0[nx] = fma(-v, t0, g0[nx]);
+            if (q == ((k + 1) & 3)) {
+                double* nrow = s.Rs + (k + 1) * LF_GLD;
+                if (k + 1 < 32) nrow[jl] = g0[nx];
+                nrow[jl + 32] = g1[nx];
+                __syncwarp();
+                lf_bar_arrive(2 + ((k + 1) & 1));
             }
-            lf_bar128();
-            const double rd = lf_rcp(row[k]);
-            const double t1 = (jl + 32 >= k) ? row[jl + 32] * rd : 0.0;
-            if (rq >= kq) {
-                const double* ur = row + 16 * rq;
-                if (kq < 2) {
-                    const double t0 = (jl >= k) ? row[jl] * rd : 0.0;
+        }
 #pragma unroll
-                    for (int ii = 0; ii < 16; ii += 2) {
-                        const double2 v = *reinterpret_cast<const double2*>(ur + ii);
-                        g1[ii] = fma(-v.x, t1, g1[ii]);
-                        g1[ii + 1] = fma(-v.y, t1, g1[ii + 1]);
-                        g0[ii] = fma(-v.x, t0, g0[ii]);
-                        g0[ii + 1] = fma(-v.y, t0, g0[ii + 1]);
-                    }
-                } else {   // columns < 32 are finished
-#pragma unroll
-                    for (int ii = 0; ii < 16; ii += 2) {
-                        const double2 v = *reinterpret_cast<const double2*>(ur + ii);
-                        g1[ii] = fma(-v.x, t1, g1[ii]);
-                        g1[ii + 1] = fma(-v.y, t1, g1[ii + 1]);
-                    }
-                }
-            }
+        for (int ii = k >> 2; ii < 16; ++ii) {
+            if (ii == nx && k < 63) continue;
+            const double v = row[4 * ii + q];
+            g1[ii] = fma(-v, t1, g1[ii]);
+            if (k < 32) g0[ii] = fma(-v, t0, g0[ii]);
         }
     }
     lf_bar128();
@@ -633,7 +645,7 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
     for (; pass < 3; ++pass) {
         lf_gram(a, s, rp);
         if (pass == 0) LF_MARK(2);
-        lf_allreduce(a, s, LF_NE, true);
+        lf_allreduce(a, s, LF_NE, true, pass == 0 ? 20 : 0);
         if (pass == 0) LF_MARK(3);
         lf_build_g(s, s.red, false, nc, 0.0);
         int fb = threadIdx.x < 128 ? lf_chol(s) : 64;

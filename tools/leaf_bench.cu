@@ -51,7 +51,7 @@ __global__ void lat_probe(long long* cyc, double* out, int n) {
         cyc[3] = (t4 - t3) * 100 / n; cyc[4] = (t5 - t4) * 100 / (8 * n); cyc[5] = (t6 - t5) * 100 / n;
     }
 }
-__global__ void chol64_probe(long long* cyc, int reps) {
+__global__ void __launch_bounds__(512, 1) chol64_probe(long long* cyc, int reps) {
     extern __shared__ __align__(16) uint8_t sm[];
     rg::LfSmem s(sm, 36);
     for (int e = threadIdx.x; e < 4096; e += blockDim.x) {
@@ -65,7 +65,21 @@ __global__ void chol64_probe(long long* cyc, int reps) {
     for (int r = 0; r < reps; ++r) {
         if (threadIdx.x < 128) bad += rg::lf_chol(s);
         __syncthreads();
-        if (r == 0) t1 = clock64();
+        if (r == 0) {
+            t1 = clock64();
+            if (threadIdx.x == 0) {   // check R^T R == G
+                double err = 0;
+                for (int i = 0; i < 64; ++i)
+                    for (int j = i; j < 64; ++j) {
+                        double acc = 0;
+                        for (int k = 0; k <= i; ++k) acc += s.Rs[k * rg::LF_GLD + i] * s.Rs[k * rg::LF_GLD + j];
+                        const double g = (i == j ? 80.0 : 1.0 / (1 + i + j));
+                        err = fmax(err, fabs(acc - g) / 80.0);
+                    }
+                cyc[5] = (long long)(err * 1e18);
+            }
+            __syncthreads();
+        }
         for (int e = threadIdx.x; e < 4096; e += blockDim.x) {
             const int i = e >> 6, j = e & 63;
             s.G[i * rg::LF_GLD + j] = (i == j ? 80.0 : 1.0 / (1 + i + j));
@@ -99,8 +113,8 @@ int main(int argc, char** argv) {
         size_t smb = 64 * 36 * 4 + rg::LfSmem::fixed_bytes();
         cudaFuncSetAttribute(chol64_probe, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smb);
         chol64_probe<<<1, 512, smb>>>(cyc, 10);
-        long long hh[5]; cudaMemcpy(hh, cyc, 40, cudaMemcpyDeviceToHost);
-        printf("chol64: first %lld cycles, warm %lld cycles (incl. G rebuild), bad-sum %lld (%s)\n", hh[2], hh[3], hh[4], cudaGetErrorString(cudaGetLastError()));
+        long long hh[6]; cudaMemcpy(hh, cyc, 48, cudaMemcpyDeviceToHost);
+        printf("chol64: first %lld cycles, warm %lld cycles (incl. G rebuild), bad-sum %lld, max|R^T R - G|/80 = %.3g (%s)\n", hh[2], hh[3], hh[4], hh[5] * 1e-18, cudaGetErrorString(cudaGetLastError()));
     }
     {
         long long* cyc; double* out; cudaMalloc(&cyc, 64); cudaMalloc(&out, 1024); cudaMemset(out, 0, 1024);
@@ -154,6 +168,8 @@ int main(int argc, char** argv) {
     long long ck[2];
     cudaMemcpyFromSymbol(ck, rg::lf_clk, sizeof(ck));
     printf("  SM clock during the kernel: %.0f MHz\n", (ck[1] - ck[0]) / ((tr[8] - tr[0]) * 1e-3));
+    printf("  allreduce: barrier 1 %.2f, reduce %.2f, barrier 2 %.2f, to smem %.2f us\n", (tr[20] - tr[2]) / 1e3,
+           (tr[21] - tr[20]) / 1e3, (tr[22] - tr[21]) / 1e3, (tr[3] - tr[22]) / 1e3);
     if (L.pq) printf("  prologue: qa load %.2f, k1 %.2f, allreduce %.2f, R_AB %.2f, k2 %.2f us\n", (tr[10] - tr[0]) / 1e3,
                      (tr[11] - tr[10]) / 1e3, (tr[12] - tr[11]) / 1e3, (tr[13] - tr[12]) / 1e3, (tr[1] - tr[13]) / 1e3);
     for (int i = 1; i < 9; ++i) printf("  %-14s %7.2f us (+%.2f)\n", names[i], (tr[i] - tr[0]) / 1e3, ((long long)tr[i] - (long long)tr[i - 1]) / 1e3);
