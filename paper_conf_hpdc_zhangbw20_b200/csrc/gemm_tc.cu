@@ -18,6 +18,8 @@
 // Split precision (reading #9, reorthogonalisation passes): operands are held as
 // hi = fp16(X) and lo = fp16((X - hi) 2^11); three MMA groups accumulate hi*hi into
 // accumulator 0 and hi*lo + lo*hi into accumulator 1; D = D0 + 2^-11 D1 in the epilogue.
+#include <cstdlib>
+
 #include <cuda.h>
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
@@ -33,7 +35,9 @@ constexpr int kBK = 64;     // k extent of one pipeline stage (one 128B swizzle 
 constexpr int kUK = 16;     // UMMA K for kind::f16
 constexpr int kEpiLd = 36;  // per-warp transpose buffer row stride (floats, 16B aligned)
 
-template <int BN, int STAGES, bool SPLIT, int EPI_WG>
+// TE = number of C chunk slots (128 rows x 32 columns, fp32) of the TMA epilogue, split evenly
+// between the epilogue warpgroups; 0 = register epilogue
+template <int BN, int STAGES, bool SPLIT, int EPI_WG, int TE = 0>
 struct GemmCfg {
     static constexpr int kABytes = kBM * kBK * 2;           // 16 KB
     static constexpr int kBBytes = BN * kBK * 2;
@@ -41,7 +45,8 @@ struct GemmCfg {
     static constexpr int kStageBytes = kOps * (kABytes + kBBytes);
     static constexpr int kDataBytes = STAGES * kStageBytes;
     static constexpr int kEpiWarps = 4 * EPI_WG;
-    static constexpr int kEpiBytes = kEpiWarps * 32 * kEpiLd * 4;
+    static constexpr int kCSlot = kBM * 32 * 4;               // fp32 C chunk, [32 cols][128 rows]
+    static constexpr int kEpiBytes = TE ? TE * kCSlot : kEpiWarps * 32 * kEpiLd * 4;
     static constexpr int kBarOffset = kDataBytes + kEpiBytes;
     static constexpr int kTotal = kBarOffset + 512 + 1024;   // barriers + 1 KB alignment slack
     static constexpr int kThreads = 128 + 32 * kEpiWarps;
@@ -73,6 +78,7 @@ struct GemmArgs {
     int bf16;
     int vec_ok;            // C / Ch / Cl accesses may use 16-byte (8-byte) vectors
     int overwrite;         // K2 only: C = D instead of C -= D (plain product, lowrank_approx)
+    int h0;                // K2 only: 16-bit image written for columns >= h0 only
 };
 
 __device__ __forceinline__ uint16_t f2h_bits(float x, int bf16) {
@@ -113,12 +119,39 @@ __device__ __forceinline__ void unit_coords(const GemmArgs& a, int u, int& t0, i
 }
 
 // MODE 0 = K1 projection (A, B K-major), MODE 1 = K2 update (A MN-major, B K-major)
-template <int MODE, int BN, int STAGES, bool SPLIT, int EPI_WG>
-__global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 1)
+// TMA-epilogue slot of chunk ch of the cnt-th tile of this CTA: warpgroup g = ch % EPI_WG owns
+// slots [g * NCW, (g + 1) * NCW) and fills them round-robin in its own chunk order.
+template <int KCH, int EPI_WG, int NCW>
+__device__ __forceinline__ void te_slot(int cnt, int ch, int& s, uint32_t& round) {
+    const int g = ch % EPI_WG;
+    const int per = (KCH - g + EPI_WG - 1) / EPI_WG;   // chunks per tile of warpgroup g
+    const int k = cnt * per + ch / EPI_WG;
+    s = g * NCW + k % NCW;
+    round = (uint32_t)(k / NCW);
+}
+
+// TE (K2 only): TMA epilogue.  Warp 3 streams the fp32 C chunks (128 rows x 32 columns, 16 KB)
+// of the tiles into per-warpgroup rings of shared-memory slots ahead of the accumulators; each
+// epilogue warp subtracts its TMEM rows from the slot in place (and stores the 16-bit image of
+// its rows directly, 64 contiguous bytes per column and warp); warp 2 (idle after the TMEM
+// allocation) issues the TMA stores and recycles the slots.  Several C chunks per SM are in
+// flight (the register-staged epilogue kept one chunk ahead and reached ~3.5-4 TB/s on the
+// HBM-bound levels).
+template <int MODE, int BN, int STAGES, bool SPLIT, int EPI_WG, int TE = 0>
+__global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThreads, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const __grid_constant__ CUtensorMap tmA_lo, const __grid_constant__ CUtensorMap tmB_lo,
-                   GemmArgs args) {
-    using C = GemmCfg<BN, STAGES, SPLIT, EPI_WG>;
+                   const __grid_constant__ CUtensorMap tmC, GemmArgs args) {
+    using C = GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>;
+    static_assert(!TE || (MODE == 1 && !SPLIT), "TMA epilogue: K2, single precision");
+    // Chunk ch of a tile belongs to warpgroup ch % EPI_WG, which owns TE / EPI_WG slots and uses
+    // them round-robin in its own chunk order, so every slot has one consumer that waits its
+    // rounds in order.  (A ring shared by both warpgroups lets one wait on round r + 1 of a slot
+    // while the other's round r -- a TMA load completing out of order -- is still pending:
+    // mbarrier parity aliasing, measured as sporadic hangs / launch failures.)
+    static_assert(TE % EPI_WG == 0, "C ring slots split evenly between the epilogue warpgroups");
+    constexpr int kNcw = TE > 0 ? TE / EPI_WG : 1;   // slots per warpgroup
+    constexpr int kCRing = TE > 0 ? TE : 1;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     float* epi_buf = reinterpret_cast<float*>(smem + C::kDataBytes);
@@ -127,6 +160,9 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
     uint64_t* tfull_bar = empty_bar + STAGES;
     uint64_t* tempty_bar = tfull_bar + 2;
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty_bar + 2);
+    uint64_t* cfull_bar = reinterpret_cast<uint64_t*>(smem + C::kBarOffset + 256);
+    uint64_t* cempty_bar = cfull_bar + kCRing;
+    uint64_t* cready_bar = cempty_bar + kCRing;
 
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -145,6 +181,14 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
         for (int a = 0; a < 2; ++a) {
             mbar_init(&tfull_bar[a], 1);
             mbar_init(&tempty_bar[a], C::kEpiWarps);
+        }
+        if (TE) {
+            for (int s = 0; s < kCRing; ++s) {
+                mbar_init(&cfull_bar[s], 1);
+                mbar_init(&cempty_bar[s], 1);
+                mbar_init(&cready_bar[s], 4);   // the four warps of the epilogue warpgroup
+            }
+            tma_prefetch_desc(&tmC);
         }
         fence_barrier_init();
     }
@@ -240,7 +284,109 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
             }
         }
         __syncwarp();
-    } else if (warp >= 4) {
+    } else if (TE && warp == 3) {
+        if (elect_one()) {
+            // ---------------- C producer: fp32 C chunks into the slot ring (chunk order = t)
+            constexpr int kChunks = BN / 32;
+            int cnt = 0;
+            for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+                int t0, tj, z, kb0, kb1;
+                unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
+                for (int ch = 0; ch < kChunks; ++ch) {
+                    int s;
+                    uint32_t round;
+                    te_slot<kChunks, EPI_WG, kNcw>(cnt, ch, s, round);
+                    mbar_wait(&cempty_bar[s], (round & 1u) ^ 1u);
+                    if (args.overwrite) {
+                        mbar_arrive(&cfull_bar[s]);
+                    } else {
+                        mbar_arrive_expect_tx(&cfull_bar[s], C::kCSlot);
+                        tma_load_2d(epi_buf + s * (C::kCSlot / 4), &tmC, &cfull_bar[s], t0, tj * BN + ch * 32);
+                    }
+                }
+            }
+        }
+        __syncwarp();
+    } else if (TE && warp == 2) {
+        if (elect_one()) {
+            // ---------------- C store issuer: slot -> global (fp32 + 16-bit image), recycle
+            constexpr int kChunks = BN / 32;
+            int cnt = 0, prev = -1;
+            for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+                int t0, tj, z, kb0, kb1;
+                unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
+                for (int ch = 0; ch < kChunks; ++ch) {
+                    int s;
+                    uint32_t round;
+                    te_slot<kChunks, EPI_WG, kNcw>(cnt, ch, s, round);
+                    mbar_wait(&cready_bar[s], round & 1u);
+                    tma_store_2d(&tmC, epi_buf + s * (C::kCSlot / 4), t0, tj * BN + ch * 32);
+                    bulk_commit();
+                    bulk_wait_read<1>();   // the previous chunk's slot has been read out: recycle it
+                    if (prev >= 0) mbar_arrive(&cempty_bar[prev]);
+                    prev = s;
+                }
+            }
+            bulk_wait<0>();
+        }
+        __syncwarp();
+    } else if (TE && warp >= 4) {
+        // ---------------- TMA epilogue warps: ew = TMEM lane quarter (32 rows), wg = chunk interleave
+        constexpr int kChunks = BN / 32;
+        const int ew = warp & 3;
+        const int wg = (warp - 4) >> 2;
+        const uint32_t lane_off = static_cast<uint32_t>(ew * 32) << 16;
+        const bool hv = args.Ch != nullptr;
+        int cnt = 0;
+        for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+            int t0, tj, z, kb0, kb1;
+            unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
+            const int64_t row = (int64_t)t0 + ew * 32 + lane;
+            const int acc = cnt % C::kAcc;
+            const uint32_t aphase = (uint32_t)(cnt / C::kAcc) & 1u;
+            bool waited = false;
+            for (int ch = wg; ch < kChunks; ch += EPI_WG) {
+                int s;
+                uint32_t round;
+                te_slot<kChunks, EPI_WG, kNcw>(cnt, ch, s, round);
+                if (!waited) {
+                    mbar_wait(&tfull_bar[acc], aphase);
+                    tc_fence_after();
+                    waited = true;
+                }
+                uint32_t v[32];
+                tmem_ld32(tmem_base + acc * C::kAccCols + lane_off + ch * 32, v);
+                tmem_ld_wait();
+                if (ch + EPI_WG >= kChunks) {
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&tempty_bar[acc]);
+                }
+                mbar_wait(&cfull_bar[s], round & 1u);
+                float* cs = epi_buf + s * (C::kCSlot / 4) + ew * 32 + lane;   // [col][128 rows]
+                const int j0 = tj * BN + ch * 32;
+                uint16_t* hp = hv ? reinterpret_cast<uint16_t*>(args.Ch) + row + (int64_t)j0 * args.ldh : nullptr;
+                const int jmax = (row < args.m && j0 + 32 > args.h0) ? min(32, args.w - j0) : 0;
+                const int jmin = args.h0 - j0;
+#pragma unroll
+                for (int jj = 0; jj < 32; ++jj) {
+                    const float d = __uint_as_float(v[jj]);
+                    const float x = args.overwrite ? d : cs[jj * kBM] - d;
+                    cs[jj * kBM] = x;
+                    if (hv && jj < jmax && jj >= jmin) hp[(int64_t)jj * args.ldh] = f2h_bits(x, args.bf16);
+                }
+                fence_proxy_async_smem();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&cready_bar[s]);
+            }
+            if (!waited) {
+                mbar_wait(&tfull_bar[acc], aphase);
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&tempty_bar[acc]);
+            }
+        }
+    } else if (!TE && warp >= 4) {
         // ---------------- epilogue warps: ew = TMEM lane quarter, wg = column interleave
         const int ew = warp & 3;
         const int wg = (warp - 4) >> 2;
@@ -347,7 +493,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG>::kThreads, 
                             nv.w = old[k].w - dv.w;
                         }
                         float* cp = args.C + row0 + (int64_t)j * args.ldc;
-                        uint16_t* hp = args.Ch ? reinterpret_cast<uint16_t*>(args.Ch) + row0 + (int64_t)j * args.ldh
+                        uint16_t* hp = (args.Ch && j >= args.h0) ? reinterpret_cast<uint16_t*>(args.Ch) + row0 + (int64_t)j * args.ldh
                                                : nullptr;
                         uint16_t* lp = args.Cl ? reinterpret_cast<uint16_t*>(args.Cl) + row0 + (int64_t)j * args.ldh
                                                : nullptr;
@@ -535,12 +681,13 @@ static int num_sms() {
     return g_num_sms;
 }
 
-template <int MODE, int BN, int STAGES, bool SPLIT, int EPI_WG>
+template <int MODE, int BN, int STAGES, bool SPLIT, int EPI_WG, int TE = 0>
 static cudaError_t launch_gemm(int units, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& al,
-                               const CUtensorMap& bl, const GemmArgs& args, cudaStream_t st) {
-    using C = GemmCfg<BN, STAGES, SPLIT, EPI_WG>;
+                               const CUtensorMap& bl, const GemmArgs& args, cudaStream_t st,
+                               const CUtensorMap* mc = nullptr) {
+    using C = GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>;
     static_assert(C::kTotal <= 227 * 1024, "shared memory budget");
-    auto kern = gemm_tc_kernel<MODE, BN, STAGES, SPLIT, EPI_WG>;
+    auto kern = gemm_tc_kernel<MODE, BN, STAGES, SPLIT, EPI_WG, TE>;
     static bool attr_set = false;
     if (!attr_set) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::kTotal);
@@ -551,8 +698,26 @@ static cudaError_t launch_gemm(int units, const CUtensorMap& a, const CUtensorMa
     const int per_sm = (C::kTotal <= 113 * 1024 && C::kTmemCols <= 256) ? 2 : 1;
     int grid = num_sms() * per_sm;
     if (grid > units) grid = units;
-    RG_LAUNCH((kern), grid, C::kThreads, C::kTotal, st, a, b, al, bl, args);
+    RG_LAUNCH((kern), grid, C::kThreads, C::kTotal, st, a, b, al, bl, mc ? *mc : a, args);
     return cudaGetLastError();
+}
+
+// K2 with the TMA epilogue.  Shared memory (<= 227 KB) is split between the operand ring and
+// the C-chunk ring (16 KB per slot): the HBM-bound levels (few k-blocks per tile) trade operand
+// stages for C chunks in flight, the tensor-bound top level (K = 2048) keeps three stages.
+static cudaError_t dispatch_bn_te(int bn, int units, const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& args,
+                                  cudaStream_t st, const CUtensorMap* mc) {
+    static const int deep_kb = getenv("RGSQR_K2_DEEP_KB") ? atoi(getenv("RGSQR_K2_DEEP_KB")) : 8;
+    const bool deep = args.kb_h <= deep_kb;
+    switch (bn) {
+        case 32: return launch_gemm<1, 32, 3, false, 2, 8>(units, a, b, a, b, args, st, mc);
+        case 64: return launch_gemm<1, 64, 2, false, 2, 10>(units, a, b, a, b, args, st, mc);
+        case 128: return launch_gemm<1, 128, 2, false, 2, 10>(units, a, b, a, b, args, st, mc);
+        case 256:
+            if (deep) return launch_gemm<1, 256, 2, false, 2, 8>(units, a, b, a, b, args, st, mc);
+            return launch_gemm<1, 256, 3, false, 2, 4>(units, a, b, a, b, args, st, mc);
+        default: return cudaErrorInvalidValue;
+    }
 }
 
 template <int MODE, bool SPLIT>
@@ -595,9 +760,10 @@ cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int s
 cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, const CUtensorMap& q1_mn,
                                const CUtensorMap& r12, const CUtensorMap& q1_mn_lo, const CUtensorMap& r12_lo,
                                float* C, int64_t ldc, void* Ch, void* Cl, int64_t ldh, int bf16, cudaStream_t st,
-                               int overwrite) {
+                               int overwrite, const CUtensorMap* mc, int h0) {
     GemmArgs args{};
     args.overwrite = overwrite;
+    args.h0 = h0;
     args.C = C;
     args.ldc = ldc;
     args.Ch = Ch;
@@ -612,6 +778,8 @@ cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, cons
     args.units = args.tiles_i * args.tiles_j;
     args.vec_ok = ((ldc & 3) == 0) && ((reinterpret_cast<uintptr_t>(C) & 15) == 0) && ((ldh & 3) == 0) &&
                   ((reinterpret_cast<uintptr_t>(Ch) & 7) == 0) && ((reinterpret_cast<uintptr_t>(Cl) & 7) == 0);
+    if (!split && mc && !Cl && !getenv("RGSQR_NO_TMA_EPI"))
+        return dispatch_bn_te(bn, args.units, q1_mn, r12, args, st, mc);
     return split ? dispatch_bn<1, true>(bn, args.units, q1_mn, r12, q1_mn_lo, r12_lo, args, st)
                  : dispatch_bn<1, false>(bn, args.units, q1_mn, r12, q1_mn, r12, args, st);
 }

@@ -147,7 +147,9 @@ cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int s
 cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, const CUtensorMap& q1_mn,
                                const CUtensorMap& r12, const CUtensorMap& q1_mn_lo, const CUtensorMap& r12_lo,
                                float* C, int64_t ldc, void* Ch, void* Cl, int64_t ldh, int bf16, cudaStream_t st,
-                               int overwrite = 0);
+                               int overwrite = 0, const CUtensorMap* mc = nullptr, int h0 = 0);
+// (mc: fp32 C, box 128 rows x 32 columns, no swizzle: K2 runs with the TMA epilogue.  h0: the
+// 16-bit image of C is written for columns >= h0 only.)
 cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, int splits, int h, int w, float* R,
                                int64_t ldr, float* Rf, int64_t ldf, uint16_t* Rh, uint16_t* Rl, int64_t ldh, int bf16,
                                cudaStream_t st);

@@ -75,6 +75,24 @@ bool encode_map(CUtensorMap* map, const void* base, int64_t inner, int64_t outer
     return r == CUDA_SUCCESS;
 }
 
+// plain (unswizzled) 2-D map for the K2 TMA epilogue: fp32 (elem 4) or 16-bit (elem 2)
+bool encode_plain(CUtensorMap* map, const void* base, int64_t inner, int64_t outer, int64_t ld_elems, int elem,
+                  bool bf16, int box_inner, int box_outer) {
+    if (!g_encode) return false;
+    if ((reinterpret_cast<uintptr_t>(base) & 15) != 0 || ((ld_elems * elem) & 15) != 0) return false;
+    cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld_elems * elem)};
+    cuuint32_t box[2] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer};
+    cuuint32_t estr[2] = {1, 1};
+    const CUtensorMapDataType dt = elem == 4 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                   : bf16    ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                             : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+    CUresult r = g_encode(map, dt, 2, const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
 int pick_bn(int w) { return w <= 32 ? 32 : w <= 64 ? 64 : w <= 128 ? 128 : 256; }
 
 enum ProfClass { PC_UPDATE = 0, PC_PROJ = 1, PC_PANEL = 2, PC_SCALE = 3, PC_CGLS = 4, PC_OTHER = 5, PC_N = 6 };
@@ -116,6 +134,9 @@ struct Op {
     int c0, h, w;
     int bn = 0, tiles_i = 0, tiles_j = 0, splits = 0, kb_total = 0, kb_per_split = 0;
     CUtensorMap ma, mb, ma_lo, mb_lo;
+    CUtensorMap mc;        // UPDATE: fp32 A2 for the TMA epilogue
+    bool te = false;
+    int h0 = 0;            // UPDATE: first output column whose 16-bit image a later K1 reads
 };
 
 struct Plan {
@@ -288,6 +309,16 @@ void build_ops(std::vector<Op>& ops, int c0, int ncols, int nb, bool pair, bool 
     build_ops(ops, c0 + h, w, nb, pair, leaf);
 }
 
+// PROJ op oi (and the UPDATE after it) of the level just above a leaf, run as the leaf's prologue
+bool folded_into_leaf(const Plan& pl, size_t oi) {
+static const bool no_fold64 = getenv("RGSQR_NO_FOLD64") != nullptr;
+const auto& ops = pl.ops;
+const Op& o = ops[oi];
+return pl.leaf && !no_fold64 && rg::leaf_prologue_fits(pl.m) && o.kind == Op::PROJ && o.h <= 64 && o.w <= 64 &&
+       oi + 2 < ops.size() && ops[oi + 1].kind == Op::UPDATE && ops[oi + 1].c0 == o.c0 &&
+       ops[oi + 2].kind == Op::PAIR && ops[oi + 2].c0 == o.c0 + o.h && ops[oi + 2].h + ops[oi + 2].w == o.w;
+}
+
 int make_plan(rg_handle h, Plan& pl) {
     if (!ensure_encode()) return RG_CUDA_ERROR;
     const int64_t m = pl.m;
@@ -305,6 +336,31 @@ int make_plan(rg_handle h, Plan& pl) {
                       (wide ? rg::cholqr_fused_fits(m, 64) : (rg::leaf_fits(m) && !pl.split));
     pl.leaf = pair && !wide;
     build_ops(pl.ops, 0, n, pl.nb, pair, pl.leaf);
+    // 16-bit images written by K2 that nothing reads: a column's image is read only as A2 of a
+    // later K1 before the leaf / panel that factors the column (those read fp32 and write the
+    // image of Q).  In leaf mode that drops the image for the first 128 columns of every K2
+    // output (the w = 128 level writes none).
+    {
+        std::vector<int> last((size_t)n, -1);   // UPDATE op that last wrote the column's image
+        std::vector<int> need(pl.ops.size(), INT_MAX);
+        for (size_t i = 0; i < pl.ops.size(); ++i) {
+            const Op& o = pl.ops[i];
+            if (o.kind == Op::PROJ && !folded_into_leaf(pl, i)) {   // (a folded prologue reads fp32)
+                for (int c = o.c0 + o.h; c < o.c0 + o.h + o.w; ++c)
+                    if (last[c] >= 0) need[last[c]] = std::min(need[last[c]], c);
+            } else if (o.kind == Op::UPDATE) {
+                for (int c = o.c0 + o.h; c < o.c0 + o.h + o.w; ++c) last[c] = (int)i;
+            } else {
+                const int c1 = o.kind == Op::PAIR ? o.c0 + o.h + o.w : o.c0 + o.w;
+                for (int c = o.c0; c < c1; ++c) last[c] = -2;
+            }
+        }
+        for (size_t i = 0; i < pl.ops.size(); ++i)
+            if (pl.ops[i].kind == Op::UPDATE) {
+                Op& o = pl.ops[i];
+                o.h0 = need[i] == INT_MAX ? o.w : std::max(0, need[i] - (o.c0 + o.h));
+            }
+    }
     int max_h = 0, max_w = 0;
     size_t pmax = 0;
     for (auto& o : pl.ops)
@@ -325,6 +381,7 @@ int make_plan(rg_handle h, Plan& pl) {
         const uint16_t* q1l = pl.split ? ql + (int64_t)o.c0 * pl.ldh : q1;
         const uint16_t* a2l = pl.split ? ql + (int64_t)(o.c0 + o.h) * pl.ldh : a2;
         o.bn = pick_bn(o.w);
+        if (o.kind == Op::UPDATE && getenv("RGSQR_K2_BN")) o.bn = std::min(o.bn, atoi(getenv("RGSQR_K2_BN")));
         if (o.kind == Op::PROJ) {
             o.tiles_i = (o.h + 127) / 128;
             o.tiles_j = (o.w + o.bn - 1) / o.bn;
@@ -355,6 +412,7 @@ int make_plan(rg_handle h, Plan& pl) {
                       encode_map(&o.mb_lo, a2l, m, o.w, pl.ldh, 64, o.bn, bf);
             if (!ok) return RG_CUDA_ERROR;
         } else {
+            o.te = !pl.split && encode_plain(&o.mc, pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq, m, o.w, pl.ldq, 4, bf, 128, 32);
             bool ok = encode_map(&o.ma, q1, m, o.h, pl.ldh, 64, 64, bf) &&
                       encode_map(&o.mb, r12h, o.h, o.w, pl.ldr12, 64, o.bn, bf) &&
                       encode_map(&o.ma_lo, q1l, m, o.h, pl.ldh, 64, 64, bf) &&
@@ -423,12 +481,9 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     }
     const Op* pending_update = nullptr;   // leaf-level K2 folded into the next panel's load
     const Op* pending_pro = nullptr;      // K1 + K2 of the level above a leaf, folded into it
-    static const bool no_fold64 = getenv("RGSQR_NO_FOLD64") != nullptr;
     for (size_t oi = 0; oi < pl.ops.size(); ++oi) {
         const Op& o = pl.ops[oi];
-        if (pl.leaf && !no_fold64 && rg::leaf_prologue_fits(m) && o.kind == Op::PROJ && o.h <= 64 && o.w <= 64 && oi + 2 < pl.ops.size() &&
-            pl.ops[oi + 1].kind == Op::UPDATE && pl.ops[oi + 1].c0 == o.c0 && pl.ops[oi + 2].kind == Op::PAIR &&
-            pl.ops[oi + 2].c0 == o.c0 + o.h && pl.ops[oi + 2].h + pl.ops[oi + 2].w == o.w) {
+        if (folded_into_leaf(pl, oi)) {
             pending_pro = &o;
             ++oi;   // the UPDATE too
             continue;
@@ -597,7 +652,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             uint16_t* Ch = qh + (int64_t)(o.c0 + o.h) * pl.ldh;
             uint16_t* Cl = ql ? ql + (int64_t)(o.c0 + o.h) * pl.ldh : nullptr;
             RG_CUDA(rg::launch_update_gemm(o.bn, pl.split != 0, m, o.w, o.h, o.ma, o.mb, o.ma_lo, o.mb_lo, C, pl.ldq, Ch,
-                                           Cl, pl.ldh, pl.bf16, st));
+                                           Cl, pl.ldh, pl.bf16, st, 0, o.te ? &o.mc : nullptr, o.h0));
         }
     }
     {

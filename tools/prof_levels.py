@@ -14,6 +14,8 @@ if os.environ.get("_PROF_CHILD") is None:
         a = agg.setdefault(k, [0, 0.0, []])
         a[0] += 1; a[1] += float(mm.group(3)); a[2].append((float(mm.group(4)), float(mm.group(5))))
     print(p.stdout)
+    if p.returncode != 0:
+        print("child failed, rc", p.returncode, "\n", "\n".join(p.stderr.splitlines()[-20:]))
     tot = sum(v[1] for v in agg.values())
     for (c, w), (n, us, tg) in sorted(agg.items(), key=lambda kv: (kv[0][0], -kv[0][1])):
         tf = sum(t for t, _ in tg) / len(tg); gb = sum(g for _, g in tg) / len(tg)
