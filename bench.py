@@ -29,6 +29,8 @@ sys.path.insert(0, ROOT)
 
 M, N = 65536, 4096                 # BASELINE config 2
 LS_M, LS_N, LS_KAPPA = 131072, 1024, 1e4  # BASELINE config 3
+ORTH_M, ORTH_N = 2097152, 256     # BASELINE config 4
+LR_M, LR_RANK = 32768, 512         # BASELINE config 5
 SAMPLE_COLS_CPU = 640              # cpu_baseline: oracle Householder on 65536 x 640 (~10 s)
 SAMPLE_COLS_REF = 256              # --impl reference: per-step sample 65536 x 256
 
@@ -154,6 +156,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-ls", action="store_true")
+    ap.add_argument("--no-orth", action="store_true")
+    ap.add_argument("--no-lowrank", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
     args = ap.parse_args()
@@ -277,9 +281,22 @@ def main():
     ls = None
     if not args.no_ls and ws == 1 and hasattr(rg.lib(), "ls_solve_refined") and not callable(getattr(rg.lib().ls_solve_refined, "__wrapped__", None)):
         try:
-            ls = bench_ls(rg, torch, h)
+            ls = bench_ls(rg, torch, h, pk)
         except Exception as ex:  # keep the headline line even if the LS leg fails
             ls = {"error": str(ex)[:200]}
+
+    orth = None
+    if not args.no_orth:
+        try:
+            orth = bench_orth(rg, torch, h, ws, rank, dist, pk)
+        except Exception as ex:
+            orth = {"error": str(ex)[:200]}
+    lowrank = None
+    if not args.no_lowrank and ws == 1:
+        try:
+            lowrank = bench_lowrank(rg, torch, h, pk)
+        except Exception as ex:
+            lowrank = {"error": str(ex)[:200]}
 
     cpu = None
     if rank == 0 and not args.no_cpu:
@@ -305,6 +322,8 @@ def main():
             "cpu_baseline": cpu,
             "e2e": e2e,
             "ls": ls,
+            "orthogonalize": orth,
+            "lowrank": lowrank,
             "gpu_launches": (launches * args.steps) if launches else None,
             "clocks": clk.summary(),
         }
@@ -326,7 +345,97 @@ def accuracy_probe(rg, torch, A, Q, R, p=8):
     return {"backward_error": be, "orthogonality_F": orth, "method": "8 Hutchinson probes, fp64 (torch, check only)"}
 
 
-def bench_ls(rg, torch, h):
+def _time_calls(torch, call, restore, reps):
+    """CUDA events around each call on the current stream; the untimed restore runs before it."""
+    st = torch.cuda.current_stream()
+    ts = []
+    for _ in range(reps):
+        restore()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(st)
+        out = call()
+        e1.record(st)
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    return ts, out
+
+
+def bench_orth(rg, torch, h, ws, rank, dist, pk):
+    """BASELINE config 4: orthogonalisation of 2,097,152 x 256 N(0,1), row-sharded over the ws ranks
+    (strong scaling: 2,097,152 / ws rows per rank), reortho until orth <= 1e-5.  Time = max over
+    ranks of the median of 5 calls.  HBM roofline: 8 m n bytes per pass (read A, write Q)."""
+    m_all, n = ORTH_M, ORTH_N
+    m = m_all // ws
+    g = torch.Generator(device="cuda").manual_seed(20200623 + 4 + rank)
+    A0 = torch.randn(n, m, generator=g, device="cuda", dtype=torch.float32).t()
+    A = torch.empty_like(A0.t()).t()
+    R = torch.zeros(n, n, device="cuda").t()
+    res = {}
+
+    def call():
+        _, _, passes, est = rg.orthogonalize(A, R, orth_tol=1e-5, max_passes=3, handle=h)
+        res["passes"], res["est"] = passes, est
+
+    ts, _ = _time_calls(torch, call, lambda: A.copy_(A0), 2 + 5)
+    ms = statistics.median(ts[2:])
+    if dist is not None:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    passes = res["passes"]
+    alg_bytes = 8.0 * m_all * n * passes
+    gbs = alg_bytes / (ms * 1e-3) / 1e9
+    peak = pk["hbm_gbs"] * ws
+    del A0, A
+    return {"workload": f"orthogonalize {m_all}x{n} N(0,1), reortho to 1e-5 (BASELINE config 4), "
+                        f"{'row-sharded x' + str(ws) if ws > 1 else '1 GPU'}",
+            "ms": ms, "passes": passes, "orth_est": res["est"],
+            "tflops": passes * qr_flops(m_all, n) / (ms * 1e-3) / 1e12,
+            "roofline": {"bound": "hbm", "achieved": gbs, "peak": peak, "unit": "GB/s", "frac": gbs / peak,
+                         "alg_bytes": alg_bytes, "note": "8 m n bytes per pass (read A fp32, write Q fp32)"}}
+
+
+def bench_lowrank(rg, torch, h, pk):
+    """BASELINE config 5: randomized rank-512 approximation of a 32768 x 32768 matrix (p = 16,
+    q = 1).  Roofline: max(HBM, tensor) over the (2 + 2q) passes over A, each 2 m n l flops and
+    4 m n bytes (fp32 A read)."""
+    import numpy as np
+    import synth
+    m = n = LR_M
+    rank, p, q = LR_RANK, 16, 1
+    At, s = synth.lowrank_matrix(m, n, 2048, "geometric", 1e6, seed=synth.SEED_BASE + 5, device="cuda")
+    A = At.t()
+    U = torch.empty(rank, m, device="cuda").t()
+    S = torch.empty(rank, device="cuda")
+    V = torch.empty(rank, n, device="cuda").t()
+
+    def call():
+        rg.lowrank_approx(A, rank, oversample=p, power_iters=q, seed=7, U=U, S=S, V=V, handle=h)
+
+    ts, _ = _time_calls(torch, call, lambda: None, 2 + 5)
+    ms = statistics.median(ts[2:])
+    l = rank + p
+    passes = 2 + 2 * q
+    t_tc = passes * 2.0 * m * n * l / (pk["bf16_tflops_sustained"] * 1e12)
+    t_hbm = passes * 4.0 * m * n / (pk["hbm_gbs"] * 1e9)
+    roof_ms = max(t_tc, t_hbm) * 1e3
+    # accuracy: ||A - U S V^T||_F / ||A||_F against the closed-form optimum (check only)
+    U64, V64, S64 = U.double(), V.double(), S.double()
+    num = 0.0
+    for j0 in range(0, n, 4096):
+        num += torch.linalg.norm(A[:, j0:j0 + 4096].double() - (U64 * S64) @ V64[j0:j0 + 4096].t()).item() ** 2
+    err = (num / float(np.sum(s ** 2))) ** 0.5
+    opt = float(np.sqrt(np.sum(s[rank:] ** 2) / np.sum(s ** 2)))
+    del A, At, U64, V64
+    return {"workload": f"randomized low rank {m}x{n}, rank {rank}, p {p}, q {q} (BASELINE config 5)",
+            "ms": ms, "lr_error": err, "lr_optimal": opt, "ratio_to_optimal": err / opt,
+            "roofline": {"bound": "hbm" if t_hbm >= t_tc else "tensor", "roofline_ms": roof_ms,
+                         "frac": roof_ms / ms,
+                         "note": f"{passes} passes over fp32 A: max({passes} x 2mnl flops at the sustained bf16 peak, "
+                                 f"{passes} x 4mn bytes at the copy bandwidth)"}}
+
+
+def bench_ls(rg, torch, h, pk):
     import numpy as np
     import synth
     A = synth.svd_matrix(LS_M, LS_N, "geometric", LS_KAPPA, seed=synth.SEED_BASE + 2)
@@ -351,7 +460,14 @@ def bench_ls(rg, torch, h):
     x_ref32 = np.linalg.lstsq(A.astype(np.float32).astype(np.float64), b.astype(np.float32).astype(np.float64),
                               rcond=None)[0]
     xv = x.cpu().numpy()
+    # roofline: k CGLS iterations x 8mn bytes at the copy bandwidth + the two
+    # RGSQR passes (factor + 1 reortho) at the sustained tensor peak
+    roof_ms = (it * 8.0 * LS_M * LS_N / (pk["hbm_gbs"] * 1e9)
+               + 2 * qr_flops(LS_M, LS_N) / (pk["bf16_tflops_sustained"] * 1e12)) * 1e3
     return {"workload": f"LS {LS_M}x{LS_N} cond 1e4 geometric, b ~ N(0,1) (BASELINE config 3)", "ms": ms,
+            "roofline": {"roofline_ms": roof_ms, "frac": roof_ms / ms,
+                         "note": "iters x 8mn bytes (A read twice per CGLS iteration) at the copy bandwidth "
+                                 "+ 2 RGSQR passes at the sustained tensor peak"},
             "iters": it, "relres": rel, "status": status,
             "fe_vs_fp32_problem": float(np.linalg.norm(xv - x_ref32) / np.linalg.norm(x_ref32)),
             "fe_vs_fp64_problem": float(np.linalg.norm(xv - x_ref) / np.linalg.norm(x_ref))}

@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "kernels.h"
 
@@ -157,6 +158,165 @@ __global__ void __launch_bounds__(256) jacobi_sweeps_kernel(double* __restrict__
     if (gwarp == 0 && lane == 0) flags[1] = sweep;
 }
 
+// ------------------------------------------------------------------ cluster Jacobi (l <= 576)
+// Same rotations, Brent-Luk parallel ordering, but the columns live in registers: warp k of a
+// thread-block cluster (<= 16 CTAs) holds the pair (top_k, bot_k), NPL doubles per lane per column
+// (element u * 32 + lane).  After each round the pairs move along the ring
+//   top_1 <- bot_0, top_k <- top_{k-1} (k >= 2), bot_k <- bot_{k+1} (k <= P - 2), bot_{P-1} <- top_{P-1}
+// through the receivers' shared-memory slots (distributed shared memory stores), two cluster
+// barriers per round; P (P - 1) ... every pair of the 2P columns meets once per 2P - 1 rounds.
+// V is not accumulated: V_b = R^T W S^{-2} afterwards (jacobi_rank_rt_kernel).  Replaces the
+// grid-synchronised kernel above, whose L2-latency-bound rounds cost ~14 us each (70 ms at l = 528).
+template <int NPL>
+__global__ void __launch_bounds__(576, 1) jacobi_cluster_kernel(double* __restrict__ W, int l, int P, int wper,
+                                                                int max_sweeps, double tol, int* flags) {
+    cg::cluster_group cl = cg::this_cluster();
+    extern __shared__ __align__(16) double jc_smem[];
+    double* slot = jc_smem;                                              // [wper][2][NPL * 32]
+    int* sid = reinterpret_cast<int*>(slot + (size_t)wper * 2 * NPL * 32);   // [wper][2]
+    __shared__ int rot_flag;
+    const int crank = (int)cl.block_rank();
+    const int csize = (int)cl.num_blocks();
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int gw = crank * wper + warp;
+    const bool active = warp < wper && gw < P;
+    double x[NPL], y[NPL];
+    int ix = 2 * gw, iy = 2 * gw + 1;
+#pragma unroll
+    for (int u = 0; u < NPL; ++u) {
+        const int i = u * 32 + lane;
+        x[u] = (active && ix < l && i < l) ? W[(int64_t)ix * l + i] : 0.0;
+        y[u] = (active && iy < l && i < l) ? W[(int64_t)iy * l + i] : 0.0;
+    }
+    // where this warp's outgoing columns go: (cta, warp, slot 0 = top / 1 = bot)
+    auto slot_ptr = [&](int g, int which) -> double* {
+        double* local = slot + ((size_t)(g % wper) * 2 + which) * NPL * 32;
+        return cl.map_shared_rank(local, g / wper);
+    };
+    auto sid_ptr = [&](int g, int which) -> int* { return cl.map_shared_rank(sid + (g % wper) * 2 + which, g / wper); };
+    int sweep = 0;
+    for (; sweep < max_sweeps; ++sweep) {
+        if (threadIdx.x == 0) rot_flag = 0;
+        int any = 0;
+        cl.sync();
+        for (int r = 0; r < 2 * P - 1; ++r) {
+            if (active && ix < l && iy < l) {
+                double a = 0.0, b = 0.0, g = 0.0;
+#pragma unroll
+                for (int u = 0; u < NPL; ++u) {
+                    a = fma(x[u], x[u], a);
+                    b = fma(y[u], y[u], b);
+                    g = fma(x[u], y[u], g);
+                }
+                a = wsum(a);
+                b = wsum(b);
+                g = wsum(g);
+                if (!(fabs(g) <= tol * sqrt(a * b) || g == 0.0)) {
+                    any = 1;
+                    const double zeta = (b - a) / (2.0 * g);
+                    const double t = (zeta >= 0.0 ? 1.0 : -1.0) / (fabs(zeta) + sqrt(1.0 + zeta * zeta));
+                    const double c = 1.0 / sqrt(1.0 + t * t), sn = c * t;
+#pragma unroll
+                    for (int u = 0; u < NPL; ++u) {
+                        const double xv = x[u], yv = y[u];
+                        x[u] = c * xv - sn * yv;
+                        y[u] = sn * xv + c * yv;
+                    }
+                }
+            }
+            if (P == 1) continue;
+            if (active) {
+                if (gw >= 1 && gw <= P - 2) {   // top -> top slot of gw + 1
+                    double* d = slot_ptr(gw + 1, 0);
+#pragma unroll
+                    for (int u = 0; u < NPL; ++u) d[u * 32 + lane] = x[u];
+                    if (lane == 0) *sid_ptr(gw + 1, 0) = ix;
+                }
+                {   // bot -> bot slot of gw - 1, or (gw = 0) the top slot of warp 1
+                    double* d = gw >= 1 ? slot_ptr(gw - 1, 1) : slot_ptr(1, 0);
+#pragma unroll
+                    for (int u = 0; u < NPL; ++u) d[u * 32 + lane] = y[u];
+                    if (lane == 0) *(gw >= 1 ? sid_ptr(gw - 1, 1) : sid_ptr(1, 0)) = iy;
+                }
+            }
+            cl.sync();
+            if (active) {
+                const double* mt = slot + ((size_t)warp * 2 + 0) * NPL * 32;
+                const double* mb = slot + ((size_t)warp * 2 + 1) * NPL * 32;
+                if (gw == P - 1) {   // bot <- own top, top <- slot
+#pragma unroll
+                    for (int u = 0; u < NPL; ++u) y[u] = x[u];
+                    iy = ix;
+                } else {
+#pragma unroll
+                    for (int u = 0; u < NPL; ++u) y[u] = mb[u * 32 + lane];
+                    iy = sid[warp * 2 + 1];
+                }
+                if (gw >= 1) {
+#pragma unroll
+                    for (int u = 0; u < NPL; ++u) x[u] = mt[u * 32 + lane];
+                    ix = sid[warp * 2 + 0];
+                }
+            }
+            cl.sync();
+        }
+        if (any && lane == 0) atomicOr(&rot_flag, 1);
+        cl.sync();
+        int tot = 0;
+        for (int c = 0; c < csize; ++c) tot |= *cl.map_shared_rank(&rot_flag, c);
+        cl.sync();
+        if (!tot) {
+            ++sweep;
+            break;
+        }
+    }
+    if (active) {
+#pragma unroll
+        for (int u = 0; u < NPL; ++u) {
+            const int i = u * 32 + lane;
+            if (i < l) {
+                if (ix < l) W[(int64_t)ix * l + i] = x[u];
+                if (iy < l) W[(int64_t)iy * l + i] = y[u];
+            }
+        }
+    }
+    if (crank == 0 && threadIdx.x == 0) flags[1] = sweep;
+}
+
+// Ranks by descending sigma_j = |w_j| (ties by index); for rank < r: S, Ub(:, rank) = w_j / sigma_j,
+// Vb(:, rank) = R^T w_j / sigma_j^2 (R = U_b S V_b^T => V_b = R^T U_b S^{-1}); fp64, one CTA per j.
+__global__ void jacobi_rank_rt_kernel(const double* __restrict__ W, const float* __restrict__ R, int64_t ldr, int l,
+                                      int r, const double* __restrict__ sig, float* __restrict__ S,
+                                      float* __restrict__ Ub, float* __restrict__ Vb) {
+    RG_PDL_ENTRY();
+    extern __shared__ double wcol[];
+    const int j = blockIdx.x;
+    __shared__ int s_rank;
+    if (threadIdx.x == 0) {
+        const double sj = sig[j];
+        int rank = 0;
+        for (int i = 0; i < l; ++i) {
+            const double si = sig[i];
+            rank += (si > sj) || (si == sj && i < j);
+        }
+        s_rank = rank;
+    }
+    for (int i = threadIdx.x; i < l; i += blockDim.x) wcol[i] = W[i + (int64_t)j * l];
+    __syncthreads();
+    const int rank = s_rank;
+    if (rank >= r) return;
+    const double sj = sig[j];
+    if (threadIdx.x == 0) S[rank] = (float)sj;
+    const double inv = sj > 0.0 ? 1.0 / sj : 0.0;
+    for (int i = threadIdx.x; i < l; i += blockDim.x) {
+        Ub[i + (int64_t)rank * l] = (float)(wcol[i] * inv);
+        const float* rc = R + (int64_t)i * ldr;   // column i of R: R(k, i), k <= i
+        double v = 0.0;
+        for (int k = 0; k <= i; ++k) v = fma((double)rc[k], wcol[k], v);
+        Vb[i + (int64_t)rank * l] = (float)(v * inv * inv);
+    }
+}
+
 // sigma_j = |w_j|; rank by descending sigma (ties by index); for rank < r write
 // S[rank], Ub[:, rank] = w_j / sigma_j (fp32, ld l), Vb[:, rank] = v_j (fp32, ld l).
 __global__ void jacobi_extract_kernel(const double* __restrict__ W, const double* __restrict__ V, int l, int r,
@@ -236,6 +396,47 @@ cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double*
                                                                                                              W, V);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
+    if (l <= 576 && getenv("RGSQR_JACOBI_GRID") == nullptr) {
+        const int P = (l + 1) / 2;
+        const int cs = std::max(1, std::min(16, (P + 17) / 18));   // <= 18 warps (576 threads) per CTA
+        const int wper = (P + cs - 1) / cs;
+        const int npl = (l + 31) / 32;
+        int max_sweeps = 40;
+        double tol = 1e-13;
+        cudaLaunchConfig_t cfg{};
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = cs;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.gridDim = dim3(cs);
+        cfg.blockDim = dim3(32 * wper);
+        cfg.stream = st;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        auto go = [&](auto kern, int np) -> cudaError_t {
+            cfg.dynamicSmemBytes = (size_t)wper * 2 * np * 32 * 8 + (size_t)wper * 2 * 4 + 16;
+            cudaError_t e2 = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                  (int)cfg.dynamicSmemBytes);
+            if (e2 != cudaSuccess) return e2;
+            if (cs > 8) {
+                e2 = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+                if (e2 != cudaSuccess) return e2;
+            }
+            ++g_launches;
+            return cudaLaunchKernelEx(&cfg, kern, W, l, P, wper, max_sweeps, tol, flags);
+        };
+        if (npl <= 4) e = go(jacobi_cluster_kernel<4>, 4);
+        else if (npl <= 8) e = go(jacobi_cluster_kernel<8>, 8);
+        else if (npl <= 12) e = go(jacobi_cluster_kernel<12>, 12);
+        else e = go(jacobi_cluster_kernel<18>, 18);
+        if (e != cudaSuccess) return e;
+        RG_LAUNCH((jacobi_extract_kernel), l, 256, 0, st, W, V, l, r, S, Ub, Vb, sig);
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        RG_LAUNCH((jacobi_rank_rt_kernel), l, 256, (size_t)l * 8, st, W, R, ldr, l, r, sig, S, Ub, Vb);
+        return cudaGetLastError();
+    }
     int dev = 0, sms = 148, per_sm = 1;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);

@@ -60,3 +60,25 @@ def test_lowrank_config5_scaled(rg):
     opt = np.sqrt(np.sum(sfull[256:] ** 2) / np.sum(sfull ** 2))
     err = oracle.lowrank_error(A.astype(np.float64), U, S, V)
     assert err / opt < 1.05, (err, opt)   # reading #17: ~1.016 with q = 1
+
+
+def test_lowrank_cluster_jacobi_matches_grid_jacobi(rg, monkeypatch):
+    """The register/cluster Jacobi (V_b = R^T U_b S^-2) and the grid-synchronised Jacobi (V_b
+    accumulated) give the same factorisation up to rounding."""
+    m, n = 4096, 1024
+    A, s = synth.lowrank_matrix(m, n, 300, "geometric", 1e4, seed=77)
+    outs = []
+    for env in (None, "1"):
+        if env:
+            monkeypatch.setenv("RGSQR_JACOBI_GRID", env)
+        U, S, V = rg.lowrank_approx(_dev(A), 200, oversample=16, power_iters=1, seed=3)
+        outs.append([x.cpu().numpy().astype(np.float64) for x in (U, S, V)])
+    (U1, S1, V1), (U2, S2, V2) = outs
+    np.testing.assert_allclose(S1, S2, rtol=1e-5)
+    # singular vectors up to sign
+    for X1, X2 in ((U1, U2), (V1, V2)):
+        d = np.sign(np.sum(X1 * X2, axis=0))
+        assert np.linalg.norm(X1 - X2 * d) / np.linalg.norm(X1) < 1e-3
+    err1 = oracle.lowrank_error(A.astype(np.float64), U1, S1, V1)
+    err2 = oracle.lowrank_error(A.astype(np.float64), U2, S2, V2)
+    assert abs(err1 - err2) <= 1e-4 * err2

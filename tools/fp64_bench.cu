@@ -30,6 +30,32 @@ __global__ void dmma_tp(double* out, int n) {
     }
     out[blockIdx.x * blockDim.x + threadIdx.x] = c0 + c1 + d0 + d1 + e0 + e1 + f0 + f1;
 }
+// larger fp64 shapes (sm_90+): m16n8k4 (A 2 regs, B 1, C 4), m16n8k8 (A 4, B 2), m16n8k16 (A 8, B 4)
+__global__ void dmma16_tp(double* out, int n) {
+    double a = threadIdx.x * 1e-3, b = 1.0 + threadIdx.x * 1e-4;
+    double c[4][4] = {};
+    for (int i = 0; i < n; ++i) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            asm volatile("mma.sync.aligned.m16n8k4.row.col.f64.f64.f64.f64 {%0,%1,%2,%3}, {%4,%5}, {%6}, {%0,%1,%2,%3};"
+                         : "+d"(c[u][0]), "+d"(c[u][1]), "+d"(c[u][2]), "+d"(c[u][3]) : "d"(a), "d"(a), "d"(b));
+    }
+    double s = 0; for (int u = 0; u < 4; ++u) for (int v = 0; v < 4; ++v) s += c[u][v];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+__global__ void dmma16k16_tp(double* out, int n) {
+    double a = threadIdx.x * 1e-3, b = 1.0 + threadIdx.x * 1e-4;
+    double c[4][4] = {};
+    for (int i = 0; i < n; ++i) {
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            asm volatile("mma.sync.aligned.m16n8k16.row.col.f64.f64.f64.f64 {%0,%1,%2,%3}, {%4,%5,%6,%7,%8,%9,%10,%11}, {%12,%13,%14,%15}, {%0,%1,%2,%3};"
+                         : "+d"(c[u][0]), "+d"(c[u][1]), "+d"(c[u][2]), "+d"(c[u][3])
+                         : "d"(a), "d"(a), "d"(a), "d"(a), "d"(a), "d"(a), "d"(a), "d"(a), "d"(b), "d"(b), "d"(b), "d"(b));
+    }
+    double s = 0; for (int u = 0; u < 4; ++u) for (int v = 0; v < 4; ++v) s += c[u][v];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
 int main() {
     double* out; float* in;
     cudaMalloc(&out, 148 * 1024 * 8 * 4); cudaMalloc(&in, 4096);
@@ -50,6 +76,16 @@ int main() {
     cudaEventElapsedTime(&ms, a, b);
     fl = 148.0 * 4 * 8 * n * 4 * 256;   // warps * mma * 256 FMA
     printf("DMMA m8n8k4: %.2f TFMA/s -> %.1f FMA/clk/SM (%s)\n", fl / ms / 1e9, fl / ms / 1e-3 / 148 / 1.9e9,
+           cudaGetErrorString(cudaGetLastError()));
+    cudaEventRecord(a); dmma16_tp<<<148 * 4, 256>>>(out, n); cudaEventRecord(b); cudaEventSynchronize(b);
+    cudaEventElapsedTime(&ms, a, b);
+    fl = 148.0 * 4 * 8 * n * 4 * 512;
+    printf("DMMA m16n8k4: %.2f TFMA/s -> %.1f FMA/clk/SM (%s)\n", fl / ms / 1e9, fl / ms / 1e-3 / 148 / 1.9e9,
+           cudaGetErrorString(cudaGetLastError()));
+    cudaEventRecord(a); dmma16k16_tp<<<148 * 4, 256>>>(out, n / 4); cudaEventRecord(b); cudaEventSynchronize(b);
+    cudaEventElapsedTime(&ms, a, b);
+    fl = 148.0 * 4 * 8 * (n / 4) * 4 * 2048;
+    printf("DMMA m16n8k16: %.2f TFMA/s -> %.1f FMA/clk/SM (%s)\n", fl / ms / 1e9, fl / ms / 1e-3 / 148 / 1.9e9,
            cudaGetErrorString(cudaGetLastError()));
     return 0;
 }

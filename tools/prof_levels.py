@@ -1,4 +1,7 @@
-"""Per-op event profile of one RGSQR call at BASELINE config 2, summarised per (class, width)."""
+"""Per-op event profile of one call, summarised per (class, width).
+
+RG_CALL=factor (default, BASELINE config 2: RG_M x RG_N) | orth (orthogonalize, config 4 with
+RG_M=2097152 RG_N=256) | lowrank (config 5, RG_M x RG_M, rank 512)."""
 import os, sys, subprocess, collections, re
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 if os.environ.get("_PROF_CHILD") is None:
@@ -25,14 +28,35 @@ if os.environ.get("_PROF_CHILD") is None:
 import torch
 import paper_conf_hpdc_zhangbw20_b200 as rg
 m = int(os.environ.get("RG_M", 65536)); n = int(os.environ.get("RG_N", 4096))
+call = os.environ.get("RG_CALL", "factor")
 h = rg.Handle(0)
+if call == "lowrank":
+    n = m
 A = torch.randn(n, m, device="cuda").t()
-Q = torch.empty(n, m, device="cuda").t(); R = torch.empty(n, n, device="cuda").t()
+A0 = A.clone() if call == "orth" else None
+Q = torch.empty(n, m, device="cuda").t() if call == "factor" else None
+R = torch.empty(n, n, device="cuda").t() if call != "lowrank" else None
 o = rg.make_opts(sync=False)
+
+
+def run():
+    if call == "factor":
+        rg.rgsqr_factor(A, Q=Q, R=R, handle=h, opts=o, check=False)
+    elif call == "orth":
+        A.copy_(A0)
+        print("passes", rg.orthogonalize(A, R, orth_tol=1e-5, max_passes=3, handle=h)[2:])
+    else:
+        rg.lowrank_approx(A, 512, oversample=16, power_iters=1, seed=7, handle=h)
+
+
 for _ in range(3):
-    rg.rgsqr_factor(A, Q=Q, R=R, handle=h, opts=o, check=False)
+    run()
 torch.cuda.synchronize()
 h.profile(True); h.profile_reset()
-rg.rgsqr_factor(A, Q=Q, R=R, handle=h, opts=o, check=False)
+ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+ev[0].record()
+run()
+ev[1].record()
 torch.cuda.synchronize()
+print("call ms (events, profiling on)", ev[0].elapsed_time(ev[1]))
 print({c: h.profile_get(c) for c in ("update", "proj", "panel", "scale", "other")})
