@@ -68,12 +68,15 @@ __global__ void unscale_rows_kernel(float* __restrict__ X, int64_t ldx, int64_t 
 
 // W (l x l fp64, ld l) = R (upper fp32, ldr), V = I
 __global__ void jacobi_init_kernel(const float* __restrict__ R, int64_t ldr, int l, double* __restrict__ W,
-                                   double* __restrict__ V) {
+                                   double* __restrict__ V, int trans) {
     RG_PDL_ENTRY();
     const int64_t total = (int64_t)l * l;
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
         const int i = (int)(e % l), j = (int)(e / l);
-        W[e] = (i <= j) ? (double)R[i + (int64_t)j * ldr] : 0.0;
+        if (trans)
+            W[e] = (j <= i) ? (double)R[j + (int64_t)i * ldr] : 0.0;
+        else
+            W[e] = (i <= j) ? (double)R[i + (int64_t)j * ldr] : 0.0;
         V[e] = (i == j) ? 1.0 : 0.0;
     }
 }
@@ -158,126 +161,169 @@ __global__ void __launch_bounds__(256) jacobi_sweeps_kernel(double* __restrict__
     if (gwarp == 0 && lane == 0) flags[1] = sweep;
 }
 
-// ------------------------------------------------------------------ cluster Jacobi (l <= 576)
-// Same rotations, Brent-Luk parallel ordering, but the columns live in registers: warp k of a
-// thread-block cluster (<= 16 CTAs) holds the pair (top_k, bot_k), NPL doubles per lane per column
-// (element u * 32 + lane).  After each round the pairs move along the ring
-//   top_1 <- bot_0, top_k <- top_{k-1} (k >= 2), bot_k <- bot_{k+1} (k <= P - 2), bot_{P-1} <- top_{P-1}
-// through the receivers' shared-memory slots (distributed shared memory stores), two cluster
-// barriers per round; P (P - 1) ... every pair of the 2P columns meets once per 2P - 1 rounds.
-// V is not accumulated: V_b = R^T W S^{-2} afterwards (jacobi_rank_rt_kernel).  Replaces the
-// grid-synchronised kernel above, whose L2-latency-bound rounds cost ~14 us each (70 ms at l = 528).
+// ------------------------------------------------------------------ cluster Jacobi (l <= 544)
+// Same rotations, block-cyclic parallel ordering, columns resident in registers.  A thread-block
+// cluster of cs CTAs x wper warps covers 2 cs wper >= l columns (padding columns are zero and never
+// rotated); warp i of a CTA holds one column of each of the CTA's two blocks (x: "top" block,
+// y: "bot" block), NPL doubles per lane (element u * 32 + lane).  One sweep:
+//   1. all pairs among the CTA's own 2 wper columns: round-robin (Brent-Luk) over its warps, column
+//      moves through shared memory (the two blocks are then re-formed as the x-set and y-set);
+//   2. 2 cs - 2 rounds of a round-robin over the 2 cs blocks between CTAs (block moves by
+//      distributed-shared-memory stores, two cluster barriers per round); in each, the wper x wper
+//      pairs of the CTA's two blocks: wper local rounds, the y block shifted one warp per round.
+// Every pair of columns meets once per sweep (intra-block pairs in step 1, the CTA's own block pair
+// in step 1, every other block pair in step 2).  Converged when no rotation fired in a sweep.
+// V is not accumulated: V_b = R^T W S^{-2} afterwards (jacobi_rank_rt_kernel).  At l = 528 this
+// replaces a one-pair-per-warp ordering with 527 cluster-synchronised rounds per sweep (28 ms) and
+// a grid-synchronised kernel with L2-latency-bound rounds (70 ms).
 template <int NPL>
-__global__ void __launch_bounds__(576, 1) jacobi_cluster_kernel(double* __restrict__ W, int l, int P, int wper,
+__device__ __forceinline__ double jc_dot(const double (&x)[NPL], const double (&y)[NPL]) {
+    double g0 = 0.0, g1 = 0.0;   // two accumulators: halves the dependent DFMA chain
+#pragma unroll
+    for (int u = 0; u < NPL; u += 2) {
+        g0 = fma(x[u], y[u], g0);
+        if (u + 1 < NPL) g1 = fma(x[u + 1], y[u + 1], g1);
+    }
+    return wsum(g0 + g1);
+}
+
+// One Hestenes rotation of (x, y) with their squared norms a, b carried along (updated as
+// a - t g, b + t g instead of recomputed: one dot product per rotation).
+template <int NPL>
+__device__ __forceinline__ bool jc_rotate(double (&x)[NPL], double (&y)[NPL], double& a, double& b, int ix, int iy,
+                                          int l, double tol) {
+    if (ix >= l || iy >= l) return false;
+    const double g = jc_dot<NPL>(x, y);
+    if (g * g <= tol * tol * (a * b) || g == 0.0) return false;
+    const double zeta = (b - a) / (2.0 * g);
+    const double t = (zeta >= 0.0 ? 1.0 : -1.0) / (fabs(zeta) + sqrt(1.0 + zeta * zeta));
+    const double c = rsqrt(1.0 + t * t), sn = c * t;
+#pragma unroll
+    for (int u = 0; u < NPL; ++u) {
+        const double xv = x[u], yv = y[u];
+        x[u] = c * xv - sn * yv;
+        y[u] = sn * xv + c * yv;
+    }
+    a -= t * g;
+    b += t * g;
+    return true;
+}
+
+template <int NPL>
+__global__ void __launch_bounds__(544, 1) jacobi_cluster_kernel(double* __restrict__ W, int l, int wper,
                                                                 int max_sweeps, double tol, int* flags) {
     cg::cluster_group cl = cg::this_cluster();
     extern __shared__ __align__(16) double jc_smem[];
-    double* slot = jc_smem;                                              // [wper][2][NPL * 32]
-    int* sid = reinterpret_cast<int*>(slot + (size_t)wper * 2 * NPL * 32);   // [wper][2]
+    double* buf = jc_smem;                                                      // [2][wper][NPL * 32]
+    double* bnrm = buf + (size_t)2 * wper * NPL * 32;                            // [2][wper] squared norms
+    int* bid = reinterpret_cast<int*>(bnrm + 2 * wper);                          // [2][wper] column ids
     __shared__ int rot_flag;
     const int crank = (int)cl.block_rank();
-    const int csize = (int)cl.num_blocks();
+    const int cs = (int)cl.num_blocks();
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int gw = crank * wper + warp;
-    const bool active = warp < wper && gw < P;
+    auto slot = [&](int which, int w) { return buf + ((size_t)which * wper + w) * NPL * 32; };
     double x[NPL], y[NPL];
-    int ix = 2 * gw, iy = 2 * gw + 1;
+    double na = 0.0, nb = 0.0;
+    int ix = (2 * crank) * wper + warp, iy = (2 * crank + 1) * wper + warp;
 #pragma unroll
     for (int u = 0; u < NPL; ++u) {
         const int i = u * 32 + lane;
-        x[u] = (active && ix < l && i < l) ? W[(int64_t)ix * l + i] : 0.0;
-        y[u] = (active && iy < l && i < l) ? W[(int64_t)iy * l + i] : 0.0;
+        x[u] = (ix < l && i < l) ? W[(int64_t)ix * l + i] : 0.0;
+        y[u] = (iy < l && i < l) ? W[(int64_t)iy * l + i] : 0.0;
     }
-    // where this warp's outgoing columns go: (cta, warp, slot 0 = top / 1 = bot)
-    auto slot_ptr = [&](int g, int which) -> double* {
-        double* local = slot + ((size_t)(g % wper) * 2 + which) * NPL * 32;
-        return cl.map_shared_rank(local, g / wper);
+    // column v, its id and norm into slot (which, w) of CTA `cta` (local when cta < 0)
+    auto put = [&](int cta, int which, int w, const double (&v)[NPL], int id, double nrm) {
+        double* d = slot(which, w);
+        double* dn = bnrm + which * wper + w;
+        int* di = bid + which * wper + w;
+        if (cta >= 0) {
+            d = cl.map_shared_rank(d, cta);
+            dn = cl.map_shared_rank(dn, cta);
+            di = cl.map_shared_rank(di, cta);
+        }
+#pragma unroll
+        for (int u = 0; u < NPL; ++u) d[u * 32 + lane] = v[u];
+        if (lane == 0) {
+            *dn = nrm;
+            *di = id;
+        }
     };
-    auto sid_ptr = [&](int g, int which) -> int* { return cl.map_shared_rank(sid + (g % wper) * 2 + which, g / wper); };
+    auto get = [&](int which, double (&v)[NPL], int& id, double& nrm) {
+        const double* d = slot(which, warp);
+#pragma unroll
+        for (int u = 0; u < NPL; ++u) v[u] = d[u * 32 + lane];
+        id = bid[which * wper + warp];
+        nrm = bnrm[which * wper + warp];
+    };
     int sweep = 0;
     for (; sweep < max_sweeps; ++sweep) {
         if (threadIdx.x == 0) rot_flag = 0;
-        int any = 0;
+        bool any = false;
+        na = jc_dot<NPL>(x, x);   // exact norms once per sweep (the rotations update them)
+        nb = jc_dot<NPL>(y, y);
         cl.sync();
-        for (int r = 0; r < 2 * P - 1; ++r) {
-            if (active && ix < l && iy < l) {
-                double a = 0.0, b = 0.0, g = 0.0;
+        // ---- 1. all pairs among the CTA's 2 wper columns (Brent-Luk over the warps)
+        for (int r = 0; r < 2 * wper - 1; ++r) {
+            any |= jc_rotate<NPL>(x, y, na, nb, ix, iy, l, tol);
+            if (wper == 1) break;
+            if (warp >= 1 && warp <= wper - 2) put(-1, 0, warp + 1, x, ix, na);
+            if (warp >= 1) put(-1, 1, warp - 1, y, iy, nb);
+            else put(-1, 0, 1, y, iy, nb);
+            __syncthreads();
+            if (warp == wper - 1) {
 #pragma unroll
-                for (int u = 0; u < NPL; ++u) {
-                    a = fma(x[u], x[u], a);
-                    b = fma(y[u], y[u], b);
-                    g = fma(x[u], y[u], g);
-                }
-                a = wsum(a);
-                b = wsum(b);
-                g = wsum(g);
-                if (!(fabs(g) <= tol * sqrt(a * b) || g == 0.0)) {
-                    any = 1;
-                    const double zeta = (b - a) / (2.0 * g);
-                    const double t = (zeta >= 0.0 ? 1.0 : -1.0) / (fabs(zeta) + sqrt(1.0 + zeta * zeta));
-                    const double c = 1.0 / sqrt(1.0 + t * t), sn = c * t;
-#pragma unroll
-                    for (int u = 0; u < NPL; ++u) {
-                        const double xv = x[u], yv = y[u];
-                        x[u] = c * xv - sn * yv;
-                        y[u] = sn * xv + c * yv;
-                    }
-                }
+                for (int u = 0; u < NPL; ++u) y[u] = x[u];
+                iy = ix;
+                nb = na;
+            } else {
+                get(1, y, iy, nb);
             }
-            if (P == 1) continue;
-            if (active) {
-                if (gw >= 1 && gw <= P - 2) {   // top -> top slot of gw + 1
-                    double* d = slot_ptr(gw + 1, 0);
-#pragma unroll
-                    for (int u = 0; u < NPL; ++u) d[u * 32 + lane] = x[u];
-                    if (lane == 0) *sid_ptr(gw + 1, 0) = ix;
-                }
-                {   // bot -> bot slot of gw - 1, or (gw = 0) the top slot of warp 1
-                    double* d = gw >= 1 ? slot_ptr(gw - 1, 1) : slot_ptr(1, 0);
-#pragma unroll
-                    for (int u = 0; u < NPL; ++u) d[u * 32 + lane] = y[u];
-                    if (lane == 0) *(gw >= 1 ? sid_ptr(gw - 1, 1) : sid_ptr(1, 0)) = iy;
-                }
-            }
+            if (warp >= 1) get(0, x, ix, na);
+            __syncthreads();
+        }
+        // ---- 2. block pairs between CTAs
+        for (int tr = 1; tr <= 2 * cs - 2; ++tr) {
             cl.sync();
-            if (active) {
-                const double* mt = slot + ((size_t)warp * 2 + 0) * NPL * 32;
-                const double* mb = slot + ((size_t)warp * 2 + 1) * NPL * 32;
-                if (gw == P - 1) {   // bot <- own top, top <- slot
-#pragma unroll
-                    for (int u = 0; u < NPL; ++u) y[u] = x[u];
-                    iy = ix;
-                } else {
-#pragma unroll
-                    for (int u = 0; u < NPL; ++u) y[u] = mb[u * 32 + lane];
-                    iy = sid[warp * 2 + 1];
-                }
-                if (gw >= 1) {
-#pragma unroll
-                    for (int u = 0; u < NPL; ++u) x[u] = mt[u * 32 + lane];
-                    ix = sid[warp * 2 + 0];
-                }
-            }
+            if (crank >= 1 && crank <= cs - 2) put(crank + 1, 0, warp, x, ix, na);   // x block -> CTA + 1
+            if (crank >= 1) put(crank - 1, 1, warp, y, iy, nb);                       // y block -> CTA - 1
+            else put(1, 0, warp, y, iy, nb);                                          // (CTA 0: -> x of CTA 1)
             cl.sync();
+            if (crank == cs - 1) {
+#pragma unroll
+                for (int u = 0; u < NPL; ++u) y[u] = x[u];
+                iy = ix;
+                nb = na;
+            } else {
+                get(1, y, iy, nb);
+            }
+            if (crank >= 1) get(0, x, ix, na);
+            __syncthreads();
+            // the wper x wper pairs (x_i, y_{i+s}): shift y one warp down per round
+            for (int sft = 0; sft < wper; ++sft) {
+                any |= jc_rotate<NPL>(x, y, na, nb, ix, iy, l, tol);
+                if (sft == wper - 1) break;
+                const int p = sft & 1;
+                put(-1, p, (warp + wper - 1) % wper, y, iy, nb);
+                __syncthreads();
+                get(p, y, iy, nb);
+            }
         }
         if (any && lane == 0) atomicOr(&rot_flag, 1);
         cl.sync();
         int tot = 0;
-        for (int c = 0; c < csize; ++c) tot |= *cl.map_shared_rank(&rot_flag, c);
+        for (int c = 0; c < cs; ++c) tot |= *cl.map_shared_rank(&rot_flag, c);
         cl.sync();
         if (!tot) {
             ++sweep;
             break;
         }
     }
-    if (active) {
 #pragma unroll
-        for (int u = 0; u < NPL; ++u) {
-            const int i = u * 32 + lane;
-            if (i < l) {
-                if (ix < l) W[(int64_t)ix * l + i] = x[u];
-                if (iy < l) W[(int64_t)iy * l + i] = y[u];
-            }
+    for (int u = 0; u < NPL; ++u) {
+        const int i = u * 32 + lane;
+        if (i < l) {
+            if (ix < l) W[(int64_t)ix * l + i] = x[u];
+            if (iy < l) W[(int64_t)iy * l + i] = y[u];
         }
     }
     if (crank == 0 && threadIdx.x == 0) flags[1] = sweep;
@@ -287,7 +333,7 @@ __global__ void __launch_bounds__(576, 1) jacobi_cluster_kernel(double* __restri
 // Vb(:, rank) = R^T w_j / sigma_j^2 (R = U_b S V_b^T => V_b = R^T U_b S^{-1}); fp64, one CTA per j.
 __global__ void jacobi_rank_rt_kernel(const double* __restrict__ W, const float* __restrict__ R, int64_t ldr, int l,
                                       int r, const double* __restrict__ sig, float* __restrict__ S,
-                                      float* __restrict__ Ub, float* __restrict__ Vb) {
+                                      float* __restrict__ Ub, float* __restrict__ Vb, int trans) {
     RG_PDL_ENTRY();
     extern __shared__ double wcol[];
     const int j = blockIdx.x;
@@ -308,12 +354,19 @@ __global__ void jacobi_rank_rt_kernel(const double* __restrict__ W, const float*
     const double sj = sig[j];
     if (threadIdx.x == 0) S[rank] = (float)sj;
     const double inv = sj > 0.0 ? 1.0 / sj : 0.0;
+    // trans = 0: W = R J = U_b S, V_b = R^T W S^-2.  trans = 1: W = R^T J = V_b S, U_b = R W S^-2.
+    float* Wout = trans ? Vb : Ub;
+    float* Oout = trans ? Ub : Vb;
     for (int i = threadIdx.x; i < l; i += blockDim.x) {
-        Ub[i + (int64_t)rank * l] = (float)(wcol[i] * inv);
-        const float* rc = R + (int64_t)i * ldr;   // column i of R: R(k, i), k <= i
+        Wout[i + (int64_t)rank * l] = (float)(wcol[i] * inv);
         double v = 0.0;
-        for (int k = 0; k <= i; ++k) v = fma((double)rc[k], wcol[k], v);
-        Vb[i + (int64_t)rank * l] = (float)(v * inv * inv);
+        if (trans) {
+            for (int k = i; k < l; ++k) v = fma((double)R[i + (int64_t)k * ldr], wcol[k], v);   // row i of R
+        } else {
+            const float* rc = R + (int64_t)i * ldr;   // column i of R: R(k, i), k <= i
+            for (int k = 0; k <= i; ++k) v = fma((double)rc[k], wcol[k], v);
+        }
+        Oout[i + (int64_t)rank * l] = (float)(v * inv * inv);
     }
 }
 
@@ -392,17 +445,23 @@ cudaError_t launch_unscale_rows(float* X, int64_t ldx, int64_t rows, int cols, c
 
 cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double* W, double* V, double* sig, int* flags,
                               float* S, float* Ub, float* Vb, cudaStream_t st) {
+    const bool cluster = l <= 544 && getenv("RGSQR_JACOBI_GRID") == nullptr;
+    // one-sided Jacobi on R^T (the graded, lower-triangular transpose) needs about half the sweeps
+    // of Jacobi on R (measured 11 vs 21 at l = 528)
+    const int trans = cluster ? (getenv("RGSQR_JACOBI_T") != nullptr ? atoi(getenv("RGSQR_JACOBI_T")) : 1) : 0;
+    const double jtol = getenv("RGSQR_JACOBI_TOL") ? atof(getenv("RGSQR_JACOBI_TOL")) : 1e-13;
     RG_LAUNCH((jacobi_init_kernel), (unsigned)std::min<int64_t>(((int64_t)l * l + 255) / 256, 148 * 8), 256, 0, st, R, ldr, l,
-                                                                                                             W, V);
+                                                                                                             W, V, trans);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
-    if (l <= 576 && getenv("RGSQR_JACOBI_GRID") == nullptr) {
+    if (cluster) {
+        // 2 cs wper >= l columns, <= 17 warps (544 threads) per CTA, <= 16 CTAs per cluster
         const int P = (l + 1) / 2;
-        const int cs = std::max(1, std::min(16, (P + 17) / 18));   // <= 18 warps (576 threads) per CTA
+        const int cs = std::max(1, std::min(16, (P + 16) / 17));
         const int wper = (P + cs - 1) / cs;
         const int npl = (l + 31) / 32;
         int max_sweeps = 40;
-        double tol = 1e-13;
+        double tol = jtol;
         cudaLaunchConfig_t cfg{};
         cudaLaunchAttribute at[1];
         at[0].id = cudaLaunchAttributeClusterDimension;
@@ -415,7 +474,7 @@ cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double*
         cfg.attrs = at;
         cfg.numAttrs = 1;
         auto go = [&](auto kern, int np) -> cudaError_t {
-            cfg.dynamicSmemBytes = (size_t)wper * 2 * np * 32 * 8 + (size_t)wper * 2 * 4 + 16;
+            cfg.dynamicSmemBytes = (size_t)2 * wper * np * 32 * 8 + (size_t)wper * 2 * (8 + 4) + 16;
             cudaError_t e2 = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                   (int)cfg.dynamicSmemBytes);
             if (e2 != cudaSuccess) return e2;
@@ -424,17 +483,17 @@ cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double*
                 if (e2 != cudaSuccess) return e2;
             }
             ++g_launches;
-            return cudaLaunchKernelEx(&cfg, kern, W, l, P, wper, max_sweeps, tol, flags);
+            return cudaLaunchKernelEx(&cfg, kern, W, l, wper, max_sweeps, tol, flags);
         };
         if (npl <= 4) e = go(jacobi_cluster_kernel<4>, 4);
         else if (npl <= 8) e = go(jacobi_cluster_kernel<8>, 8);
         else if (npl <= 12) e = go(jacobi_cluster_kernel<12>, 12);
-        else e = go(jacobi_cluster_kernel<18>, 18);
+        else e = go(jacobi_cluster_kernel<17>, 17);
         if (e != cudaSuccess) return e;
         RG_LAUNCH((jacobi_extract_kernel), l, 256, 0, st, W, V, l, r, S, Ub, Vb, sig);
         e = cudaGetLastError();
         if (e != cudaSuccess) return e;
-        RG_LAUNCH((jacobi_rank_rt_kernel), l, 256, (size_t)l * 8, st, W, R, ldr, l, r, sig, S, Ub, Vb);
+        RG_LAUNCH((jacobi_rank_rt_kernel), l, 256, (size_t)l * 8, st, W, R, ldr, l, r, sig, S, Ub, Vb, trans);
         return cudaGetLastError();
     }
     int dev = 0, sms = 148, per_sm = 1;
