@@ -124,6 +124,33 @@ __device__ __forceinline__ void gram_block_accum(const float* tile, int rows, in
     }
 }
 
+// fp64 tensor-core (DMMA m8n8k4) variant for the streaming passes: warp w takes the 4-row
+// k-steps w, w + 8, ... of the 128-row tile and accumulates all 10 upper 8x8 blocks of the 32x32
+// Gram (block t: (bi, bj) row by row); fragment b of a k-step is P[k0 + c][8 b + g] (lane = 4 g +
+// c), converted once and used as both the A (P_bi^T) and B (P_bj) operand.  Replaces 4x4 DFMA
+// blocks fed by 8 LDS + 8 F2F per 16 DFMA, which stalled on shared-memory latency (ncu:
+// short_scoreboard, 12 % of DRAM peak).
+__host__ __device__ constexpr int cq_blk_i(int t) { return t < 4 ? 0 : t < 7 ? 1 : t < 9 ? 2 : 3; }
+__host__ __device__ constexpr int cq_blk_j(int t) { return t < 4 ? t : t < 7 ? t - 3 : t < 9 ? t - 5 : 3; }
+template <int T>
+__device__ __forceinline__ void cq_dmma(double (&acc)[10][2], const double (&f)[4]) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                 : "+d"(acc[T][0]), "+d"(acc[T][1])
+                 : "d"(f[cq_blk_i(T)]), "d"(f[cq_blk_j(T)]));
+}
+__device__ __forceinline__ void gram_dmma_accum(const float* tile, int rows, int warp, int lane, double (&acc)[10][2]) {
+    const int g = lane >> 2, c = lane & 3;
+    const float* col = tile + g * CQ_LD + c;
+#pragma unroll 2
+    for (int k0 = 4 * warp; k0 < rows; k0 += 32) {   // rows beyond `rows` in the last k-step are zero
+        double f[4];
+#pragma unroll
+        for (int b = 0; b < 4; ++b) f[b] = (double)col[8 * b * CQ_LD + k0];
+        cq_dmma<0>(acc, f); cq_dmma<1>(acc, f); cq_dmma<2>(acc, f); cq_dmma<3>(acc, f); cq_dmma<4>(acc, f);
+        cq_dmma<5>(acc, f); cq_dmma<6>(acc, f); cq_dmma<7>(acc, f); cq_dmma<8>(acc, f); cq_dmma<9>(acc, f);
+    }
+}
+
 // ---------------------------------------------------------------- Cholesky + inverse
 // Whole CTA (blockDim.x == NT threads), N x N fp64 (N = 32 or 64), blocked by 4 columns:
 // N / 4 block steps of
@@ -482,10 +509,8 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
     }
     const bool write_q = (PASS == 2) || (PASS == 1 && single);
     const bool gram = (PASS == 0) || (PASS == 1 && !single);
-    const int g = tid / CQ_BLK, blk = tid % CQ_BLK;
-    int bi, bj;
-    blk_coords(blk, bi, bj);
-    double acc[4][4] = {};
+    const int warp = tid >> 5, lane = tid & 31;
+    double acc[10][2] = {};
     const int64_t rows_per_cta = ((a.m + gridDim.x - 1) / gridDim.x + 3) / 4 * 4;
     const int64_t r0 = (int64_t)blockIdx.x * rows_per_cta;
     const int64_t r1 = min(a.m, r0 + rows_per_cta);
@@ -535,29 +560,42 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
                 }
             }
         }
-        if (gram && g < CQ_GROUPS) gram_block_accum(tile, rows, g, bi, bj, acc);
+        if (gram) gram_dmma_accum(tile, rows, warp, lane, acc);
     }
     if (!gram) return;
-    // ---- CTA partial Gram: sum the 7 row-group accumulators (2 at a time through smem)
+    // ---- CTA partial Gram: the 8 warps' block accumulators summed in warp order (2 warps at a
+    // time through smem: slot (w & 1) * 640 + block * 64 + 2 lane + v)
     double* out = a.ws.part + (int64_t)blockIdx.x * 1024;
+    double* sw = &sred[0][0];
+    double run[4] = {0.0, 0.0, 0.0, 0.0};
     for (int round = 0; round < 4; ++round) {
-        const int g0 = round * 2;
         __syncthreads();
-        for (int e = tid; e < 2 * 1024; e += CQ_THREADS) (&sred[0][0])[e] = 0.0;
-        __syncthreads();
-        if (g >= g0 && g < g0 + 2 && g < CQ_GROUPS) {
+        if ((warp >> 1) == round) {
 #pragma unroll
-            for (int u = 0; u < 4; ++u)
-#pragma unroll
-                for (int v = 0; v < 4; ++v) sred[g - g0][(bi * 4 + u) + (bj * 4 + v) * 32] = acc[u][v];
+            for (int t = 0; t < 10; ++t) {
+                sw[(warp & 1) * 640 + t * 64 + 2 * lane] = acc[t][0];
+                sw[(warp & 1) * 640 + t * 64 + 2 * lane + 1] = acc[t][1];
+            }
         }
         __syncthreads();
-        for (int e = tid; e < 1024; e += CQ_THREADS) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const int e = tid + CQ_THREADS * q;
             const int i = e & 31, j = e >> 5;
-            double s = (round == 0) ? 0.0 : out[e];
-            s += sred[0][e] + sred[1][e];
-            out[e] = (i <= j) ? s : 0.0;
+            if (i <= j) {
+                const int bi = i >> 3, bj = j >> 3;
+                const int t = bi == 0 ? bj : bi == 1 ? 3 + bj : bi == 2 ? 5 + bj : 9;
+                const int idx = t * 64 + 2 * (4 * (i & 7) + ((j & 7) >> 1)) + (j & 1);
+                run[q] += sw[idx];
+                run[q] += sw[640 + idx];
+            }
         }
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const int e = tid + CQ_THREADS * q;
+        const int i = e & 31, j = e >> 5;
+        out[e] = (i <= j) ? run[q] : 0.0;
     }
     __syncthreads();
     reduce_and_factor(a, PASS, &sred[0][0], reinterpret_cast<double*>(tile));
