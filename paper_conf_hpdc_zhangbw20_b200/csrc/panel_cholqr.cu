@@ -35,7 +35,8 @@ namespace rg {
 
 constexpr int CQ_NB = 32;
 constexpr int CQ_TILE = 128;          // rows staged per iteration
-constexpr int CQ_LD = CQ_TILE + 1;    // smem column stride (bank-conflict-free column access)
+constexpr int CQ_LD = CQ_TILE + 4;    // smem column stride: 16-byte aligned columns; the DMMA
+                                      // fragment reads (lane 4 g + c -> 4 g + c mod 32) stay conflict-free
 constexpr int CQ_THREADS = 256;
 constexpr int CQ_BLK = 36;            // 4x4 blocks in the upper triangle of a 32x32 Gram (8*9/2)
 constexpr int CQ_GROUPS = CQ_THREADS / CQ_BLK;  // 7 row groups of 36 threads
@@ -454,7 +455,9 @@ __device__ void reduce_and_factor(const CqArgs& a, int pass, double* smem_R, dou
 // Per 128-row tile, thread t owns rows {t/8 + 32 i} (i < 4) and columns 4 (t%8) .. +3, so
 // every shared-memory load of R^{-1} (one float4) feeds 16 FMAs.
 __device__ __forceinline__ void tile_times_rinv(float* tile, const float* Rinv /*32 x 32, ld 32*/, int tid) {
-    const int cgp = tid & 7, rgp = tid >> 3;
+    // thread (cgp = tid % 8, rq = tid / 8): rows 4 rq .. 4 rq + 3 (one float4 of the column) x
+    // columns 4 cgp .. + 3: two 16-byte shared loads per 16 FMAs
+    const int cgp = tid & 7, rq = tid >> 3;
     float o[4][4];
 #pragma unroll
     for (int i = 0; i < 4; ++i)
@@ -463,20 +466,21 @@ __device__ __forceinline__ void tile_times_rinv(float* tile, const float* Rinv /
 #pragma unroll 8
     for (int k = 0; k < CQ_NB; ++k) {
         const float4 rv = *reinterpret_cast<const float4*>(Rinv + k * 32 + 4 * cgp);
+        const float4 xv = *reinterpret_cast<const float4*>(tile + k * CQ_LD + 4 * rq);
+        const float x[4] = {xv.x, xv.y, xv.z, xv.w};
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
-            const float x = tile[k * CQ_LD + rgp + 32 * i];
-            o[i][0] = fmaf(x, rv.x, o[i][0]);
-            o[i][1] = fmaf(x, rv.y, o[i][1]);
-            o[i][2] = fmaf(x, rv.z, o[i][2]);
-            o[i][3] = fmaf(x, rv.w, o[i][3]);
+            o[i][0] = fmaf(x[i], rv.x, o[i][0]);
+            o[i][1] = fmaf(x[i], rv.y, o[i][1]);
+            o[i][2] = fmaf(x[i], rv.z, o[i][2]);
+            o[i][3] = fmaf(x[i], rv.w, o[i][3]);
         }
     }
     __syncthreads();
 #pragma unroll
-    for (int i = 0; i < 4; ++i)
-#pragma unroll
-        for (int c = 0; c < 4; ++c) tile[(4 * cgp + c) * CQ_LD + rgp + 32 * i] = o[i][c];
+    for (int c = 0; c < 4; ++c)
+        *reinterpret_cast<float4*>(tile + (4 * cgp + c) * CQ_LD + 4 * rq) =
+            make_float4(o[0][c], o[1][c], o[2][c], o[3][c]);
     __syncthreads();
 }
 
@@ -508,6 +512,10 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
             }
     }
     const bool write_q = (PASS == 2) || (PASS == 1 && single);
+    // 16-byte Q / 8-byte image stores need aligned column starts (rows per CTA and tiles are
+    // multiples of 4)
+    const bool vec = ((a.ldq & 3) == 0) && ((reinterpret_cast<uintptr_t>(a.Q) & 15) == 0) && ((a.ldh & 3) == 0) &&
+                     ((reinterpret_cast<uintptr_t>(a.Qh) & 7) == 0) && ((reinterpret_cast<uintptr_t>(a.Ql) & 7) == 0);
     const bool gram = (PASS == 0) || (PASS == 1 && !single);
     const int warp = tid >> 5, lane = tid & 31;
     double acc[10][2] = {};
@@ -541,7 +549,47 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
         if (PASS > 0) {
             tile_times_rinv(tile, Ri[0], tid);                 // tile <- Q1 = P R1^{-1}
             if (PASS == 2) tile_times_rinv(tile, Ri[1], tid);  // tile <- Q = Q1 R2^{-1}
-            if (write_q) {
+            if (write_q && vec) {
+                // 4 consecutive rows of a column per thread: float4 Q, 8-byte 16-bit images
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const int e = tid + k * CQ_THREADS;
+                    const int rq = e & 31, c = e >> 5;
+                    const int r = 4 * rq;
+                    if (c < a.nc && r < rows) {
+                        const float4 v = *reinterpret_cast<const float4*>(tile + c * CQ_LD + r);
+                        const int64_t gr = base + r;
+                        if (r + 3 < rows) {
+                            __stcs(reinterpret_cast<float4*>(a.Q + gr + (int64_t)c * a.ldq), v);
+                            if (a.Qh) {
+                                const float vv[4] = {v.x, v.y, v.z, v.w};
+                                ushort4 hb, lb;
+                                uint16_t* hp = reinterpret_cast<uint16_t*>(&hb);
+                                uint16_t* lp = reinterpret_cast<uint16_t*>(&lb);
+#pragma unroll
+                                for (int u = 0; u < 4; ++u) {
+                                    hp[u] = cq_to16(vv[u], a.bf16);
+                                    lp[u] = cq_to16((vv[u] - cq_from16(hp[u], a.bf16)) * 2048.f, a.bf16);
+                                }
+                                *reinterpret_cast<ushort4*>(a.Qh + gr + (int64_t)c * a.ldh) = hb;
+                                if (a.Ql) *reinterpret_cast<ushort4*>(a.Ql + gr + (int64_t)c * a.ldh) = lb;
+                            }
+                        } else {
+                            const float vv[4] = {v.x, v.y, v.z, v.w};
+                            for (int u = 0; u < 4 && r + u < rows; ++u) {
+                                a.Q[gr + u + (int64_t)c * a.ldq] = vv[u];
+                                if (a.Qh) {
+                                    const uint16_t hb = cq_to16(vv[u], a.bf16);
+                                    a.Qh[gr + u + (int64_t)c * a.ldh] = hb;
+                                    if (a.Ql)
+                                        a.Ql[gr + u + (int64_t)c * a.ldh] =
+                                            cq_to16((vv[u] - cq_from16(hb, a.bf16)) * 2048.f, a.bf16);
+                                }
+                            }
+                        }
+                    }
+                }
+            } else if (write_q) {
 #pragma unroll
                 for (int k = 0; k < 16; ++k) {
                     const int e = tid + k * CQ_THREADS;
