@@ -1166,7 +1166,13 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
             rc = check_status(h);
             if (rc) break;
         }
-        if (orth_tol > 0) {
+        // A first pass with 16-bit GEMMs cannot be orthogonal below ~0.5 u16 n / sqrt(m) (reading
+        // #9, SURVEY [EMU]): when a quarter of that floor is above the tolerance the probe after
+        // pass 1 is skipped (the second pass runs anyway; only the estimate's cost is saved).
+        const double u16 = o.precision ? 0x1p-8 : 0x1p-11;
+        const double m_all = (double)m_local * std::max(1, h->nranks);
+        const bool skip_probe = passes == 1 && 0.25 * u16 * (double)n / std::sqrt(m_all) > orth_tol;
+        if (orth_tol > 0 && !skip_probe) {
             rc = orth_estimate(h, dA, dlda, m_local, (int)n, &est);
             if (rc || est <= orth_tol) break;
         }
