@@ -28,6 +28,7 @@
 #include <cooperative_groups.h>
 
 #include "kernels.h"
+#include "ptx.cuh"
 
 namespace cg = cooperative_groups;
 
@@ -38,6 +39,8 @@ constexpr int CQ_TILE = 128;          // rows staged per iteration
 constexpr int CQ_LD = CQ_TILE + 4;    // smem column stride: 16-byte aligned columns; the DMMA
                                       // fragment reads (lane 4 g + c -> 4 g + c mod 32) stay conflict-free
 constexpr int CQ_THREADS = 256;
+constexpr int CQ_STAGES = 3;                        // cp.async ring depth of the streaming passes
+constexpr int CQ_TILE_FLOATS = 32 * (CQ_TILE + 4);  // one 128 x 32 tile (column stride CQ_LD)
 constexpr int CQ_BLK = 36;            // 4x4 blocks in the upper triangle of a 32x32 Gram (8*9/2)
 constexpr int CQ_GROUPS = CQ_THREADS / CQ_BLK;  // 7 row groups of 36 threads
 constexpr int CQ_FAN = 16;            // CTAs per reduction group
@@ -487,7 +490,8 @@ __device__ __forceinline__ void tile_times_rinv(float* tile, const float* Rinv /
 template <int PASS>
 __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
     RG_PDL_ENTRY();
-    __shared__ __align__(16) float tile[CQ_NB * CQ_LD + 64];   // also R1 scratch (32 x 33 doubles)
+    __shared__ __align__(16) float tile_static[CQ_NB * CQ_LD + 64];   // also R1 scratch (32 x 33 doubles)
+    extern __shared__ __align__(16) float ring[];                       // [CQ_STAGES][CQ_TILE_FLOATS]
     __shared__ __align__(16) float Ri[2][32 * 32];
     __shared__ __align__(16) double sred[2][1024];   // CTA partial-sum scratch (2 row groups at a time); reused
                                        // as the 32 x 33 Cholesky scratch by the last CTA
@@ -522,29 +526,59 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
     const int64_t rows_per_cta = ((a.m + gridDim.x - 1) / gridDim.x + 3) / 4 * 4;
     const int64_t r0 = (int64_t)blockIdx.x * rows_per_cta;
     const int64_t r1 = min(a.m, r0 + rows_per_cta);
-    // register prefetch of the next tile: thread loads element (r = e % 128, c = e / 128)
-    float pre[16];
+    // Tiles of 128 rows x 32 columns.  Aligned panels: a CQ_STAGES-deep cp.async ring in dynamic
+    // shared memory (48 KB of loads in flight per CTA); otherwise a one-tile register prefetch.
+    const bool async_ld = ((a.ldp & 3) == 0) && ((reinterpret_cast<uintptr_t>(a.P) & 15) == 0);
+    auto issue = [&](int64_t tb, float* dst) {   // rows [tb, tb + 128) of the panel, 16-byte copies
 #pragma unroll
-    for (int k = 0; k < 16; ++k) {
-        const int e = tid + k * CQ_THREADS;
-        const int r = e % CQ_TILE, c = e / CQ_TILE;
-        pre[k] = (r0 + r < r1 && c < a.nc) ? a.P[r0 + r + (int64_t)c * a.ldp] : 0.f;
-    }
-    for (int64_t base = r0; base < r1; base += CQ_TILE) {
-        const int rows = (int)((r1 - base) < CQ_TILE ? (r1 - base) : CQ_TILE);
-        __syncthreads();
-#pragma unroll
-        for (int k = 0; k < 16; ++k) {
+        for (int k = 0; k < 4; ++k) {
             const int e = tid + k * CQ_THREADS;
-            tile[(e / CQ_TILE) * CQ_LD + (e % CQ_TILE)] = pre[k];
+            const int rq = e & 31, c = e >> 5;
+            const int64_t gr = tb + 4 * rq;
+            const int avail = (c < a.nc && gr < r1) ? (int)(r1 - gr < 4 ? r1 - gr : 4) : 0;
+            const float* src = avail > 0 ? a.P + gr + (int64_t)c * a.ldp : a.P;
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst + c * CQ_LD + 4 * rq)),
+                         "l"(src), "r"(avail * 4)
+                         : "memory");
         }
-        __syncthreads();
-        const int64_t nb = base + CQ_TILE;
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    float pre[16];
+    if (async_ld) {
+#pragma unroll
+        for (int sidx = 0; sidx < CQ_STAGES - 1; ++sidx) issue(r0 + (int64_t)sidx * CQ_TILE, ring + sidx * CQ_TILE_FLOATS);
+    } else {
 #pragma unroll
         for (int k = 0; k < 16; ++k) {
             const int e = tid + k * CQ_THREADS;
             const int r = e % CQ_TILE, c = e / CQ_TILE;
-            pre[k] = (nb + r < r1 && c < a.nc) ? a.P[nb + r + (int64_t)c * a.ldp] : 0.f;
+            pre[k] = (r0 + r < r1 && c < a.nc) ? a.P[r0 + r + (int64_t)c * a.ldp] : 0.f;
+        }
+    }
+    int it = 0;
+    for (int64_t base = r0; base < r1; base += CQ_TILE, ++it) {
+        const int rows = (int)((r1 - base) < CQ_TILE ? (r1 - base) : CQ_TILE);
+        float* tile = tile_static;
+        if (async_ld) {
+            issue(base + (int64_t)(CQ_STAGES - 1) * CQ_TILE, ring + ((it + CQ_STAGES - 1) % CQ_STAGES) * CQ_TILE_FLOATS);
+            asm volatile("cp.async.wait_group %0;" ::"n"(CQ_STAGES - 1) : "memory");
+            __syncthreads();
+            tile = ring + (it % CQ_STAGES) * CQ_TILE_FLOATS;
+        } else {
+            __syncthreads();
+#pragma unroll
+            for (int k = 0; k < 16; ++k) {
+                const int e = tid + k * CQ_THREADS;
+                tile[(e / CQ_TILE) * CQ_LD + (e % CQ_TILE)] = pre[k];
+            }
+            __syncthreads();
+            const int64_t nb = base + CQ_TILE;
+#pragma unroll
+            for (int k = 0; k < 16; ++k) {
+                const int e = tid + k * CQ_THREADS;
+                const int r = e % CQ_TILE, c = e / CQ_TILE;
+                pre[k] = (nb + r < r1 && c < a.nc) ? a.P[nb + r + (int64_t)c * a.ldp] : 0.f;
+            }
         }
         if (PASS > 0) {
             tile_times_rinv(tile, Ri[0], tid);                 // tile <- Q1 = P R1^{-1}
@@ -561,18 +595,37 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
                         const int64_t gr = base + r;
                         if (r + 3 < rows) {
                             __stcs(reinterpret_cast<float4*>(a.Q + gr + (int64_t)c * a.ldq), v);
-                            if (a.Qh) {
-                                const float vv[4] = {v.x, v.y, v.z, v.w};
-                                ushort4 hb, lb;
-                                uint16_t* hp = reinterpret_cast<uint16_t*>(&hb);
-                                uint16_t* lp = reinterpret_cast<uint16_t*>(&lb);
-#pragma unroll
-                                for (int u = 0; u < 4; ++u) {
-                                    hp[u] = cq_to16(vv[u], a.bf16);
-                                    lp[u] = cq_to16((vv[u] - cq_from16(hp[u], a.bf16)) * 2048.f, a.bf16);
+                            if (a.Qh) {   // packed (two-wide) conversions
+                                uint2 hb, lb;
+                                float2 h01, h23;
+                                if (a.bf16) {
+                                    const __nv_bfloat162 b01 = __floats2bfloat162_rn(v.x, v.y), b23 = __floats2bfloat162_rn(v.z, v.w);
+                                    hb.x = *reinterpret_cast<const uint32_t*>(&b01);
+                                    hb.y = *reinterpret_cast<const uint32_t*>(&b23);
+                                    h01 = __bfloat1622float2(b01);
+                                    h23 = __bfloat1622float2(b23);
+                                } else {
+                                    const __half2 b01 = __floats2half2_rn(v.x, v.y), b23 = __floats2half2_rn(v.z, v.w);
+                                    hb.x = *reinterpret_cast<const uint32_t*>(&b01);
+                                    hb.y = *reinterpret_cast<const uint32_t*>(&b23);
+                                    h01 = __half22float2(b01);
+                                    h23 = __half22float2(b23);
                                 }
-                                *reinterpret_cast<ushort4*>(a.Qh + gr + (int64_t)c * a.ldh) = hb;
-                                if (a.Ql) *reinterpret_cast<ushort4*>(a.Ql + gr + (int64_t)c * a.ldh) = lb;
+                                *reinterpret_cast<uint2*>(a.Qh + gr + (int64_t)c * a.ldh) = hb;
+                                if (a.Ql) {
+                                    const float l0 = (v.x - h01.x) * 2048.f, l1 = (v.y - h01.y) * 2048.f;
+                                    const float l2 = (v.z - h23.x) * 2048.f, l3 = (v.w - h23.y) * 2048.f;
+                                    if (a.bf16) {
+                                        const __nv_bfloat162 c01 = __floats2bfloat162_rn(l0, l1), c23 = __floats2bfloat162_rn(l2, l3);
+                                        lb.x = *reinterpret_cast<const uint32_t*>(&c01);
+                                        lb.y = *reinterpret_cast<const uint32_t*>(&c23);
+                                    } else {
+                                        const __half2 c01 = __floats2half2_rn(l0, l1), c23 = __floats2half2_rn(l2, l3);
+                                        lb.x = *reinterpret_cast<const uint32_t*>(&c01);
+                                        lb.y = *reinterpret_cast<const uint32_t*>(&c23);
+                                    }
+                                    *reinterpret_cast<uint2*>(a.Ql + gr + (int64_t)c * a.ldh) = lb;
+                                }
                             }
                         } else {
                             const float vv[4] = {v.x, v.y, v.z, v.w};
@@ -609,6 +662,7 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
             }
         }
         if (gram) gram_dmma_accum(tile, rows, warp, lane, acc);
+        if (async_ld) __syncthreads();   // this ring slot is refilled by the next iteration
     }
     if (!gram) return;
     // ---- CTA partial Gram: the 8 warps' block accumulators summed in warp order (2 warps at a
@@ -646,7 +700,7 @@ __global__ void __launch_bounds__(CQ_THREADS, 2) cq_pass_kernel(CqArgs a) {
         out[e] = (i <= j) ? run[q] : 0.0;
     }
     __syncthreads();
-    reduce_and_factor(a, PASS, &sred[0][0], reinterpret_cast<double*>(tile));
+    reduce_and_factor(a, PASS, &sred[0][0], reinterpret_cast<double*>(tile_static));
 }
 
 
@@ -1324,10 +1378,18 @@ cudaError_t launch_panel_cholqr(const CholqrLaunch& L, bool* handles_failure, cu
     }
     if (handles_failure) *handles_failure = false;      // the guarded MGS/TSQR kernels must follow
     cudaError_t e;
+    constexpr size_t ring_bytes = (size_t)CQ_STAGES * CQ_TILE_FLOATS * 4;
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaFuncSetAttribute(cq_pass_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ring_bytes);
+        cudaFuncSetAttribute(cq_pass_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ring_bytes);
+        cudaFuncSetAttribute(cq_pass_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ring_bytes);
+        attr_set = true;
+    }
     for (int pass = 0; pass < 3; ++pass) {
-        if (pass == 0) RG_LAUNCH((cq_pass_kernel<0>), grid, CQ_THREADS, 0, st, a);
-        if (pass == 1) RG_LAUNCH((cq_pass_kernel<1>), grid, CQ_THREADS, 0, st, a);
-        if (pass == 2) RG_LAUNCH((cq_pass_kernel<2>), grid, CQ_THREADS, 0, st, a);
+        if (pass == 0) RG_LAUNCH((cq_pass_kernel<0>), grid, CQ_THREADS, ring_bytes, st, a);
+        if (pass == 1) RG_LAUNCH((cq_pass_kernel<1>), grid, CQ_THREADS, ring_bytes, st, a);
+        if (pass == 2) RG_LAUNCH((cq_pass_kernel<2>), grid, CQ_THREADS, ring_bytes, st, a);
         e = cudaGetLastError();
         if (e != cudaSuccess) return e;
         if (a.distributed && pass < 2) {
