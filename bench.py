@@ -157,6 +157,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-ls", action="store_true")
     ap.add_argument("--no-orth", action="store_true")
+    ap.add_argument("--no-bf16", action="store_true")
     ap.add_argument("--no-lowrank", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -285,6 +286,32 @@ def main():
         except Exception as ex:  # keep the headline line even if the LS leg fails
             ls = {"error": str(ex)[:200]}
 
+    # the same factorization with bf16 tensor-core operands (
+    # reading #20): time and accuracy next to the fp16 headline
+    bf16 = None
+    if not args.no_bf16:
+        try:
+            ob = rg.make_opts(precision="bf16", sync=False)
+            for _ in range(3):
+                rg.rgsqr_factor(A, Q=Q, R=R, handle=h, opts=ob, check=False)
+            torch.cuda.synchronize()
+            b0, b1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            b0.record(st)
+            for _ in range(5):
+                rg.rgsqr_factor(A, Q=Q, R=R, handle=h, opts=ob, check=False)
+            b1.record(st)
+            torch.cuda.synchronize()
+            bms = b0.elapsed_time(b1) / 5
+            if dist is not None:
+                t = torch.tensor([bms], device="cuda")
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                bms = float(t.item())
+            bf16 = {"ms": bms, "tflops": flops / (bms * 1e-3) / 1e12,
+                    "accuracy": accuracy_probe(rg, torch, A, Q, R) if ws == 1 else None,
+                    "note": "rgsqr_factor(precision=bf16), same input and options otherwise"}
+        except Exception as ex:
+            bf16 = {"error": str(ex)[:200]}
+
     orth = None
     if not args.no_orth:
         try:
@@ -323,6 +350,7 @@ def main():
             "e2e": e2e,
             "ls": ls,
             "orthogonalize": orth,
+            "bf16": bf16,
             "lowrank": lowrank,
             "gpu_launches": (launches * args.steps) if launches else None,
             "clocks": clk.summary(),

@@ -176,6 +176,12 @@ __global__ void __launch_bounds__(256) jacobi_sweeps_kernel(double* __restrict__
 // V is not accumulated: V_b = R^T W S^{-2} afterwards (jacobi_rank_rt_kernel).  At l = 528 this
 // replaces a one-pair-per-warp ordering with 527 cluster-synchronised rounds per sweep (28 ms) and
 // a grid-synchronised kernel with L2-latency-bound rounds (70 ms).
+// Cluster barrier with cluster-scope release/acquire (orders the DSMEM column stores before the
+// receivers' loads).  cooperative_groups' cluster.sync() emitted a GPU-scope MEMBAR per call.
+__device__ __forceinline__ void jc_cluster_sync() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 template <int NPL>
 __device__ __forceinline__ double jc_dot(const double (&x)[NPL], const double (&y)[NPL]) {
     double g0 = 0.0, g1 = 0.0;   // two accumulators: halves the dependent DFMA chain
@@ -261,7 +267,7 @@ __global__ void __launch_bounds__(544, 1) jacobi_cluster_kernel(double* __restri
         bool any = false;
         na = jc_dot<NPL>(x, x);   // exact norms once per sweep (the rotations update them)
         nb = jc_dot<NPL>(y, y);
-        cl.sync();
+        jc_cluster_sync();
         // ---- 1. all pairs among the CTA's 2 wper columns (Brent-Luk over the warps)
         for (int r = 0; r < 2 * wper - 1; ++r) {
             any |= jc_rotate<NPL>(x, y, na, nb, ix, iy, l, tol);
@@ -283,11 +289,11 @@ __global__ void __launch_bounds__(544, 1) jacobi_cluster_kernel(double* __restri
         }
         // ---- 2. block pairs between CTAs
         for (int tr = 1; tr <= 2 * cs - 2; ++tr) {
-            cl.sync();
+            jc_cluster_sync();
             if (crank >= 1 && crank <= cs - 2) put(crank + 1, 0, warp, x, ix, na);   // x block -> CTA + 1
             if (crank >= 1) put(crank - 1, 1, warp, y, iy, nb);                       // y block -> CTA - 1
             else put(1, 0, warp, y, iy, nb);                                          // (CTA 0: -> x of CTA 1)
-            cl.sync();
+            jc_cluster_sync();
             if (crank == cs - 1) {
 #pragma unroll
                 for (int u = 0; u < NPL; ++u) y[u] = x[u];
@@ -309,10 +315,10 @@ __global__ void __launch_bounds__(544, 1) jacobi_cluster_kernel(double* __restri
             }
         }
         if (any && lane == 0) atomicOr(&rot_flag, 1);
-        cl.sync();
+        jc_cluster_sync();
         int tot = 0;
         for (int c = 0; c < cs; ++c) tot |= *cl.map_shared_rank(&rot_flag, c);
-        cl.sync();
+        jc_cluster_sync();
         if (!tot) {
             ++sweep;
             break;
