@@ -215,103 +215,210 @@ __device__ __forceinline__ bool jc_rotate(double (&x)[NPL], double (&y)[NPL], do
     return true;
 }
 
+// Rotation angle from (a, b, g) = (|x|^2, |y|^2, x^T y); false when the pair is already
+// orthogonal to tol (or involves a padding column).
+// fp64 reciprocal / reciprocal square root: hardware approximation (MUFU, ~2^-23) + Newton
+// steps.  The rotation's dependent chain is latency-bound (one rotation per warp per round), and
+// the IEEE div / sqrt sequences dominated it.  t only steers convergence; c is refined to ~2^-50 so
+// that c^2 (1 + t^2) = 1 keeps the column norms (the singular values) intact.
+__device__ __forceinline__ double jc_rcp(double x) {
+    double y;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
+    double e = fma(-x, y, 1.0);
+    y = fma(y, e, y);
+    e = fma(-x, y, 1.0);
+    return fma(y, e, y);
+}
+__device__ __forceinline__ double jc_rsqrt(double x) {
+    double y;
+    asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
+    y = y * fma(-0.5 * x * y, y, 1.5);
+    return y * fma(-0.5 * x * y, y, 1.5);
+}
+__device__ __forceinline__ bool jc_angle(double a, double b, double g, double tol, double& c, double& sn, double& t) {
+    if (g * g <= tol * tol * (a * b) || g == 0.0) return false;
+    const double zeta = (b - a) * jc_rcp(2.0 * g);
+    const double az = fabs(zeta);
+    const double q = 1.0 + zeta * zeta;
+    const double sq = q * jc_rsqrt(q);   // sqrt(1 + zeta^2)
+    t = (zeta >= 0.0 ? 1.0 : -1.0) * jc_rcp(az + sq);
+    c = jc_rsqrt(1.0 + t * t);
+    sn = c * t;
+    return true;
+}
+
+// Rotation of the register column x (squared norm a) with the shared-memory column yc (norm *nb).
+// y is streamed from shared memory twice (dot, then update) instead of held in registers: the
+// 17-warp CTAs of l = 528 have 96 registers per thread.
+template <int NPL>
+__device__ __forceinline__ bool jc_rotate_smem(double (&x)[NPL], double& a, int ix, double* yc, double* nb, int iy,
+                                               int l, double tol, int lane) {
+    if (ix >= l || iy >= l) return false;
+    double g0 = 0.0, g1 = 0.0;
+#pragma unroll
+    for (int u = 0; u < NPL; u += 2) {
+        g0 = fma(x[u], yc[u * 32 + lane], g0);
+        if (u + 1 < NPL) g1 = fma(x[u + 1], yc[(u + 1) * 32 + lane], g1);
+    }
+    const double g = wsum(g0 + g1);
+    const double b = *nb;
+    double c, sn, t;
+    if (!jc_angle(a, b, g, tol, c, sn, t)) return false;
+#pragma unroll
+    for (int u = 0; u < NPL; ++u) {
+        const double xv = x[u], yv = yc[u * 32 + lane];
+        x[u] = c * xv - sn * yv;
+        yc[u * 32 + lane] = sn * xv + c * yv;
+    }
+    a -= t * g;
+    __syncwarp();
+    if (lane == 0) *nb = b + t * g;
+    return true;
+}
+
+// Rotation of two shared-memory columns (norms *na, *nb), streamed.
+template <int NPL>
+__device__ __forceinline__ bool jc_rotate_2smem(double* xc, double* na, int ix, double* yc, double* nb, int iy, int l,
+                                                double tol, int lane) {
+    if (ix >= l || iy >= l) return false;
+    double g0 = 0.0, g1 = 0.0;
+#pragma unroll
+    for (int u = 0; u < NPL; u += 2) {
+        g0 = fma(xc[u * 32 + lane], yc[u * 32 + lane], g0);
+        if (u + 1 < NPL) g1 = fma(xc[(u + 1) * 32 + lane], yc[(u + 1) * 32 + lane], g1);
+    }
+    const double g = wsum(g0 + g1);
+    const double a = *na, b = *nb;
+    double c, sn, t;
+    if (!jc_angle(a, b, g, tol, c, sn, t)) return false;
+#pragma unroll
+    for (int u = 0; u < NPL; ++u) {
+        const double xv = xc[u * 32 + lane], yv = yc[u * 32 + lane];
+        xc[u * 32 + lane] = c * xv - sn * yv;
+        yc[u * 32 + lane] = sn * xv + c * yv;
+    }
+    __syncwarp();
+    if (lane == 0) {
+        *na = a - t * g;
+        *nb = b + t * g;
+    }
+    return true;
+}
+
 template <int NPL>
 __global__ void __launch_bounds__(544, 1) jacobi_cluster_kernel(double* __restrict__ W, int l, int wper,
                                                                 int max_sweeps, double tol, int* flags) {
     cg::cluster_group cl = cg::this_cluster();
     extern __shared__ __align__(16) double jc_smem[];
-    double* buf = jc_smem;                                                      // [2][wper][NPL * 32]
-    double* bnrm = buf + (size_t)2 * wper * NPL * 32;                            // [2][wper] squared norms
-    int* bid = reinterpret_cast<int*>(bnrm + 2 * wper);                          // [2][wper] column ids
+    // slots 0 .. wper - 1: the x block, wper .. 2 wper - 1: the y block (NPL * 32 doubles each)
+    double* buf = jc_smem;
+    double* snrm = buf + (size_t)2 * wper * NPL * 32;   // [2 wper] squared norms
+    int* sid = reinterpret_cast<int*>(snrm + 2 * wper); // [2 wper] column ids
     __shared__ int rot_flag;
     const int crank = (int)cl.block_rank();
     const int cs = (int)cl.num_blocks();
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    auto slot = [&](int which, int w) { return buf + ((size_t)which * wper + w) * NPL * 32; };
-    double x[NPL], y[NPL];
-    double na = 0.0, nb = 0.0;
-    int ix = (2 * crank) * wper + warp, iy = (2 * crank + 1) * wper + warp;
+    auto col = [&](int slot) { return buf + (size_t)slot * NPL * 32; };
+    // x (this warp's column of the x block) in registers; the y block in shared memory
+    double x[NPL];
+    int ix = (2 * crank) * wper + warp;
+    double na = 0.0;
+    {
+        const int iy = (2 * crank + 1) * wper + warp;
+        double* yc = col(wper + warp);
 #pragma unroll
-    for (int u = 0; u < NPL; ++u) {
-        const int i = u * 32 + lane;
-        x[u] = (ix < l && i < l) ? W[(int64_t)ix * l + i] : 0.0;
-        y[u] = (iy < l && i < l) ? W[(int64_t)iy * l + i] : 0.0;
+        for (int u = 0; u < NPL; ++u) {
+            const int i = u * 32 + lane;
+            x[u] = (ix < l && i < l) ? W[(int64_t)ix * l + i] : 0.0;
+            yc[u * 32 + lane] = (iy < l && i < l) ? W[(int64_t)iy * l + i] : 0.0;
+        }
+        if (lane == 0) sid[wper + warp] = iy;
     }
-    // column v, its id and norm into slot (which, w) of CTA `cta` (local when cta < 0)
-    auto put = [&](int cta, int which, int w, const double (&v)[NPL], int id, double nrm) {
-        double* d = slot(which, w);
-        double* dn = bnrm + which * wper + w;
-        int* di = bid + which * wper + w;
-        if (cta >= 0) {
-            d = cl.map_shared_rank(d, cta);
-            dn = cl.map_shared_rank(dn, cta);
-            di = cl.map_shared_rank(di, cta);
-        }
-#pragma unroll
-        for (int u = 0; u < NPL; ++u) d[u * 32 + lane] = v[u];
-        if (lane == 0) {
-            *dn = nrm;
-            *di = id;
-        }
-    };
-    auto get = [&](int which, double (&v)[NPL], int& id, double& nrm) {
-        const double* d = slot(which, warp);
-#pragma unroll
-        for (int u = 0; u < NPL; ++u) v[u] = d[u * 32 + lane];
-        id = bid[which * wper + warp];
-        nrm = bnrm[which * wper + warp];
-    };
     int sweep = 0;
     for (; sweep < max_sweeps; ++sweep) {
         if (threadIdx.x == 0) rot_flag = 0;
         bool any = false;
-        na = jc_dot<NPL>(x, x);   // exact norms once per sweep (the rotations update them)
-        nb = jc_dot<NPL>(y, y);
-        jc_cluster_sync();
-        // ---- 1. all pairs among the CTA's 2 wper columns (Brent-Luk over the warps)
-        for (int r = 0; r < 2 * wper - 1; ++r) {
-            any |= jc_rotate<NPL>(x, y, na, nb, ix, iy, l, tol);
-            if (wper == 1) break;
-            if (warp >= 1 && warp <= wper - 2) put(-1, 0, warp + 1, x, ix, na);
-            if (warp >= 1) put(-1, 1, warp - 1, y, iy, nb);
-            else put(-1, 0, 1, y, iy, nb);
-            __syncthreads();
-            if (warp == wper - 1) {
+        // ---- 1. all pairs among the CTA's 2 wper columns: x block to shared memory, circle-method
+        // round robin over the 2 wper slots (pairs of slots, no column moves)
+        {
+            double* xc = col(warp);
 #pragma unroll
-                for (int u = 0; u < NPL; ++u) y[u] = x[u];
-                iy = ix;
-                nb = na;
-            } else {
-                get(1, y, iy, nb);
+            for (int u = 0; u < NPL; ++u) xc[u * 32 + lane] = x[u];
+            double yy = 0.0;
+            const double* yc = col(wper + warp);
+#pragma unroll
+            for (int u = 0; u < NPL; ++u) yy = fma(yc[u * 32 + lane], yc[u * 32 + lane], yy);
+            yy = wsum(yy);
+            na = jc_dot<NPL>(x, x);   // exact norms once per sweep (rotations update them)
+            if (lane == 0) {
+                sid[warp] = ix;
+                snrm[warp] = na;
+                snrm[wper + warp] = yy;
             }
-            if (warp >= 1) get(0, x, ix, na);
+        }
+        __syncthreads();
+        for (int r = 0; r < 2 * wper - 1; ++r) {
+            int p, q;
+            rr_pair(2 * wper, r, warp, p, q);
+            any |= jc_rotate_2smem<NPL>(col(p), snrm + p, sid[p], col(q), snrm + q, sid[q], l, tol, lane);
             __syncthreads();
         }
-        // ---- 2. block pairs between CTAs
-        for (int tr = 1; tr <= 2 * cs - 2; ++tr) {
-            jc_cluster_sync();
-            if (crank >= 1 && crank <= cs - 2) put(crank + 1, 0, warp, x, ix, na);   // x block -> CTA + 1
-            if (crank >= 1) put(crank - 1, 1, warp, y, iy, nb);                       // y block -> CTA - 1
-            else put(1, 0, warp, y, iy, nb);                                          // (CTA 0: -> x of CTA 1)
-            jc_cluster_sync();
-            if (crank == cs - 1) {
+        {
+            const double* xc = col(warp);
 #pragma unroll
-                for (int u = 0; u < NPL; ++u) y[u] = x[u];
-                iy = ix;
-                nb = na;
-            } else {
-                get(1, y, iy, nb);
+            for (int u = 0; u < NPL; ++u) x[u] = xc[u * 32 + lane];
+            na = snrm[warp];
+        }
+        // ---- 2. block pairs between CTAs (pull form of the block round robin):
+        //   new x(c) = x(0) (c = 0), y(0) (c = 1), x(c - 1);   new y(c) = y(c + 1), x(cs - 1) (c = cs - 1)
+        for (int tr = 1; tr <= 2 * cs - 2; ++tr) {
+            {
+                double* xc = col(warp);
+#pragma unroll
+                for (int u = 0; u < NPL; ++u) xc[u * 32 + lane] = x[u];
+                if (lane == 0) {
+                    sid[warp] = ix;
+                    snrm[warp] = na;
+                }
             }
-            if (crank >= 1) get(0, x, ix, na);
+            jc_cluster_sync();
+            double ny[NPL];
+            int iny;
+            double nny;
+            {
+                const int src_c = crank == cs - 1 ? crank : crank + 1;
+                const int src_s = crank == cs - 1 ? warp : wper + warp;
+                const double* ycr = cl.map_shared_rank(col(src_s), src_c);
+#pragma unroll
+                for (int u = 0; u < NPL; ++u) ny[u] = ycr[u * 32 + lane];
+                iny = *cl.map_shared_rank(sid + src_s, src_c);
+                nny = *cl.map_shared_rank(snrm + src_s, src_c);
+            }
+            if (crank >= 1) {
+                const int src_c = crank - 1;
+                const int src_s = crank == 1 ? wper + warp : warp;
+                const double* xcr = cl.map_shared_rank(col(src_s), src_c);
+#pragma unroll
+                for (int u = 0; u < NPL; ++u) x[u] = xcr[u * 32 + lane];
+                ix = *cl.map_shared_rank(sid + src_s, src_c);
+                na = *cl.map_shared_rank(snrm + src_s, src_c);
+            }
+            jc_cluster_sync();
+            {
+                double* yc = col(wper + warp);
+#pragma unroll
+                for (int u = 0; u < NPL; ++u) yc[u * 32 + lane] = ny[u];
+                if (lane == 0) {
+                    sid[wper + warp] = iny;
+                    snrm[wper + warp] = nny;
+                }
+            }
             __syncthreads();
-            // the wper x wper pairs (x_i, y_{i+s}): shift y one warp down per round
+            // the wper x wper pairs (x_i, y_{(i + s) mod wper})
             for (int sft = 0; sft < wper; ++sft) {
-                any |= jc_rotate<NPL>(x, y, na, nb, ix, iy, l, tol);
-                if (sft == wper - 1) break;
-                const int p = sft & 1;
-                put(-1, p, (warp + wper - 1) % wper, y, iy, nb);
+                const int ys = wper + (warp + sft) % wper;
+                any |= jc_rotate_smem<NPL>(x, na, ix, col(ys), snrm + ys, sid[ys], l, tol, lane);
                 __syncthreads();
-                get(p, y, iy, nb);
             }
         }
         if (any && lane == 0) atomicOr(&rot_flag, 1);
@@ -324,12 +431,16 @@ __global__ void __launch_bounds__(544, 1) jacobi_cluster_kernel(double* __restri
             break;
         }
     }
+    {
+        const double* yc = col(wper + warp);
+        const int iy = sid[wper + warp];
 #pragma unroll
-    for (int u = 0; u < NPL; ++u) {
-        const int i = u * 32 + lane;
-        if (i < l) {
-            if (ix < l) W[(int64_t)ix * l + i] = x[u];
-            if (iy < l) W[(int64_t)iy * l + i] = y[u];
+        for (int u = 0; u < NPL; ++u) {
+            const int i = u * 32 + lane;
+            if (i < l) {
+                if (ix < l) W[(int64_t)ix * l + i] = x[u];
+                if (iy < l) W[(int64_t)iy * l + i] = yc[u * 32 + lane];
+            }
         }
     }
     if (crank == 0 && threadIdx.x == 0) flags[1] = sweep;
@@ -480,7 +591,7 @@ cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double*
         cfg.attrs = at;
         cfg.numAttrs = 1;
         auto go = [&](auto kern, int np) -> cudaError_t {
-            cfg.dynamicSmemBytes = (size_t)2 * wper * np * 32 * 8 + (size_t)wper * 2 * (8 + 4) + 16;
+            cfg.dynamicSmemBytes = (size_t)2 * wper * np * 32 * 8 + (size_t)wper * 2 * (8 + 4) + 16;   // x + y blocks
             cudaError_t e2 = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                   (int)cfg.dynamicSmemBytes);
             if (e2 != cudaSuccess) return e2;

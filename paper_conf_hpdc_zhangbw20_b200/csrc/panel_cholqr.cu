@@ -41,8 +41,6 @@ constexpr int CQ_LD = CQ_TILE + 4;    // smem column stride: 16-byte aligned col
 constexpr int CQ_THREADS = 256;
 constexpr int CQ_STAGES = 3;                        // cp.async ring depth of the streaming passes
 constexpr int CQ_TILE_FLOATS = 32 * (CQ_TILE + 4);  // one 128 x 32 tile (column stride CQ_LD)
-constexpr int CQ_BLK = 36;            // 4x4 blocks in the upper triangle of a 32x32 Gram (8*9/2)
-constexpr int CQ_GROUPS = CQ_THREADS / CQ_BLK;  // 7 row groups of 36 threads
 constexpr int CQ_FAN = 16;            // CTAs per reduction group
 
 __device__ __forceinline__ uint16_t cq_to16(float x, int bf16) {
@@ -102,33 +100,7 @@ __device__ __forceinline__ void cq_signal_fail(const CqArgs& a) {
 }
 
 // ---------------------------------------------------------------- Gram accumulation
-__device__ __forceinline__ void blk_coords(int blk, int& bi, int& bj) {
-    int b = 0, rem = blk;
-    while (rem >= 8 - b) {
-        rem -= 8 - b;
-        ++b;
-    }
-    bi = b;
-    bj = b + rem;
-}
-
-__device__ __forceinline__ void gram_block_accum(const float* tile, int rows, int g, int bi, int bj,
-                                                 double (&acc)[4][4]) {
-    for (int r = g; r < rows; r += CQ_GROUPS) {
-        double x[4], y[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            x[u] = (double)tile[(bi * 4 + u) * CQ_LD + r];
-            y[u] = (double)tile[(bj * 4 + u) * CQ_LD + r];
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u)
-#pragma unroll
-            for (int v = 0; v < 4; ++v) acc[u][v] = fma(x[u], y[v], acc[u][v]);
-    }
-}
-
-// fp64 tensor-core (DMMA m8n8k4) variant for the streaming passes: warp w takes the 4-row
+// Streaming passes, on the fp64 tensor cores (DMMA m8n8k4): warp w takes the 4-row
 // k-steps w, w + 8, ... of the 128-row tile and accumulates all 10 upper 8x8 blocks of the 32x32
 // Gram (block t: (bi, bj) row by row); fragment b of a k-step is P[k0 + c][8 b + g] (lane = 4 g +
 // c), converted once and used as both the A (P_bi^T) and B (P_bj) operand.  Replaces 4x4 DFMA

@@ -124,6 +124,26 @@ def test_rgsqr_tall_panel_streaming_path(rg):
     _check_qr(A, Q, R, kappa=np.linalg.cond(A))
 
 
+@pytest.mark.parametrize("pad", [0, 3])
+def test_rgsqr_tall_streaming_aligned_and_unaligned(rg, pad):
+    """Streaming passes (m = 200000) through both load paths: lda = m (16-byte aligned columns:
+    cp.async ring, vector stores) and lda = m + 3 (register prefetch, scalar stores); the two
+    must agree to rounding and meet the factorization bounds."""
+    m, n = 200000, 64
+    A = synth.gaussian(m, n, seed=43).astype(np.float32)
+    big = np.zeros((n, m + pad), dtype=np.float32)
+    big[:, :m] = A.T
+    Ad = torch.from_numpy(big).cuda().t()[:m]          # column-major view, lda = m + pad
+    Q = torch.zeros(n, m + pad, device="cuda").t()[:m]
+    Q, R = rg.rgsqr_factor(Ad, Q=Q)
+    torch.cuda.synchronize()
+    Qn = Q.cpu().numpy().astype(np.float64)
+    Rn = R.cpu().numpy().astype(np.float64)
+    _check_qr(A, Qn, Rn, kappa=np.linalg.cond(A))
+    Q0, R0 = _run(rg, A)
+    assert np.linalg.norm(Rn - R0) / np.linalg.norm(R0) < 1e-5
+
+
 def test_rgsqr_config1(rg):
     """BASELINE config 1: 1024 x 64, cond ~ 10 (geometric spectrum), vs the fp64 oracle."""
     A = synth.svd_matrix(1024, 64, "geometric", 10.0, seed=synth.SEED_BASE + 0).astype(np.float32)
