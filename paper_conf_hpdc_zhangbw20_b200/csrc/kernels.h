@@ -174,6 +174,12 @@ size_t gemv_n_work_doubles(int64_t m, int n);
 cudaError_t launch_gemv_t(const float* A, int64_t lda, int64_t m, int n, const double* r, double* s, double* work,
                           const double* done, cudaStream_t st);
 size_t gemv_t_work_doubles(int64_t m, int n);
+// one-pass q = A t, w = A^T q (CGLS, NEXT-4); sc[1] = |q|^2
+size_t gemv_nt_work_doubles(int n);
+bool gemv_nt_ok(const float* A, int64_t lda, int n);
+cudaError_t launch_gemv_nt(const float* A, int64_t lda, int64_t m, int n, const double* t, double* q, double* w,
+                           double* work, double* sc, cudaStream_t st);
+cudaError_t launch_cgls_sv(double* sv, const double* w, int n, const double* sc, cudaStream_t st);
 // Rinv: 2 n^2 doubles -- R^{-1} column-major, then its row-major copy (read by launch_trmv(.., 0, ..))
 cudaError_t launch_trinv_upper(const float* R, int64_t ldr, int n, double* Rinv, cudaStream_t st);
 cudaError_t launch_trmv(const double* Rinv, int n, const double* x, double* y, int transpose, const double* done,

@@ -827,8 +827,27 @@ int enqueue_cgls_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int 
     double* r = sv + n;
     double* q = r + m;
     double* work = q + m;
-    double* sqp = work + std::max(rg::gemv_n_work_doubles(m, n), rg::gemv_t_work_doubles(m, n));
+    double* sqp = work + std::max({rg::gemv_n_work_doubles(m, n), rg::gemv_t_work_doubles(m, n),
+                                   rg::gemv_nt_work_doubles(n) + (size_t)n});
     const double* done = sc + 6;
+    if (rg::gemv_nt_ok(A, lda, n)) {
+        // one pass over A per iteration: q = A t and w = A^T q together; A^T r by recurrence
+        double* w = work + rg::gemv_nt_work_doubles(n);
+        for (int k = 0; k < iters; ++k) {
+            ProfScope _s(h, PC_CGLS, 4.0 * m * n, 4.0 * m * n);
+            RG_CUDA(rg::launch_trmv(Rinv, n, p, t, 0, done, st));                 // t = R \ p
+            RG_CUDA(rg::launch_gemv_nt(A, lda, m, n, t, q, w, work, sc, st));    // q = A t, w = A^T q, delta
+            int rc = nccl_allreduce(h, sc + 1, 1, ncclFloat64);
+            if (rc) return rc;
+            rc = nccl_allreduce(h, w, n, ncclFloat64);
+            if (rc) return rc;
+            RG_CUDA(rg::launch_cgls_xr(x, t, r, q, m, n, sc, st));                 // lines 13-15 (alpha)
+            RG_CUDA(rg::launch_cgls_sv(sv, w, n, sc, st));                         // A^T r -= alpha A^T q
+            RG_CUDA(rg::launch_trmv(Rinv, n, sv, s, 1, done, st));                // line 16: s = R^-T A^T r
+            RG_CUDA(rg::launch_cgls_p(s, p, n, sc, 0, st));                        // lines 17-21
+        }
+        return RG_OK;
+    }
     for (int k = 0; k < iters; ++k) {
         ProfScope _s(h, PC_CGLS, 4.0 * m * n, 8.0 * m * n);
         RG_CUDA(rg::launch_trmv(Rinv, n, p, t, 0, done, st));                 // t = R \ p
@@ -1246,7 +1265,8 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     if (!h->rinv.ensure((size_t)2 * n * n * 8 + 64)) return RG_ALLOC;   // Rinv + its row-major copy
     RG_CUDA(rg::launch_trinv_upper(Rw, n, (int)n, h->rinv.as<double>(), h->stream));
     // ---- CGLS state: sc[16] | x p s t sv (n each) | r q (m each) | gemv work
-    const size_t work = std::max(rg::gemv_n_work_doubles(m_local, (int)n), rg::gemv_t_work_doubles(m_local, (int)n));
+    const size_t work = std::max({rg::gemv_n_work_doubles(m_local, (int)n), rg::gemv_t_work_doubles(m_local, (int)n),
+                                  rg::gemv_nt_work_doubles((int)n) + (size_t)n});
     if (!h->cg.ensure((16 + 5 * (size_t)n + 2 * (size_t)m_local + work + 2048) * 8 + 256)) return RG_ALLOC;
     double* base = h->cg.as<double>();
     double* sc = base;

@@ -95,3 +95,29 @@ def test_orthogonalize_fixed_two_passes(rg):
     Q, _, passes, est = rg.orthogonalize(Ad, None, orth_tol=0.0, max_passes=2)
     assert passes == 2
     assert oracle.orthogonality(Q.cpu().numpy().astype(np.float64)) <= 1e-5
+
+
+@pytest.mark.parametrize("kappa", [1e2, 1e4])
+def test_ls_one_pass_cgls_matches_two_pass(rg, monkeypatch, kappa):
+    """The one-pass CGLS product (q = A t and A^T q in one sweep of A, A^T r by recurrence) and the
+    two-pass form (A^T r recomputed from r, the default) reach the same solution (reading #24)."""
+    m, n = 16384, 512
+    A = synth.svd_matrix(m, n, "geometric", kappa, seed=61).astype(np.float32)
+    b = synth.rhs(A.astype(np.float64), seed=61, consistent=False).astype(np.float32)
+    x_star, _ = oracle.ls_qr(A.astype(np.float64), b.astype(np.float64))
+    out = []
+    for two in (False, True):
+        if two:
+            monkeypatch.delenv("RGSQR_CGLS_ONE_PASS", raising=False)
+        else:
+            monkeypatch.setenv("RGSQR_CGLS_ONE_PASS", "1")
+        h = rg.Handle(0)   # fresh handle: its captured CGLS graph follows the current mode
+        x, it, rel, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), tol=1e-10, maxit=200, handle=h)
+        torch.cuda.synchronize()
+        out.append((x.cpu().numpy(), it, rel, st))
+        h.close()
+    (x1, it1, _, st1), (x2, it2, _, st2) = out
+    assert st1 == rg.RG_OK and st2 == rg.RG_OK
+    assert abs(it1 - it2) <= 2, (it1, it2)
+    assert np.linalg.norm(x1 - x2) / np.linalg.norm(x2) <= 1e-8
+    assert np.linalg.norm(x1 - x_star) / np.linalg.norm(x_star) <= 1e-5
