@@ -796,7 +796,8 @@ int orth_estimate(rg_handle h, const float* Q, int64_t ldq, int64_t m, int n, do
     return RG_OK;
 }
 
-// run RGSQR + `extra` split-precision reorthogonalisation passes; Q (ldq) and R (ldr) outputs
+// run RGSQR + `extra` reorthogonalisation passes (16-bit; split precision with opts.split) for the
+// least-squares preconditioner; Q (ldq) and R (ldr) outputs
 int factor_with_reortho(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq, float* R,
                         int64_t ldr, const rg_opts& o, int extra) {
     int rc = run_rgsqr(h, m, n, A, lda, Q, ldq, R, ldr, o, o.split);
@@ -807,7 +808,9 @@ int factor_with_reortho(rg_handle h, int64_t m, int64_t n, const float* A, int64
         }
         if (!h->lsR.ensure((size_t)n * n * 4 + 256)) return RG_ALLOC;
         float* R2 = h->lsR.as<float>();
-        rc = run_rgsqr(h, m, n, Q, ldq, Q, ldq, R2, n, o, 1);
+        // reading #8: for the CGLS preconditioner a plain 16-bit reortho pass suffices (kappa(A R^-1)
+        // ~ 1.8 either way, SURVEY [EMU]); split precision only when the caller asks (opts.split)
+        rc = run_rgsqr(h, m, n, Q, ldq, Q, ldq, R2, n, o, o.split);
         if (rc) return rc;
         rc = trmm_into(h, R2, n, R, ldr, (int)n);
     }
