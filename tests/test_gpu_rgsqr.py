@@ -144,6 +144,21 @@ def test_rgsqr_tall_streaming_aligned_and_unaligned(rg, pad):
     assert np.linalg.norm(Rn - R0) / np.linalg.norm(R0) < 1e-5
 
 
+def test_rgsqr_tall_streaming_breakdown(rg):
+    """Streaming panels (m = 200000): an exactly zero column in the second 32-column panel fails
+    the CholQR pivot test there, the guarded MGS/TSQR fallback reports the breakdown, and an
+    ill-conditioned tall matrix (kappa 1e3) factors to the usual bounds."""
+    m = 200000
+    A = synth.gaussian(m, 64, seed=47).astype(np.float32)
+    A[:, 40] = 0.0
+    with pytest.raises(rg.RGError) as e:
+        _run(rg, A)
+    assert e.value.status == rg.RG_BREAKDOWN
+    B = synth.svd_matrix(m, 64, "geometric", 1e3, seed=48).astype(np.float32)
+    Q, R = _run(rg, B)
+    _check_qr(B, Q, R, kappa=1e3, orth_scale=1.0)
+
+
 def test_rgsqr_config1(rg):
     """BASELINE config 1: 1024 x 64, cond ~ 10 (geometric spectrum), vs the fp64 oracle."""
     A = synth.svd_matrix(1024, 64, "geometric", 10.0, seed=synth.SEED_BASE + 0).astype(np.float32)
