@@ -494,14 +494,19 @@ __device__ double lf_inverse(const LfSmem& s, int nc) {
         for (int i = 0; i < 32; ++i) s.X32[(base + i) * 64 + base + j] = b[i];
     }
     __syncthreads();
-    // T = R12 X22 into the X21 slot (rows 32.., cols 0..31: zero afterwards)
+    // T = R12 X22 into the X21 slot (rows 32.., cols 0..31: zero afterwards).  The 32-term dots are
+    // fully unrolled over k with the triangle as predication (X22 is upper: X22(k, jj) = 0 for
+    // k > jj, stored as zero), so all loads issue back to back and four FMA chains interleave (a
+    // runtime-bounded loop waited on every shared load: ~1 us per product).
     float tv[2];
 #pragma unroll
     for (int q = 0; q < 2; ++q) {
         const int e = tid + LF_THREADS * q, i = e >> 5, jj = e & 31;
-        float acc = 0.f;
-        for (int k = 0; k <= jj; ++k) acc = fmaf(s.Rt32[(32 + k) * LF_TLD + i], s.X32[(32 + k) * 64 + 32 + jj], acc);
-        tv[q] = acc;
+        float a4[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+        for (int k = 0; k < 32; ++k)
+            a4[k & 3] = fmaf(s.Rt32[(32 + k) * LF_TLD + i], s.X32[(32 + k) * 64 + 32 + jj], a4[k & 3]);
+        tv[q] = (a4[0] + a4[1]) + (a4[2] + a4[3]);
     }
     __syncthreads();
 #pragma unroll
@@ -510,13 +515,14 @@ __device__ double lf_inverse(const LfSmem& s, int nc) {
         s.X32[(32 + i) * 64 + jj] = tv[q];
     }
     __syncthreads();
-    // X12 = -X11 T
+    // X12 = -X11 T (X11 upper: X11(i, k) = 0 for k < i, stored as zero; unrolled as above)
 #pragma unroll
     for (int q = 0; q < 2; ++q) {
         const int e = tid + LF_THREADS * q, i = e >> 5, jj = e & 31;
-        float acc = 0.f;
-        for (int k = i; k < 32; ++k) acc = fmaf(s.X32[i * 64 + k], s.X32[(32 + k) * 64 + jj], acc);
-        tv[q] = -acc;
+        float a4[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+        for (int k = 0; k < 32; ++k) a4[k & 3] = fmaf(s.X32[i * 64 + k], s.X32[(32 + k) * 64 + jj], a4[k & 3]);
+        tv[q] = -((a4[0] + a4[1]) + (a4[2] + a4[3]));
     }
     __syncthreads();
     double xn = 0.0, rn = 0.0;
