@@ -708,6 +708,7 @@ __device__ void lf_load_qa(const LeafArgs& a, const LfSmem& s, int64_t r0, int r
 }
 
 // partial R_AB: warp w owns the 16 x 16 output block (w / 4, w % 4) over all k-steps
+template <int BF>
 __device__ void lf_pro_k1(const LeafArgs& a, const LfSmem& s, int rp16) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, c = lane & 3;
@@ -731,11 +732,11 @@ __device__ void lf_pro_k1(const LeafArgs& a, const LfSmem& s, int rp16) {
         for (int nt = 0; nt < 2; ++nt) {
             const float2 y0 = *reinterpret_cast<const float2*>(pb + 8 * nt * ld + k0);
             const float2 y1 = *reinterpret_cast<const float2*>(pb + 8 * nt * ld + k0 + 8);
-            bfr[nt][0] = lf_pack2(y0.x, y0.y, a.bf16);
-            bfr[nt][1] = lf_pack2(y1.x, y1.y, a.bf16);
+            bfr[nt][0] = lf_pack2(y0.x, y0.y, BF);
+            bfr[nt][1] = lf_pack2(y1.x, y1.y, BF);
         }
 #pragma unroll
-        for (int nt = 0; nt < 2; ++nt) lf_mma16816(acc[nt], af, bfr[nt], a.bf16);
+        for (int nt = 0; nt < 2; ++nt) lf_mma16816(acc[nt], af, bfr[nt], BF);
     }
     double* out = a.part + (int64_t)blockIdx.x * LF_PART;
 #pragma unroll
@@ -748,6 +749,7 @@ __device__ void lf_pro_k1(const LeafArgs& a, const LfSmem& s, int rp16) {
 }
 
 // P <- P - Q_A R_AB over the tile's 64 columns; s.RABh holds -R_AB as [n][k]
+template <int BF>
 __device__ void lf_pro_k2(const LeafArgs& a, const LfSmem& s, int rp16) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, c = lane & 3;
@@ -775,7 +777,7 @@ __device__ void lf_pro_k2(const LeafArgs& a, const LfSmem& s, int rp16) {
                 const uint16_t* bp = s.RABh + (8 * nt + g) * LF_ABLD + 16 * ks + 2 * c;
                 const uint32_t bfr[2] = {*reinterpret_cast<const uint32_t*>(bp),
                                          *reinterpret_cast<const uint32_t*>(bp + 8)};
-                lf_mma16816(d[nt], af, bfr, a.bf16);
+                lf_mma16816(d[nt], af, bfr, BF);
             }
         }
 #pragma unroll
@@ -807,6 +809,7 @@ __device__ void lf_load_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, int
     }
 }
 
+template <int BF>
 __device__ void lf_store_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, int rows) {
     const int nq = (rows + 3) >> 2;
     for (int e = threadIdx.x; e < a.nc * nq; e += LF_THREADS) {
@@ -819,9 +822,10 @@ __device__ void lf_store_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, in
         uint16_t* hbp = reinterpret_cast<uint16_t*>(&hb);
         uint16_t* lbp = reinterpret_cast<uint16_t*>(&lb);
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            hbp[u] = lf_to16(vv[u], a.bf16);
-            lbp[u] = lf_to16((vv[u] - lf_from16(hbp[u], a.bf16)) * 2048.f, a.bf16);
+        for (int u = 0; u < 4; ++u) hbp[u] = lf_to16(vv[u], BF);
+        if (a.Ql) {   // lo image (split mode) only when requested
+#pragma unroll
+            for (int u = 0; u < 4; ++u) lbp[u] = lf_to16((vv[u] - lf_from16(hbp[u], BF)) * 2048.f, BF);
         }
         uint16_t* dh = a.Qh ? a.Qh + gr + (int64_t)cc * a.ldh : nullptr;
         uint16_t* dl = a.Ql ? a.Ql + gr + (int64_t)cc * a.ldh : nullptr;
@@ -842,7 +846,7 @@ __device__ void lf_store_cols(const LeafArgs& a, const LfSmem& s, int64_t r0, in
 }
 
 // ------------------------------------------------------------------ the kernel
-template <int NI>
+template <int NI, int BF>
 __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
     extern __shared__ __align__(16) uint8_t lf_smem[];
     const LfSmem s(lf_smem, a.ldt);
@@ -862,19 +866,19 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
     if (a.pq) {
         // ---- prologue: the level above (R_AB = Q_A^T P, P -= Q_A R_AB)
         LF_MARK(10);
-        lf_pro_k1(a, s, rp16);
+        lf_pro_k1<BF>(a, s, rp16);
         LF_MARK(11);
         lf_allreduce(a, s, 4096, false);
         LF_MARK(12);
         for (int e = threadIdx.x; e < 4096; e += LF_THREADS) {
             const int i = e >> 6, j = e & 63;   // R_AB(i, j)
             const float v = (i < a.ph && j < a.nc) ? (float)__ldcg(a.red + e) : 0.f;
-            s.RABh[j * LF_ABLD + i] = lf_to16(-v, a.bf16);
+            s.RABh[j * LF_ABLD + i] = lf_to16(-v, BF);
             if (blockIdx.x == 0 && i < a.ph && j < a.nc) a.R[(int64_t)(i - a.ph) + (int64_t)j * a.ldr] = v;
         }
         __syncthreads();
         LF_MARK(13);
-        lf_pro_k2(a, s, rp16);
+        lf_pro_k2<BF>(a, s, rp16);
     }
     LF_MARK(1);
     int npass = 0;
@@ -884,7 +888,7 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
         return;
     }
     LF_MARK(7);
-    lf_store_cols(a, s, r0, rows);
+    lf_store_cols<BF>(a, s, r0, rows);
     if (blockIdx.x == 0) {   // R (fp32) from the fp64 factor (s.Rs for one pass, else the accumulated one)
         const double* racc = a.racc + (((npass - 1) & 1) ? 64 * 64 : 0);
         for (int e = threadIdx.x; e < a.nc * a.nc; e += LF_THREADS) {
@@ -981,12 +985,15 @@ cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st) {
             ((reinterpret_cast<uintptr_t>(L.Qh) & 7) == 0) && ((reinterpret_cast<uintptr_t>(L.Ql) & 7) == 0);
     const size_t smem = leaf_smem_bytes(L.m);
     const bool small = ((a.rows_per + 15) & ~15) <= 448;
-    void (*kern)(LeafArgs) = small ? leaf_kernel<7> : leaf_kernel<LF_MAXI>;
-    static size_t attr[2] = {0, 0};
-    if (smem > attr[small]) {
+    // the 16-bit format is a template parameter: runtime bf16 branches in the prologue's mma.sync /
+    // pack loops and the image stores cost convergence-barrier (BSSY) overhead
+    void (*kern)(LeafArgs) = a.bf16 ? (small ? leaf_kernel<7, 1> : leaf_kernel<LF_MAXI, 1>)
+                                    : (small ? leaf_kernel<7, 0> : leaf_kernel<LF_MAXI, 0>);
+    static size_t attr[2][2] = {{0, 0}, {0, 0}};
+    if (smem > attr[a.bf16 ? 1 : 0][small]) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
-        attr[small] = smem;
+        attr[a.bf16 ? 1 : 0][small] = smem;
     }
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(grid);

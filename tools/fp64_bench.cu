@@ -56,6 +56,26 @@ __global__ void dmma16k16_tp(double* out, int n) {
     double s = 0; for (int u = 0; u < 4; ++u) for (int v = 0; v < 4; ++v) s += c[u][v];
     out[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
+// mma.sync m16n8k16 f16 -> f32: throughput (4 independent accumulators) and latency (1 chain)
+__global__ void hmma_tp(float* out, int n, int chains) {
+    unsigned a0 = threadIdx.x, a1 = a0 + 1, a2 = a0 + 2, a3 = a0 + 3, b0 = a0 ^ 5, b1 = a0 ^ 7;
+    float c[4][4] = {};
+    long long t0 = clock64();
+    for (int i = 0; i < n; ++i) {
+        if (chains == 4) {
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+                asm volatile("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, {%0,%1,%2,%3};"
+                             : "+f"(c[u][0]), "+f"(c[u][1]), "+f"(c[u][2]), "+f"(c[u][3]) : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+        } else {
+            asm volatile("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, {%0,%1,%2,%3};"
+                         : "+f"(c[0][0]), "+f"(c[0][1]), "+f"(c[0][2]), "+f"(c[0][3]) : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+        }
+    }
+    long long t1 = clock64();
+    float s = 0; for (int u = 0; u < 4; ++u) for (int v = 0; v < 4; ++v) s += c[u][v];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = s + (threadIdx.x == 0 && blockIdx.x == 0 ? (float)(t1 - t0) : 0.f);
+}
 int main() {
     double* out; float* in;
     cudaMalloc(&out, 148 * 1024 * 8 * 4); cudaMalloc(&in, 4096);
@@ -87,5 +107,16 @@ int main() {
     fl = 148.0 * 4 * 8 * (n / 4) * 4 * 2048;
     printf("DMMA m16n8k16: %.2f TFMA/s -> %.1f FMA/clk/SM (%s)\n", fl / ms / 1e9, fl / ms / 1e-3 / 148 / 1.9e9,
            cudaGetErrorString(cudaGetLastError()));
+    {
+        float* fo; cudaMalloc(&fo, 148 * 1024 * 4 * 4);
+        hmma_tp<<<148 * 4, 256>>>(fo, 64, 4);
+        cudaEventRecord(a); hmma_tp<<<148 * 4, 256>>>(fo, n, 4); cudaEventRecord(b); cudaEventSynchronize(b);
+        cudaEventElapsedTime(&ms, a, b);
+        fl = 148.0 * 4 * 8 * n * 4 * 4096.0;   // warps * mma * (16*8*16*2 flops)
+        printf("HMMA m16n8k16 (mma.sync): %.1f TFLOP/s -> %.0f flop/clk/SM\n", fl / ms / 1e9, fl / ms / 1e-3 / 148 / 1.9e9);
+        hmma_tp<<<1, 32>>>(fo, 4096, 1);
+        float h0; cudaMemcpy(&h0, fo, 4, cudaMemcpyDeviceToHost);
+        printf("HMMA dependent-chain latency: %.1f cycles per mma\n", h0 / 4096.0);
+    }
     return 0;
 }
