@@ -259,7 +259,20 @@ __device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne, bool to
     lf_grid_sync(a.bar);
     if (mk) LF_MARK(mk + 2);
     if (!to_smem) return;
-    for (int e = threadIdx.x; e < ne; e += LF_THREADS) s.red[e] = __ldcg(a.red + e);
+    // every thread's loads in flight at once (a load-then-store loop paid one L2 round trip per
+    // iteration: ~1.4 us for the 2080-entry Gram)
+    constexpr int MQ = (LF_PART + LF_THREADS - 1) / LF_THREADS;
+    double v[MQ];
+#pragma unroll
+    for (int u = 0; u < MQ; ++u) {
+        const int e = threadIdx.x + u * LF_THREADS;
+        v[u] = e < ne ? __ldcg(a.red + e) : 0.0;
+    }
+#pragma unroll
+    for (int u = 0; u < MQ; ++u) {
+        const int e = threadIdx.x + u * LF_THREADS;
+        if (e < ne) s.red[e] = v[u];
+    }
     __syncthreads();
 }
 
@@ -870,11 +883,20 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
         LF_MARK(11);
         lf_allreduce(a, s, 4096, false);
         LF_MARK(12);
-        for (int e = threadIdx.x; e < 4096; e += LF_THREADS) {
-            const int i = e >> 6, j = e & 63;   // R_AB(i, j)
-            const float v = (i < a.ph && j < a.nc) ? (float)__ldcg(a.red + e) : 0.f;
-            s.RABh[j * LF_ABLD + i] = lf_to16(-v, BF);
-            if (blockIdx.x == 0 && i < a.ph && j < a.nc) a.R[(int64_t)(i - a.ph) + (int64_t)j * a.ldr] = v;
+        {
+            constexpr int MQ = 4096 / LF_THREADS;   // all loads in flight, then convert / store
+            float v[MQ];
+#pragma unroll
+            for (int u = 0; u < MQ; ++u) {
+                const int e = threadIdx.x + u * LF_THREADS, i = e >> 6, j = e & 63;   // R_AB(i, j)
+                v[u] = (i < a.ph && j < a.nc) ? (float)__ldcg(a.red + e) : 0.f;
+            }
+#pragma unroll
+            for (int u = 0; u < MQ; ++u) {
+                const int e = threadIdx.x + u * LF_THREADS, i = e >> 6, j = e & 63;
+                s.RABh[j * LF_ABLD + i] = lf_to16(-v[u], BF);
+                if (blockIdx.x == 0 && i < a.ph && j < a.nc) a.R[(int64_t)(i - a.ph) + (int64_t)j * a.ldr] = v[u];
+            }
         }
         __syncthreads();
         LF_MARK(13);
