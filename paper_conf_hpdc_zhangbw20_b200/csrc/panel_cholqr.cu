@@ -923,10 +923,23 @@ __device__ void cf_allreduce(const CqArgs& a, double* Gs) {
         while (ld_acquire_gpu(flag) == s_gen) __nanosleep(100);
     __syncthreads();
     fence_acq_rel_gpu();
-    for (int e = tid; e < NE; e += CF_THREADS) {
-        int i, j;
-        tri_unpack(e, i, j);
-        Gs[i + NC * j] = __ldcg(w.G + e);
+    {   // all of this thread's loads in flight before the unpack/stores (one L2 round trip)
+        constexpr int MQ = (NE + CF_THREADS - 1) / CF_THREADS;
+        double v[MQ];
+#pragma unroll
+        for (int u = 0; u < MQ; ++u) {
+            const int e = tid + u * CF_THREADS;
+            v[u] = e < NE ? __ldcg(w.G + e) : 0.0;
+        }
+#pragma unroll
+        for (int u = 0; u < MQ; ++u) {
+            const int e = tid + u * CF_THREADS;
+            if (e < NE) {
+                int i, j;
+                tri_unpack(e, i, j);
+                Gs[i + NC * j] = v[u];
+            }
+        }
     }
     __syncthreads();
 }
