@@ -237,22 +237,33 @@ __device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne, bool to
     const int grid = gridDim.x;
     const int slice = (ne + grid - 1) / grid;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    for (int q = warp; q < slice; q += LF_NW) {
-        const int e = blockIdx.x * slice + q;
-        if (e < ne) {
-            constexpr int NB = (LF_MAX_GRID + 31) / 32;   // all loads in flight, summed in CTA order
-            double p[NB];
+    // two entries per warp per round, all 2 NB loads in flight (the 4096-entry prologue reduction
+    // has ~28 entries per CTA: one round instead of two dependent ones)
+    for (int q = warp; q < slice; q += 2 * LF_NW) {
+        constexpr int NB = (LF_MAX_GRID + 31) / 32;   // summed in CTA order (deterministic)
+        const int e0 = blockIdx.x * slice + q, e1 = e0 + LF_NW;
+        const bool v0 = e0 < ne, v1 = (q + LF_NW < slice) && e1 < ne;
+        double p0[NB], p1[NB];
 #pragma unroll
-            for (int u = 0; u < NB; ++u) {
-                const int b = lane + 32 * u;
-                p[u] = b < grid ? __ldcg(a.part + (int64_t)b * LF_PART + e) : 0.0;
-            }
-            double v = p[0];
+        for (int u = 0; u < NB; ++u) {
+            const int b = lane + 32 * u;
+            p0[u] = (v0 && b < grid) ? __ldcg(a.part + (int64_t)b * LF_PART + e0) : 0.0;
+            p1[u] = (v1 && b < grid) ? __ldcg(a.part + (int64_t)b * LF_PART + e1) : 0.0;
+        }
+        double s0 = p0[0], s1 = p1[0];
 #pragma unroll
-            for (int u = 1; u < NB; ++u) v += p[u];
+        for (int u = 1; u < NB; ++u) {
+            s0 += p0[u];
+            s1 += p1[u];
+        }
 #pragma unroll
-            for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-            if (lane == 0) __stcg(a.red + e, v);
+        for (int o = 16; o > 0; o >>= 1) {
+            s0 += __shfl_xor_sync(0xffffffffu, s0, o);
+            s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+        }
+        if (lane == 0) {
+            if (v0) __stcg(a.red + e0, s0);
+            if (v1) __stcg(a.red + e1, s1);
         }
     }
     if (mk) LF_MARK(mk + 1);
