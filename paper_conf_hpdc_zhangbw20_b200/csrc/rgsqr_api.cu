@@ -139,6 +139,21 @@ struct Op {
     int h0 = 0;            // UPDATE: first output column whose 16-bit image a later K1 reads
 };
 
+// Host-pointer pipeline of rgsqr_factor (pinned host A/Q/R, one pass, one rank): A arrives in
+// column chunks on a copy stream and each chunk is scaled (section 3.5) just before the first op
+// that touches it; Q columns go back to the host as soon as their panel has run, because the
+// recursion (Alg 1, eqs 4-5) only reads Q1 after its panel -- later levels write columns to the
+// right of it.  Both PCIe directions then overlap the factorization instead of bracketing it.
+struct HostPipe {
+    float* hQ = nullptr;
+    int64_t hldq = 0;
+    int chunk = 128;                  // H2D / scaling granularity (columns)
+    int scaled = 0, copied = 0;       // columns scaled on the device / enqueued for D2H
+    std::vector<cudaEvent_t>* in_ev = nullptr;   // H2D chunk k landed
+    cudaStream_t cs_out = nullptr;
+    cudaEvent_t ev = nullptr;         // main-stream progress marker for the D2H stream
+};
+
 struct Plan {
     // key
     int64_t m = 0, n = 0, lda = 0, ldq = 0, ldr = 0;
@@ -154,12 +169,15 @@ struct Plan {
     size_t p_floats = 0;
     long long launches = 0;  // kernels per pass (counted while enqueueing)
     cudaGraphExec_t exec = nullptr;
+    HostPipe* pipe = nullptr;  // set for one eager enqueue of the host-pointer pipeline
 };
 
 struct rg_handle_s {
     int device = 0;
     cudaStream_t stream = nullptr;
     cudaStream_t capture_stream = nullptr;  // private stream used only to capture plans into graphs
+    cudaStream_t cs_in = nullptr, cs_out = nullptr;   // host-pointer pipeline copy streams (lazy)
+    std::vector<cudaEvent_t> pipe_ev;               // [0] progress, [1] start, [2] end, [3..] H2D chunks
     ncclComm_t comm = nullptr;
     int rank = 0, nranks = 1;
     int64_t last_info = -1;
@@ -267,6 +285,16 @@ bool ensure_encode() {
 }
 
 enum PtrSide { SIDE_DEVICE, SIDE_HOST };
+// page-locked (cudaHostAlloc / cudaHostRegister) host memory: copies to and from it are async DMA
+bool is_pinned(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeHost;
+}
+
 PtrSide ptr_side(const void* p) {
     cudaPointerAttributes a;
     if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
@@ -467,7 +495,38 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     uint16_t* ql = pl.split ? h->ql.as<uint16_t>() : nullptr;
     int* status = h->status.as<int>();
     const bool dist = pl.nranks > 1 && h->comm;
-    {
+    HostPipe* pp = pl.pipe;
+    // pipeline: scale the columns [pp->scaled, cend) rounded up to whole chunks, each after its H2D
+    auto pipe_need = [&](int cend) -> int {
+        while (pp && pp->scaled < cend) {
+            const int c = pp->scaled, nc = std::min(pp->chunk, n - c);
+            RG_CUDA(cudaStreamWaitEvent(st, (*pp->in_ev)[c / pp->chunk], 0));
+            RG_CUDA(rg::launch_colnorm(pl.A + (int64_t)c * pl.lda, pl.lda, m, nc, h->partial.as<double>(),
+                                       h->norm2.as<double>() + c, st));
+            RG_CUDA(rg::launch_colscale(h->norm2.as<double>() + c, nc, pl.scale, h->scale.as<float>() + c, status,
+                                        c, st));
+            RG_CUDA(rg::launch_scale_cast(pl.A + (int64_t)c * pl.lda, pl.lda, pl.Q + (int64_t)c * pl.ldq, pl.ldq,
+                                          qh + (int64_t)c * pl.ldh, ql ? ql + (int64_t)c * pl.ldh : nullptr, pl.ldh,
+                                          m, nc, h->scale.as<float>() + c, pl.bf16, st));
+            pp->scaled += nc;
+        }
+        return RG_OK;
+    };
+    // pipeline: Q columns [0, cend) are final; send the new ones home in >= 256-column pieces
+    auto pipe_done = [&](int cend, bool flush) -> int {
+        if (!pp || cend - pp->copied <= 0 || (!flush && cend - pp->copied < 256)) return RG_OK;
+        RG_CUDA(cudaEventRecord(pp->ev, st));
+        RG_CUDA(cudaStreamWaitEvent(pp->cs_out, pp->ev, 0));
+        RG_CUDA(cudaMemcpy2DAsync(pp->hQ + (int64_t)pp->copied * pp->hldq, pp->hldq * 4,
+                                  pl.Q + (int64_t)pp->copied * pl.ldq, pl.ldq * 4, m * 4, cend - pp->copied,
+                                  cudaMemcpyDeviceToHost, pp->cs_out));
+        pp->copied = cend;
+        return RG_OK;
+    };
+    int panel_end = 0;   // columns left of this have had their panel enqueued
+    if (pp) {
+        RG_CUDA(cudaMemset2DAsync(pl.R, pl.ldr * sizeof(float), 0, n * sizeof(float), n, st));
+    } else {
         ProfScope _s(h, PC_SCALE, 0, (double)m * n * (pl.split ? 16 : 14));
         RG_CUDA(rg::launch_colnorm(pl.A, pl.lda, m, n, h->partial.as<double>(), h->norm2.as<double>(), st));
         if (dist) {
@@ -483,6 +542,11 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     const Op* pending_pro = nullptr;      // K1 + K2 of the level above a leaf, folded into it
     for (size_t oi = 0; oi < pl.ops.size(); ++oi) {
         const Op& o = pl.ops[oi];
+        if (pp) {
+            int rc = pipe_done(panel_end, false);
+            if (!rc) rc = pipe_need(o.c0 + (o.kind == Op::PANEL ? o.w : o.h + o.w));
+            if (rc) return rc;
+        }
         if (folded_into_leaf(pl, oi)) {
             pending_pro = &o;
             ++oi;   // the UPDATE too
@@ -495,6 +559,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             continue;
         }
         if (o.kind == Op::PAIR) {
+            panel_end = o.c0 + o.h + o.w;
             // two panels + R12 = Q1^T A2 + A2 -= Q1 R12 of a (h + w)-column block; algorithmic bytes:
             // read the block (fp32), write Q (fp32) + shadow(s)
             const double wt = o.h + o.w;
@@ -547,6 +612,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             continue;
         }
         if (o.kind == Op::PANEL) {
+            panel_end = o.c0 + o.w;
             // algorithmic bytes: read the panel (fp32), write Q (fp32) + 16-bit shadow (+ lo shadow)
             ProfScope _s(h, PC_PANEL, 2.0 * m * o.w * o.w, (double)m * o.w * (pl.split ? 12 : 10), o.w);
             rg::PanelLaunch p{};
@@ -655,6 +721,11 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
                                            Cl, pl.ldh, pl.bf16, st, 0, o.te ? &o.mc : nullptr, o.h0));
         }
     }
+    if (pp) {
+        int rc = pipe_need(n);
+        if (!rc) rc = pipe_done(n, true);
+        if (rc) return rc;
+    }
     {
         ProfScope _s(h, PC_OTHER);
         RG_CUDA(rg::launch_unscale_r(pl.R, pl.ldr, n, pl.scale ? h->scale.as<float>() : nullptr, st));
@@ -694,7 +765,7 @@ int check_status(rg_handle h) {
 // local = true forces the single-GPU path even in row-sharded mode (used for the small
 // replicated factorizations of lowrank_approx).
 int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq, float* R,
-              int64_t ldr, const rg_opts& o, int split, bool local = false) {
+              int64_t ldr, const rg_opts& o, int split, bool local = false, HostPipe* pipe = nullptr) {
     if (!ensure_workspace(h, m, n, split)) return RG_ALLOC;
     const int nb = (o.nb <= 0 || o.nb > 32) ? 32 : o.nb;
     const int nranks = local ? 1 : h->nranks;
@@ -739,6 +810,14 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
     }
     int rc = reset_status(h);
     if (rc) return rc;
+    if (pipe) {   // eager: the copy-stream waits sit between the plan's kernels
+        const long long graph_launches = pl->launches;
+        pl->pipe = pipe;
+        rc = enqueue_rgsqr(h, *pl);
+        pl->pipe = nullptr;
+        pl->launches = graph_launches;
+        return rc;
+    }
     const bool use_graph = !h->prof && getenv("RGSQR_NO_GRAPH") == nullptr;
     if (!use_graph) return enqueue_rgsqr(h, *pl);
     if (!pl->exec) {
@@ -1011,6 +1090,9 @@ int rg_destroy(rg_handle h) {
     if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
     if (h->status_host) cudaFreeHost(h->status_host);
     if (h->capture_stream) cudaStreamDestroy(h->capture_stream);
+    if (h->cs_in) cudaStreamDestroy(h->cs_in);
+    if (h->cs_out) cudaStreamDestroy(h->cs_out);
+    for (auto e : h->pipe_ev) cudaEventDestroy(e);
     delete h;
     return RG_OK;
 }
@@ -1093,6 +1175,56 @@ int rg_profile_get(rg_handle h, int cls, double* ms, int64_t* launches, double* 
     return RG_OK;
 }
 
+// rgsqr_factor on pinned host buffers, one pass: column-chunked H2D of A on cs_in, the plan
+// enqueued eagerly with a wait per chunk (HostPipe), Q columns D2H on cs_out as their panels
+// finish, R D2H after the unscale; the user's stream joins cs_out before the status check.
+int factor_host_pipelined(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq,
+                          float* R, int64_t ldr, const rg_opts& o) {
+    if (!h->stageQ.ensure((size_t)m * n * 4) || !h->stageR.ensure((size_t)n * n * 4)) return RG_ALLOC;
+    if (!h->cs_in) RG_CUDA(cudaStreamCreateWithFlags(&h->cs_in, cudaStreamNonBlocking));
+    if (!h->cs_out) RG_CUDA(cudaStreamCreateWithFlags(&h->cs_out, cudaStreamNonBlocking));
+    HostPipe pp;
+    pp.chunk = 128;
+    const int nchunks = (int)((n + pp.chunk - 1) / pp.chunk);
+    while ((int)h->pipe_ev.size() < 3 + nchunks) {
+        cudaEvent_t e;
+        RG_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        h->pipe_ev.push_back(e);
+    }
+    std::vector<cudaEvent_t> in_ev(h->pipe_ev.begin() + 3, h->pipe_ev.begin() + 3 + nchunks);
+    float* dQ = h->stageQ.as<float>();
+    float* dR = h->stageR.as<float>();
+    cudaStream_t st = h->stream;
+    // the staging buffer is free once everything before this call on the user's stream is done
+    RG_CUDA(cudaEventRecord(h->pipe_ev[1], st));
+    RG_CUDA(cudaStreamWaitEvent(h->cs_in, h->pipe_ev[1], 0));
+    RG_CUDA(cudaStreamWaitEvent(h->cs_out, h->pipe_ev[1], 0));
+    for (int k = 0; k < nchunks; ++k) {
+        const int64_t c = (int64_t)k * pp.chunk, nc = std::min<int64_t>(pp.chunk, n - c);
+        RG_CUDA(cudaMemcpy2DAsync(dQ + c * m, m * 4, A + c * lda, lda * 4, m * 4, nc, cudaMemcpyHostToDevice,
+                                  h->cs_in));
+        RG_CUDA(cudaEventRecord(in_ev[k], h->cs_in));
+    }
+    pp.hQ = Q;
+    pp.hldq = ldq;
+    pp.in_ev = &in_ev;
+    pp.cs_out = h->cs_out;
+    pp.ev = h->pipe_ev[0];
+    int rc = run_rgsqr(h, m, n, dQ, m, dQ, m, dR, n, o, o.split, false, &pp);
+    if (rc == RG_OK)
+        RG_CUDA(cudaMemcpy2DAsync(R, ldr * 4, dR, n * 4, n * 4, n, cudaMemcpyDeviceToHost, st));
+    // join both copy streams (also on error: nothing may still be in flight into the staging buffer)
+    RG_CUDA(cudaEventRecord(h->pipe_ev[2], h->cs_out));
+    RG_CUDA(cudaStreamWaitEvent(st, h->pipe_ev[2], 0));
+    RG_CUDA(cudaEventRecord(h->pipe_ev[2], h->cs_in));
+    RG_CUDA(cudaStreamWaitEvent(st, h->pipe_ev[2], 0));
+    if (rc) {
+        cudaStreamSynchronize(st);
+        return rc;
+    }
+    return check_status(h);
+}
+
 int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq,
                  float* R, int64_t ldr, const rg_opts* opts) {
     if (!h) return -1;
@@ -1115,6 +1247,13 @@ int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_
     float* dQ = Q;
     float* dR = R;
     int64_t dlda = lda, dldq = ldq, dldr = ldr;
+    if (host && o.reortho <= 0 && h->nranks <= 1 && !h->prof && is_pinned(A) && is_pinned(Q) && is_pinned(R) &&
+        getenv("RGSQR_NO_PIPE") == nullptr) {
+        int rc = factor_host_pipelined(h, m_local, n, A, lda, Q, ldq, R, ldr, o);
+        end_call(h);
+        prof_collect(h);
+        return rc;
+    }
     if (host) {
         // stage: A -> device Q buffer (factor in place), results copied back
         if (!h->stageQ.ensure((size_t)m_local * n * 4) || !h->stageR.ensure((size_t)n * n * 4)) return RG_ALLOC;

@@ -268,3 +268,41 @@ def test_rgsqr_invalid_arguments(rg):
     assert L.rgsqr_factor(h.ptr, 20, 10, None, 20, p, 20, p, 20, ctypes.byref(o)) == -4
     assert L.rgsqr_factor(h.ptr, 20, 10, p, 19, p, 20, p, 20, ctypes.byref(o)) == -5
     assert L.rgsqr_factor(h.ptr, 20, 10, p, 20, p, 20, p, 9, ctypes.byref(o)) == -9
+
+
+@pytest.mark.parametrize("m,n,pad", [(3000, 96, 0), (5000, 300, 7), (20000, 1000, 0), (4099, 640, 3)])
+def test_rgsqr_pinned_host_pipeline(rg, m, n, pad):
+    """Pinned host A/Q/R take the pipelined path (column-chunked H2D, chunked scaling, Q columns
+    D2H as their panels finish); per-column scaling and per-column norms make it the same
+    arithmetic as the device path, so Q and R must be bit-identical to it."""
+    A = synth.gaussian(m, n, seed=synth.SEED_BASE + 31 + n).astype(np.float32)
+    Ah = torch.zeros(n, m + pad, dtype=torch.float32, pin_memory=True)
+    Ah[:, :m].copy_(torch.from_numpy(np.ascontiguousarray(A.T)))
+    Ah = Ah.t()[:m]
+    Qh = torch.full((n, m + pad), -1.0, dtype=torch.float32, pin_memory=True).t()[:m]
+    Rh = torch.full((n, n), -1.0, dtype=torch.float32, pin_memory=True).t()
+    for _ in range(2):   # second call reuses the staging buffers and copy streams
+        rg.rgsqr_factor(Ah, Q=Qh, R=Rh)
+        Qd, Rd = rg.rgsqr_factor(_dev(A))
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(Qh.numpy(), Qd.cpu().numpy())
+        np.testing.assert_array_equal(Rh.numpy(), Rd.cpu().numpy())
+    _check_qr(A, Qh.numpy().astype(np.float64), Rh.numpy().astype(np.float64), kappa=np.linalg.cond(A))
+
+
+def test_rgsqr_pinned_host_pipeline_breakdown(rg):
+    A = synth.gaussian(2048, 300, seed=13).astype(np.float32)
+    A[:, 257] = 0.0   # a zero column in the third H2D chunk
+    Ah = torch.from_numpy(np.ascontiguousarray(A.T)).pin_memory().t()
+    Qh = torch.empty(300, 2048, dtype=torch.float32, pin_memory=True).t()
+    Rh = torch.empty(300, 300, dtype=torch.float32, pin_memory=True).t()
+    with pytest.raises(rg.RGError) as e:
+        rg.rgsqr_factor(Ah, Q=Qh, R=Rh)
+    with pytest.raises(rg.RGError) as ed:
+        _run(rg, A)
+    assert e.value.status == ed.value.status == rg.RG_BREAKDOWN
+    assert e.value.info == ed.value.info
+    B = synth.gaussian(2048, 300, seed=14).astype(np.float32)
+    Bh = torch.from_numpy(np.ascontiguousarray(B.T)).pin_memory().t()
+    rg.rgsqr_factor(Bh, Q=Qh, R=Rh)
+    _check_qr(B, Qh.numpy().astype(np.float64), Rh.numpy().astype(np.float64), kappa=np.linalg.cond(B))
