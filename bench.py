@@ -276,7 +276,7 @@ def main():
         dt = (time.perf_counter() - t0) / args.e2e_steps
         e2e = {"value": flops / dt / 1e12, "unit": "TFLOP/s", "ms_per_step": dt * 1e3,
                "h2d_bytes_per_step": M * N * 4, "d2h_bytes_per_step": M * N * 4 + N * N * 4,
-               "note": "rgsqr_factor on pinned host A/Q/R: H2D of A, factor, D2H of Q and R, status sync"}
+               "note": "rgsqr_factor on pinned host A/Q/R: column-chunked H2D of A overlapped with the factorization, Q/R columns D2H as their panels finish, status sync"}
         del Ah, Qh, Rh
 
     ls = None

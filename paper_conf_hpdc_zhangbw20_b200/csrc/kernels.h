@@ -44,7 +44,8 @@ cudaError_t launch_colscale(const double* norm2, int n, int do_scale, float* sca
 size_t colnorm_partial_doubles(int64_t m, int n);
 cudaError_t launch_scale_cast(const float* A, int64_t lda, float* Q, int64_t ldq, uint16_t* Qh, uint16_t* Ql,
                               int64_t ldh, int64_t m, int n, const float* scale, int bf16, cudaStream_t st);
-cudaError_t launch_unscale_r(float* R, int64_t ldr, int n, const float* scale, cudaStream_t st);
+cudaError_t launch_unscale_r(float* R, int64_t ldr, int n, const float* scale, cudaStream_t st, int c0 = 0,
+                             int nc = -1);
 
 // ---- panel.cu (eq 8 + Alg 2)
 struct PanelLaunch {

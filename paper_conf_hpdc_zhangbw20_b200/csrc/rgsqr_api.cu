@@ -147,6 +147,8 @@ struct Op {
 struct HostPipe {
     float* hQ = nullptr;
     int64_t hldq = 0;
+    float* hR = nullptr;
+    int64_t hldr = 0;
     int chunk = 128;                  // H2D / scaling granularity (columns)
     int scaled = 0, copied = 0;       // columns scaled on the device / enqueued for D2H
     std::vector<cudaEvent_t>* in_ev = nullptr;   // H2D chunk k landed
@@ -515,10 +517,17 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     // pipeline: Q columns [0, cend) are final; send the new ones home in >= 256-column pieces
     auto pipe_done = [&](int cend, bool flush) -> int {
         if (!pp || cend - pp->copied <= 0 || (!flush && cend - pp->copied < 256)) return RG_OK;
+        // R(:, j) is final once column j's panel has run too (eq 6: R12 blocks of column j come
+        // from K1s of levels where j lies in A2, all enqueued before that panel)
+        RG_CUDA(rg::launch_unscale_r(pl.R, pl.ldr, n, pl.scale ? h->scale.as<float>() : nullptr, st, pp->copied,
+                                     cend - pp->copied));
         RG_CUDA(cudaEventRecord(pp->ev, st));
         RG_CUDA(cudaStreamWaitEvent(pp->cs_out, pp->ev, 0));
         RG_CUDA(cudaMemcpy2DAsync(pp->hQ + (int64_t)pp->copied * pp->hldq, pp->hldq * 4,
                                   pl.Q + (int64_t)pp->copied * pl.ldq, pl.ldq * 4, m * 4, cend - pp->copied,
+                                  cudaMemcpyDeviceToHost, pp->cs_out));
+        RG_CUDA(cudaMemcpy2DAsync(pp->hR + (int64_t)pp->copied * pp->hldr, pp->hldr * 4,
+                                  pl.R + (int64_t)pp->copied * pl.ldr, pl.ldr * 4, n * 4, cend - pp->copied,
                                   cudaMemcpyDeviceToHost, pp->cs_out));
         pp->copied = cend;
         return RG_OK;
@@ -724,7 +733,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     if (pp) {
         int rc = pipe_need(n);
         if (!rc) rc = pipe_done(n, true);
-        if (rc) return rc;
+        return rc;   // R unscaled and sent home piecewise
     }
     {
         ProfScope _s(h, PC_OTHER);
@@ -1177,7 +1186,8 @@ int rg_profile_get(rg_handle h, int cls, double* ms, int64_t* launches, double* 
 
 // rgsqr_factor on pinned host buffers, one pass: column-chunked H2D of A on cs_in, the plan
 // enqueued eagerly with a wait per chunk (HostPipe), Q columns D2H on cs_out as their panels
-// finish, R D2H after the unscale; the user's stream joins cs_out before the status check.
+// finish (with the matching columns of R, unscaled piecewise); the user's stream joins cs_out
+// before the status check.
 int factor_host_pipelined(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq,
                           float* R, int64_t ldr, const rg_opts& o) {
     if (!h->stageQ.ensure((size_t)m * n * 4) || !h->stageR.ensure((size_t)n * n * 4)) return RG_ALLOC;
@@ -1207,12 +1217,12 @@ int factor_host_pipelined(rg_handle h, int64_t m, int64_t n, const float* A, int
     }
     pp.hQ = Q;
     pp.hldq = ldq;
+    pp.hR = R;
+    pp.hldr = ldr;
     pp.in_ev = &in_ev;
     pp.cs_out = h->cs_out;
     pp.ev = h->pipe_ev[0];
     int rc = run_rgsqr(h, m, n, dQ, m, dQ, m, dR, n, o, o.split, false, &pp);
-    if (rc == RG_OK)
-        RG_CUDA(cudaMemcpy2DAsync(R, ldr * 4, dR, n * 4, n * 4, n, cudaMemcpyDeviceToHost, st));
     // join both copy streams (also on error: nothing may still be in flight into the staging buffer)
     RG_CUDA(cudaEventRecord(h->pipe_ev[2], h->cs_out));
     RG_CUDA(cudaStreamWaitEvent(st, h->pipe_ev[2], 0));
