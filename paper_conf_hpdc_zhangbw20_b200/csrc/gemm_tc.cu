@@ -788,8 +788,14 @@ cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, in
                                int64_t ldr, float* Rf, int64_t ldf, uint16_t* Rh, uint16_t* Rl, int64_t ldh, int bf16,
                                cudaStream_t st) {
     const int64_t total = (int64_t)h * w;
-    if (total >= 65536 && (ldp & 3) == 0 && (p_stride & 3) == 0 && (reinterpret_cast<uintptr_t>(P) & 15) == 0) {
-        const int64_t units = (int64_t)((h + 127) / 128) * w;
+    const bool aligned = (ldp & 3) == 0 && (p_stride & 3) == 0 && (reinterpret_cast<uintptr_t>(P) & 15) == 0;
+    const int64_t units = (int64_t)((h + 127) / 128) * w;
+    if (aligned && splits > 32 && units <= (int64_t)num_sms() * 2) {
+        // narrow levels (many splits, few outputs): one wave of 1024-thread CTAs, 128 x 1 outputs per
+        // CTA, every split lane's float4 loads in flight at once
+        RG_LAUNCH((proj_reduce4_kernel<32>), (unsigned)units, dim3(32, 32), 0, st, P, ldp, p_stride, splits, h, w, R,
+                  ldr, Rf, ldf, Rh, Rl, ldh, bf16);
+    } else if (total >= 65536 && aligned) {
         const int grid = (int)std::min<int64_t>(units, (int64_t)num_sms() * 8);
         RG_LAUNCH((proj_reduce4_kernel<8>), grid, dim3(32, 8), 0, st, P, ldp, p_stride, splits, h, w, R, ldr, Rf, ldf,
                   Rh, Rl, ldh, bf16);
