@@ -652,6 +652,51 @@ __global__ void __launch_bounds__(32 * LANES) proj_reduce4_kernel(const float* _
     }
 }
 
+// Few splits (the wide levels, where the tile count already fills the machine): a plain
+// grid-stride pass, 4 consecutive rows i per thread (float4, the partial buffers are padded to
+// whole 128-row tiles), all splits summed in order z = 0, 1, ... by that thread (deterministic).
+// The split-lane kernel above leaves most lanes idle here and pays two block barriers per
+// 128-row unit.
+__global__ void __launch_bounds__(256) proj_reduce_few_kernel(const float* __restrict__ P, int64_t ldp,
+                                                              int64_t p_stride, int splits, int h, int w,
+                                                              float* __restrict__ R, int64_t ldr,
+                                                              float* __restrict__ Rf, int64_t ldf,
+                                                              uint16_t* __restrict__ Rh, uint16_t* __restrict__ Rl,
+                                                              int64_t ldh, int bf16) {
+    RG_PDL_ENTRY();
+    const int h4 = (h + 3) >> 2;
+    const int64_t groups = (int64_t)h4 * w;
+    for (int64_t gi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; gi < groups;
+         gi += (int64_t)gridDim.x * blockDim.x) {
+        const int i0 = 4 * (int)(gi % h4), j = (int)(gi / h4);
+        const float* p = P + (int64_t)j * ldp + i0;
+        float4 v[8];
+#pragma unroll
+        for (int z = 0; z < 8; ++z)
+            if (z < splits) v[z] = __ldcg(reinterpret_cast<const float4*>(p + (int64_t)z * p_stride));
+        float4 t = v[0];
+#pragma unroll
+        for (int z = 1; z < 8; ++z)
+            if (z < splits) {
+                t.x += v[z].x; t.y += v[z].y; t.z += v[z].z; t.w += v[z].w;
+            }
+        const float tv[4] = {t.x, t.y, t.z, t.w};
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+            const int i = i0 + e;
+            if (i < h) {
+                if (R) R[i + (int64_t)j * ldr] = tv[e];
+                if (Rf) Rf[i + (int64_t)j * ldf] = tv[e];
+                if (Rh) {
+                    const uint16_t hb = f2h_bits(tv[e], bf16);
+                    Rh[i + (int64_t)j * ldh] = hb;
+                    if (Rl) Rl[i + (int64_t)j * ldh] = f2h_bits((tv[e] - h2f_bits(hb, bf16)) * 2048.0f, bf16);
+                }
+            }
+        }
+    }
+}
+
 // After a cross-rank allreduce of Rf: write R and the 16-bit images.
 __global__ void proj_finish_kernel(const float* __restrict__ Rf, int64_t ldf, int h, int w, float* __restrict__ R,
                                    int64_t ldr, uint16_t* __restrict__ Rh, uint16_t* __restrict__ Rl, int64_t ldh,
@@ -790,7 +835,12 @@ cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, in
     const int64_t total = (int64_t)h * w;
     const bool aligned = (ldp & 3) == 0 && (p_stride & 3) == 0 && (reinterpret_cast<uintptr_t>(P) & 15) == 0;
     const int64_t units = (int64_t)((h + 127) / 128) * w;
-    if (aligned && splits > 32 && units <= (int64_t)num_sms() * 2) {
+    if (aligned && splits <= 8) {
+        const int64_t groups = (int64_t)((h + 3) / 4) * w;
+        const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((groups + 255) / 256, (int64_t)num_sms() * 8));
+        RG_LAUNCH((proj_reduce_few_kernel), grid, 256, 0, st, P, ldp, p_stride, splits, h, w, R, ldr, Rf, ldf, Rh, Rl,
+                  ldh, bf16);
+    } else if (aligned && splits > 32 && units <= (int64_t)num_sms() * 2) {
         // narrow levels (many splits, few outputs): one wave of 1024-thread CTAs, 128 x 1 outputs per
         // CTA, every split lane's float4 loads in flight at once
         RG_LAUNCH((proj_reduce4_kernel<32>), (unsigned)units, dim3(32, 32), 0, st, P, ldp, p_stride, splits, h, w, R,
