@@ -150,14 +150,16 @@ __global__ void __launch_bounds__(256) scale_cast_kernel(const float* __restrict
 }
 
 // R(:, j) <- R(:, j) / scale[j] (exact: powers of two) for j in [c0, c0 + nc); strictly-lower
-// part zeroed.
-__global__ void unscale_r_kernel(float* R, int64_t ldr, int n, const float* __restrict__ scale, int c0, int nc) {
+// part zeroed.  grid.y walks the columns, grid.x x 256 threads the rows (coalesced, no division).
+__global__ void __launch_bounds__(256) unscale_r_kernel(float* R, int64_t ldr, int n, const float* __restrict__ scale,
+                                                        int c0, int nc) {
     RG_PDL_ENTRY();
-    const int64_t total = (int64_t)n * nc;
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
-        const int i = (int)(e % n), j = c0 + (int)(e / n);
-        float* r = R + i + (int64_t)j * ldr;
-        *r = (i <= j) ? (scale ? *r / scale[j] : *r) : 0.f;
+    for (int jj = blockIdx.y; jj < nc; jj += gridDim.y) {
+        const int j = c0 + jj;
+        const float s = scale ? scale[j] : 1.0f;
+        float* r = R + (int64_t)j * ldr;
+        for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
+            r[i] = (i <= j) ? (scale ? r[i] / s : r[i]) : 0.f;
     }
 }
 
@@ -196,11 +198,10 @@ cudaError_t launch_scale_cast(const float* A, int64_t lda, float* Q, int64_t ldq
 
 cudaError_t launch_unscale_r(float* R, int64_t ldr, int n, const float* scale, cudaStream_t st, int c0, int nc) {
     if (nc < 0) nc = n - c0;
-    const int64_t total = (int64_t)n * nc;
-    int blocks = (int)((total + 255) / 256);
-    if (blocks > 148 * 8) blocks = 148 * 8;
-    if (blocks < 1) return cudaSuccess;
-    RG_LAUNCH((unscale_r_kernel), blocks, 256, 0, st, R, ldr, n, scale, c0, nc);
+    if (nc <= 0 || n <= 0) return cudaSuccess;
+    const int bx = (n + 255) / 256 < 4 ? (n + 255) / 256 : 4;
+    const int by = nc < 65535 ? nc : 65535;
+    RG_LAUNCH((unscale_r_kernel), dim3(bx, by), 256, 0, st, R, ldr, n, scale, c0, nc);
     return cudaGetLastError();
 }
 
