@@ -498,18 +498,23 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     int* status = h->status.as<int>();
     const bool dist = pl.nranks > 1 && h->comm;
     HostPipe* pp = pl.pipe;
+    // section 3.5 on columns [c, c + nc): norms, power-of-two scales, scaled fp32 + 16-bit images
+    auto scale_cols = [&](int c, int nc) -> int {
+        RG_CUDA(rg::launch_colnorm(pl.A + (int64_t)c * pl.lda, pl.lda, m, nc, h->partial.as<double>(),
+                                   h->norm2.as<double>() + c, st));
+        RG_CUDA(rg::launch_colscale(h->norm2.as<double>() + c, nc, pl.scale, h->scale.as<float>() + c, status, c, st));
+        RG_CUDA(rg::launch_scale_cast(pl.A + (int64_t)c * pl.lda, pl.lda, pl.Q + (int64_t)c * pl.ldq, pl.ldq,
+                                      qh + (int64_t)c * pl.ldh, ql ? ql + (int64_t)c * pl.ldh : nullptr, pl.ldh, m, nc,
+                                      h->scale.as<float>() + c, pl.bf16, st));
+        return RG_OK;
+    };
     // pipeline: scale the columns [pp->scaled, cend) rounded up to whole chunks, each after its H2D
     auto pipe_need = [&](int cend) -> int {
         while (pp && pp->scaled < cend) {
             const int c = pp->scaled, nc = std::min(pp->chunk, n - c);
             RG_CUDA(cudaStreamWaitEvent(st, (*pp->in_ev)[c / pp->chunk], 0));
-            RG_CUDA(rg::launch_colnorm(pl.A + (int64_t)c * pl.lda, pl.lda, m, nc, h->partial.as<double>(),
-                                       h->norm2.as<double>() + c, st));
-            RG_CUDA(rg::launch_colscale(h->norm2.as<double>() + c, nc, pl.scale, h->scale.as<float>() + c, status,
-                                        c, st));
-            RG_CUDA(rg::launch_scale_cast(pl.A + (int64_t)c * pl.lda, pl.lda, pl.Q + (int64_t)c * pl.ldq, pl.ldq,
-                                          qh + (int64_t)c * pl.ldh, ql ? ql + (int64_t)c * pl.ldh : nullptr, pl.ldh,
-                                          m, nc, h->scale.as<float>() + c, pl.bf16, st));
+            int rc = scale_cols(c, nc);
+            if (rc) return rc;
             pp->scaled += nc;
         }
         return RG_OK;

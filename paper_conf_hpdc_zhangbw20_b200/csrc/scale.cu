@@ -14,7 +14,8 @@
 
 namespace rg {
 
-constexpr int kNormChunk = 32768;  // rows per CTA of the column-norm pass
+constexpr int kNormChunk = 32768;     // rows per CTA of the column-norm pass
+constexpr int kNormChunkMin = 2048;   // ... at most this short (narrow column ranges)
 
 __device__ __forceinline__ uint16_t s_to16(float x, int bf16) {
     if (bf16) {
@@ -31,11 +32,11 @@ __device__ __forceinline__ float s_from16(uint16_t u, int bf16) {
 
 // partial[y * n + j] = sum_{i in chunk y} A(i, j)^2   (fp64 accumulation)
 __global__ void __launch_bounds__(256) colnorm_partial_kernel(const float* __restrict__ A, int64_t lda, int64_t m,
-                                                              int n, double* __restrict__ partial) {
+                                                              int n, double* __restrict__ partial, int rows_per) {
     RG_PDL_ENTRY();
     const int j = blockIdx.x;
-    const int64_t i0 = (int64_t)blockIdx.y * kNormChunk;
-    const int64_t i1 = min(m, i0 + kNormChunk);
+    const int64_t i0 = (int64_t)blockIdx.y * rows_per;
+    const int64_t i1 = min(m, i0 + rows_per);
     const float* a = A + (int64_t)j * lda;
     double s = 0.0;
     const bool vec = ((reinterpret_cast<uintptr_t>(a + i0) & 15) == 0);
@@ -165,9 +166,13 @@ __global__ void __launch_bounds__(256) unscale_r_kernel(float* R, int64_t ldr, i
 
 cudaError_t launch_colnorm(const float* A, int64_t lda, int64_t m, int n, double* partial, double* norm2,
                            cudaStream_t st) {
-    const int chunks = (int)((m + kNormChunk - 1) / kNormChunk);
+    // kNormChunk rows per CTA; narrow column ranges (the chunked scaling pass) use shorter row
+    // chunks (down to kNormChunkMin) so that the grid still covers ~8 CTAs per SM
+    int rows_per = kNormChunk;
+    while (rows_per > kNormChunkMin && (int64_t)n * ((m + rows_per - 1) / rows_per) < 148 * 8) rows_per >>= 1;
+    const int chunks = (int)((m + rows_per - 1) / rows_per);
     dim3 grid(n, chunks);
-    RG_LAUNCH((colnorm_partial_kernel), grid, 256, 0, st, A, lda, m, n, partial);
+    RG_LAUNCH((colnorm_partial_kernel), grid, 256, 0, st, A, lda, m, n, partial, rows_per);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
     RG_LAUNCH((colnorm_sum_kernel), (n + 127) / 128, 128, 0, st, partial, chunks, n, norm2);
@@ -181,7 +186,7 @@ cudaError_t launch_colscale(const double* norm2, int n, int do_scale, float* sca
 }
 
 size_t colnorm_partial_doubles(int64_t m, int n) {
-    return (size_t)((m + kNormChunk - 1) / kNormChunk) * (size_t)n;
+    return (size_t)((m + kNormChunkMin - 1) / kNormChunkMin) * (size_t)n;
 }
 
 cudaError_t launch_scale_cast(const float* A, int64_t lda, float* Q, int64_t ldq, uint16_t* Qh, uint16_t* Ql,
