@@ -12,7 +12,10 @@
  *     asynchronous on the handle's stream apart from the final status check) or HOST
  *     pointers (pageable or pinned; the library stages them through device workspace and the
  *     call returns when the results are back in host memory).  All matrix arguments of one
- *     call must be on the same side.
+ *     call must be on the same side.  rgsqr_factor on PINNED host A, Q and R (single rank,
+ *     reortho = 0) overlaps the copies with the factorization: A goes up in column chunks and
+ *     Q / R columns come back as soon as their panel has run; the results are bit-identical to
+ *     the device-pointer call.
  *   - The caller owns every input and output.  The library owns only the workspace inside the
  *     handle (grown lazily, freed by rg_destroy).
  *   - Return value: 0 = RG_OK; a NEGATIVE value -i means argument i (1-based, the handle is
