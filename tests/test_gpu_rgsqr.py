@@ -306,3 +306,23 @@ def test_rgsqr_pinned_host_pipeline_breakdown(rg):
     Bh = torch.from_numpy(np.ascontiguousarray(B.T)).pin_memory().t()
     rg.rgsqr_factor(Bh, Q=Qh, R=Rh)
     _check_qr(B, Qh.numpy().astype(np.float64), Rh.numpy().astype(np.float64), kappa=np.linalg.cond(B))
+
+
+@pytest.mark.parametrize("kw", [dict(precision="bf16"), dict(split=True), dict(panel="mgs"), dict(scale=False),
+                                dict(reortho=1), dict(nb=16)])
+def test_rgsqr_pinned_host_options(rg, kw):
+    """Every option through pinned host buffers (pipelined when reortho = 0, staged otherwise)
+    gives the device-pointer call's Q and R bit for bit."""
+    m, n = 6000, 200
+    A = synth.gaussian(m, n, seed=synth.SEED_BASE + 77).astype(np.float32) * np.float32(3e-3)
+    Ah = torch.from_numpy(np.ascontiguousarray(A.T)).pin_memory().t()
+    Qh = torch.empty(n, m, dtype=torch.float32, pin_memory=True).t()
+    Rh = torch.empty(n, n, dtype=torch.float32, pin_memory=True).t()
+    o = rg.make_opts(**kw)
+    rg.rgsqr_factor(Ah, Q=Qh, R=Rh, opts=o)
+    Qd, Rd = rg.rgsqr_factor(_dev(A), opts=o)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(Qh.numpy(), Qd.cpu().numpy())
+    np.testing.assert_array_equal(Rh.numpy(), Rd.cpu().numpy())
+    _check_qr(A, Qh.numpy().astype(np.float64), Rh.numpy().astype(np.float64), kappa=np.linalg.cond(A),
+              orth_scale=1.0 if kw.get("precision") == "bf16" or kw.get("scale") is False else 1e-2)
