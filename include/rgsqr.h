@@ -60,7 +60,11 @@ enum {
 /* Options.  rg_opts_default() fills the defaults listed here. */
 typedef struct {
     int precision;  /* tensor-core operand type: 0 = fp16 (default), 1 = bf16 */
-    int nb;         /* recursion leaf width (panel columns), 1..32; 0 = auto (32) */
+    int nb;         /* panel width of the recursion's base case, 1..32; 0 = auto (32).  With the
+                       default nb = 32 and a single-GPU, non-split pass whose rows fit on chip
+                       (m <= ~85K), the base case is a 64-column block factored by one leaf
+                       kernel (CholQR2, fp64 Gram; reading #2) -- the same unique Q, R as two
+                       32-column panels + K1 + K2 in exact arithmetic */
     int scale;      /* 1 = automatic power-of-two column scaling (default, section 3.5 P:L357-361,
                        reading #4); 0 = off */
     int reortho;    /* extra reorthogonalisation passes: for rgsqr_factor default 0; for
@@ -90,21 +94,47 @@ RG_API int64_t rg_last_launches(rg_handle h);
 /* Build identity, e.g. "rgsqr sm_100a tcgen05"; never NULL. */
 RG_API const char* rg_version(void);
 
-/* ---- row-sharded multi-GPU mode --------------------------------------------
+/* ---- row-sharded multi-GPU mode (the row split of eq 8) ----------
+ * Each rank holds a contiguous block of rows; the collectives combine only small pieces (column
+ * norms, the K1 blocks R12, the panel Gram matrices or TSQR R factors, CGLS vectors).  At most
+ * RG_MAX_RANKS ranks (one 8-GPU node; the TSQR panel stacks <= 8 32 x 32 R factors).
+ * Three ways to attach a handle to a group (each replaces the previous one and drops the
+ * handle's cached plans):
+ *   rg_comm_init  -- the library creates its own NCCL communicator from a ncclUniqueId that
+ *                    rg_comm_unique_id wrote on the root rank (broadcast it, e.g. with
+ *                    torch.distributed); destroyed with the handle.  nranks == 1 is allowed.
+ *   rg_set_comm   -- use a CALLER-OWNED ncclComm_t (e.g. torch.distributed's); NULL detaches
+ *                    (back to single-GPU mode).  The communicator must come from the same
+ *                    libnccl the library loaded (rg_nccl_load with that path) and outlive the
+ *                    handle's use of it.
+ *   rg_set_vcomm  -- in-process "virtual ranks": P handles on ONE device share a group made by
+ *                    rg_vgroup_create; each rank's API call must run on its own host thread,
+ *                    concurrently.  Collectives are a host rendezvous + a fixed-order reduction
+ *                    kernel; plans run eagerly (no CUDA graphs).  For testing the row-sharded
+ *                    branches on one GPU; a rank that never arrives makes its peers fail with
+ *                    RG_NCCL_ERROR after 120 s.
  * NCCL is loaded at run time (dlopen) from `nccl_path` (NULL = "libnccl.so.2").
- * rg_comm_unique_id writes a 128-byte ncclUniqueId on the root rank; broadcast it (e.g. with
- * torch.distributed) and call rg_comm_init on every rank.  nranks == 1 is allowed. */
+ * Errors: -3 rank outside [0, nranks), -4 nranks outside [1, RG_MAX_RANKS]; rg_set_vcomm -2 the
+ * group was created on another device; rg_vgroup_destroy -1 while handles are attached. */
+#define RG_MAX_RANKS 8
 RG_API int rg_nccl_load(const char* nccl_path);
 RG_API int rg_comm_unique_id(void* id128);
 RG_API int rg_comm_init(rg_handle h, const void* id128, int rank, int nranks);
+RG_API int rg_set_comm(rg_handle h, void* nccl_comm, int rank, int nranks);
+RG_API int rg_vgroup_create(void** group, int nranks);   /* on the current CUDA device */
+RG_API int rg_vgroup_destroy(void* group);
+RG_API int rg_set_vcomm(rg_handle h, void* group, int rank);
 
 /* ---- rgsqr_factor: A = Q R (Algorithm 1) -------------------------------------
  * A (m_local x n, lda) is not modified unless Q aliases it (Q == A and ldq == lda: in place).
  * Q (m_local x n, ldq): orthonormal columns.  R (n x n, ldr): upper triangular with
  * positive diagonal, strictly-lower part zeroed, replicated on all ranks.
  * Recursive trailing updates R12 = Q1^T A2 and A2 -= Q1 R12 on tcgen05 tensor cores with
- * 16-bit operands and fp32 accumulation; the 32-column leaves are the fp32
- * CAQR/MGS panel of eq 8 / Alg 2.  Requires m (global) >= n >= 1.
+ * 16-bit operands and fp32 accumulation.  Base case (reading #2, #20): 64-column
+ * leaves factored by CholQR2 with an fp64 Gram (rows resident on chip, m <= ~85K rows), else
+ * 32-column CholQR2 panels (fused or streaming); opts->panel = 1 selects the paper's fp32
+ * TSQR/MGS panel of eq 8 / Alg 2, which is also the automatic fallback when a
+ * Cholesky pivot fails.  Requires m (global) >= n >= 1.
  * Errors: -2 m_local < 1 (or m < n single-GPU), -3 n < 1, -4 A NULL, -5 lda < m_local,
  * -6 Q NULL, -7 ldq < m_local, -8 R NULL, -9 ldr < n; RG_BREAKDOWN, RG_NONFINITE. */
 RG_API int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq,
@@ -115,7 +145,8 @@ RG_API int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A,
  * estimate ||I - Q^T Q||_F > orth_tol and passes < max_passes: [Q2, R2] = RGSQR(Q) with the
  * split-precision GEMMs (reading #9) and R <- R2 R ("twice is enough").
  * R (n x n, ldr) receives the accumulated triangular factor if non-NULL.  passes_out: number
- * of RGSQR passes run; orth_est_out: final ||I - Q^T Q||_F (exact, via a Gram matrix).
+ * of RGSQR passes run; orth_est_out: final ||I - Q^T Q||_F, a Hutchinson estimate with 8 fixed
+ * Gaussian probes (E||M g||^2 = ||M||_F^2; within a few % of the exact value).
  * orth_tol <= 0 means "run exactly max_passes passes".
  * Errors: -2..-6 as above (A is arg 4, lda arg 5, R arg 6, ldr arg 7 (< n with R non-NULL)),
  * -9 max_passes < 1; RG_NOT_CONVERGED if the final estimate is above orth_tol > 0. */
@@ -153,6 +184,17 @@ RG_API int lowrank_approx(rg_handle h, int64_t m_local, int64_t n, const float* 
 RG_API int rg_profile_enable(rg_handle h, int enable);
 RG_API int rg_profile_reset(rg_handle h);
 RG_API int rg_profile_get(rg_handle h, int cls, double* ms, int64_t* launches, double* flops, double* bytes);
+
+/* ---- generator access for parity tests -----------------------------------------------------
+ * The seeded Gaussian stream behind lowrank_approx's Omega (seed = its `seed`) and the
+ * orthogonality probes: element e takes Philox4x32-10 call e >> 1 with counter
+ * {call lo32, call hi32, 0, 0} and key {seed lo32, seed hi32}; words (0, 1) for even e, (2, 3)
+ * for odd e give u1 = (w_a + 1) 2^-32, u2 = w_b 2^-32, z = sqrt(-2 ln u1) cos(2 pi u2) (fp64).
+ * rg_debug_philox writes the 4 raw words of calls 0 .. ncalls-1 (4 * ncalls uint32, DEVICE
+ * pointer); rg_debug_gaussian writes z for e = 0 .. n-1 (n doubles, DEVICE pointer).  Both
+ * synchronise.  Errors: -2 negative count, -4 pointer NULL or not device memory. */
+RG_API int rg_debug_philox(rg_handle h, int64_t ncalls, uint64_t seed, uint32_t* words);
+RG_API int rg_debug_gaussian(rg_handle h, int64_t n, uint64_t seed, double* out);
 
 #ifdef __cplusplus
 }

@@ -30,7 +30,9 @@ EXPORTS = [
     "rg_opts_default", "rg_create", "rg_set_stream", "rg_destroy", "rg_status_string", "rg_last_info",
     "rg_version", "rg_last_launches", "rg_nccl_load", "rg_comm_unique_id", "rg_comm_init", "rgsqr_factor", "orthogonalize",
     "ls_solve_refined", "lowrank_approx", "rg_profile_enable", "rg_profile_reset", "rg_profile_get",
+    "rg_set_comm", "rg_vgroup_create", "rg_vgroup_destroy", "rg_set_vcomm", "rg_debug_gaussian", "rg_debug_philox",
 ]
+RG_MAX_RANKS = 8
 
 PROFILE_CLASSES = {"update": 0, "proj": 1, "panel": 2, "scale": 3, "cgls": 4, "other": 5}
 
@@ -80,6 +82,12 @@ def _lib():
         L.rg_nccl_load.argtypes = [ctypes.c_char_p]
         L.rg_comm_unique_id.argtypes = [vp]
         L.rg_comm_init.argtypes = [vp, vp, i32, i32]
+        L.rg_set_comm.argtypes = [vp, vp, i32, i32]
+        L.rg_vgroup_create.argtypes = [ctypes.POINTER(vp), i32]
+        L.rg_vgroup_destroy.argtypes = [vp]
+        L.rg_set_vcomm.argtypes = [vp, vp, i32]
+        L.rg_debug_gaussian.argtypes = [vp, i64, ctypes.c_uint64, vp]
+        L.rg_debug_philox.argtypes = [vp, i64, ctypes.c_uint64, vp]
         L.rgsqr_factor.argtypes = [vp, i64, i64, vp, i64, vp, i64, vp, i64, ctypes.POINTER(rg_opts)]
         L.orthogonalize.argtypes = [vp, i64, i64, vp, i64, vp, i64, ctypes.c_double, i32,
                                     ctypes.POINTER(i32), f64p, ctypes.POINTER(rg_opts)]
@@ -223,6 +231,18 @@ class Handle:
         _check("rg_comm_init", _lib().rg_comm_init(self._h, buf, int(rank), int(nranks)), self)
         self.rank, self.nranks = rank, nranks
 
+    def set_comm(self, nccl_comm_ptr: int, rank: int, nranks: int):
+        """Row-sharded mode on a caller-owned ncclComm_t (0 detaches)."""
+        _check("rg_set_comm", _lib().rg_set_comm(self._h, ctypes.c_void_p(int(nccl_comm_ptr)), int(rank),
+                                                 int(nranks)), self)
+        self.rank, self.nranks = (rank, nranks) if nccl_comm_ptr else (0, 1)
+
+    def set_vcomm(self, group, rank: int):
+        """Attach to an in-process virtual-rank group (VGroup); None detaches."""
+        _check("rg_set_vcomm", _lib().rg_set_vcomm(self._h, group.ptr if group is not None else None, int(rank)),
+               self)
+        self.rank, self.nranks = (rank, group.nranks) if group is not None else (0, 1)
+
     # ---- profiling -------------------------------------------------------------------------
     def profile(self, enable=True):
         _lib().rg_profile_enable(self._h, int(bool(enable)))
@@ -236,6 +256,76 @@ class Handle:
         c = PROFILE_CLASSES[cls] if isinstance(cls, str) else int(cls)
         _lib().rg_profile_get(self._h, c, ctypes.byref(ms), ctypes.byref(n), ctypes.byref(fl), ctypes.byref(by))
         return {"ms": ms.value, "launches": n.value, "flops": fl.value, "bytes": by.value}
+
+
+class VGroup:
+    """In-process virtual ranks on one device (rg_vgroup_create): P handles, one host thread per
+    rank, run the library's row-sharded code path with fixed-order on-device collectives."""
+
+    def __init__(self, nranks: int, device: int = 0):
+        import torch
+        torch.cuda.set_device(device)
+        self._g = ctypes.c_void_p()
+        st = _lib().rg_vgroup_create(ctypes.byref(self._g), int(nranks))
+        if st != RG_OK:
+            raise RGError("rg_vgroup_create", st)
+        self.nranks = nranks
+        self.device = device
+
+    @property
+    def ptr(self):
+        return self._g
+
+    def close(self):
+        if self._g:
+            _lib().rg_vgroup_destroy(self._g)
+            self._g = ctypes.c_void_p()
+
+
+def run_ranks(fns):
+    """Run fns[r]() on one host thread per rank (the library releases the GIL in every call);
+    returns their results, re-raising the first exception."""
+    import threading
+    out = [None] * len(fns)
+    err = [None] * len(fns)
+
+    def body(r):
+        try:
+            out[r] = fns[r]()
+        except BaseException as e:  # noqa: BLE001
+            err[r] = e
+
+    ts = [threading.Thread(target=body, args=(r,)) for r in range(len(fns))]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    for e in err:
+        if e is not None:
+            raise e
+    return out
+
+
+def debug_gaussian(n: int, seed: int, out=None, handle=None):
+    """The device Philox4x32-10 + Box-Muller generator behind lowrank_approx's Omega and the
+    Hutchinson probes, exposed for bit-exact parity tests: n fp64 values into a CUDA tensor."""
+    import torch
+    h = _handle(handle)
+    if out is None:
+        out = torch.empty(n, dtype=torch.float64, device="cuda")
+    _check("rg_debug_gaussian", _lib().rg_debug_gaussian(h.ptr, int(n), ctypes.c_uint64(int(seed) & (2**64 - 1)),
+                                                        ctypes.c_void_p(out.data_ptr())), h)
+    return out
+
+
+def debug_philox(ncalls: int, seed: int, handle=None):
+    """Raw Philox4x32-10 words (ncalls x 4 uint32 as int64 numpy) of the device generator."""
+    import torch
+    h = _handle(handle)
+    out = torch.empty(ncalls * 4, dtype=torch.int32, device="cuda")
+    _check("rg_debug_philox", _lib().rg_debug_philox(h.ptr, int(ncalls), ctypes.c_uint64(int(seed) & (2**64 - 1)),
+                                                    ctypes.c_void_p(out.data_ptr())), h)
+    return out.cpu().numpy().view(np.uint32).astype(np.int64).reshape(ncalls, 4)
 
 
 def _find_nccl():

@@ -715,16 +715,7 @@ __global__ void proj_finish_kernel(const float* __restrict__ Rf, int64_t ldf, in
 }
 
 // ------------------------------------------------------------------ host launchers
-static int g_num_sms = 0;
-static int num_sms() {
-    if (!g_num_sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
-        if (g_num_sms <= 0) g_num_sms = 148;
-    }
-    return g_num_sms;
-}
+static int num_sms() { return dev_sms(); }
 
 template <int MODE, int BN, int STAGES, bool SPLIT, int EPI_WG, int TE = 0>
 static cudaError_t launch_gemm(int units, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& al,
@@ -733,11 +724,9 @@ static cudaError_t launch_gemm(int units, const CUtensorMap& a, const CUtensorMa
     using C = GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>;
     static_assert(C::kTotal <= 227 * 1024, "shared memory budget");
     auto kern = gemm_tc_kernel<MODE, BN, STAGES, SPLIT, EPI_WG, TE>;
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::kTotal);
+    {
+        cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), C::kTotal);
         if (e != cudaSuccess) return e;
-        attr_set = true;
     }
     // persistent grid: one CTA per SM (two when the footprint allows), never more than units
     const int per_sm = (C::kTotal <= 113 * 1024 && C::kTmemCols <= 256) ? 2 : 1;

@@ -23,6 +23,14 @@ namespace rg {
 
 bool pdl_enabled();
 
+// Per-device properties of the CURRENT device (cached per device ordinal, thread-safe): one process
+// may drive several GPUs (one handle per device, or in-process virtual ranks).
+int dev_sms();              // multiprocessor count
+int dev_smem_optin();       // cudaDevAttrMaxSharedMemoryPerBlockOptin
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per (device, kernel) and whenever a larger
+// size is needed on that device; the attribute is per device context.
+cudaError_t ensure_smem_attr(const void* kernel, size_t bytes);
+
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
                             Args&&... args);
@@ -191,6 +199,7 @@ cudaError_t launch_cgls_xr(double* x, const double* t, double* r, const double* 
                            cudaStream_t st);
 cudaError_t launch_cgls_p(const double* s, double* p, int n, double* sc, int first, cudaStream_t st);
 cudaError_t launch_gaussian_philox(int64_t total, uint64_t seed, double* out64, float* out32, cudaStream_t st);
+cudaError_t launch_philox_words(int64_t ncalls, uint64_t seed, uint32_t* words, cudaStream_t st);
 size_t probe_work_doubles(int64_t m, int n, int p);
 cudaError_t launch_orth_probe_z(const float* Q, int64_t ldq, int64_t m, int n, const double* G, double* work,
                                 double* Z, cudaStream_t st);

@@ -937,26 +937,8 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
 }
 
 // ------------------------------------------------------------------ host side
-static int lf_sms() {
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (sms <= 0) sms = 148;
-    }
-    return sms;
-}
-static int lf_smem_max() {
-    static int v = 0;
-    if (!v) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-        v -= 1024;   // static shared memory + slack
-    }
-    return v;
-}
+static int lf_sms() { return dev_sms(); }
+static int lf_smem_max() { return dev_smem_optin() - 1024; }   // static shared memory + slack
 static void lf_geometry(int64_t m, int& grid, int& rows_per, int& ldt) {
     grid = lf_sms() < LF_MAX_GRID ? lf_sms() : LF_MAX_GRID;
     rows_per = (int)(((m + grid - 1) / grid + 7) & ~int64_t(7));
@@ -1022,11 +1004,9 @@ cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st) {
     // pack loops and the image stores cost convergence-barrier (BSSY) overhead
     void (*kern)(LeafArgs) = a.bf16 ? (small ? leaf_kernel<7, 1> : leaf_kernel<LF_MAXI, 1>)
                                     : (small ? leaf_kernel<7, 0> : leaf_kernel<LF_MAXI, 0>);
-    static size_t attr[2][2] = {{0, 0}, {0, 0}};
-    if (smem > attr[a.bf16 ? 1 : 0][small]) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    {
+        cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), smem);
         if (e != cudaSuccess) return e;
-        attr[a.bf16 ? 1 : 0][small] = smem;
     }
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(grid);

@@ -1269,15 +1269,7 @@ size_t cholqr_counter_ints(int64_t m) {
 }
 
 
-static int sm_count() {
-    static int sms = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    }
-    return sms;
-}
+static int sm_count() { return dev_sms(); }
 
 bool cholqr_fused_fits(int64_t m, int ncols) {
     const int64_t rows_per = (m + sm_count() - 1) / sm_count();
@@ -1325,19 +1317,13 @@ static cudaError_t launch_fused(CqArgs a, cudaStream_t st) {
     const int64_t rows_per = (a.m + sms - 1) / sms;
     const int ld = (int)(rows_per | 1);   // odd leading dimension: conflict-free column walks
     // all of shared memory: the tile, Gs, and the rest for Rs / Ri / Gram staging
-    static int smem_max = 0;
-    if (!smem_max) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
-        smem_max -= 2048;   // static shared memory of the kernel + slack
-    }
+    const int smem_max = dev_smem_optin() - 2048;   // static shared memory of the kernel + slack
     const size_t tile_bytes = (((size_t)NC * ld * 4 + 15) & ~(size_t)15);
     const size_t gs_bytes = (size_t)NC * (NC + 2) * 8;
     if (tile_bytes + CfBufs<NC>::fixed_bytes > (size_t)smem_max) return cudaErrorInvalidValue;
     const int s_cap = (int)(((size_t)smem_max - tile_bytes - gs_bytes) / 8);
     const size_t smem = (size_t)smem_max;
-    cudaError_t e = cudaFuncSetAttribute(cq_fused_kernel<NC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(cq_fused_kernel<NC>), smem);
     if (e != cudaSuccess) return e;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(sms);
@@ -1364,13 +1350,10 @@ cudaError_t launch_panel_cholqr(const CholqrLaunch& L, bool* handles_failure, cu
     if (handles_failure) *handles_failure = false;      // the guarded MGS/TSQR kernels must follow
     cudaError_t e;
     constexpr size_t ring_bytes = (size_t)CQ_STAGES * CQ_TILE_FLOATS * 4;
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaFuncSetAttribute(cq_pass_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ring_bytes);
-        cudaFuncSetAttribute(cq_pass_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ring_bytes);
-        cudaFuncSetAttribute(cq_pass_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ring_bytes);
-        attr_set = true;
-    }
+    if ((e = ensure_smem_attr(reinterpret_cast<const void*>(cq_pass_kernel<0>), ring_bytes)) != cudaSuccess ||
+        (e = ensure_smem_attr(reinterpret_cast<const void*>(cq_pass_kernel<1>), ring_bytes)) != cudaSuccess ||
+        (e = ensure_smem_attr(reinterpret_cast<const void*>(cq_pass_kernel<2>), ring_bytes)) != cudaSuccess)
+        return e;
     for (int pass = 0; pass < 3; ++pass) {
         if (pass == 0) RG_LAUNCH((cq_pass_kernel<0>), grid, CQ_THREADS, ring_bytes, st, a);
         if (pass == 1) RG_LAUNCH((cq_pass_kernel<1>), grid, CQ_THREADS, ring_bytes, st, a);

@@ -14,6 +14,11 @@
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <condition_variable>
+#include <map>
+#include <mutex>
 #include <climits>
 #include <cmath>
 #include <cstdio>
@@ -100,19 +105,36 @@ enum ProfClass { PC_UPDATE = 0, PC_PROJ = 1, PC_PANEL = 2, PC_SCALE = 3, PC_CGLS
 }  // namespace
 
 // ------------------------------------------------------------------ device buffers
-static int g_alloc_epoch = 0;  // bumped whenever any workspace buffer moves (plans/graphs embed addresses)
-
+// Workspace buffer of one handle.  A buffer is bound to its handle's stream and allocation epoch
+// (rg_create): growing it bumps the epoch (plans / graphs embed addresses and are rebuilt) and
+// zeroes the new memory in stream order on the handle's stream, then waits for it -- counters,
+// flags and the leaf's grid-barrier word rely on zero-initialised workspace, and the handle's
+// stream may be a non-blocking stream that the legacy-stream cudaMemset would not order against.
 struct DevBuf {
     void* p = nullptr;
     size_t bytes = 0;
+    int* epoch = nullptr;                 // owning handle's allocation epoch
+    const cudaStream_t* stream = nullptr; // owning handle's stream
     bool ensure(size_t b) {
         if (b <= bytes) return true;
-        ++g_alloc_epoch;
-        if (p) cudaFree(p);
+        if (epoch) ++*epoch;
+        if (p) {
+            if (stream) cudaStreamSynchronize(*stream);   // nothing in flight may still use it
+            cudaFree(p);
+        }
         p = nullptr;
         bytes = 0;
-        if (cudaMalloc(&p, b) != cudaSuccess) return false;
-        cudaMemset(p, 0, b);  // counters / flags rely on zero-initialised workspace
+        if (cudaMalloc(&p, b) != cudaSuccess) {
+            cudaGetLastError();
+            p = nullptr;
+            return false;
+        }
+        const cudaStream_t st = stream ? *stream : nullptr;
+        if (cudaMemsetAsync(p, 0, b, st) != cudaSuccess || cudaStreamSynchronize(st) != cudaSuccess) {
+            cudaFree(p);
+            p = nullptr;
+            return false;
+        }
         bytes = b;
         return true;
     }
@@ -164,7 +186,7 @@ struct Plan {
     float* R = nullptr;
     int nb = 0, bf16 = 0, split = 0, scale = 1, nranks = 1, rank = 0, panel = 0;
     bool leaf = false;       // last level runs as leaf.cu kernels
-    int epoch = -1;          // g_alloc_epoch the plan was built against
+    int epoch = -1;          // handle allocation epoch the plan was built against
     // derived
     int64_t ldh = 0, ldr12 = 0;
     std::vector<Op> ops;
@@ -174,13 +196,133 @@ struct Plan {
     HostPipe* pipe = nullptr;  // set for one eager enqueue of the host-pointer pipeline
 };
 
+
+// ------------------------------------------------------------------ in-process virtual ranks
+// P handles on ONE device form a group; each rank's collective calls come from its own host
+// thread (the API calls of the P ranks run concurrently, one thread per handle).  A collective
+// is a host rendezvous: every rank records a "ready" event on its stream; the last to arrive
+// makes its stream wait for all of them, reduces the P buffers in fixed rank order (0, 1, ..)
+// into the group scratch with one kernel and copies the result to every rank's buffer (or, for
+// an allgather, copies every rank's block into every rank's receive buffer), records "done",
+// and wakes the others, which make their streams wait for "done".  Deterministic, no NCCL:
+// it exists so that the row-sharded branches of the library can run and be
+// checked on a single GPU (NCCL refuses two ranks on one device).
+__global__ void vsum_kernel(const void* const* in, int P, size_t count, int f64, void* out) {
+    const size_t stride = (size_t)gridDim.x * blockDim.x;
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < count; i += stride) {
+        if (f64) {
+            double s = reinterpret_cast<const double*>(in[0])[i];
+            for (int r = 1; r < P; ++r) s += reinterpret_cast<const double*>(in[r])[i];
+            reinterpret_cast<double*>(out)[i] = s;
+        } else {
+            float s = reinterpret_cast<const float*>(in[0])[i];
+            for (int r = 1; r < P; ++r) s += reinterpret_cast<const float*>(in[r])[i];
+            reinterpret_cast<float*>(out)[i] = s;
+        }
+    }
+}
+
+struct VGroup {
+    int P = 0;
+    int device = -1;
+    std::mutex mu;
+    std::condition_variable cv;
+    int arrived = 0;
+    unsigned long long gen = 0;
+    int failed = 0;                      // a rank timed out or saw a mismatch: all later calls fail
+    struct Slot {
+        const void* send = nullptr;
+        void* recv = nullptr;
+        size_t count = 0;
+        int kind = 0;                    // 0 allreduce (in place), 1 allgather
+        int f64 = 0;
+        cudaStream_t st = nullptr;
+    };
+    std::vector<Slot> slots;
+    std::vector<cudaEvent_t> ready;
+    cudaEvent_t done = nullptr;
+    void* scratch = nullptr;             // reduction result
+    size_t scratch_bytes = 0;
+    void** dptrs = nullptr;              // device array of the P input pointers
+    int attached = 0;
+};
+
+int vgroup_collective(VGroup* g, int rank, VGroup::Slot slot) {
+    using namespace std::chrono;
+    std::unique_lock<std::mutex> lk(g->mu);
+    if (g->failed) return RG_NCCL_ERROR;
+    if (cudaEventRecord(g->ready[rank], slot.st) != cudaSuccess) return RG_CUDA_ERROR;
+    g->slots[rank] = slot;
+    const unsigned long long my = g->gen;
+    if (++g->arrived == g->P) {
+        int rc = RG_OK;
+        for (int r = 0; r < g->P; ++r)
+            if (g->slots[r].count != slot.count || g->slots[r].kind != slot.kind || g->slots[r].f64 != slot.f64)
+                rc = RG_NCCL_ERROR;   // ranks disagree on the collective: a library bug
+        cudaStream_t st = slot.st;
+        const size_t esz = slot.f64 ? 8 : 4, bytes = slot.count * esz;
+        for (int r = 0; r < g->P && rc == RG_OK; ++r)
+            if (cudaStreamWaitEvent(st, g->ready[r], 0) != cudaSuccess) rc = RG_CUDA_ERROR;
+        if (rc == RG_OK && slot.kind == 0 && bytes > 0) {
+            if (bytes > g->scratch_bytes) {
+                cudaStreamSynchronize(st);
+                if (g->scratch) cudaFree(g->scratch);
+                g->scratch = nullptr;
+                g->scratch_bytes = 0;
+                if (cudaMalloc(&g->scratch, bytes) != cudaSuccess) rc = RG_ALLOC;
+                else g->scratch_bytes = bytes;
+            }
+            std::vector<const void*> in((size_t)g->P);
+            for (int r = 0; r < g->P; ++r) in[r] = g->slots[r].recv;
+            if (rc == RG_OK &&
+                cudaMemcpyAsync(g->dptrs, in.data(), sizeof(void*) * g->P, cudaMemcpyHostToDevice, st) != cudaSuccess)
+                rc = RG_CUDA_ERROR;
+            if (rc == RG_OK) {
+                // (the host array `in` must outlive the async copy: synchronise before it goes away)
+                const int blocks = (int)std::min<size_t>(1024, (slot.count + 255) / 256);
+                vsum_kernel<<<blocks, 256, 0, st>>>(const_cast<const void* const*>(g->dptrs), g->P, slot.count,
+                                                    slot.f64, g->scratch);
+                ++rg::g_launches;
+                if (cudaGetLastError() != cudaSuccess || cudaStreamSynchronize(st) != cudaSuccess) rc = RG_CUDA_ERROR;
+            }
+            for (int r = 0; r < g->P && rc == RG_OK; ++r)
+                if (cudaMemcpyAsync(g->slots[r].recv, g->scratch, bytes, cudaMemcpyDeviceToDevice, st) != cudaSuccess)
+                    rc = RG_CUDA_ERROR;
+        } else if (rc == RG_OK && slot.kind == 1 && bytes > 0) {
+            for (int r = 0; r < g->P && rc == RG_OK; ++r)
+                for (int q = 0; q < g->P && rc == RG_OK; ++q) {
+                    char* dst = reinterpret_cast<char*>(g->slots[r].recv) + (size_t)q * bytes;
+                    if (dst == g->slots[q].send) continue;
+                    if (cudaMemcpyAsync(dst, g->slots[q].send, bytes, cudaMemcpyDeviceToDevice, st) != cudaSuccess)
+                        rc = RG_CUDA_ERROR;
+                }
+        }
+        if (rc == RG_OK && cudaEventRecord(g->done, st) != cudaSuccess) rc = RG_CUDA_ERROR;
+        if (rc) g->failed = 1;
+        g->arrived = 0;
+        ++g->gen;
+        g->cv.notify_all();
+        return rc;
+    }
+    if (!g->cv.wait_for(lk, seconds(120), [&] { return g->gen != my; })) {
+        g->failed = 1;   // a peer rank never arrived (it returned early with an error)
+        g->cv.notify_all();
+        return RG_NCCL_ERROR;
+    }
+    if (g->failed) return RG_NCCL_ERROR;
+    return cudaStreamWaitEvent(slot.st, g->done, 0) == cudaSuccess ? RG_OK : RG_CUDA_ERROR;
+}
+
 struct rg_handle_s {
     int device = 0;
     cudaStream_t stream = nullptr;
     cudaStream_t capture_stream = nullptr;  // private stream used only to capture plans into graphs
     cudaStream_t cs_in = nullptr, cs_out = nullptr;   // host-pointer pipeline copy streams (lazy)
     std::vector<cudaEvent_t> pipe_ev;               // [0] progress, [1] start, [2] end, [3..] H2D chunks
-    ncclComm_t comm = nullptr;
+    ncclComm_t comm = nullptr;       // NCCL communicator (row-sharded mode)
+    bool own_comm = false;           // created by rg_comm_init (destroyed with the handle)
+    VGroup* vgroup = nullptr;        // in-process virtual ranks (rg_set_vcomm)
+    bool dist() const { return nranks > 1 && (comm || vgroup); }
     int rank = 0, nranks = 1;
     int64_t last_info = -1;
     // workspace
@@ -195,6 +337,20 @@ struct rg_handle_s {
     const void* cgls_key[4] = {nullptr, nullptr, nullptr, nullptr};
     int64_t cgls_key_mn[3] = {0, 0, 0};
     DevBuf aux;                                     // misc (orthogonalize / lowrank)
+    DevBuf vscratch;                                // virtual-rank collectives (rank 0 of a group)
+    int alloc_epoch = 0;                            // bumped whenever a workspace buffer moves
+    std::vector<DevBuf*> bufs() {
+        return {&qh, &ql, &P, &r12h, &r12l, &r12f, &partial, &norm2, &scale, &status, &pws, &pcnt,
+                &rgather, &rstackq, &stageA, &stageQ, &stageR, &stageB, &stageX, &cg, &aux, &lsQ, &lsR, &rinv,
+                &probeG, &probeW, &cq_ws, &cq_flags, &leaf_bar, &lrA16, &lrB16, &lrB16l, &lrY, &lrZ, &lrQ16,
+                &lrQ16l, &lrR, &lrW, &lrV, &lrUb, &lrVb, &lrSig, &lrOm, &lrScale, &lrFlags, &vscratch};
+    }
+    void bind_bufs() {
+        for (DevBuf* b : bufs()) {
+            b->epoch = &alloc_epoch;
+            b->stream = &stream;
+        }
+    }
     int* status_host = nullptr;                     // pinned
     long long last_launches = 0;                    // kernels launched by the last API call
     long long call_g0 = 0;                          // rg::g_launches at the start of the call
@@ -362,7 +518,7 @@ int make_plan(rg_handle h, Plan& pl) {
     const bool wide = getenv("RGSQR_WIDE") != nullptr;
     // (split-precision passes keep the tensor-core K1/K2 at the last level: the leaf kernel's
     // mma.sync K1/K2 are single 16-bit products)
-    const bool pair = pl.panel == 0 && pl.nb == 32 && !(pl.nranks > 1 && h->comm) &&
+    const bool pair = pl.panel == 0 && pl.nb == 32 && !(pl.nranks > 1 && h->dist()) &&
                       (wide ? rg::cholqr_fused_fits(m, 64) : (rg::leaf_fits(m) && !pl.split));
     pl.leaf = pair && !wide;
     build_ops(pl.ops, 0, n, pl.nb, pair, pl.leaf);
@@ -475,9 +631,36 @@ bool ensure_workspace(rg_handle h, int64_t m, int64_t n, int split) {
     return ok;
 }
 
+// in-place sum over the ranks (no-op on one rank)
 int nccl_allreduce(rg_handle h, void* buf, size_t count, ncclDataType_t t) {
-    if (h->nranks <= 1 || !h->comm) return RG_OK;
+    if (!h->dist()) return RG_OK;
+    if (h->vgroup) {
+        VGroup::Slot sl;
+        sl.send = buf;
+        sl.recv = buf;
+        sl.count = count;
+        sl.kind = 0;
+        sl.f64 = t == ncclFloat64;
+        sl.st = h->stream;
+        return vgroup_collective(h->vgroup, h->rank, sl);
+    }
     if (g_nccl.AllReduce(buf, buf, count, t, ncclSum, h->comm, h->stream) != ncclSuccess) return RG_NCCL_ERROR;
+    return RG_OK;
+}
+
+// recv[r * count ..] = rank r's send (count elements each, fp32)
+int coll_allgather_f32(rg_handle h, const float* send, float* recv, size_t count) {
+    if (h->vgroup) {
+        VGroup::Slot sl;
+        sl.send = send;
+        sl.recv = recv;
+        sl.count = count;
+        sl.kind = 1;
+        sl.f64 = 0;
+        sl.st = h->stream;
+        return vgroup_collective(h->vgroup, h->rank, sl);
+    }
+    if (g_nccl.AllGather(send, recv, count, ncclFloat32, h->comm, h->stream) != ncclSuccess) return RG_NCCL_ERROR;
     return RG_OK;
 }
 
@@ -496,7 +679,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     uint16_t* qh = h->qh.as<uint16_t>();
     uint16_t* ql = pl.split ? h->ql.as<uint16_t>() : nullptr;
     int* status = h->status.as<int>();
-    const bool dist = pl.nranks > 1 && h->comm;
+    const bool dist = pl.nranks > 1 && h->dist();
     HostPipe* pp = pl.pipe;
     // section 3.5 on columns [c, c + nc): norms, power-of-two scales, scaled fp32 + 16-bit images
     auto scale_cols = [&](int c, int nc) -> int {
@@ -697,8 +880,8 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
                 p.ldr = o.w;
                 p.distributed = 1;
                 RG_CUDA(rg::launch_panel(p, st));
-                if (g_nccl.AllGather(p.R, rg_all, (size_t)o.w * o.w, ncclFloat32, h->comm, st) != ncclSuccess)
-                    return RG_NCCL_ERROR;
+                int rc = coll_allgather_f32(h, p.R, rg_all, (size_t)o.w * o.w);
+                if (rc) return rc;
                 float* qb = h->rstackq.as<float>();
                 RG_CUDA(rg::launch_panel_stack(rg_all, h->nranks, o.w, Rdiag, pl.ldr, qb, status, o.c0, p.guard, st));
                 RG_CUDA(rg::launch_panel_apply(p, qb + (int64_t)h->rank * 32 * 32, st));
@@ -789,7 +972,7 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
         if (c->m == m && c->n == n && c->lda == lda && c->ldq == ldq && c->ldr == ldr && c->A == A && c->Q == Q &&
             c->R == R && c->nb == nb && c->bf16 == o.precision && c->split == split && c->scale == o.scale &&
             c->nranks == nranks && c->rank == h->rank && c->panel == o.panel) {
-            if (c->epoch != g_alloc_epoch) {   // a workspace buffer moved: rebuild this plan
+            if (c->epoch != h->alloc_epoch) {   // a workspace buffer moved: rebuild this plan
                 if (c->exec) cudaGraphExecDestroy(c->exec);
                 h->plans.erase(h->plans.begin() + i);
                 break;
@@ -808,10 +991,10 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
         int rc = make_plan(h, *np);
         if (rc) return rc;
         if (!h->P.ensure(np->p_floats * 4 + 4096)) return RG_ALLOC;
-        np->epoch = g_alloc_epoch;
+        np->epoch = h->alloc_epoch;
         // invalidate older plans if P just moved (their graphs captured the old pointer)
         for (auto& c : h->plans)
-            if (c->epoch != g_alloc_epoch && c->exec) {
+            if (c->epoch != h->alloc_epoch && c->exec) {
                 cudaGraphExecDestroy(c->exec);
                 c->exec = nullptr;
             }
@@ -832,7 +1015,7 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
         pl->launches = graph_launches;
         return rc;
     }
-    const bool use_graph = !h->prof && getenv("RGSQR_NO_GRAPH") == nullptr;
+    const bool use_graph = !h->prof && !h->vgroup && getenv("RGSQR_NO_GRAPH") == nullptr;
     if (!use_graph) return enqueue_rgsqr(h, *pl);
     if (!pl->exec) {
         // capture on the private stream (the user's may be the legacy stream, which cannot
@@ -1011,6 +1194,43 @@ bool pdl_enabled() {   // opt-in: measured slower than plain graph edges for thi
     static const bool on = getenv("RGSQR_PDL") != nullptr;
     return on;
 }
+
+namespace {
+std::mutex g_dev_mu;
+std::map<int, std::pair<int, int>> g_dev_props;               // device -> (SMs, opt-in smem)
+std::map<std::pair<int, const void*>, size_t> g_smem_attr;    // (device, kernel) -> bytes set
+int cur_device() {
+    int d = 0;
+    cudaGetDevice(&d);
+    return d;
+}
+std::pair<int, int> dev_props() {
+    const int d = cur_device();
+    std::lock_guard<std::mutex> lk(g_dev_mu);
+    auto it = g_dev_props.find(d);
+    if (it != g_dev_props.end()) return it->second;
+    int sms = 0, smem = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, d);
+    cudaDeviceGetAttribute(&smem, cudaDevAttrMaxSharedMemoryPerBlockOptin, d);
+    if (sms <= 0) sms = 148;
+    if (smem <= 0) smem = 227 * 1024;
+    g_dev_props[d] = {sms, smem};
+    return {sms, smem};
+}
+}  // namespace
+
+int dev_sms() { return dev_props().first; }
+int dev_smem_optin() { return dev_props().second; }
+
+cudaError_t ensure_smem_attr(const void* kernel, size_t bytes) {
+    const int d = cur_device();
+    std::lock_guard<std::mutex> lk(g_dev_mu);
+    size_t& cur = g_smem_attr[{d, kernel}];
+    if (bytes <= cur) return cudaSuccess;
+    cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+    if (e == cudaSuccess) cur = bytes;
+    return e;
+}
 }
 
 // ====================================================================== C-ABI
@@ -1058,6 +1278,7 @@ int rg_create(rg_handle* out, int device, void* stream) {
     rg_handle h = new rg_handle_s();
     h->device = device;
     h->stream = reinterpret_cast<cudaStream_t>(stream);
+    h->bind_bufs();
     if (cudaMallocHost(&h->status_host, 64) != cudaSuccess) {
         delete h;
         return RG_ALLOC;
@@ -1082,26 +1303,21 @@ int rg_set_stream(rg_handle h, void* stream) {
     return RG_OK;
 }
 
+static void detach_comm(rg_handle h);
+
 int rg_destroy(rg_handle h) {
     if (!h) return -1;
     cudaSetDevice(h->device);
     cudaStreamSynchronize(h->stream);
     for (auto& p : h->plans)
         if (p->exec) cudaGraphExecDestroy(p->exec);
-    DevBuf* bufs[] = {&h->qh, &h->ql, &h->P, &h->r12h, &h->r12l, &h->r12f, &h->partial, &h->norm2, &h->scale,
-                      &h->status, &h->pws, &h->pcnt, &h->rgather, &h->rstackq, &h->stageA, &h->stageQ,
-                      &h->stageR, &h->stageB, &h->stageX, &h->cg, &h->aux,
-                      &h->lsQ, &h->lsR, &h->rinv, &h->probeG, &h->probeW, &h->cq_ws, &h->lrA16, &h->lrB16, &h->lrB16l, &h->lrY,
-                      &h->lrZ, &h->lrQ16, &h->lrQ16l, &h->lrR, &h->lrW, &h->lrV, &h->lrUb, &h->lrVb, &h->lrSig,
-                      &h->lrOm, &h->lrScale, &h->lrFlags,
-                      &h->cq_flags};
     if (h->cgls_exec) cudaGraphExecDestroy(h->cgls_exec);
-    for (auto* b : bufs) b->release();
+    for (DevBuf* b : h->bufs()) b->release();
     for (auto& e : h->ev_pool) {
         cudaEventDestroy(e.first);
         cudaEventDestroy(e.second);
     }
-    if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
+    detach_comm(h);
     if (h->status_host) cudaFreeHost(h->status_host);
     if (h->capture_stream) cudaStreamDestroy(h->capture_stream);
     if (h->cs_in) cudaStreamDestroy(h->cs_in);
@@ -1141,10 +1357,33 @@ int rg_comm_unique_id(void* id128) {
     return RG_OK;
 }
 
+// drop every cached plan / graph (their collectives and split decisions depend on the mode)
+static void reset_plans(rg_handle h) {
+    for (auto& p : h->plans)
+        if (p->exec) cudaGraphExecDestroy(p->exec);
+    h->plans.clear();
+    if (h->cgls_exec) cudaGraphExecDestroy(h->cgls_exec);
+    h->cgls_exec = nullptr;
+    h->cgls_key[0] = nullptr;
+}
+
+static void detach_comm(rg_handle h) {
+    if (h->comm && h->own_comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
+    h->comm = nullptr;
+    h->own_comm = false;
+    if (h->vgroup) {
+        std::lock_guard<std::mutex> lk(h->vgroup->mu);
+        --h->vgroup->attached;
+    }
+    h->vgroup = nullptr;
+    h->rank = 0;
+    h->nranks = 1;
+}
+
 int rg_comm_init(rg_handle h, const void* id128, int rank, int nranks) {
     if (!h) return -1;
     if (!id128) return -2;
-    if (nranks < 1 || nranks > 64) return -4;
+    if (nranks < 1 || nranks > RG_MAX_RANKS) return -4;
     if (rank < 0 || rank >= nranks) return -3;
     if (!g_nccl.lib && rg_nccl_load(nullptr) != RG_OK) return RG_NCCL_ERROR;
     ncclUniqueId id;
@@ -1152,13 +1391,98 @@ int rg_comm_init(rg_handle h, const void* id128, int rank, int nranks) {
     cudaSetDevice(h->device);
     ncclComm_t c = nullptr;
     if (g_nccl.CommInitRank(&c, nranks, id, rank) != ncclSuccess) return RG_NCCL_ERROR;
-    if (h->comm && g_nccl.CommDestroy) g_nccl.CommDestroy(h->comm);
+    detach_comm(h);
     h->comm = c;
+    h->own_comm = true;
     h->rank = rank;
     h->nranks = nranks;
-    for (auto& p : h->plans)
-        if (p->exec) cudaGraphExecDestroy(p->exec);
-    h->plans.clear();
+    reset_plans(h);
+    return RG_OK;
+}
+
+int rg_set_comm(rg_handle h, void* nccl_comm, int rank, int nranks) {
+    if (!h) return -1;
+    if (nccl_comm && (nranks < 1 || nranks > RG_MAX_RANKS)) return -4;
+    if (nccl_comm && (rank < 0 || rank >= nranks)) return -3;
+    if (nccl_comm && !g_nccl.lib && rg_nccl_load(nullptr) != RG_OK) return RG_NCCL_ERROR;
+    detach_comm(h);
+    if (nccl_comm) {
+        h->comm = reinterpret_cast<ncclComm_t>(nccl_comm);
+        h->own_comm = false;
+        h->rank = rank;
+        h->nranks = nranks;
+    }
+    reset_plans(h);
+    return RG_OK;
+}
+
+int rg_vgroup_create(void** group, int nranks) {
+    if (!group) return -1;
+    *group = nullptr;
+    if (nranks < 1 || nranks > RG_MAX_RANKS) return -2;
+    VGroup* g = new VGroup();
+    g->P = nranks;
+    g->slots.resize(nranks);
+    g->ready.resize(nranks, nullptr);
+    for (int r = 0; r < nranks; ++r)
+        if (cudaEventCreateWithFlags(&g->ready[r], cudaEventDisableTiming) != cudaSuccess) return RG_CUDA_ERROR;
+    if (cudaEventCreateWithFlags(&g->done, cudaEventDisableTiming) != cudaSuccess) return RG_CUDA_ERROR;
+    if (cudaMalloc(&g->dptrs, sizeof(void*) * RG_MAX_RANKS) != cudaSuccess) return RG_ALLOC;
+    cudaGetDevice(&g->device);
+    *group = g;
+    return RG_OK;
+}
+
+int rg_vgroup_destroy(void* group) {
+    VGroup* g = reinterpret_cast<VGroup*>(group);
+    if (!g) return -1;
+    {
+        std::lock_guard<std::mutex> lk(g->mu);
+        if (g->attached > 0) return -1;   // detach (rg_set_vcomm(h, NULL, 0) / rg_destroy) first
+    }
+    cudaDeviceSynchronize();
+    for (auto e : g->ready) cudaEventDestroy(e);
+    cudaEventDestroy(g->done);
+    if (g->scratch) cudaFree(g->scratch);
+    if (g->dptrs) cudaFree(g->dptrs);
+    delete g;
+    return RG_OK;
+}
+
+int rg_set_vcomm(rg_handle h, void* group, int rank) {
+    if (!h) return -1;
+    VGroup* g = reinterpret_cast<VGroup*>(group);
+    if (g && (rank < 0 || rank >= g->P)) return -3;
+    if (g && g->device != h->device) return -2;
+    detach_comm(h);
+    if (g) {
+        std::lock_guard<std::mutex> lk(g->mu);
+        ++g->attached;
+        h->vgroup = g;
+        h->rank = rank;
+        h->nranks = g->P;
+    }
+    reset_plans(h);
+    return RG_OK;
+}
+
+int rg_debug_gaussian(rg_handle h, int64_t n, uint64_t seed, double* out) {
+    if (!h) return -1;
+    if (n < 0) return -2;
+    if (!out || ptr_side(out) != SIDE_DEVICE) return -4;
+    cudaSetDevice(h->device);
+    RG_CUDA(rg::launch_gaussian_philox(n, seed, out, nullptr, h->stream));
+    RG_CUDA(cudaStreamSynchronize(h->stream));
+    return RG_OK;
+}
+
+int rg_debug_philox(rg_handle h, int64_t ncalls, uint64_t seed, uint32_t* words) {
+    if (!h) return -1;
+    if (ncalls < 0) return -2;
+    if (!words || ptr_side(words) != SIDE_DEVICE) return -4;
+    cudaSetDevice(h->device);
+    RG_CUDA(rg::launch_philox_words(ncalls, seed, words, h->stream));
+    RG_CUDA(cudaStreamSynchronize(h->stream));
     return RG_OK;
 }
 
@@ -1448,7 +1772,7 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     const int blk = 8;
     int done_iters = 0;
     double hsc[16];
-    const bool use_graph = !h->prof && getenv("RGSQR_NO_GRAPH") == nullptr;
+    const bool use_graph = !h->prof && !h->vgroup && getenv("RGSQR_NO_GRAPH") == nullptr;
     while (done_iters < maxit) {
         const int cnt = std::min(blk, maxit - done_iters);
         if (use_graph && cnt == blk) {
@@ -1570,7 +1894,7 @@ int lowrank_approx(rg_handle h, int64_t m_local, int64_t n, const float* A, int6
     if (rc) return rc;
     // ---- power-of-two column scaling of A into fp16 range (section 3.5): A16 = fp16(A P)
     RG_CUDA(rg::launch_colnorm(dA, dlda, m_local, (int)n, h->partial.as<double>(), h->norm2.as<double>(), st));
-    if (h->nranks > 1 && h->comm) {
+    if (h->dist()) {
         rc = nccl_allreduce(h, h->norm2.p, n, ncclFloat64);
         if (rc) return rc;
     }
@@ -1589,7 +1913,7 @@ int lowrank_approx(rg_handle h, int64_t m_local, int64_t n, const float* A, int6
         int r2 = gemm_tn(h, m_local, (int)n, l, A16, ldm16, h->qh.as<uint16_t>(), round_up(std::max<int64_t>(m_local, 8), 8),
                          out, n, bf);
         if (r2) return r2;
-        if (h->nranks > 1 && h->comm) {
+        if (h->dist()) {
             r2 = nccl_allreduce(h, out, (size_t)n * l, ncclFloat32);
             if (r2) return r2;
         }

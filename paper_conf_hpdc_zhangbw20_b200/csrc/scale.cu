@@ -87,7 +87,12 @@ __global__ void colscale_kernel(const double* __restrict__ norm2, int n, int do_
     if (do_scale && s > 0.0 && isfinite(s)) {
         int e;
         frexp(sqrt(s), &e);              // ||a_j|| = frac * 2^e, frac in [0.5, 1)
-        f = ldexpf(1.0f, 9 - e);         // scaled norm in [256, 512)
+        // scaled norm in [256, 512); the exponent is clamped to normal fp32 powers of two
+        // (2^-126 .. 2^127) so the scale stays exact and finite: a column with a norm below
+        // 2^-118 or above 2^135 is scaled as far as an exact power of two allows (a finite fp32
+        // column norm is below 2^136, so only the tiny end can be left short of the target)
+        const int ex = min(127, max(-126, 9 - e));
+        f = ldexpf(1.0f, ex);
     }
     scale[j] = f;
 }

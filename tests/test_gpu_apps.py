@@ -58,18 +58,25 @@ def test_ls_host_pointers(rg):
 
 
 def test_ls_paper_faithful_mode_converges(rg):
-    """reortho = 0 (paper-faithful, one RGSQR pass) and reortho = 1 both converge to the LS
-    solution (Alg 3); the one-pass R is a usable preconditioner even though its Q is far from
-    orthogonal at kappa = 1e4."""
+    """Paper-faithful preconditioner (reortho = 0 and the paper's fp32 TSQR/MGS panel, eq 8 +
+    Alg 2; reading #8) against the default (one reortho pass, CholQR2 panels): both reach the
+    LS solution (Alg 3), and the reorthogonalised R needs no more CGLS iterations than the
+    one-pass R (the one-pass preconditioner is what makes the paper's kappa = 1e4
+    geometric case slow)."""
     A = synth.svd_matrix(8192, 128, "geometric", 1e4, seed=5).astype(np.float32)
     b = synth.rhs(A.astype(np.float64), seed=5, consistent=True).astype(np.float32)
     x_star, _ = oracle.ls_qr(A.astype(np.float64), b.astype(np.float64))
-    for reo in (0, 1):
-        x, it, _, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), opts=rg.make_opts(reortho=reo),
-                                           maxit=400)
-        assert st == rg.RG_OK and it < 100, (reo, it, st)
+    iters = {}
+    for name, o in (("faithful", rg.make_opts(reortho=0, panel="mgs")), ("one-pass", rg.make_opts(reortho=0)),
+                    ("reortho", rg.make_opts(reortho=1))):
+        x, it, _, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), opts=o, maxit=400)
+        assert st == rg.RG_OK, (name, it, st)
         xv = x.cpu().numpy()
-        assert np.linalg.norm(xv - x_star) / np.linalg.norm(x_star) <= 1e-5
+        assert np.linalg.norm(xv - x_star) / np.linalg.norm(x_star) <= 1e-5, name
+        iters[name] = it
+    assert iters["reortho"] <= iters["faithful"], iters
+    assert iters["reortho"] <= iters["one-pass"], iters
+    assert iters["reortho"] <= 30, iters
 
 
 @pytest.mark.parametrize("kappa", [1.0, 1e3, 1e4])

@@ -34,6 +34,13 @@ def _run(rg, A32, **kw):
 
 
 def _check_qr(A32, Q, R, kappa=10.0, orth_scale=1e-2):
+    """Identities and distance to the UNIQUE factors Q*, R* of the oracle's Householder QR
+    (positive diagonal).  Tolerance (reading #25): the computed pair is the exact QR
+    U (T R) of A - dA with Q = U T, T^T T = Q^T Q = I - E, so to first order
+        ||R - R*||_F / ||R*||_F <= sqrt(2) kappa be + ||E||_F / sqrt(2),
+        ||Q - Q*||_F / ||Q*||_F <= (1 + sqrt(2)) kappa be + ||E||_F / sqrt(2 n)
+    (Sun's perturbation bounds of the QR factors; be = ||dA||_F / ||A||_F); the tests use
+    10 kappa be + orth and 10 kappa be + orth / sqrt(n)."""
     A = np.asarray(A32, dtype=np.float64)
     m, n = A.shape
     assert np.all(np.isfinite(Q)) and np.all(np.isfinite(R))
@@ -45,10 +52,9 @@ def _check_qr(A32, Q, R, kappa=10.0, orth_scale=1e-2):
     assert orth <= orth_scale * np.sqrt(n), orth
     Qo, Ro, _ = oracle.householder(A)
     dr = np.linalg.norm(R - Ro) / np.linalg.norm(Ro)
-    # first-order perturbation of the unique R: kappa(A) times (backward error + loss of
-    # orthogonality); the 16-bit K1 rounding shows up in orth, not in be, when the update that
-    # follows it is done in fp32 (leaf-level K2 folded into the panel)
-    assert dr <= max(10 * kappa * (be + orth / np.sqrt(n)), 1e-5), (dr, be, orth)
+    dq = np.linalg.norm(Q - Qo) / np.linalg.norm(Qo)
+    assert dr <= 10 * kappa * be + orth + 1e-6, (dr, be, orth, kappa)
+    assert dq <= 10 * kappa * be + orth / np.sqrt(n) + 1e-6, (dq, be, orth, kappa)
     return be, orth, dr
 
 
@@ -63,12 +69,25 @@ def test_rgsqr_gaussian_parity(rg, m, n, panel):
 
 @pytest.mark.parametrize("kappa", [1e2, 1e4, 1e6])
 def test_rgsqr_ill_conditioned_backward_error(rg, kappa):
-    """Backward error independent of cond(A) (Fig 3); orthogonality grows ~kappa u_h."""
+    """Backward error independent of cond(A) (Fig 3); orthogonality grows ~kappa u_h.
+    The distance to the unique factors is checked where its first-order bound (reading #25) is
+    informative (kappa be < 0.05, i.e. kappa = 1e2 here); beyond that the QR factors of A are
+    not determined to working accuracy by any 16-bit-update method and only be is meaningful."""
     A = synth.svd_matrix(4096, 128, "geometric", kappa, seed=21).astype(np.float32)
     Q, R = _run(rg, A)
     A64 = A.astype(np.float64)
-    assert oracle.backward_error(A64, Q, R) < 5e-3
-    assert np.all(np.diag(R) > 0)
+    be = oracle.backward_error(A64, Q, R)
+    assert be < 5e-3
+    assert np.all(np.diag(R) > 0) and np.all(np.tril(R, -1) == 0)
+    if kappa * be < 0.05:
+        _check_qr(A, Q, R, kappa=kappa, orth_scale=1.0)
+    else:
+        # the leading columns are well conditioned: their block of R is still pinned
+        k = 16
+        Ak = A64[:, :k]
+        _, Rk, _ = oracle.householder(Ak)
+        kk = np.linalg.cond(Ak)
+        assert np.linalg.norm(R[:k, :k] - Rk) / np.linalg.norm(Rk) <= 10 * kk * be + 1e-2
 
 
 @pytest.mark.parametrize("kappa", [10.0, 1e5])
@@ -325,4 +344,4 @@ def test_rgsqr_pinned_host_options(rg, kw):
     np.testing.assert_array_equal(Qh.numpy(), Qd.cpu().numpy())
     np.testing.assert_array_equal(Rh.numpy(), Rd.cpu().numpy())
     _check_qr(A, Qh.numpy().astype(np.float64), Rh.numpy().astype(np.float64), kappa=np.linalg.cond(A),
-              orth_scale=1.0 if kw.get("precision") == "bf16" or kw.get("scale") is False else 1e-2)
+              orth_scale=5e-2 if kw.get("precision") == "bf16" or kw.get("scale") is False else 1e-2)

@@ -285,3 +285,25 @@ def test_generator_spectra():
     for kind in ("geometric", "arithmetic", "cluster"):
         A = synth.svd_matrix(200, 20, kind, 1e4, seed=1)
         np.testing.assert_allclose(np.linalg.svd(A, compute_uv=False), synth.sigma(20, kind, 1e4), rtol=1e-12)
+
+
+def test_gaussian_philox_box_muller_mapping():
+    """The word -> Gaussian mapping of the sketch stream (reading #17) pinned
+    against the KAT-pinned Philox words: element e takes call e >> 1 with counter
+    {e >> 1, 0, 0, 0} and key {seed lo, seed hi}; even e uses words (0, 1), odd e words (2, 3);
+    u1 = (w_a + 1) 2^-32 in (0, 1], u2 = w_b 2^-32, z = sqrt(-2 ln u1) cos(2 pi u2).  A swapped
+    word pair, a dropped +1 (ln 0 at w_a = 0), a column-major / row-major mix-up of the (rows x
+    cols) fill or a 2^-31 scale all fail here."""
+    seed = 0x1234_5678_9ABC_DEF0
+    rows, cols = 37, 3
+    Z = oracle.gaussian_philox(rows, cols, seed)
+    flat = Z.reshape(-1, order="F")
+    for e in range(rows * cols):
+        w = oracle.philox4x32_10([e >> 1, 0, 0, 0], [seed & 0xFFFFFFFF, seed >> 32])
+        a, b = (w[0], w[1]) if e % 2 == 0 else (w[2], w[3])
+        u1 = (a + 1.0) * 2.0 ** -32
+        u2 = b * 2.0 ** -32
+        z = np.sqrt(-2.0 * np.log(u1)) * np.cos(2.0 * np.pi * u2)
+        assert abs(flat[e] - z) <= 4e-16 * max(1.0, abs(z)), (e, flat[e], z)
+    # the stream does not depend on the shape it is read into (element index = e)
+    np.testing.assert_array_equal(oracle.gaussian_philox(rows * cols, 1, seed)[:, 0], flat)
