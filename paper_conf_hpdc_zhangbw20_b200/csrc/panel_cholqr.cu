@@ -1240,7 +1240,10 @@ __global__ void cq_factor_kernel(CqArgs a, int pass) {
     RG_PDL_ENTRY();
     __shared__ __align__(16) double Rs[32 * CH_LD];
     __shared__ __align__(16) double R1s[32 * CH_LD];
-    if (pass > 0 && *(volatile int*)a.ws.fail) return;
+    // pass 1 runs only for two-pass panels: a single-pass panel (ws.fail[1], decided after pass
+    // 0) has already written Q and R, and its second Gram was never formed (the host allreduce
+    // of that slot is issued regardless and carries stale data)
+    if (pass > 0 && (*(volatile int*)a.ws.fail || *(volatile int*)(a.ws.fail + 1))) return;
     const bool ok = chol_inv_cta<256, false>(a.ws.G + pass * 1024, a.nc, Rs, R1s, a.ws.R + pass * 1024,
                                              a.ws.Rinv + pass * 1024, false);
     if (!ok && threadIdx.x == 0) cq_signal_fail(a);
