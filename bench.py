@@ -161,6 +161,8 @@ def main():
     ap.add_argument("--no-lowrank", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--comm", default="own", choices=["own", "torch"],
+                    help="N > 1: the library's own NCCL communicator or torch's (rg_set_comm)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "ours" else args.warmup
     ws, rank, local = dist_env()
@@ -178,8 +180,14 @@ def main():
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     h = rg.Handle(local)
+    comm = None
     if ws > 1:
-        h.init_comm(rank, ws)
+        if args.comm == "torch":
+            h.attach_torch_comm()           # rg_set_comm on torch's ProcessGroupNCCL communicator
+            comm = "torch ProcessGroupNCCL communicator (rg_set_comm)"
+        else:
+            h.init_comm(rank, ws)           # the library's own NCCL communicator (rg_comm_init)
+            comm = "library NCCL communicator (rg_comm_init)"
 
     m_global = M * ws
     # synthetic input: N(0,1) fp32 drawn on the device (seeded per rank; > L2 so no flush needed)
@@ -340,7 +348,7 @@ def main():
             "config": {"workload": f"RGSQR {m_global}x{N} fp32 N(0,1), fp16 tensor-core updates (BASELINE config 2"
                                    f"{'' if ws == 1 else ', row-sharded ' + str(M) + ' rows per GPU'})",
                        "m": m_global, "n": N, "nb": 32, "l2": "inputs (1 GiB per GPU) larger than L2, no flush",
-                       "parallelism": f"row-sharded x{ws}" if ws > 1 else "single GPU"},
+                       "parallelism": f"row-sharded x{ws}" if ws > 1 else "single GPU", "comm": comm},
             "frac_of_spec_2250": tflops / 2250.0,
             "frac_of_measured_matmul": tflops / pk["bf16_tflops"],
             "accuracy": acc,

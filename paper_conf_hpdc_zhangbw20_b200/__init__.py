@@ -237,6 +237,24 @@ class Handle:
                                                  int(nranks)), self)
         self.rank, self.nranks = (rank, nranks) if nccl_comm_ptr else (0, 1)
 
+    def attach_torch_comm(self, group=None):
+        """Row-sharded mode on torch.distributed's own NCCL communicator (ProcessGroupNCCL of
+        `group`, default the world) through rg_set_comm: no second communicator.  torch loads
+        libnccl dynamically from nvidia/nccl/lib; the library dlopens the same file, so the
+        ncclComm_t is valid for its calls.  Collectives of torch and of the library on this
+        communicator must not overlap in time (synchronise between them)."""
+        import torch
+        import torch.distributed as dist
+        pg = group or dist.distributed_c10d._get_default_group()
+        backend = pg._get_backend(torch.device("cuda", self.device))
+        dist.barrier(group=pg)          # the communicator exists once a collective has run
+        torch.cuda.synchronize(self.device)
+        path = _find_nccl()
+        st = _lib().rg_nccl_load(path.encode() if path else None)
+        if st != RG_OK:
+            raise RGError("rg_nccl_load", st)
+        self.set_comm(backend._comm_ptr(), dist.get_rank(pg), dist.get_world_size(pg))
+
     def set_vcomm(self, group, rank: int):
         """Attach to an in-process virtual-rank group (VGroup); None detaches."""
         _check("rg_set_vcomm", _lib().rg_set_vcomm(self._h, group.ptr if group is not None else None, int(rank)),
