@@ -73,11 +73,17 @@ struct LeafArgs {
     // prologue (Algorithm 1 lines 8-9 of the level above, folded in): R_AB = Q_A^T P, P -= Q_A R_AB
     const uint16_t* pq;  // Q_A, 16-bit image (ld ldh), m x ph; null: no prologue
     int ph;              // columns of Q_A (<= 64)
+    int fast;            // first Gram on the 16-bit tensor cores (split fp16, see lf_gram16)
 };
 
 #ifdef LF_TRACE
 __device__ unsigned long long lf_trace[32];
 __device__ long long lf_clk[2];
+__device__ int lf_count[4];   // [0] fast-Gram fallbacks, [1] passes
+#define LF_COUNT(i, v)                                              \
+    do {                                                            \
+        if (blockIdx.x == 0 && threadIdx.x == 0) lf_count[i] += v;  \
+    } while (0)
 #define LF_MARK(i)                                                                     \
     do {                                                                               \
         if (blockIdx.x == 0 && threadIdx.x == 0) {                                     \
@@ -87,6 +93,9 @@ __device__ long long lf_clk[2];
         }                                                                              \
     } while (0)
 #else
+#define LF_COUNT(i, v) \
+    do {               \
+    } while (0)
 #define LF_MARK(i) \
     do {           \
     } while (0)
@@ -193,8 +202,10 @@ struct LfSmem {
     float* rdiag32;   // 64
     uint16_t* RABh;   // 64 x LF_ABLD: -R_AB as the prologue K2 B operand, [n][k]
     int* flag;        // 8 ints
+    float* dsc;       // 64: 1 / (power-of-two column scale of X) in the tensor-core apply
+    uint4* xfrag;     // 32 (k-step, n-tile) x 32 lanes: split fp16 B fragments of X = R^-1 (16 KB)
     static constexpr size_t fixed_bytes() {
-        return 2 * LF_REGION + 2 * 64 * 8 + 64 * 8 + 64 * 8 + 64 * 4 + 64 * LF_ABLD * 2 + 64;
+        return 2 * LF_REGION + 2 * 64 * 8 + 64 * 8 + 64 * 8 + 64 * 4 + 64 * LF_ABLD * 2 + 64 + 64 * 4 + 16384;
     }
     __device__ LfSmem(uint8_t* base, int ldt) {
         tile = reinterpret_cast<float*>(base);
@@ -219,6 +230,10 @@ struct LfSmem {
         RABh = reinterpret_cast<uint16_t*>(p);
         p += 64 * LF_ABLD * 2;
         flag = reinterpret_cast<int*>(p);
+        p += 64;
+        dsc = reinterpret_cast<float*>(p);
+        p += 64 * 4;
+        xfrag = reinterpret_cast<uint4*>(p);
     }
 };
 static_assert(LF_NENT * 8 <= LF_REGION && LF_NE * 8 <= LF_REGION, "region A");
@@ -387,6 +402,123 @@ __device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int rp) {
     }
 }
 
+// ------------------------------------------------------------------ Gram (16-bit tensor cores)
+// G = P^T P from a two-term fp16 split of every entry x: hi = fp16(x), lo = fp16((x - hi) 2^11),
+// x_i x_j = hi_i hi_j + 2^-11 (hi_i lo_j + lo_i hi_j) + O(2^-22 |x_i x_j|) -- three products on
+// mma.sync m16n8k16 with fp32 accumulation (1024 FMA/clk/SM measured vs 64 for the fp64 DMMA of
+// lf_gram).  The entries are the column-scaled (section 3.5, reading #4) and projected block:
+// |x| <= 512, so nothing overflows fp16; a column whose norm has dropped below 0.01 (entries near
+// the fp16 subnormal range) or any non-finite value sends the pass back to the fp64 Gram
+// (lf_cholqr).  20 upper 16 x 8 tiles of the 64 x 64 Gram; warp = tile group q (5 tiles) x
+// k-quarter kq; per element v = hh + 2^-11 mx in fp32, the four k-quarters summed in fixed
+// order, stored as fp64 in the packed-upper-triangle partial of lf_gram.  Relative error ~1e-6
+// of |P_i||P_j|: used for a single CholQR pass only when R is well conditioned (lf_cholqr).
+__device__ __forceinline__ void lf_split2(float2 v, uint32_t& hi, uint32_t& lo) {
+    const __half2 h = __floats2half2_rn(v.x, v.y);
+    const float2 hf = __half22float2(h);
+    const __half2 l = __floats2half2_rn((v.x - hf.x) * 2048.f, (v.y - hf.y) * 2048.f);
+    hi = *reinterpret_cast<const uint32_t*>(&h);
+    lo = *reinterpret_cast<const uint32_t*>(&l);
+}
+
+__device__ __forceinline__ void lf_mma_f16(float (&d)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
+                                           uint32_t b0, uint32_t b1) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, {%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+}
+
+// Tile groups (16 x 8 tiles (bi, cb): Gram rows 16 bi.., columns 8 cb..), chosen so that the work
+// per k-step -- 3 mma per tile + one split of every 8-column block a tile touches -- is balanced:
+//   q0: 16x16 blocks (0,0) (0,1) (1,1)  -> 6 tiles, column blocks 0-3
+//   q1: 16x16 blocks (2,2) (2,3) (3,3)  -> 6 tiles, column blocks 4-7
+//   q2: 16x16 blocks (0,2) (0,3)        -> 4 tiles, column blocks 0, 1, 4-7
+//   q3: 16x16 blocks (1,2) (1,3)        -> 4 tiles, column blocks 2-7
+__host__ __device__ constexpr int lf_t16_n(int q) { return q < 2 ? 6 : 4; }
+__host__ __device__ constexpr int lf_t16_bi(int q, int t) {
+    return q == 0 ? (t < 4 ? 0 : 1) : q == 1 ? (t < 4 ? 2 : 3) : q == 2 ? 0 : 1;
+}
+__host__ __device__ constexpr int lf_t16_cb(int q, int t) {
+    return q == 0 ? (t < 4 ? t : t - 2) : q == 1 ? (t < 4 ? 4 + t : t + 2) : 4 + t;
+}
+__host__ __device__ constexpr bool lf_t16_need(int q, int cb) {
+    bool need = false;
+    for (int t = 0; t < lf_t16_n(q); ++t)
+        need |= (lf_t16_cb(q, t) == cb) || (2 * lf_t16_bi(q, t) == cb) || (2 * lf_t16_bi(q, t) + 1 == cb);
+    return need;
+}
+
+constexpr int LF_G16LD = 65;   // dense fp32 64 x 64 per k-quarter in the epilogue (odd: conflict-free)
+
+// Partial Gram of the CTA's rows, group Q of k-quarter kq, written to the dense k-quarter slab.
+template <int Q>
+__device__ __forceinline__ void lf_gram16_group(const LfSmem& s, int ldt, int rp16, int kq, int lane, float* slab) {
+    constexpr int NT = lf_t16_n(Q);
+    const int g = lane >> 2, c = lane & 3;
+    float hh[NT][4], mx[NT][4];
+#pragma unroll
+    for (int t = 0; t < NT; ++t)
+#pragma unroll
+        for (int u = 0; u < 4; ++u) hh[t][u] = mx[t][u] = 0.f;
+#pragma unroll 1
+    for (int k0 = 16 * kq; k0 < rp16; k0 += 64) {
+        uint32_t fh[8][2], fl[8][2];
+#pragma unroll
+        for (int cb = 0; cb < 8; ++cb) {
+            if (!lf_t16_need(Q, cb)) continue;   // compile-time: only the blocks this group's tiles touch
+            const float* col = s.tile + (8 * cb + g) * ldt + k0 + 2 * c;
+            lf_split2(*reinterpret_cast<const float2*>(col), fh[cb][0], fl[cb][0]);
+            lf_split2(*reinterpret_cast<const float2*>(col + 8), fh[cb][1], fl[cb][1]);
+        }
+#pragma unroll
+        for (int t = 0; t < NT; ++t) {
+            const int bi = lf_t16_bi(Q, t), cb = lf_t16_cb(Q, t);
+            const int r0 = 2 * bi, r1 = 2 * bi + 1;
+            lf_mma_f16(hh[t], fh[r0][0], fh[r1][0], fh[r0][1], fh[r1][1], fh[cb][0], fh[cb][1]);
+            lf_mma_f16(mx[t], fh[r0][0], fh[r1][0], fh[r0][1], fh[r1][1], fl[cb][0], fl[cb][1]);
+            lf_mma_f16(mx[t], fl[r0][0], fl[r1][0], fl[r0][1], fl[r1][1], fh[cb][0], fh[cb][1]);
+        }
+    }
+#pragma unroll
+    for (int t = 0; t < NT; ++t) {
+        const int bi = lf_t16_bi(Q, t), cb = lf_t16_cb(Q, t);
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int i = 16 * bi + g + 8 * (u >> 1), j = 8 * cb + 2 * c + (u & 1);
+            slab[i * LF_G16LD + j] = fmaf(mx[t][u], 0x1p-11f, hh[t][u]);
+        }
+    }
+}
+
+__device__ void lf_gram16(const LeafArgs& a, const LfSmem& s, int rp16) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int q = warp & 3, kq = warp >> 2;
+    static_assert(4 * 64 * LF_G16LD * 4 <= 2 * LF_REGION, "scratch");   // regions A + B are adjacent
+    float* slabs = reinterpret_cast<float*>(s.scr);
+    float* slab = slabs + kq * 64 * LF_G16LD;
+    switch (q) {
+        case 0: lf_gram16_group<0>(s, a.ldt, rp16, kq, lane, slab); break;
+        case 1: lf_gram16_group<1>(s, a.ldt, rp16, kq, lane, slab); break;
+        case 2: lf_gram16_group<2>(s, a.ldt, rp16, kq, lane, slab); break;
+        default: lf_gram16_group<3>(s, a.ldt, rp16, kq, lane, slab); break;
+    }
+    LF_MARK(25);
+    __syncthreads();
+    // the four k-quarters in fixed order -> fp64 packed upper triangle of the CTA partial
+    double* out = a.part + (int64_t)blockIdx.x * LF_PART;
+#pragma unroll 2
+    for (int e = threadIdx.x; e < 64 * 64; e += LF_THREADS) {
+        const int i = e >> 6, j = e & 63;
+        if (i <= j) {
+            const int o = i * LF_G16LD + j;
+            constexpr int S = 64 * LF_G16LD;
+            const float sum = ((slabs[o] + slabs[S + o]) + slabs[2 * S + o]) + slabs[3 * S + o];
+            __stcg(out + j * (j + 1) / 2 + i, (double)sum);
+        }
+    }
+}
+
 // ------------------------------------------------------------------ Cholesky (warps 0-3)
 // s.G holds the full symmetric 64 x 64 Gram (identity beyond nc).  Warp q (< 4) keeps the rows
 // i = 4 ii + q (ii < 16; cyclic, so the live rows stay balanced over the four SMSPs as the
@@ -491,9 +623,9 @@ __device__ int lf_chol(const LfSmem& s) {
 //                                    looking: each step one multiply + independent FMAs)
 //   T   = R12 X22,  X12 = -X11 T     all threads, 1024 outputs each
 // Writes s.X32 (row-major) and returns |R|_F^2 |R^{-1}|_F^2 over the nc x nc block (all threads).
-__device__ double lf_inverse(const LfSmem& s, int nc) {
+__device__ double lf_inverse(const LfSmem& s, int nc, double* keq = nullptr) {
     const int tid = threadIdx.x;
-    __shared__ double s_norm[2][LF_NW];
+    __shared__ double s_norm[3][LF_NW];
     if (tid < 64) {
         const int base = tid < 32 ? 0 : 32, j = tid & 31;
         float b[32];
@@ -549,7 +681,7 @@ __device__ double lf_inverse(const LfSmem& s, int nc) {
         tv[q] = -((a4[0] + a4[1]) + (a4[2] + a4[3]));
     }
     __syncthreads();
-    double xn = 0.0, rn = 0.0;
+    double xn = 0.0, rn = 0.0, en = 0.0;
 #pragma unroll
     for (int q = 0; q < 2; ++q) {
         const int e = tid + LF_THREADS * q, i = e >> 5, jj = e & 31;
@@ -563,24 +695,30 @@ __device__ double lf_inverse(const LfSmem& s, int nc) {
             const double x = s.X32[e], r = s.Rs[i * LF_GLD + jj];
             xn = fma(x, x, xn);
             rn = fma(r, r, rn);
+            en = fma(x * x, s.gdiag[i], en);   // (|p_i| X_ij)^2: R^-1 of the column-equilibrated block
         }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         xn += __shfl_xor_sync(0xffffffffu, xn, o);
         rn += __shfl_xor_sync(0xffffffffu, rn, o);
+        en += __shfl_xor_sync(0xffffffffu, en, o);
     }
     if ((tid & 31) == 0) {
         s_norm[0][tid >> 5] = xn;
         s_norm[1][tid >> 5] = rn;
+        s_norm[2][tid >> 5] = en;
     }
     __syncthreads();
-    double sx = 0.0, sr = 0.0;
+    double sx = 0.0, sr = 0.0, se = 0.0;
 #pragma unroll
     for (int w = 0; w < LF_NW; ++w) {
         sx += s_norm[0][w];
         sr += s_norm[1][w];
+        se += s_norm[2][w];
     }
+    // kappa_F^2 of the column-equilibrated block R D^-1 (D = diag |p_j|): |R D^-1|_F^2 = nc
+    if (keq) *keq = (double)nc * se;
     return sx * sr;
 }
 
@@ -631,6 +769,81 @@ __device__ void lf_apply(const LeafArgs& a, const LfSmem& s, int rp) {
     __syncthreads();
 }
 
+// tile rows [0, rp) <- tile * R^{-1} on the 16-bit tensor cores (fast path only): Q = P X with the
+// two-term fp16 split of both operands, Q ~ Ph Xh + 2^-11 (Ph Xl + Pl Xh) (mma.sync m16n8k16, fp32
+// accumulation; relative error ~1e-6 like the split Gram).  X's columns carry power-of-two scales
+// c_j (largest |X_ij c_j| in [2^7, 2^8)), undone exactly on the output.  X is pre-split once into
+// fragment-ordered hi/lo B operands (s.xfrag); warp w owns the 16-row blocks w, w + 16, .. and
+// computes all 64 output columns of them (only the k-steps ks <= nt / 2 the triangle needs), so
+// it reads and overwrites only its own rows: no block-wide barrier inside.
+__device__ void lf_apply16(const LeafArgs& a, const LfSmem& s, int rp16) {
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int g = lane >> 2, c = lane & 3;
+    if (tid < 64) {   // column scales of X (upper triangular: rows 0..j)
+        float mx = 0.f;
+        for (int k = 0; k <= tid; ++k) mx = fmaxf(mx, fabsf(s.X32[k * 64 + tid]));
+        int e = 0;
+        if (mx > 0.f) frexpf(mx, &e);
+        const int ex = min(120, max(-120, 8 - e));
+        s.dsc[tid] = ldexpf(1.f, -ex);                       // 1 / c_j
+        reinterpret_cast<float*>(s.U)[tid] = ldexpf(1.f, ex);   // c_j (scratch)
+    }
+    __syncthreads();
+    const float* cs = reinterpret_cast<const float*>(s.U);
+    for (int e = tid; e < 32 * 32; e += LF_THREADS) {
+        const int pi = e >> 5, ln = e & 31, ks = pi >> 3, nt = pi & 7;
+        const int gg = ln >> 2, cc = ln & 3;
+        const int n = 8 * nt + gg;
+        const float sc = cs[n];
+        const int k0 = 16 * ks + 2 * cc;
+        const float2 v0 = make_float2(s.X32[k0 * 64 + n] * sc, s.X32[(k0 + 1) * 64 + n] * sc);
+        const float2 v1 = make_float2(s.X32[(k0 + 8) * 64 + n] * sc, s.X32[(k0 + 9) * 64 + n] * sc);
+        uint4 f;
+        lf_split2(v0, f.x, f.z);
+        lf_split2(v1, f.y, f.w);
+        s.xfrag[e] = f;   // {hi b0, hi b1, lo b0, lo b1}
+    }
+    __syncthreads();
+    const int ld = a.ldt;
+    for (int rb = warp; 16 * rb < rp16; rb += LF_NW) {
+        const int r0 = 16 * rb;
+        float hh[8][4], mx[8][4];
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+            for (int u = 0; u < 4; ++u) hh[nt][u] = mx[nt][u] = 0.f;
+#pragma unroll
+        for (int ks = 0; ks < 4; ++ks) {
+            const float* pc = s.tile + (16 * ks + 2 * c) * ld + r0 + g;
+            // A = P rows r0 .., k = columns 16 ks ..: a0 (g, 2c..), a1 (g + 8, 2c..), a2 (g, 2c + 8..), a3 (g + 8, 2c + 8..)
+            uint32_t ah[4], al[4];
+            lf_split2(make_float2(pc[0], pc[ld]), ah[0], al[0]);
+            lf_split2(make_float2(pc[8], pc[ld + 8]), ah[1], al[1]);
+            lf_split2(make_float2(pc[8 * ld], pc[9 * ld]), ah[2], al[2]);
+            lf_split2(make_float2(pc[8 * ld + 8], pc[9 * ld + 8]), ah[3], al[3]);
+#pragma unroll
+            for (int nt = 2 * ks; nt < 8; ++nt) {
+                const uint4 f = s.xfrag[(ks * 8 + nt) * 32 + lane];
+                lf_mma_f16(hh[nt], ah[0], ah[1], ah[2], ah[3], f.x, f.y);
+                lf_mma_f16(mx[nt], ah[0], ah[1], ah[2], ah[3], f.z, f.w);
+                lf_mma_f16(mx[nt], al[0], al[1], al[2], al[3], f.x, f.y);
+            }
+        }
+        __syncwarp();   // every lane of the warp has read its rows before any of them is overwritten
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt) {
+            const int j = 8 * nt + 2 * c;
+            const float i0 = s.dsc[j], i1 = s.dsc[j + 1];
+            float* o = s.tile + j * ld + r0 + g;
+            o[0] = fmaf(mx[nt][0], 0x1p-11f, hh[nt][0]) * i0;
+            o[ld] = fmaf(mx[nt][1], 0x1p-11f, hh[nt][1]) * i1;
+            o[8] = fmaf(mx[nt][2], 0x1p-11f, hh[nt][2]) * i0;
+            o[ld + 8] = fmaf(mx[nt][3], 0x1p-11f, hh[nt][3]) * i1;
+        }
+    }
+    __syncthreads();
+}
+
 // Racc <- R_pass Racc (CTA 0, fp64, global ping-pong buffers); first pass: Racc = R_pass.
 __device__ void lf_racc(const LeafArgs& a, const LfSmem& s, int pass) {
     const double* src = a.racc + (pass & 1 ? 0 : 64 * 64);
@@ -670,18 +883,43 @@ __device__ void lf_build_g(const LfSmem& s, const double* packed, bool global, i
 template <int NI>
 __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int* npass) {
     bool shifted = false;
+    bool fast = a.fast != 0;   // first pass on the split-fp16 Gram (lf_gram16)
     int bad = -1;
     int pass = 0;
     for (; pass < 3; ++pass) {
-        lf_gram(a, s, rp);
+        if (fast && pass == 0) lf_gram16(a, s, rp);
+        else lf_gram(a, s, rp);
         if (pass == 0) LF_MARK(2);
         lf_allreduce(a, s, LF_NE, true, pass == 0 ? 20 : 0);
         if (pass == 0) LF_MARK(3);
         lf_build_g(s, s.red, false, nc, 0.0);
+        if (fast && pass == 0) {
+            // split-Gram validity: every column norm in [0.01, 2^15] (entries far from the fp16
+            // subnormal and overflow ranges) and finite
+            if (threadIdx.x == 0) s.flag[1] = 0;
+            __syncthreads();
+            if (threadIdx.x < nc) {
+                const double d = s.gdiag[threadIdx.x];
+                if (!(d >= 1e-4 && d <= 0x1p30)) s.flag[1] = 1;
+            }
+            __syncthreads();
+            if (s.flag[1]) {
+                LF_COUNT(0, 1);
+                fast = false;
+                pass = -1;
+                continue;
+            }
+        }
         int fb = threadIdx.x < 128 ? lf_chol(s) : 64;
         if (threadIdx.x == 0) s.flag[0] = fb;
         __syncthreads();
         fb = s.flag[0];
+        if (fb < 64 && pass == 0 && fast) {   // redo the pass on the fp64 Gram
+            LF_COUNT(0, 1);
+            fast = false;
+            pass = -1;
+            continue;
+        }
         if (fb < 64 && pass == 0) {
             // shifted CholQR: G + sh I, sh = 11 (m nc + nc (nc + 1)) u ||P||_F^2
             double tr = 0.0;
@@ -700,17 +938,29 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
             bad = fb;
             break;
         }
-        const double kk = lf_inverse(s, nc);   // every thread: same value
+        double keq = 0.0;
+        const double kk = lf_inverse(s, nc, &keq);   // every thread: same values
+        if (pass == 0 && fast && keq > 1.21 * nc * nc) {
+            // kappa_F of the column-equilibrated block > 1.1 nc: the split Gram's ~1e-6 error
+            // relative to |p_i||p_j| would cost ~kappa^2 1e-6 of orthogonality in a single pass --
+            // redo the pass on the fp64 Gram
+            LF_COUNT(0, 1);
+            fast = false;
+            pass = -1;
+            continue;
+        }
         const bool stop = (pass == 0) ? (!shifted && kk <= 4.0 * nc * nc)
                                       : ((pass == 1 && !shifted) || pass == 2);
         // R = R_p ... R_1: a single pass keeps R in s.Rs; otherwise CTA 0 accumulates in global
         if (blockIdx.x == 0 && !(pass == 0 && stop)) lf_racc(a, s, pass);
         if (pass == 0) LF_MARK(5);
-        lf_apply<NI>(a, s, rp);
+        if (fast && pass == 0) lf_apply16(a, s, rp);
+        else lf_apply<NI>(a, s, rp);
         if (pass == 0) LF_MARK(6);
         if (stop) break;
     }
     *npass = pass + 1;
+    LF_COUNT(1, pass + 1);
     return bad;
 }
 
@@ -991,6 +1241,8 @@ cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st) {
     a.bf16 = L.bf16;
     a.pq = L.pq;
     a.ph = L.pq ? L.ph : 0;
+    static const bool fp64_gram = getenv("RGSQR_LEAF_FP64_GRAM") != nullptr;
+    a.fast = fp64_gram ? 0 : 1;
     if (a.pq && (a.ph < 1 || a.ph > 64 || (L.ldh & 7) != 0 || (reinterpret_cast<uintptr_t>(L.pq) & 15) != 0 ||
                  !leaf_prologue_fits(L.m)))
         return cudaErrorInvalidValue;

@@ -761,7 +761,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             // read the block (fp32), write Q (fp32) + shadow(s)
             const double wt = o.h + o.w;
             ProfScope _s(h, PC_PANEL, 2.0 * m * (o.h * o.h + o.w * o.w) + 4.0 * m * o.h * o.w,
-                         (double)m * wt * (pl.split ? 12 : 10));
+                         (double)m * wt * (pl.split ? 12 : 10), pending_pro ? 1 : 0);   // tag 1: folded prologue
             int* cq_fail = h->cq_flags.as<int>();
             rg::CholqrLaunch c{};
             c.P = pl.Q + (int64_t)o.c0 * pl.ldq;

@@ -4,9 +4,17 @@
 #include <cstdlib>
 #include <vector>
 #include <cuda_runtime.h>
+#include <cuda_fp16.h>
+#include <cmath>
 #define LF_TRACE 1
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/kernels.h"
-namespace rg { thread_local long long g_launches = 0; bool pdl_enabled() { return false; } }
+namespace rg {
+thread_local long long g_launches = 0;
+bool pdl_enabled() { return false; }
+int dev_sms() { int d = 0, v = 0; cudaGetDevice(&d); cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, d); return v; }
+int dev_smem_optin() { int d = 0, v = 0; cudaGetDevice(&d); cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, d); return v; }
+cudaError_t ensure_smem_attr(const void* k, size_t b) { return cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)b); }
+}
 #include "../paper_conf_hpdc_zhangbw20_b200/csrc/leaf.cu"
 __global__ void lat_probe(long long* cyc, double* out, int n) {
     __shared__ double sm[1024];
@@ -127,7 +135,12 @@ int main(int argc, char** argv) {
     const int nc = argc > 2 ? atoi(argv[2]) : 64;
     std::vector<float> h((size_t)m * nc);
     srand(1);
-    for (auto& x : h) x = (rand() / (float)RAND_MAX) - 0.5f;
+    // N(0,1) columns (Box-Muller), scaled like the library's column scaling (norm ~300)
+    for (size_t i = 0; i < h.size(); ++i) {
+        const double u1 = (rand() + 1.0) / ((double)RAND_MAX + 2.0), u2 = rand() / ((double)RAND_MAX + 1.0);
+        const double norm = 256.0 + 256.0 * (double)((i / m) * 37 % 64) / 64.0;   // like the column scaling
+        h[i] = (float)(sqrt(-2 * log(u1)) * cos(6.283185307179586 * u2) * norm / sqrt((double)m));
+    }
     float *P, *Q, *R; uint16_t* Qh; double* ws; unsigned* bar; int* status;
     cudaMalloc(&P, m * nc * 4); cudaMalloc(&Q, m * nc * 4); cudaMalloc(&R, 64 * 64 * 4);
     cudaMalloc(&Qh, m * nc * 2); cudaMalloc(&ws, rg::leaf_ws_doubles() * 8); cudaMalloc(&bar, 4096);
@@ -139,7 +152,12 @@ int main(int argc, char** argv) {
     uint16_t* qa16 = nullptr;
     if (argc > 3 && atoi(argv[3])) {   // prologue with a random 64-column 16-bit Q_A
         std::vector<uint16_t> hq((size_t)m * 64);
-        for (size_t i = 0; i < hq.size(); ++i) hq[i] = 0x2000 + (uint16_t)(rand() & 0x3ff);   // small positive halves
+        // a nearly orthonormal Q_A: N(0, 1/m) entries as fp16
+        for (size_t i = 0; i < hq.size(); ++i) {
+            const double u1 = (rand() + 1.0) / ((double)RAND_MAX + 2.0), u2 = rand() / ((double)RAND_MAX + 1.0);
+            const __half hv = __float2half((float)(sqrt(-2 * log(u1)) * cos(6.283185307179586 * u2) / sqrt((double)m)));
+            hq[i] = *reinterpret_cast<const uint16_t*>(&hv);
+        }
         cudaMalloc(&qa16, hq.size() * 2);
         cudaMemcpy(qa16, hq.data(), hq.size() * 2, cudaMemcpyHostToDevice);
         L.pq = qa16; L.ph = 64;
@@ -167,6 +185,10 @@ int main(int argc, char** argv) {
     const char* names[9] = {"start", "loaded", "gram", "allreduce", "chol", "inverse+racc", "apply", "cholqr done", "stored"};
     long long ck[2];
     cudaMemcpyFromSymbol(ck, rg::lf_clk, sizeof(ck));
+    int cnt[4];
+    cudaMemcpyFromSymbol(cnt, rg::lf_count, sizeof(cnt));
+    printf("  per launch: fast-Gram fallbacks %.2f, CholQR passes %.2f\n", cnt[0] / (double)(iters + 3), cnt[1] / (double)(iters + 3));
+    printf("  gram16: mma %.2f, epilogue %.2f us\n", (tr[25] - tr[1]) / 1e3, (tr[2] - tr[25]) / 1e3);
     printf("  SM clock during the kernel: %.0f MHz\n", (ck[1] - ck[0]) / ((tr[8] - tr[0]) * 1e-3));
     printf("  allreduce: barrier 1 %.2f, reduce %.2f, barrier 2 %.2f, to smem %.2f us\n", (tr[20] - tr[2]) / 1e3,
            (tr[21] - tr[20]) / 1e3, (tr[22] - tr[21]) / 1e3, (tr[3] - tr[22]) / 1e3);
