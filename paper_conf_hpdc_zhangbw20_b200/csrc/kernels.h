@@ -146,6 +146,7 @@ struct LeafLaunch {
 bool leaf_fits(int64_t m);          // rows per SM fit in shared memory (and RGSQR_NO_LEAF unset)
 bool leaf_prologue_fits(int64_t m); // ... and the 16-bit staging copy of the prologue's Q_A
 size_t leaf_ws_doubles();
+size_t leaf_stats_offset();   // doubles into the leaf workspace: 3 uint64 counters (launches, fast-Gram fallbacks, passes)
 cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st);
 
 // ---- gemm_tc.cu (Alg 1 lines 8-9 on tcgen05)

@@ -74,16 +74,18 @@ struct LeafArgs {
     const uint16_t* pq;  // Q_A, 16-bit image (ld ldh), m x ph; null: no prologue
     int ph;              // columns of Q_A (<= 64)
     int fast;            // first Gram on the 16-bit tensor cores (split fp16, see lf_gram16)
+    unsigned long long* stats;   // [0] launches, [1] fast-Gram fallbacks, [2] CholQR passes (CTA 0)
 };
 
+// Per-handle counters (CTA 0, thread 0; read with RGSQR_LEAF_STATS=1): launches, fast-Gram
+// fallbacks to the fp64 Gram, CholQR passes.
+#define LF_COUNT(i, v)                                                        \
+    do {                                                                      \
+        if (blockIdx.x == 0 && threadIdx.x == 0) a.stats[(i) + 1] += (v);     \
+    } while (0)
 #ifdef LF_TRACE
 __device__ unsigned long long lf_trace[32];
 __device__ long long lf_clk[2];
-__device__ int lf_count[4];   // [0] fast-Gram fallbacks, [1] passes
-#define LF_COUNT(i, v)                                              \
-    do {                                                            \
-        if (blockIdx.x == 0 && threadIdx.x == 0) lf_count[i] += v;  \
-    } while (0)
 #define LF_MARK(i)                                                                     \
     do {                                                                               \
         if (blockIdx.x == 0 && threadIdx.x == 0) {                                     \
@@ -93,9 +95,6 @@ __device__ int lf_count[4];   // [0] fast-Gram fallbacks, [1] passes
         }                                                                              \
     } while (0)
 #else
-#define LF_COUNT(i, v) \
-    do {               \
-    } while (0)
 #define LF_MARK(i) \
     do {           \
     } while (0)
@@ -617,6 +616,125 @@ __device__ int lf_chol(const LfSmem& s) {
     return min(s_bad[0], s_bad[1]);
 }
 
+// Fast path (after the split Gram): Cholesky AND inverse in one pivot loop, fp32.  The elimination
+// of lf_chol (warps 0-3, rows 4 ii + q in registers, pivot rows published through shared memory
+// with producer / consumer named barriers, look-ahead on row k + 1) is applied to the augmented
+// [S | W] with W = I: after step k, S = U = L^{-1} G (upper) and W = L^{-1} (unit lower), G = L D L^T,
+// so R = D^{-1/2} U and R^{-1} = W^T D^{-1/2} come out together -- the separate blocked inverse
+// (lf_inverse) leaves the critical path.  fp32 is enough here: the split Gram carries ~1e-6
+// relative error and the fast path is taken only for kappa_F(equilibrated) <= 1.1 nc.
+// Writes s.X32 = R^{-1} (row-major), s.Rs = R (fp64 row-major, for the output / racc),
+// s.rdiag32; *keq = kappa_F^2 of the column-equilibrated block.  Returns the first failed pivot
+// (64 if none): a pivot fails unless finite and > 1e-4 G(k, k) (beyond that kappa, the fp64
+// path takes over anyway).  Called by all threads.
+constexpr int LF_PUB = 129;   // published rows: S (0..63) | W (64..127), odd stride
+
+__device__ __forceinline__ float lf_rcp32(float x) {
+    float y;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+
+__device__ int lf_chol_inv32(const LfSmem& s, int nc, double* keq) {
+    static_assert(64 * LF_PUB * 4 <= LF_REGION, "region B");
+    float* pub = reinterpret_cast<float*>(s.G);
+    const int t = threadIdx.x, jl = t & 31, q = t >> 5;
+    __shared__ int s_bad2[2];
+    __shared__ double s_en[LF_NW];
+    if (t < 128) {
+        float g0[16], g1[16], w0[16], w1[16];
+#pragma unroll
+        for (int ii = 0; ii < 16; ++ii) {
+            const int i = 4 * ii + q;
+            g0[ii] = (float)s.G[i * LF_GLD + jl];
+            g1[ii] = (float)s.G[i * LF_GLD + jl + 32];
+            w0[ii] = (i == jl) ? 1.f : 0.f;
+            w1[ii] = (i == jl + 32) ? 1.f : 0.f;
+        }
+        lf_bar128();   // every thread has its part of G before the rows overwrite it
+        if (q == 0) {
+            pub[jl] = g0[0];
+            pub[jl + 32] = g1[0];
+            pub[64 + jl] = w0[0];
+            pub[96 + jl] = w1[0];
+            __syncwarp();
+            lf_bar_arrive(2);
+        }
+#pragma unroll
+        for (int k = 0; k < 64; ++k) {
+            const float* row = pub + k * LF_PUB;
+            if (q != (k & 3)) lf_bar_sync(2 + (k & 1));
+            const float rd = lf_rcp32(row[k]);
+            const float t1 = (jl + 32 > k) ? row[jl + 32] * rd : 0.f;
+            const float t0 = (k < 32 && jl > k) ? row[jl] * rd : 0.f;
+            const float u0 = (jl <= k) ? row[64 + jl] * rd : 0.f;
+            const float u1 = (k >= 32 && jl + 32 <= k) ? row[96 + jl] * rd : 0.f;
+            const int nx = (k + 1) >> 2;   // register row of pivot k + 1 in its owner warp
+            if (k < 63) {
+                const float v = row[4 * nx + q];
+                g1[nx] = fmaf(-v, t1, g1[nx]);
+                if (k < 32) g0[nx] = fmaf(-v, t0, g0[nx]);
+                w0[nx] = fmaf(-v, u0, w0[nx]);
+                if (k >= 32) w1[nx] = fmaf(-v, u1, w1[nx]);
+                if (q == ((k + 1) & 3)) {
+                    float* nrow = pub + (k + 1) * LF_PUB;
+                    if (k + 1 < 32) nrow[jl] = g0[nx];
+                    nrow[jl + 32] = g1[nx];
+                    nrow[64 + jl] = w0[nx];
+                    nrow[96 + jl] = w1[nx];
+                    __syncwarp();
+                    lf_bar_arrive(2 + ((k + 1) & 1));
+                }
+            }
+#pragma unroll
+            for (int ii = k >> 2; ii < 16; ++ii) {
+                if (ii == nx && k < 63) continue;
+                const float v = row[4 * ii + q];
+                g1[ii] = fmaf(-v, t1, g1[ii]);
+                if (k < 32) g0[ii] = fmaf(-v, t0, g0[ii]);
+                w0[ii] = fmaf(-v, u0, w0[ii]);
+                if (k >= 32) w1[ii] = fmaf(-v, u1, w1[ii]);
+            }
+        }
+    }
+    __syncthreads();
+    if (t < 64) {
+        const float d = pub[t * LF_PUB + t];
+        const bool good = (d > (float)s.gdiag[t] * 1e-4f) && isfinite(d);
+        s.rdiag32[t] = good ? rsqrtf(d) : 1.f;
+        const unsigned badm = __ballot_sync(0xffffffffu, !good);
+        if (jl == 0) s_bad2[t >> 5] = badm ? (__ffs(badm) - 1 + 32 * (t >> 5)) : 64;
+    }
+    __syncthreads();
+    // X(i, j) = W(j, i) / sqrt(d_j) (i <= j),  R(i, j) = U(i, j) / sqrt(d_i) (j >= i)
+    constexpr int PER = 64 * 64 / LF_THREADS;
+    float rr[PER];
+    double en = 0.0;
+#pragma unroll
+    for (int u = 0; u < PER; ++u) {
+        const int e = t + u * LF_THREADS, i = e >> 6, j = e & 63;
+        const float x = (i <= j) ? pub[j * LF_PUB + 64 + i] * s.rdiag32[j] : 0.f;
+        s.X32[e] = x;
+        rr[u] = (j >= i) ? pub[i * LF_PUB + j] * s.rdiag32[i] : 0.f;
+        if (i < nc && j < nc && i <= j) en = fma((double)x * x, s.gdiag[i], en);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) en += __shfl_xor_sync(0xffffffffu, en, o);
+    if (jl == 0) s_en[t >> 5] = en;
+    __syncthreads();   // pub (region B) fully read: R may overwrite it
+    double se = 0.0;
+#pragma unroll
+    for (int w = 0; w < LF_NW; ++w) se += s_en[w];
+    *keq = (double)nc * se;
+#pragma unroll
+    for (int u = 0; u < PER; ++u) {
+        const int e = t + u * LF_THREADS, i = e >> 6, j = e & 63;
+        s.Rs[i * LF_GLD + j] = (double)rr[u];
+    }
+    __syncthreads();
+    return min(s_bad2[0], s_bad2[1]);
+}
+
 // X = R^{-1} (upper, fp32: it only feeds the fp32 product P R^{-1} and the kappa test), blocked
 // on 32 x 32 blocks, whole CTA:
 //   X11 = R11^{-1}, X22 = R22^{-1}   threads 0..63, column-parallel back substitution (right-
@@ -910,16 +1028,27 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
                 continue;
             }
         }
+        if (fast && pass == 0) {
+            // fp32 Cholesky + inverse in one loop; a failed pivot or a kappa above the fast-path
+            // bound redoes the pass on the fp64 Gram
+            double keq = 0.0;
+            const int fb32 = lf_chol_inv32(s, nc, &keq);
+            LF_MARK(4);
+            if (fb32 < 64 || !(keq <= 1.21 * nc * nc)) {
+                LF_COUNT(0, 1);
+                fast = false;
+                pass = -1;
+                continue;
+            }
+            LF_MARK(5);
+            lf_apply16(a, s, rp);
+            LF_MARK(6);
+            break;   // single pass: R in s.Rs
+        }
         int fb = threadIdx.x < 128 ? lf_chol(s) : 64;
         if (threadIdx.x == 0) s.flag[0] = fb;
         __syncthreads();
         fb = s.flag[0];
-        if (fb < 64 && pass == 0 && fast) {   // redo the pass on the fp64 Gram
-            LF_COUNT(0, 1);
-            fast = false;
-            pass = -1;
-            continue;
-        }
         if (fb < 64 && pass == 0) {
             // shifted CholQR: G + sh I, sh = 11 (m nc + nc (nc + 1)) u ||P||_F^2
             double tr = 0.0;
@@ -938,24 +1067,13 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
             bad = fb;
             break;
         }
-        double keq = 0.0;
-        const double kk = lf_inverse(s, nc, &keq);   // every thread: same values
-        if (pass == 0 && fast && keq > 1.21 * nc * nc) {
-            // kappa_F of the column-equilibrated block > 1.1 nc: the split Gram's ~1e-6 error
-            // relative to |p_i||p_j| would cost ~kappa^2 1e-6 of orthogonality in a single pass --
-            // redo the pass on the fp64 Gram
-            LF_COUNT(0, 1);
-            fast = false;
-            pass = -1;
-            continue;
-        }
+        const double kk = lf_inverse(s, nc);   // every thread: same value
         const bool stop = (pass == 0) ? (!shifted && kk <= 4.0 * nc * nc)
                                       : ((pass == 1 && !shifted) || pass == 2);
         // R = R_p ... R_1: a single pass keeps R in s.Rs; otherwise CTA 0 accumulates in global
         if (blockIdx.x == 0 && !(pass == 0 && stop)) lf_racc(a, s, pass);
         if (pass == 0) LF_MARK(5);
-        if (fast && pass == 0) lf_apply16(a, s, rp);
-        else lf_apply<NI>(a, s, rp);
+        lf_apply<NI>(a, s, rp);
         if (pass == 0) LF_MARK(6);
         if (stop) break;
     }
@@ -1129,6 +1247,7 @@ __global__ void __launch_bounds__(LF_THREADS, 1) leaf_kernel(LeafArgs a) {
     const int rows = rem <= 0 ? 0 : (rem < a.rows_per ? (int)rem : a.rows_per);
     const int rp16 = (rows + 15) & ~15;
     LF_MARK(0);
+    if (blockIdx.x == 0 && threadIdx.x == 0) a.stats[0] += 1;
 #ifdef LF_TRACE
     if (blockIdx.x == 0 && threadIdx.x == 0) lf_clk[0] = clock64();
 #endif
@@ -1219,6 +1338,7 @@ bool leaf_prologue_fits(int64_t m) {
 }
 
 size_t leaf_ws_doubles() { return (size_t)(LF_MAX_GRID + 1) * LF_PART + 2 * 64 * 64 + 64; }
+size_t leaf_stats_offset() { return (size_t)(LF_MAX_GRID + 1) * LF_PART + 2 * 64 * 64; }
 
 cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st) {
     if (L.nc < 1 || L.nc > 64 || !leaf_fits(L.m)) return cudaErrorInvalidValue;
@@ -1235,6 +1355,7 @@ cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st) {
     a.part = L.ws;
     a.red = L.ws + (size_t)LF_MAX_GRID * LF_PART;
     a.racc = a.red + LF_PART;
+    a.stats = reinterpret_cast<unsigned long long*>(a.racc + 2 * 64 * 64);
     a.bar = L.bar;
     a.status = L.status;
     a.col0 = L.col0;

@@ -1628,6 +1628,13 @@ int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_
         RG_CUDA(cudaMemcpy2DAsync(R, ldr * 4, dR, dldr * 4, n * 4, n, cudaMemcpyDeviceToHost, h->stream));
     }
     if (o.sync || host) rc = check_status(h);
+    if (getenv("RGSQR_LEAF_STATS") && h->cq_ws.p) {   // development: leaf-kernel counters so far
+        unsigned long long c[3] = {0, 0, 0};
+        cudaMemcpyAsync(c, h->cq_ws.as<double>() + rg::leaf_stats_offset(), sizeof(c), cudaMemcpyDeviceToHost,
+                        h->stream);
+        cudaStreamSynchronize(h->stream);
+        fprintf(stderr, "[rgsqr leaf] launches %llu fast-Gram fallbacks %llu CholQR passes %llu\n", c[0], c[1], c[2]);
+    }
     end_call(h);
     prof_collect(h);
     return rc;

@@ -143,7 +143,7 @@ int main(int argc, char** argv) {
     }
     float *P, *Q, *R; uint16_t* Qh; double* ws; unsigned* bar; int* status;
     cudaMalloc(&P, m * nc * 4); cudaMalloc(&Q, m * nc * 4); cudaMalloc(&R, 64 * 64 * 4);
-    cudaMalloc(&Qh, m * nc * 2); cudaMalloc(&ws, rg::leaf_ws_doubles() * 8); cudaMalloc(&bar, 4096);
+    cudaMalloc(&Qh, m * nc * 2); cudaMalloc(&ws, rg::leaf_ws_doubles() * 8); cudaMemset(ws, 0, rg::leaf_ws_doubles() * 8); cudaMalloc(&bar, 4096);
     cudaMalloc(&status, 64); cudaMemset(bar, 0, 4096); cudaMemset(status, 0x7f, 64);
     cudaMemcpy(P, h.data(), m * nc * 4, cudaMemcpyHostToDevice);
     rg::LeafLaunch L{};
@@ -185,9 +185,9 @@ int main(int argc, char** argv) {
     const char* names[9] = {"start", "loaded", "gram", "allreduce", "chol", "inverse+racc", "apply", "cholqr done", "stored"};
     long long ck[2];
     cudaMemcpyFromSymbol(ck, rg::lf_clk, sizeof(ck));
-    int cnt[4];
-    cudaMemcpyFromSymbol(cnt, rg::lf_count, sizeof(cnt));
-    printf("  per launch: fast-Gram fallbacks %.2f, CholQR passes %.2f\n", cnt[0] / (double)(iters + 3), cnt[1] / (double)(iters + 3));
+    unsigned long long cnt[3];
+    cudaMemcpy(cnt, ws + rg::leaf_stats_offset(), sizeof(cnt), cudaMemcpyDeviceToHost);
+    printf("  per launch: fast-Gram fallbacks %.2f, CholQR passes %.2f (%llu launches)\n", cnt[1] / (double)cnt[0], cnt[2] / (double)cnt[0], cnt[0]);
     printf("  gram16: mma %.2f, epilogue %.2f us\n", (tr[25] - tr[1]) / 1e3, (tr[2] - tr[25]) / 1e3);
     printf("  SM clock during the kernel: %.0f MHz\n", (ck[1] - ck[0]) / ((tr[8] - tr[0]) * 1e-3));
     printf("  allreduce: barrier 1 %.2f, reduce %.2f, barrier 2 %.2f, to smem %.2f us\n", (tr[20] - tr[2]) / 1e3,
