@@ -176,6 +176,17 @@ RG_API int lowrank_approx(rg_handle h, int64_t m_local, int64_t n, const float* 
                    int power_iters, uint64_t seed, float* U, int64_t ldu, float* S, float* V, int64_t ldv,
                    const rg_opts* opts);
 
+/* ---- lowrank_qrsvd: deterministic QR-SVD low rank of a tall-skinny A (section 3.4) --
+ * A = Q R (one RGSQR pass, no reorthogonalisation: "the roundoff errors in RGSQRF is insignificant"
+ * next to the truncation error), R = U_R S V_R^T (one-sided Jacobi in fp64 on the n x n R),
+ * A_r = Q U_R(:, 1:r) S_r V_R(:, 1:r)^T (Table 4).  U: m_local x rank (ldu, row-local in
+ * row-sharded mode), S: rank (descending), V: n x rank (ldv, replicated).  Workspace: an m_local x n
+ * fp32 Q plus its two 16-bit images and n x n fp64 Jacobi matrices.  Requires m (global) >= n,
+ * n <= 4096.  Errors: -2 m_local, -3 n, -4 A NULL, -5 lda, -6 rank outside [1, n], -7 U NULL,
+ * -8 ldu, -9 S NULL, -10 V NULL, -11 ldv < n; RG_BREAKDOWN, RG_NONFINITE. */
+RG_API int lowrank_qrsvd(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_t lda, int rank, float* U,
+                         int64_t ldu, float* S, float* V, int64_t ldv, const rg_opts* opts);
+
 /* ---- profiling (bench.py's roofline) -------------------------------------------------------
  * When enabled, each kernel class is bracketed by CUDA events on the handle's stream and the
  * per-class device time / launch count / algorithmic work accumulate until reset.

@@ -30,7 +30,7 @@ EXPORTS = [
     "rg_opts_default", "rg_create", "rg_set_stream", "rg_destroy", "rg_status_string", "rg_last_info",
     "rg_version", "rg_last_launches", "rg_nccl_load", "rg_comm_unique_id", "rg_comm_init", "rgsqr_factor", "orthogonalize",
     "ls_solve_refined", "lowrank_approx", "rg_profile_enable", "rg_profile_reset", "rg_profile_get",
-    "rg_set_comm", "rg_vgroup_create", "rg_vgroup_destroy", "rg_set_vcomm", "rg_debug_gaussian", "rg_debug_philox",
+    "rg_set_comm", "rg_vgroup_create", "rg_vgroup_destroy", "rg_set_vcomm", "rg_debug_gaussian", "rg_debug_philox", "lowrank_qrsvd",
 ]
 RG_MAX_RANKS = 8
 
@@ -95,6 +95,7 @@ def _lib():
                                        ctypes.POINTER(i32), f64p, ctypes.POINTER(rg_opts)]
         L.lowrank_approx.argtypes = [vp, i64, i64, vp, i64, i32, i32, i32, ctypes.c_uint64, vp, i64, vp, vp, i64,
                                      ctypes.POINTER(rg_opts)]
+        L.lowrank_qrsvd.argtypes = [vp, i64, i64, vp, i64, i32, vp, i64, vp, vp, i64, ctypes.POINTER(rg_opts)]
         L.rg_profile_enable.argtypes = [vp, i32]
         L.rg_profile_reset.argtypes = [vp]
         L.rg_profile_get.argtypes = [vp, i32, f64p, ctypes.POINTER(i64), f64p, f64p]
@@ -460,6 +461,27 @@ def lowrank_approx(A, rank, *, oversample=16, power_iters=1, seed=0, U=None, S=N
                                ctypes.byref(o))
     if check:
         _check("lowrank_approx", st, h)
+    return U, S, V
+
+
+def lowrank_qrsvd(A, rank, *, U=None, S=None, V=None, handle=None, opts=None, check=True):
+    """Deterministic QR-SVD rank-`rank` approximation of a tall-skinny A (section 3.4, Table 4):
+    A = QR, R = U_R S V_R^T, U = Q U_R(:, :rank).  Returns (U, S, V)."""
+    h = _handle(handle)
+    a = _mat(A, "A")
+    m, n = a.rows, a.cols
+    if U is None:
+        U = _like(A, m, rank)
+    if S is None:
+        S = _like(A, rank, None)
+    if V is None:
+        V = _like(A, n, rank)
+    u, s, v = _mat(U, "U"), _mat(S, "S"), _mat(V, "V")
+    o = opts if opts is not None else make_opts()
+    st = _lib().lowrank_qrsvd(h.ptr, m, n, ctypes.c_void_p(a.ptr), a.ld, int(rank), ctypes.c_void_p(u.ptr), u.ld,
+                              ctypes.c_void_p(s.ptr), ctypes.c_void_p(v.ptr), v.ld, ctypes.byref(o))
+    if check:
+        _check("lowrank_qrsvd", st, h)
     return U, S, V
 
 

@@ -1972,4 +1972,88 @@ int lowrank_approx(rg_handle h, int64_t m_local, int64_t n, const float* A, int6
     return rc;
 }
 
+
+// Deterministic QR-SVD low-rank approximation of a tall-skinny A (section 3.4, Table 4):
+// A = Q R (one RGSQR pass: "the roundoff errors in RGSQRF is insignificant, thus no refinement or
+// re-orthogonalization is needed"), R = U_R S V_R^T (one-sided Jacobi, fp64), and
+// A_r = (Q U_R(:, 1:r)) S_r V_R(:, 1:r)^T.  U = Q U_R(:, 1:r) with the split-precision tensor-core
+// product (reading #9); V = V_R(:, 1:r).
+int lowrank_qrsvd(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_t lda, int rank, float* U,
+                  int64_t ldu, float* S, float* V, int64_t ldv, const rg_opts* opts) {
+    if (!h) return -1;
+    rg_opts o;
+    if (opts) o = *opts; else rg_opts_default(&o);
+    if (m_local < 1 || (h->nranks <= 1 && m_local < n)) return -2;
+    if (n < 1 || n > 4096) return -3;
+    if (!A) return -4;
+    if (lda < m_local) return -5;
+    if (rank < 1 || rank > n) return -6;
+    if (!U) return -7;
+    if (ldu < m_local) return -8;
+    if (!S) return -9;
+    if (!V) return -10;
+    if (ldv < n) return -11;
+    cudaSetDevice(h->device);
+    begin_call(h);
+    cudaStream_t st = h->stream;
+    const bool host = ptr_side(A) == SIDE_HOST;
+    const float* dA = A;
+    int64_t dlda = lda;
+    float *dU = U, *dS = S, *dV = V;
+    int64_t dldu = ldu, dldv = ldv;
+    if (host) {
+        if (!h->stageA.ensure((size_t)m_local * n * 4) || !h->stageQ.ensure((size_t)m_local * rank * 4) ||
+            !h->stageR.ensure(((size_t)n * rank + rank) * 4 + 256))
+            return RG_ALLOC;
+        RG_CUDA(cudaMemcpy2DAsync(h->stageA.p, m_local * 4, A, lda * 4, m_local * 4, n, cudaMemcpyHostToDevice, st));
+        dA = h->stageA.as<float>();
+        dlda = m_local;
+        dU = h->stageQ.as<float>();
+        dldu = m_local;
+        dV = h->stageR.as<float>();
+        dldv = n;
+        dS = dV + (size_t)n * rank;
+    }
+    const int l = (int)n;
+    const int64_t ldm16 = round_up(std::max<int64_t>(m_local, 8), 8);
+    const int64_t ldl16 = round_up(std::max(l, 8), 8);
+    bool ok = h->lsQ.ensure((size_t)m_local * n * 4) && h->lrR.ensure((size_t)l * l * 4) &&
+              h->lrW.ensure((size_t)l * l * 8) && h->lrV.ensure((size_t)l * l * 8) &&
+              h->lrUb.ensure((size_t)l * l * 4) && h->lrVb.ensure((size_t)l * l * 4) && h->lrSig.ensure(l * 8 + 64) &&
+              h->lrFlags.ensure(64) && h->lrQ16.ensure((size_t)ldm16 * l * 2) && h->lrQ16l.ensure((size_t)ldm16 * l * 2) &&
+              h->lrB16.ensure((size_t)ldl16 * rank * 2 + 64) && h->lrB16l.ensure((size_t)ldl16 * rank * 2 + 64);
+    if (!ok) return RG_ALLOC;
+    float* Qw = h->lsQ.as<float>();
+    float* Rl = h->lrR.as<float>();
+    rg_opts qo = o;
+    qo.sync = 0;
+    int rc = run_rgsqr(h, m_local, n, dA, dlda, Qw, m_local, Rl, l, qo, 0);   // A = Q R
+    if (rc) return rc;
+    rc = check_status(h);
+    if (rc) return rc;
+    // R = U_R S V_R^T: Jacobi on R (trans = 0 in the grid form gives U_R = W S^-1, V_R = J)
+    RG_CUDA(rg::launch_jacobi_svd(Rl, l, l, rank, h->lrW.as<double>(), h->lrV.as<double>(), h->lrSig.as<double>(),
+                                  h->lrFlags.as<int>(), dS, h->lrUb.as<float>(), h->lrVb.as<float>(), st));
+    // U = Q U_R(:, 1:r)  (split-precision tensor-core product, ~fp32 accurate)
+    uint16_t* q16 = h->lrQ16.as<uint16_t>();
+    uint16_t* q16l = h->lrQ16l.as<uint16_t>();
+    uint16_t* b16 = h->lrB16.as<uint16_t>();
+    uint16_t* b16l = h->lrB16l.as<uint16_t>();
+    RG_CUDA(rg::launch_cast_rows(Qw, m_local, m_local, l, nullptr, q16, q16l, ldm16, o.precision, st));
+    RG_CUDA(rg::launch_cast_rows(h->lrUb.as<float>(), l, l, rank, nullptr, b16, b16l, ldl16, o.precision, st));
+    rc = gemm_nn(h, m_local, rank, l, q16, q16l, ldm16, b16, b16l, ldl16, dU, dldu, o.precision);
+    if (rc) return rc;
+    RG_CUDA(cudaMemcpy2DAsync(dV, dldv * 4, h->lrVb.as<float>(), (size_t)l * 4, (size_t)n * 4, rank,
+                              cudaMemcpyDeviceToDevice, st));
+    if (host) {
+        RG_CUDA(cudaMemcpy2DAsync(U, ldu * 4, dU, dldu * 4, m_local * 4, rank, cudaMemcpyDeviceToHost, st));
+        RG_CUDA(cudaMemcpy2DAsync(V, ldv * 4, dV, dldv * 4, n * 4, rank, cudaMemcpyDeviceToHost, st));
+        RG_CUDA(cudaMemcpyAsync(S, dS, rank * 4, cudaMemcpyDeviceToHost, st));
+    }
+    if (o.sync || host) rc = check_status(h);
+    end_call(h);
+    prof_collect(h);
+    return rc;
+}
+
 }  // extern "C"

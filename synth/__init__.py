@@ -91,6 +91,28 @@ def lowrank_matrix(m: int, n: int, k: int, kind: str, kappa: float, seed: int, d
     return At, s
 
 
+def svd_matrix_device(m: int, n: int, kind: str, kappa: float, seed: int, device="cuda"):
+    """Large-size form of svd_matrix for the GPU tests / bench (test-harness cost only): the
+    Gaussian factors are drawn with a seeded torch generator ON the device and orthonormalised
+    there (fp64); same spectrum recipe (reading #15).  Returns (A^T row-major fp32 (n x m), i.e.
+    column-major A, and sigma)."""
+    import torch
+
+    gen = torch.Generator(device=device).manual_seed(int(seed))
+    X = torch.randn(m, n, generator=gen, device=device, dtype=torch.float64)
+    U, Ru = torch.linalg.qr(X)
+    U *= torch.sign(torch.diagonal(Ru))
+    del X, Ru
+    Y = torch.randn(n, n, generator=gen, device=device, dtype=torch.float64)
+    V, Rv = torch.linalg.qr(Y)
+    V *= torch.sign(torch.diagonal(Rv))
+    s = sigma(n, kind, kappa)
+    U *= torch.from_numpy(s).to(device)
+    At = (V @ U.T).to(torch.float32).contiguous()   # (U s V^T)^T
+    del U, V, Y
+    return At, s
+
+
 def rhs(A: np.ndarray, seed: int, consistent: bool) -> np.ndarray:
     g = rng(seed + 7919)
     m, n = A.shape
