@@ -172,8 +172,15 @@ cudaError_t launch_cast_rows(const float* src, int64_t lds, int64_t rows, int co
 cudaError_t launch_cast_rows64(const double* src, int64_t lds, int64_t rows, int cols, const float* rscale,
                                uint16_t* hi, uint16_t* lo, int64_t ldd, int bf16, cudaStream_t st);
 cudaError_t launch_unscale_rows(float* X, int64_t ldx, int64_t rows, int cols, const float* rscale, cudaStream_t st);
+// W: jacobi_w_doubles(l) (l x svd_bj_cols(l) for the block Jacobi), V: l x l, flags: >= 64 ints
 cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double* W, double* V, double* sig, int* flags,
                               float* S, float* Ub, float* Vb, cudaStream_t st);
+size_t jacobi_w_doubles(int l);
+// ---- svd.cu (block one-sided Jacobi: 64-column block pairs on thread-block clusters)
+bool svd_bj_fits(int l);
+int svd_bj_cols(int l);
+cudaError_t launch_svd_bj(double* W, int l, int max_sweeps, double tol, unsigned long long* maxoff, int* sweeps_out,
+                          cudaStream_t st);
 
 // ---- blas.cu (CGLS vectors, triangular inverse, small products)
 // y = A x (fp32 A, fp64 x, y); with sq: also sq[sq_idx] = |y|^2 via sq_part (>= 1184 doubles)

@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 
 #include "kernels.h"
@@ -560,8 +561,32 @@ cudaError_t launch_unscale_rows(float* X, int64_t ldx, int64_t rows, int cols, c
     return cudaGetLastError();
 }
 
+size_t jacobi_w_doubles(int l) { return (size_t)l * std::max(l, svd_bj_cols(l)); }
+
 cudaError_t launch_jacobi_svd(const float* R, int64_t ldr, int l, int r, double* W, double* V, double* sig, int* flags,
                               float* S, float* Ub, float* Vb, cudaStream_t st) {
+    if (svd_bj_fits(l) && getenv("RGSQR_JACOBI_GRID") == nullptr && getenv("RGSQR_JACOBI_CLUSTER") == nullptr) {
+        // block one-sided Jacobi (svd.cu) on W = R^T (reading #22): W -> V_R S, U_R = R W S^-2
+        RG_LAUNCH((jacobi_init_kernel), (unsigned)std::min<int64_t>(((int64_t)l * l + 255) / 256, 148 * 8), 256, 0, st,
+                  R, ldr, l, W, V, 1);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        const int cols = svd_bj_cols(l);
+        if (cols > l) {
+            e = cudaMemsetAsync(W + (size_t)l * l, 0, (size_t)l * (cols - l) * 8, st);
+            if (e != cudaSuccess) return e;
+        }
+        const double jtol = getenv("RGSQR_JACOBI_TOL") ? atof(getenv("RGSQR_JACOBI_TOL")) : 1e-12;
+        int sweeps = 0;
+        e = launch_svd_bj(W, l, 30, jtol, reinterpret_cast<unsigned long long*>(flags + 2), &sweeps, st);
+        if (e != cudaSuccess) return e;
+        if (getenv("RGSQR_JACOBI_TRACE")) fprintf(stderr, "[rgsqr svd] block Jacobi l = %d: %d sweeps\n", l, sweeps);
+        RG_LAUNCH((jacobi_extract_kernel), l, 256, 0, st, W, V, l, r, S, Ub, Vb, sig);
+        e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        RG_LAUNCH((jacobi_rank_rt_kernel), l, 256, (size_t)l * 8, st, W, R, ldr, l, r, sig, S, Ub, Vb, 1);
+        return cudaGetLastError();
+    }
     const bool cluster = l <= 544 && getenv("RGSQR_JACOBI_GRID") == nullptr;
     // one-sided Jacobi on R^T (the graded, lower-triangular transpose) needs about half the sweeps
     // of Jacobi on R (measured 11 vs 21 at l = 528)

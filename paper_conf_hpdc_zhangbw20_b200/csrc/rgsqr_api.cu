@@ -1886,9 +1886,9 @@ int lowrank_approx(rg_handle h, int64_t m_local, int64_t n, const float* A, int6
               h->lrB16l.ensure((size_t)ldl16 * rank * 2 + 64) && h->lrY.ensure((size_t)m_local * l * 4) &&
               h->lrZ.ensure((size_t)n * l * 4) && h->lrQ16.ensure((size_t)std::max(ldm16, ldn16) * l * 2) &&
               h->lrQ16l.ensure((size_t)std::max(ldm16, ldn16) * l * 2) && h->lrR.ensure((size_t)l * l * 4) &&
-              h->lrW.ensure((size_t)l * l * 8) && h->lrV.ensure((size_t)l * l * 8) &&
+              h->lrW.ensure(rg::jacobi_w_doubles(l) * 8) && h->lrV.ensure((size_t)l * l * 8) &&
               h->lrUb.ensure((size_t)l * l * 4) && h->lrVb.ensure((size_t)l * l * 4) && h->lrSig.ensure(l * 8 + 64) &&
-              h->lrOm.ensure((size_t)n * l * 8) && h->lrScale.ensure(n * 4 + 64) && h->lrFlags.ensure(64) &&
+              h->lrOm.ensure((size_t)n * l * 8) && h->lrScale.ensure(n * 4 + 64) && h->lrFlags.ensure(512) &&
               h->partial.ensure(rg::colnorm_partial_doubles(m_local, (int)n) * 8 + 64) && h->norm2.ensure(n * 8 + 64) &&
               h->status.ensure(64);
     if (!ok) return RG_ALLOC;
@@ -2018,9 +2018,9 @@ int lowrank_qrsvd(rg_handle h, int64_t m_local, int64_t n, const float* A, int64
     const int64_t ldm16 = round_up(std::max<int64_t>(m_local, 8), 8);
     const int64_t ldl16 = round_up(std::max(l, 8), 8);
     bool ok = h->lsQ.ensure((size_t)m_local * n * 4) && h->lrR.ensure((size_t)l * l * 4) &&
-              h->lrW.ensure((size_t)l * l * 8) && h->lrV.ensure((size_t)l * l * 8) &&
+              h->lrW.ensure(rg::jacobi_w_doubles(l) * 8) && h->lrV.ensure((size_t)l * l * 8) &&
               h->lrUb.ensure((size_t)l * l * 4) && h->lrVb.ensure((size_t)l * l * 4) && h->lrSig.ensure(l * 8 + 64) &&
-              h->lrFlags.ensure(64) && h->lrQ16.ensure((size_t)ldm16 * l * 2) && h->lrQ16l.ensure((size_t)ldm16 * l * 2) &&
+              h->lrFlags.ensure(512) && h->lrQ16.ensure((size_t)ldm16 * l * 2) && h->lrQ16l.ensure((size_t)ldm16 * l * 2) &&
               h->lrB16.ensure((size_t)ldl16 * rank * 2 + 64) && h->lrB16l.ensure((size_t)ldl16 * rank * 2 + 64);
     if (!ok) return RG_ALLOC;
     float* Qw = h->lsQ.as<float>();
