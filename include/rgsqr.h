@@ -76,6 +76,9 @@ typedef struct {
     int panel;      /* leaf panel algorithm: 0 = auto (default): CholQR2 with an fp64 Gram, falling
                        back on the device to the TSQR/MGS panel if a Cholesky pivot fails;
                        1 = TSQR/MGS only (eq 8 + Alg 2, the paper's panel) */
+    int solver;     /* ls_solve_refined iteration: 0 = CGLS (default, Algorithm 3 as corrected by
+                       reading #5), 1 = LSQR (same R preconditioner, same two passes over A
+                       per iteration, same stopping test ||(A R^-1)^T r_k|| <= tol ||(A R^-1)^T b||) */
 } rg_opts;
 
 RG_API void rg_opts_default(rg_opts* o);

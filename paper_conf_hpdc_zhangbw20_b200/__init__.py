@@ -54,7 +54,7 @@ class RGError(RuntimeError):
 class rg_opts(ctypes.Structure):
     _fields_ = [("precision", ctypes.c_int), ("nb", ctypes.c_int), ("scale", ctypes.c_int),
                 ("reortho", ctypes.c_int), ("split", ctypes.c_int), ("sync", ctypes.c_int),
-                ("panel", ctypes.c_int)]
+                ("panel", ctypes.c_int), ("solver", ctypes.c_int)]
 
 
 _LIB = None
@@ -115,7 +115,8 @@ def version() -> str:
     return _lib().rg_version().decode()
 
 
-def make_opts(precision="fp16", nb=32, scale=True, reortho=-1, split=False, sync=True, panel="auto") -> rg_opts:
+def make_opts(precision="fp16", nb=32, scale=True, reortho=-1, split=False, sync=True, panel="auto",
+              solver="cgls") -> rg_opts:
     o = rg_opts()
     _lib().rg_opts_default(ctypes.byref(o))
     o.precision = {"fp16": 0, "bf16": 1}[precision] if isinstance(precision, str) else int(precision)
@@ -125,6 +126,7 @@ def make_opts(precision="fp16", nb=32, scale=True, reortho=-1, split=False, sync
     o.split = int(bool(split))
     o.sync = int(bool(sync))
     o.panel = {"auto": 0, "cholqr2": 0, "mgs": 1, "tsqr": 1}[panel] if isinstance(panel, str) else int(panel)
+    o.solver = {"cgls": 0, "lsqr": 1}[solver] if isinstance(solver, str) else int(solver)
     return o
 
 

@@ -206,6 +206,10 @@ cudaError_t launch_sqnorm(const double* v, int64_t len, double* sc, int idx, cud
 cudaError_t launch_cgls_xr(double* x, const double* t, double* r, const double* q, int64_t m, int n, double* sc,
                            cudaStream_t st);
 cudaError_t launch_cgls_p(const double* s, double* p, int n, double* sc, int first, cudaStream_t st);
+// LSQR (right-preconditioned by R, same passes as CGLS): u = q - (alpha / beta) u, sc[1] = |u|^2
+cudaError_t launch_lsqr_u(double* u, const double* q, int64_t m, double* sc, double* sqp, cudaStream_t st);
+cudaError_t launch_lsqr_step(const double* p, double* v, double* w, double* y, int n, double* sc, int first,
+                             cudaStream_t st);
 cudaError_t launch_gaussian_philox(int64_t total, uint64_t seed, double* out64, float* out32, cudaStream_t st);
 cudaError_t launch_philox_words(int64_t ncalls, uint64_t seed, uint32_t* words, cudaStream_t st);
 size_t probe_work_doubles(int64_t m, int n, int p);

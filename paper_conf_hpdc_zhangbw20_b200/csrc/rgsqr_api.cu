@@ -336,6 +336,7 @@ struct rg_handle_s {
     cudaGraphExec_t cgls_exec = nullptr;            // captured block of CGLS iterations
     const void* cgls_key[4] = {nullptr, nullptr, nullptr, nullptr};
     int64_t cgls_key_mn[3] = {0, 0, 0};
+    int cgls_solver = -1;                           // solver the captured block was built for
     DevBuf aux;                                     // misc (orthogonalize / lowrank)
     DevBuf vscratch;                                // virtual-rank collectives (rank 0 of a group)
     int alloc_epoch = 0;                            // bumped whenever a workspace buffer moves
@@ -1145,6 +1146,39 @@ int enqueue_cgls_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int 
 }
 
 
+// LSQR iterations (NEXT-4) on the same buffers: base = sc[16] | y v w t sv p (n each) | u q (m each) |
+// work.  Two passes over A per iteration like CGLS; dist: |u|^2 and A^T u allreduced.
+int enqueue_lsqr_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int n, int iters, double* base) {
+    cudaStream_t st = h->stream;
+    double* sc = base;
+    double* y = sc + 16;
+    double* v = y + n;
+    double* w = v + n;
+    double* t = w + n;
+    double* sv = t + n;
+    double* p = sv + n;
+    double* u = p + n;
+    double* q = u + m;
+    double* work = q + m;
+    double* sqp = work + std::max(rg::gemv_n_work_doubles(m, n), rg::gemv_t_work_doubles(m, n));
+    double* Rinv = h->rinv.as<double>();
+    const double* done = sc + 6;
+    for (int k = 0; k < iters; ++k) {
+        ProfScope _s(h, PC_CGLS, 4.0 * m * n, 8.0 * m * n);
+        RG_CUDA(rg::launch_trmv(Rinv, n, v, t, 0, done, st));                       // t = R^-1 v
+        RG_CUDA(rg::launch_gemv_n(A, lda, m, n, t, q, work, done, st));            // q = A t = M v
+        RG_CUDA(rg::launch_lsqr_u(u, q, m, sc, sqp, st));                          // u = q - alpha u, |u|^2
+        int rc = nccl_allreduce(h, sc + 1, 1, ncclFloat64);
+        if (rc) return rc;
+        RG_CUDA(rg::launch_gemv_t(A, lda, m, n, u, sv, work, done, st));           // A^T u
+        rc = nccl_allreduce(h, sv, n, ncclFloat64);
+        if (rc) return rc;
+        RG_CUDA(rg::launch_trmv(Rinv, n, sv, p, 1, done, st));                     // p = R^-T A^T u
+        RG_CUDA(rg::launch_lsqr_step(p, v, w, y, n, sc, 0, st));                   // v, alpha, Givens, y, w
+    }
+    return RG_OK;
+}
+
 // ------------------------------------------------------------------ general GEMMs (lowrank)
 // C (m x N fp32, ldc) = A (m x K, MN-major 16-bit, lda16) * B (K x N, K-major 16-bit, ldb16);
 // split: A_lo / B_lo images give ~fp32 accuracy (reading #9).
@@ -1245,6 +1279,7 @@ void rg_opts_default(rg_opts* o) {
     o->reortho = -1;
     o->split = 0;
     o->sync = 1;
+    o->solver = 0;
 }
 
 const char* rg_version(void) { return "rgsqr 0.1 sm_100a tcgen05/TMA"; }
@@ -1755,7 +1790,7 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     // ---- CGLS state: sc[16] | x p s t sv (n each) | r q (m each) | gemv work
     const size_t work = std::max({rg::gemv_n_work_doubles(m_local, (int)n), rg::gemv_t_work_doubles(m_local, (int)n),
                                   rg::gemv_nt_work_doubles((int)n) + (size_t)n});
-    if (!h->cg.ensure((16 + 5 * (size_t)n + 2 * (size_t)m_local + work + 2048) * 8 + 256)) return RG_ALLOC;
+    if (!h->cg.ensure((16 + 6 * (size_t)n + 2 * (size_t)m_local + work + 2048) * 8 + 256)) return RG_ALLOC;   // (LSQR: 6 n-vectors)
     double* base = h->cg.as<double>();
     double* sc = base;
     double* xd = sc + 16;
@@ -1769,12 +1804,34 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
         init[8] = tol;
         RG_CUDA(cudaMemcpyAsync(sc, init, sizeof(init), cudaMemcpyHostToDevice, h->stream));
     }
+    const bool lsqr = o.solver == 1;
+    if (lsqr) {
+        // LSQR start: u = b, beta_1 = |b|, p = R^-T A^T u, alpha_1 v_1 = p / beta_1, w = v, y = 0
+        double* y = sc + 16;
+        double* v = y + n;
+        double* w = v + n;
+        double* t = w + n;
+        double* svl = t + n;
+        double* pl = svl + n;
+        double* u = pl + n;
+        double* wkl = u + 2 * m_local;
+        RG_CUDA(rg::launch_cgls_init(db, m_local, (int)n, u, y, h->stream));
+        RG_CUDA(rg::launch_sqnorm(u, m_local, sc, 1, h->stream));
+        rc = nccl_allreduce(h, sc + 1, 1, ncclFloat64);
+        if (rc) return rc;
+        RG_CUDA(rg::launch_gemv_t(dA, dlda, m_local, (int)n, u, svl, wkl, nullptr, h->stream));
+        rc = nccl_allreduce(h, svl, n, ncclFloat64);
+        if (rc) return rc;
+        RG_CUDA(rg::launch_trmv(h->rinv.as<double>(), (int)n, svl, pl, 1, nullptr, h->stream));
+        RG_CUDA(rg::launch_lsqr_step(pl, v, w, y, (int)n, sc, 1, h->stream));
+    } else {
     RG_CUDA(rg::launch_cgls_init(db, m_local, (int)n, r, xd, h->stream));          // lines 4-5
     RG_CUDA(rg::launch_gemv_t(dA, dlda, m_local, (int)n, r, sv, wk, nullptr, h->stream));
     rc = nccl_allreduce(h, sv, n, ncclFloat64);
     if (rc) return rc;
     RG_CUDA(rg::launch_trmv(h->rinv.as<double>(), (int)n, sv, s, 1, nullptr, h->stream));  // line 6 (corrected)
     RG_CUDA(rg::launch_cgls_p(s, p, (int)n, sc, 1, h->stream));                    // lines 7-9
+    }
     // ---- iterations in captured blocks of `blk`, convergence flag read between blocks
     const int blk = 8;
     int done_iters = 0;
@@ -1785,7 +1842,7 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
         if (use_graph && cnt == blk) {
             const bool same = h->cgls_exec && h->cgls_key[0] == dA && h->cgls_key[1] == base &&
                               h->cgls_key[2] == h->rinv.p && h->cgls_key_mn[0] == m_local && h->cgls_key_mn[1] == n &&
-                              h->cgls_key_mn[2] == dlda;
+                              h->cgls_key_mn[2] == dlda && h->cgls_solver == o.solver;
             if (!same) {
                 if (h->cgls_exec) cudaGraphExecDestroy(h->cgls_exec);
                 h->cgls_exec = nullptr;
@@ -1794,7 +1851,9 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
                 h->stream = h->capture_stream;
                 RG_CUDA(cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal));
                 const long long before = rg::g_launches;
-                rc = enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, blk, base);
+                rc = lsqr ? enqueue_lsqr_iters(h, dA, dlda, m_local, (int)n, blk, base)
+                          : enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, blk, base);
+                h->cgls_solver = o.solver;
                 const long long captured = rg::g_launches - before;
                 rg::g_launches = before;
                 h->cgls_key_mn[2] = dlda;
@@ -1816,7 +1875,8 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
             h->replayed += (long long)(intptr_t)h->cgls_key[3];
         } else {
             const long long before = rg::g_launches;
-            rc = enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, cnt, base);
+            rc = lsqr ? enqueue_lsqr_iters(h, dA, dlda, m_local, (int)n, cnt, base)
+                      : enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, cnt, base);
             if (rc) return rc;
         }
         done_iters += cnt;
@@ -1827,6 +1887,12 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     if (done_iters == 0) {
         RG_CUDA(cudaMemcpyAsync(hsc, sc, sizeof(hsc), cudaMemcpyDeviceToHost, h->stream));
         RG_CUDA(cudaStreamSynchronize(h->stream));
+    }
+    if (lsqr) {   // x = R^-1 y (y lives where CGLS keeps x)
+        double* y = sc + 16;
+        double* tt = y + 3 * n;
+        RG_CUDA(rg::launch_trmv(h->rinv.as<double>(), (int)n, y, tt, 0, nullptr, h->stream));
+        RG_CUDA(cudaMemcpyAsync(y, tt, n * 8, cudaMemcpyDeviceToDevice, h->stream));
     }
     RG_CUDA(cudaMemcpyAsync(x, xd, n * 8, host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, h->stream));
     RG_CUDA(cudaStreamSynchronize(h->stream));

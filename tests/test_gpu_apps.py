@@ -131,3 +131,34 @@ def test_ls_one_pass_cgls_matches_two_pass(rg, monkeypatch, kappa):
     assert abs(it1 - it2) <= 2, (it1, it2)
     assert np.linalg.norm(x1 - x2) / np.linalg.norm(x2) <= 1e-8
     assert np.linalg.norm(x1 - x_star) / np.linalg.norm(x_star) <= 1e-5
+
+
+@pytest.mark.parametrize("kind,kappa", [("geometric", 1e2), ("geometric", 1e4), ("arithmetic", 1e4)])
+@pytest.mark.parametrize("consistent", [False, True])
+def test_ls_lsqr_parity(rg, kind, kappa, consistent):
+    """NEXT-4: LSQR (opts.solver = 1) on the same R-preconditioned operator reaches the oracle's LS
+    solution to the north_star tolerance, in about as many iterations as CGLS (the two are
+    mathematically equivalent Krylov methods on M = A R^-1)."""
+    m, n = 8192, 256
+    A = synth.svd_matrix(m, n, kind, kappa, seed=37).astype(np.float32)
+    b = synth.rhs(A.astype(np.float64), seed=37, consistent=consistent).astype(np.float32)
+    x_star, _ = oracle.ls_qr(A.astype(np.float64), b.astype(np.float64))
+    out = {}
+    for solver in ("cgls", "lsqr"):
+        x, it, rel, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), tol=1e-10, maxit=200,
+                                             opts=rg.make_opts(solver=solver))
+        assert st == rg.RG_OK, (solver, it, rel, st)
+        xe = x.cpu().numpy()
+        fe = np.linalg.norm(xe - x_star) / np.linalg.norm(x_star)
+        assert fe <= 1e-5, (solver, fe, it)
+        out[solver] = (it, xe)
+    assert abs(out["lsqr"][0] - out["cgls"][0]) <= 3, out
+    assert np.linalg.norm(out["lsqr"][1] - out["cgls"][1]) / np.linalg.norm(x_star) <= 1e-7
+
+
+def test_ls_lsqr_4x2_closed_form(rg):
+    A = np.array([[1, 1], [1, 2], [1, 3], [1, 4]], dtype=np.float32)
+    b = np.array([1, 3, 2, 5], dtype=np.float32)
+    x, it, rel, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), tol=1e-13,
+                                         opts=rg.make_opts(solver="lsqr"))
+    np.testing.assert_allclose(x.cpu().numpy(), [0.0, 1.1], atol=1e-9)

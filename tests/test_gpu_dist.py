@@ -181,8 +181,9 @@ def test_dist_orthogonalize(rg, ranks, kappa):
     assert abs(est - orth) <= 0.5 * orth + 1e-7
 
 
+@pytest.mark.parametrize("solver", ["cgls", "lsqr"])
 @pytest.mark.parametrize("consistent", [False, True])
-def test_dist_ls_solve_refined(rg, ranks, consistent):
+def test_dist_ls_solve_refined(rg, ranks, consistent, solver):
     """ls_solve_refined: the sharded QR preconditioner + CGLS with the ||q||^2 and A^T r
     allreduces; fe <= 1e-5 at kappa = 1e4 (north_star), x replicated."""
     m, n = 12000, 128
@@ -194,8 +195,9 @@ def test_dist_ls_solve_refined(rg, ranks, consistent):
     blocks = [_dev(A[c[r]:c[r + 1]]) for r in range(P)]
     bs = [torch.from_numpy(b[c[r]:c[r + 1]].copy()).cuda() for r in range(P)]
     xs = [torch.zeros(n, dtype=torch.float64, device="cuda") for _ in range(P)]
+    o = rg.make_opts(solver=solver)
     out = ranks.run([lambda r=r: rg.ls_solve_refined(blocks[r], bs[r], xs[r], tol=1e-10, maxit=200,
-                                                     handle=ranks.h[r]) for r in range(P)])
+                                                     handle=ranks.h[r], opts=o) for r in range(P)])
     assert all(o[3] == rg.RG_OK for o in out), [o[1:] for o in out]
     assert len({o[1] for o in out}) == 1
     for r in range(1, P):
