@@ -166,6 +166,13 @@ cudaError_t launch_proj_reduce(const float* P, int64_t ldp, int64_t p_stride, in
 cudaError_t launch_proj_finish(const float* Rf, int64_t ldf, int h, int w, float* R, int64_t ldr, uint16_t* Rh,
                                uint16_t* Rl, int64_t ldh, int bf16, cudaStream_t st);
 
+// ---- sgemm.cu (fp32 SIMT K1 / K2: the Figure 7 "no TensorCore" ablation, RGSQR_NO_TC=1)
+size_t sgemm_tn_work_floats(int64_t m, int h, int w);
+cudaError_t launch_sgemm_proj(const float* Q1, const float* A2, int64_t ld, int64_t m, int h, int w, float* R,
+                              int64_t ldr, float* work, cudaStream_t st);
+cudaError_t launch_sgemm_update(const float* Q1, const float* R12, int64_t ldr, float* A2, int64_t ld, int64_t m, int h,
+                                int w, cudaStream_t st);
+
 // ---- lowrank.cu
 cudaError_t launch_cast_rows(const float* src, int64_t lds, int64_t rows, int cols, const float* rscale, uint16_t* hi,
                              uint16_t* lo, int64_t ldd, int bf16, cudaStream_t st);

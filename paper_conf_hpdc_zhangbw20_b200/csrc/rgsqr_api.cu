@@ -517,9 +517,12 @@ int make_plan(rg_handle h, Plan& pl) {
     // the paper's structure with rows resident on chip); opt-in RGSQR_WIDE=1 the 64-column
     // CholQR2 kernel (same Q, R in exact arithmetic).
     const bool wide = getenv("RGSQR_WIDE") != nullptr;
+    // Figure 7 ablation: RGSQR_NO_TC=1 runs K1 / K2 as fp32 SIMT GEMMs and the panels
+    // without the leaf's 16-bit tensor-core paths (single GPU only; development switch)
+    const bool no_tc = getenv("RGSQR_NO_TC") != nullptr && !(pl.nranks > 1 && h->dist());
     // (split-precision passes keep the tensor-core K1/K2 at the last level: the leaf kernel's
     // mma.sync K1/K2 are single 16-bit products)
-    const bool pair = pl.panel == 0 && pl.nb == 32 && !(pl.nranks > 1 && h->dist()) &&
+    const bool pair = !no_tc && pl.panel == 0 && pl.nb == 32 && !(pl.nranks > 1 && h->dist()) &&
                       (wide ? rg::cholqr_fused_fits(m, 64) : (rg::leaf_fits(m) && !pl.split));
     pl.leaf = pair && !wide;
     build_ops(pl.ops, 0, n, pl.nb, pair, pl.leaf);
@@ -607,6 +610,9 @@ int make_plan(rg_handle h, Plan& pl) {
             if (!ok) return RG_CUDA_ERROR;
         }
     }
+    if (no_tc)
+        for (auto& o : pl.ops)
+            if (o.kind == Op::PROJ) pmax = std::max(pmax, rg::sgemm_tn_work_floats(m, o.h, o.w));
     pl.p_floats = pmax;
     (void)max_w;
     return RG_OK;
@@ -681,6 +687,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     uint16_t* ql = pl.split ? h->ql.as<uint16_t>() : nullptr;
     int* status = h->status.as<int>();
     const bool dist = pl.nranks > 1 && h->dist();
+    const bool no_tc = getenv("RGSQR_NO_TC") != nullptr && !dist;
     HostPipe* pp = pl.pipe;
     // section 3.5 on columns [c, c + nc): norms, power-of-two scales, scaled fp32 + 16-bit images
     auto scale_cols = [&](int c, int nc) -> int {
@@ -887,6 +894,15 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
                 RG_CUDA(rg::launch_panel_stack(rg_all, h->nranks, o.w, Rdiag, pl.ldr, qb, status, o.c0, p.guard, st));
                 RG_CUDA(rg::launch_panel_apply(p, qb + (int64_t)h->rank * 32 * 32, st));
             }
+        } else if (o.kind == Op::PROJ && no_tc) {
+            ProfScope _s(h, PC_PROJ, 2.0 * m * o.h * o.w, (double)m * (o.h + o.w) * 4, o.w);
+            RG_CUDA(rg::launch_sgemm_proj(pl.Q + (int64_t)o.c0 * pl.ldq, pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq, pl.ldq, m,
+                                          o.h, o.w, pl.R + o.c0 + (int64_t)(o.c0 + o.h) * pl.ldr, pl.ldr,
+                                          h->P.as<float>(), st));
+        } else if (o.kind == Op::UPDATE && no_tc) {
+            ProfScope _s(h, PC_UPDATE, 2.0 * m * o.h * o.w, (double)m * o.h * 4 + (double)m * o.w * 8, o.w);
+            RG_CUDA(rg::launch_sgemm_update(pl.Q + (int64_t)o.c0 * pl.ldq, pl.R + o.c0 + (int64_t)(o.c0 + o.h) * pl.ldr,
+                                            pl.ldr, pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq, pl.ldq, m, o.h, o.w, st));
         } else if (o.kind == Op::PROJ) {
             ProfScope _s(h, PC_PROJ, 2.0 * m * o.h * o.w * (pl.split ? 3 : 1),
                              (double)m * (o.h + o.w) * (pl.split ? 4 : 2), o.w);
