@@ -2,27 +2,29 @@
 // lowrank_approx (R_b, section 3.4 / config 5) and lowrank_qrsvd (R, section 3.4 / Table 4).
 //
 // One-sided Jacobi (Hestenes) orthogonalises the columns of W (= R^T, reading #22) by plane
-// rotations; here the columns are grouped into blocks of 32 and a round-robin tournament pairs
-// blocks (I, J).  For a pair, the 64 columns W_IJ = [W_I W_J] are orthogonalised as a unit:
-//   M = W_IJ^T W_IJ (64 x 64 Gram, fp64),  U = one cyclic Jacobi sweep on M (the standard
+// rotations; here the columns are grouped into blocks of 16 and a round-robin tournament pairs
+// blocks (I, J).  For a pair, the 32 columns W_IJ = [W_I W_J] are orthogonalised as a unit:
+//   M = W_IJ^T W_IJ (32 x 32 Gram, fp64),  U = one cyclic Jacobi sweep on M (the standard
 //   "block Jacobi with one inner sweep"),  W_IJ <- W_IJ U.
 // A sweep is nblk - 1 rounds; converged when every pair's Gram has max |M_ij| / sqrt(M_ii M_jj)
 // < tol at the start of a sweep.  The column norms of the converged W are the singular values.
 //
 // B200 mapping: one round = one launch; a pair = a thread-block cluster of C CTAs splitting the
-// l rows (C = 8 for l <= 1088: 16 pairs x 8 = 128 CTAs at l = 1024).  Per CTA: its rows of W_IJ in
+// l rows (32 pairs x 4 = 128 CTAs at l = 1024).  Per CTA: its rows of W_IJ in
 // shared memory, the partial Gram on the fp64 tensor cores (DMMA m8n8k4, one fragment per 8-column
 // block serves as A and B), a deterministic cluster all-reduce through distributed shared memory
-// (reduce-scatter in rank order + all-gather), the 64 x 64 inner sweep done redundantly by every
+// (reduce-scatter in rank order + all-gather), the 32 x 32 inner sweep done redundantly by every
 // CTA of the cluster (identical inputs -> identical U, no broadcast), the update W_IJ U on DMMA
 // (each warp owns 8 rows, so it overwrites only what it read), and the store.  The scalar
 // tournament of lowrank.cu needed one grid-wide step per column pair round (1023 per sweep at
-// l = 1024); here a sweep is 31 launches.
+// l = 1024); here a sweep is 63 launches.  (64-column pairs measured 254 us per round: the two-sided
+// 64 x 64 inner sweep is shared-memory-bandwidth bound, 128 KB of M / U traffic per inner round.)
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
 #include <cstdlib>
+#include <cstdio>
 #include <cstring>
 
 #include "kernels.h"
@@ -31,14 +33,20 @@ namespace cg = cooperative_groups;
 
 namespace rg {
 
-constexpr int BJ_B = 32;                 // columns per block
-constexpr int BJ_W = 2 * BJ_B;           // 64 columns per pair
+constexpr int BJ_B = 16;                 // columns per block
+constexpr int BJ_W = 2 * BJ_B;           // 32 columns per pair
 constexpr int BJ_THREADS = 512;
 constexpr int BJ_NW = BJ_THREADS / 32;
-constexpr int BJ_MLD = 65;               // inner M row stride (doubles)
-constexpr int BJ_ULD = 68;               // inner U row stride (doubles)
-constexpr int BJ_NE = BJ_W * (BJ_W + 1) / 2;   // 2080 packed upper Gram entries
-constexpr int BJ_MAX_ROWS = 160;         // rows per CTA
+constexpr int BJ_MLD = BJ_W + 1;         // inner M row stride (doubles)
+constexpr int BJ_ULD = BJ_W + 4;         // inner U row stride (doubles)
+constexpr int BJ_NE = BJ_W * (BJ_W + 1) / 2;   // packed upper Gram entries
+constexpr int BJ_MAX_ROWS = 320;         // rows per CTA
+constexpr int BJ_NB8 = BJ_W / 8;         // 8-column blocks of a pair
+constexpr int BJ_NT = BJ_NB8 * (BJ_NB8 + 1) / 2;   // upper 8 x 8 Gram blocks (10)
+constexpr int BJ_GROUPS = 2;             // Gram warps = groups (BJ_NT / BJ_GROUPS blocks each) x k-slices
+constexpr int BJ_TPG = BJ_NT / BJ_GROUPS;
+constexpr int BJ_KS = BJ_NW / BJ_GROUPS; // 8 k-slices
+static_assert(BJ_NT % BJ_GROUPS == 0, "Gram block groups");
 
 struct BjArgs {
     double* W;            // l rows x (nblk * 32) columns, column-major, ld = l (padding columns zero)
@@ -67,21 +75,34 @@ __device__ __forceinline__ void bj_pair(int L, int r, int k, int& p, int& q) {  
     }
 }
 
-__host__ __device__ constexpr int bj_blk_i(int t) {
+__host__ __device__ constexpr int bj_blk_i(int t) {   // upper blocks row by row
     int bi = 0;
-    while (t >= 8 - bi) {
-        t -= 8 - bi;
+    while (t >= BJ_NB8 - bi) {
+        t -= BJ_NB8 - bi;
         ++bi;
     }
     return bi;
 }
 __host__ __device__ constexpr int bj_blk_j(int t) {
     int bi = 0;
-    while (t >= 8 - bi) {
-        t -= 8 - bi;
+    while (t >= BJ_NB8 - bi) {
+        t -= BJ_NB8 - bi;
         ++bi;
     }
     return bi + t;
+}
+
+__device__ __forceinline__ double bj_rcp(double d) {
+    double y;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(d));
+    const double e = fma(-d, y, 1.0);
+    return fma(y, e, y);
+}
+__device__ __forceinline__ double bj_rsqrt(double d) {
+    double y;
+    asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(d));
+    const double e = fma(-d * y, y, 1.0);
+    return fma(0.5 * y, e, y);
 }
 
 __device__ __forceinline__ void bj_dmma(double (&d)[2], double a, double b) {
@@ -91,29 +112,34 @@ __device__ __forceinline__ void bj_dmma(double (&d)[2], double a, double b) {
 }
 
 template <int T>
-__device__ __forceinline__ void bj_blk(double (&acc)[2], const double (&f)[8]) {
+__device__ __forceinline__ void bj_blk(double (&acc)[2], const double (&f)[BJ_NB8]) {
     constexpr int bi = bj_blk_i(T), bj = bj_blk_j(T);   // compile-time: f stays in registers
     bj_dmma(acc, f[bi], f[bj]);
 }
 
+template <int Q, int U>
+struct BjGroup {   // blocks Q, Q + G, Q + 2G, ... of the group
+    static __device__ __forceinline__ void run(double (&acc)[BJ_TPG][2], const double (&f)[BJ_NB8]) {
+        bj_blk<Q + BJ_GROUPS * U>(acc[U], f);
+        BjGroup<Q, U + 1>::run(acc, f);
+    }
+};
 template <int Q>
-__device__ __forceinline__ void bj_gram_group(const double* Ws, int lds, int rows4, int kq, int lane, double (&acc)[9][2]) {
+struct BjGroup<Q, BJ_TPG> {
+    static __device__ __forceinline__ void run(double (&)[BJ_TPG][2], const double (&)[BJ_NB8]) {}
+};
+
+template <int Q>
+__device__ __forceinline__ void bj_gram_group(const double* Ws, int lds, int rows4, int ks, int lane,
+                                              double (&acc)[BJ_TPG][2]) {
     const int g = lane >> 2, c = lane & 3;
     const double* col = Ws + g * lds + c;
 #pragma unroll 1
-    for (int k0 = 4 * kq; k0 < rows4; k0 += 16) {
-        double f[8];
+    for (int k0 = 4 * ks; k0 < rows4; k0 += 4 * BJ_KS) {
+        double f[BJ_NB8];
 #pragma unroll
-        for (int b = 0; b < 8; ++b) f[b] = col[8 * b * lds + k0];
-        bj_blk<Q + 0>(acc[0], f);
-        bj_blk<Q + 4>(acc[1], f);
-        bj_blk<Q + 8>(acc[2], f);
-        bj_blk<Q + 12>(acc[3], f);
-        bj_blk<Q + 16>(acc[4], f);
-        bj_blk<Q + 20>(acc[5], f);
-        bj_blk<Q + 24>(acc[6], f);
-        bj_blk<Q + 28>(acc[7], f);
-        bj_blk<Q + 32>(acc[8], f);
+        for (int b = 0; b < BJ_NB8; ++b) f[b] = col[8 * b * lds + k0];
+        BjGroup<Q, 0>::run(acc, f);
     }
 }
 
@@ -124,12 +150,12 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
         if (prev < a.tol) return;   // uniform over the grid: converged in an earlier sweep
     }
     extern __shared__ __align__(16) double bj_smem[];
-    double* Ws = bj_smem;                                   // 64 x lds
+    double* Ws = bj_smem;                                   // BJ_W x lds
     double* part = Ws + BJ_W * a.lds;                       // packed partial Gram (BJ_NE)
     double* msum = part + BJ_NE;                            // packed reduced Gram (BJ_NE)
-    double* M = msum + BJ_NE;                               // 64 x BJ_MLD
-    double* U = M + BJ_W * BJ_MLD;                          // 64 x BJ_ULD (row-major)
-    double* scr = U + BJ_W * BJ_ULD;                        // 4 x 9 x 64 (k-quarter exchange)
+    double* M = msum + BJ_NE;                               // BJ_W x BJ_MLD
+    double* U = M + BJ_W * BJ_MLD;                          // BJ_W x BJ_ULD (row-major)
+    double* scr = U + BJ_W * BJ_ULD;                        // BJ_NT x 64 (k-slice exchange)
     __shared__ double s_a[BJ_W], s_b[BJ_W];
     __shared__ int s_o[BJ_W];
     __shared__ double s_off[BJ_NW];
@@ -148,29 +174,26 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
         Ws[lc * a.lds + i] = (i < rows) ? a.W[(int64_t)gc * a.l + r0 + i] : 0.0;
     }
     __syncthreads();
-    // ---- 2. partial Gram on DMMA: warp = group q (9 of the 36 upper 8x8 blocks) x k-quarter kq
+    // ---- 2. partial Gram on DMMA: warp = group q (BJ_TPG of the upper 8x8 blocks) x k-slice ks
     {
-        const int q = warp & 3, kq = warp >> 2;
-        double acc[9][2];
+        const int q = warp % BJ_GROUPS, ks = warp / BJ_GROUPS;
+        double acc[BJ_TPG][2];
 #pragma unroll
-        for (int u = 0; u < 9; ++u) acc[u][0] = acc[u][1] = 0.0;
-        switch (q) {
-            case 0: bj_gram_group<0>(Ws, a.lds, rows4, kq, lane, acc); break;
-            case 1: bj_gram_group<1>(Ws, a.lds, rows4, kq, lane, acc); break;
-            case 2: bj_gram_group<2>(Ws, a.lds, rows4, kq, lane, acc); break;
-            default: bj_gram_group<3>(Ws, a.lds, rows4, kq, lane, acc); break;
-        }
-        constexpr int NENT = 36 * 64;
+        for (int u = 0; u < BJ_TPG; ++u) acc[u][0] = acc[u][1] = 0.0;
+        if (q == 0) bj_gram_group<0>(Ws, a.lds, rows4, ks, lane, acc);
+        else bj_gram_group<1>(Ws, a.lds, rows4, ks, lane, acc);
+        static_assert(BJ_GROUPS == 2, "group dispatch");
+        constexpr int NENT = BJ_NT * 64;
         constexpr int NQ = (NENT + BJ_THREADS - 1) / BJ_THREADS;
         double run[NQ];
 #pragma unroll
         for (int i = 0; i < NQ; ++i) run[i] = 0.0;
-        for (int r = 0; r < 4; ++r) {   // the four k-quarters summed in order
+        for (int r = 0; r < BJ_KS; ++r) {   // the k-slices summed in order
             __syncthreads();
-            if (kq == r) {
-                double* dst = scr + q * 9 * 64 + lane;
+            if (ks == r) {
+                double* dst = scr + q * BJ_TPG * 64 + lane;
 #pragma unroll
-                for (int u = 0; u < 9; ++u) {
+                for (int u = 0; u < BJ_TPG; ++u) {
                     dst[(2 * u) * 32] = acc[u][0];
                     dst[(2 * u + 1) * 32] = acc[u][1];
                 }
@@ -186,8 +209,8 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
         for (int i = 0; i < NQ; ++i) {
             const int e = tid + BJ_THREADS * i;
             if (e < NENT) {
-                const int ln = e & 31, v = (e >> 5) & 1, qu = e >> 6, qq = qu / 9, u = qu % 9;
-                const int t = qq + 4 * u;
+                const int ln = e & 31, v = (e >> 5) & 1, qu = e >> 6, qq = qu / BJ_TPG, u = qu % BJ_TPG;
+                const int t = qq + BJ_GROUPS * u;
                 const int ii = 8 * bj_blk_i(t) + (ln >> 2), jj = 8 * bj_blk_j(t) + 2 * (ln & 3) + v;
                 if (ii <= jj) part[jj * (jj + 1) / 2 + ii] = run[i];
             }
@@ -215,7 +238,7 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
     // full symmetric M, U = I; convergence measure of this pair (before its rotations)
     double off = 0.0;
     for (int e = tid; e < BJ_W * BJ_W; e += BJ_THREADS) {
-        const int i = e >> 6, j = e & 63;
+        const int i = e / BJ_W, j = e % BJ_W;
         const int lo = min(i, j), hi = max(i, j);
         M[i * BJ_MLD + j] = msum[hi * (hi + 1) / 2 + lo];
         U[i * BJ_ULD + j] = (i == j) ? 1.0 : 0.0;
@@ -241,10 +264,14 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
             bj_pair(BJ_W, rr, tid, p, q);
             const double al = M[p * BJ_MLD + p], be = M[q * BJ_MLD + q], ga = M[p * BJ_MLD + q];
             double c = 1.0, s = 0.0;
-            if (al * be > 0.0 && fabs(ga) > 1e-15 * sqrt(al * be)) {
-                const double zeta = (be - al) / (2.0 * ga);
-                const double t = (zeta >= 0.0 ? 1.0 : -1.0) / (fabs(zeta) + sqrt(1.0 + zeta * zeta));
-                c = rsqrt(1.0 + t * t);
+            // the per-round chain is latency-bound: MUFU approximations + one Newton step each
+            // instead of IEEE div / sqrt (relative error ~1e-15, far below the sweep tolerance)
+            if (al * be > 0.0 && ga * ga > 1e-30 * (al * be)) {
+                const double zeta = (be - al) * 0.5 * bj_rcp(ga);
+                const double z2 = fma(zeta, zeta, 1.0);
+                const double sq = z2 * bj_rsqrt(z2);   // sqrt(1 + zeta^2)
+                const double t = copysign(bj_rcp(fabs(zeta) + sq), zeta);
+                c = bj_rsqrt(fma(t, t, 1.0));
                 s = c * t;
             }
             // w_p' = c w_p - s w_q,  w_q' = s w_p + c w_q
@@ -258,7 +285,7 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
         __syncthreads();
         // M <- J^T M J on 2 x 2 blocks {i, o_i} x {j, o_j} (each block updated by one thread, in place)
         for (int e = tid; e < (BJ_W / 2) * (BJ_W / 2); e += BJ_THREADS) {
-            const int ti = e >> 5, tj = e & 31;
+            const int ti = e / (BJ_W / 2), tj = e % (BJ_W / 2);
             int i, oi, j, oj;
             bj_pair(BJ_W, rr, ti, i, oi);
             bj_pair(BJ_W, rr, tj, j, oj);
@@ -276,7 +303,7 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
         }
         // U <- U J (rows x pairs, in place)
         for (int e = tid; e < BJ_W * (BJ_W / 2); e += BJ_THREADS) {
-            const int r = e >> 5, t = e & 31;
+            const int r = e / (BJ_W / 2), t = e % (BJ_W / 2);
             int p, q;
             bj_pair(BJ_W, rr, t, p, q);
             const double up = U[r * BJ_ULD + p], uq = U[r * BJ_ULD + q];
@@ -288,18 +315,18 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
     // ---- 5. W_IJ <- W_IJ U on DMMA: warp w owns rows 8 w .. 8 w + 7 (all 64 output columns)
     for (int rb = warp; 8 * rb < rows4; rb += BJ_NW) {
         const int g = lane >> 2, c = lane & 3;
-        double acc[8][2];
+        double acc[BJ_NB8][2];
 #pragma unroll
-        for (int ct = 0; ct < 8; ++ct) acc[ct][0] = acc[ct][1] = 0.0;
+        for (int ct = 0; ct < BJ_NB8; ++ct) acc[ct][0] = acc[ct][1] = 0.0;
 #pragma unroll 4
         for (int k0 = 0; k0 < BJ_W; k0 += 4) {
             const double av = Ws[(k0 + c) * a.lds + 8 * rb + g];   // A(g, c) = W(row 8 rb + g, col k0 + c)
 #pragma unroll
-            for (int ct = 0; ct < 8; ++ct) bj_dmma(acc[ct], av, U[(k0 + c) * BJ_ULD + 8 * ct + g]);
+            for (int ct = 0; ct < BJ_NB8; ++ct) bj_dmma(acc[ct], av, U[(k0 + c) * BJ_ULD + 8 * ct + g]);
         }
         __syncwarp();
 #pragma unroll
-        for (int ct = 0; ct < 8; ++ct) {
+        for (int ct = 0; ct < BJ_NB8; ++ct) {
             Ws[(8 * ct + 2 * c) * a.lds + 8 * rb + g] = acc[ct][0];
             Ws[(8 * ct + 2 * c + 1) * a.lds + 8 * rb + g] = acc[ct][1];
         }
@@ -314,8 +341,11 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
     cl.sync();   // no CTA leaves while a cluster peer may still read its shared memory
 }
 
-// (l <= 544 keeps the register/cluster Jacobi of lowrank.cu, measured faster there)
-bool svd_bj_fits(int l) { return l > 544 && l <= 8 * BJ_MAX_ROWS && getenv("RGSQR_JACOBI_SCALAR") == nullptr; }
+bool svd_bj_fits(int l) {
+    if (getenv("RGSQR_JACOBI_SCALAR") != nullptr) return false;
+    const int min_l = getenv("RGSQR_JACOBI_BLOCK_MIN") ? atoi(getenv("RGSQR_JACOBI_BLOCK_MIN")) : 545;
+    return l >= min_l && l >= 2 && l <= 8 * BJ_MAX_ROWS;
+}
 
 int svd_bj_cols(int l) { return ((l + BJ_W - 1) / BJ_W) * BJ_W; }
 
@@ -327,12 +357,12 @@ cudaError_t launch_svd_bj(double* W, int l, int max_sweeps, double tol, unsigned
     const int nblk = svd_bj_cols(l) / BJ_B;
     const int P = nblk / 2;
     int C = 1;
-    while (C < 8 && (P * C * 2 <= 148 || (l + C - 1) / C > BJ_MAX_ROWS)) C *= 2;
+    while (C < 8 && (P * C * 2 <= 148 || (l + C - 1) / C > BJ_MAX_ROWS)) C *= 2;   // ~128-148 CTAs
     const int rpc = (l + C - 1) / C;
     if (rpc > BJ_MAX_ROWS) return cudaErrorInvalidValue;
     const int rows8 = (rpc + 7) & ~7;
     const int lds = ((rows8 - 4 + 15) & ~15) + 4;   // == 4 mod 16 doubles, >= rows8
-    const size_t smem = ((size_t)BJ_W * lds + 2 * BJ_NE + BJ_W * BJ_MLD + BJ_W * BJ_ULD + 4 * 9 * 64) * 8;
+    const size_t smem = ((size_t)BJ_W * lds + 2 * BJ_NE + BJ_W * BJ_MLD + BJ_W * BJ_ULD + BJ_NT * 64) * 8;
     cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(svd_bj_round_kernel), smem);
     if (e != cudaSuccess) return e;
     e = cudaMemsetAsync(maxoff, 0, sizeof(unsigned long long) * max_sweeps, st);
@@ -375,6 +405,7 @@ cudaError_t launch_svd_bj(double* W, int l, int max_sweeps, double tol, unsigned
         if (e != cudaSuccess) return e;
         double mx;
         memcpy(&mx, &bits, sizeof(mx));
+        if (getenv("RGSQR_JACOBI_TRACE")) fprintf(stderr, "[rgsqr svd] sweep %d: max off-diagonal cosine %.3e\n", sweep, mx);
         if (mx < tol) {
             ++sweep;
             break;
