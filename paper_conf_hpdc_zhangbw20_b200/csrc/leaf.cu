@@ -628,6 +628,9 @@ __device__ int lf_chol(const LfSmem& s) {
 // (64 if none): a pivot fails unless finite and > 1e-4 G(k, k) (beyond that kappa, the fp64
 // path takes over anyway).  Called by all threads.
 constexpr int LF_PUB = 129;   // published rows: S (0..63) | W (64..127), odd stride
+#ifndef LF_CHOL_WARPS
+#define LF_CHOL_WARPS 16
+#endif
 
 __device__ __forceinline__ float lf_rcp32(float x) {
     float y;
@@ -635,61 +638,67 @@ __device__ __forceinline__ float lf_rcp32(float x) {
     return y;
 }
 
+template <int CW>   // warps in the elimination (rows 4 ii + q for CW = 4, CW ii + q in general)
 __device__ int lf_chol_inv32(const LfSmem& s, int nc, double* keq) {
     static_assert(64 * LF_PUB * 4 <= LF_REGION, "region B");
+    static_assert(CW == 4 || CW == 8 || CW == 16, "elimination warps");
+    constexpr int RPW = 64 / CW;        // register rows per warp
+    constexpr int NT = 32 * CW;         // named-barrier thread count
     float* pub = reinterpret_cast<float*>(s.G);
     const int t = threadIdx.x, jl = t & 31, q = t >> 5;
     __shared__ int s_bad2[2];
     __shared__ double s_en[LF_NW];
-    if (t < 128) {
-        float g0[16], g1[16], w0[16], w1[16];
+    auto bsync = [&](int id) { asm volatile("bar.sync %0, %1;" ::"r"(id), "n"(NT) : "memory"); };
+    auto barrive = [&](int id) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "n"(NT) : "memory"); };
+    if (t < NT) {
+        float g0[RPW], g1[RPW], w0[RPW], w1[RPW];
 #pragma unroll
-        for (int ii = 0; ii < 16; ++ii) {
-            const int i = 4 * ii + q;
+        for (int ii = 0; ii < RPW; ++ii) {
+            const int i = CW * ii + q;
             g0[ii] = (float)s.G[i * LF_GLD + jl];
             g1[ii] = (float)s.G[i * LF_GLD + jl + 32];
             w0[ii] = (i == jl) ? 1.f : 0.f;
             w1[ii] = (i == jl + 32) ? 1.f : 0.f;
         }
-        lf_bar128();   // every thread has its part of G before the rows overwrite it
+        bsync(1);   // every thread has its part of G before the rows overwrite it
         if (q == 0) {
             pub[jl] = g0[0];
             pub[jl + 32] = g1[0];
             pub[64 + jl] = w0[0];
             pub[96 + jl] = w1[0];
             __syncwarp();
-            lf_bar_arrive(2);
+            barrive(2);
         }
 #pragma unroll
         for (int k = 0; k < 64; ++k) {
             const float* row = pub + k * LF_PUB;
-            if (q != (k & 3)) lf_bar_sync(2 + (k & 1));
+            if (q != (k % CW)) bsync(2 + (k & 1));
             const float rd = lf_rcp32(row[k]);
             const float t1 = (jl + 32 > k) ? row[jl + 32] * rd : 0.f;
             const float t0 = (k < 32 && jl > k) ? row[jl] * rd : 0.f;
             const float u0 = (jl <= k) ? row[64 + jl] * rd : 0.f;
             const float u1 = (k >= 32 && jl + 32 <= k) ? row[96 + jl] * rd : 0.f;
-            const int nx = (k + 1) >> 2;   // register row of pivot k + 1 in its owner warp
+            const int nx = (k + 1) / CW;   // register row of pivot k + 1 in its owner warp
             if (k < 63) {
-                const float v = row[4 * nx + q];
+                const float v = row[CW * nx + q];
                 g1[nx] = fmaf(-v, t1, g1[nx]);
                 if (k < 32) g0[nx] = fmaf(-v, t0, g0[nx]);
                 w0[nx] = fmaf(-v, u0, w0[nx]);
                 if (k >= 32) w1[nx] = fmaf(-v, u1, w1[nx]);
-                if (q == ((k + 1) & 3)) {
+                if (q == ((k + 1) % CW)) {
                     float* nrow = pub + (k + 1) * LF_PUB;
                     if (k + 1 < 32) nrow[jl] = g0[nx];
                     nrow[jl + 32] = g1[nx];
                     nrow[64 + jl] = w0[nx];
                     nrow[96 + jl] = w1[nx];
                     __syncwarp();
-                    lf_bar_arrive(2 + ((k + 1) & 1));
+                    barrive(2 + ((k + 1) & 1));
                 }
             }
 #pragma unroll
-            for (int ii = k >> 2; ii < 16; ++ii) {
+            for (int ii = k / CW; ii < RPW; ++ii) {
                 if (ii == nx && k < 63) continue;
-                const float v = row[4 * ii + q];
+                const float v = row[CW * ii + q];
                 g1[ii] = fmaf(-v, t1, g1[ii]);
                 if (k < 32) g0[ii] = fmaf(-v, t0, g0[ii]);
                 w0[ii] = fmaf(-v, u0, w0[ii]);
@@ -1032,7 +1041,7 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
             // fp32 Cholesky + inverse in one loop; a failed pivot or a kappa above the fast-path
             // bound redoes the pass on the fp64 Gram
             double keq = 0.0;
-            const int fb32 = lf_chol_inv32(s, nc, &keq);
+            const int fb32 = lf_chol_inv32<LF_CHOL_WARPS>(s, nc, &keq);
             LF_MARK(4);
             if (fb32 < 64 || !(keq <= 1.21 * nc * nc)) {
                 LF_COUNT(0, 1);
