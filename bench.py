@@ -256,7 +256,7 @@ def main():
         roof = {"kernel": label, "bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / pk["hbm_gbs"], "peak_src": f"{pk['src']} copy bandwidth"}
     roof["traffic"] = None
-    tpath = os.path.join(ROOT, "profiles", "r01d_ncu_traffic.json")
+    tpath = os.path.join(ROOT, "profiles", "r02_ncu_traffic.json")
     if os.path.exists(tpath):
         with open(tpath) as f:
             tr = json.load(f).get(dom)
