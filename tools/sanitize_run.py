@@ -1,0 +1,27 @@
+"""Small calls through every kernel family, for compute-sanitizer (development tool)."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import paper_conf_hpdc_zhangbw20_b200 as rg
+import synth
+which = sys.argv[1] if len(sys.argv) > 1 else "all"
+def dev(A):
+    return torch.from_numpy(np.ascontiguousarray(np.asarray(A, dtype=np.float32).T)).cuda().t()
+h = rg.Handle(0)
+o = rg.make_opts()
+if which in ("all", "factor"):
+    A = synth.gaussian(4096, 256, seed=1).astype(np.float32)      # leaf + tcgen05 K1/K2 (w = 128)
+    rg.rgsqr_factor(dev(A), handle=h, opts=rg.make_opts(sync=True))
+    A = synth.gaussian(20000, 96, seed=2).astype(np.float32)      # fused CholQR panels
+    rg.rgsqr_factor(dev(A), handle=h)
+    rg.rgsqr_factor(dev(A), handle=h, opts=rg.make_opts(panel="mgs"))
+if which in ("all", "apps"):
+    A = synth.svd_matrix(8192, 128, "geometric", 1e3, seed=3).astype(np.float32)
+    rg.orthogonalize(dev(A), None, orth_tol=1e-5, max_passes=3, handle=h)
+    b = synth.rhs(A.astype(np.float64), seed=3, consistent=False).astype(np.float32)
+    rg.ls_solve_refined(dev(A), torch.from_numpy(b).cuda(), handle=h)
+    rg.ls_solve_refined(dev(A), torch.from_numpy(b).cuda(), handle=h, opts=rg.make_opts(solver="lsqr"))
+    L, _ = synth.lowrank_matrix(2048, 512, 128, "geometric", 1e4, seed=4)
+    rg.lowrank_approx(dev(L), 64, oversample=16, power_iters=1, seed=5, handle=h)
+torch.cuda.synchronize()
+print("ok", which)
