@@ -60,7 +60,7 @@ struct LeafArgs {
     int nc;              // block columns, 1..64
     float* R;            // nc x nc diagonal block of R, ldr (upper written, lower zeroed)
     int64_t ldr;
-    double* part;        // [LF_MAX_GRID][LF_PART] CTA partials
+    double* part;        // [LF_PART][LF_MAX_GRID] CTA partials, entry-major (coalesced reduce reads)
     double* red;         // [LF_PART] reduced result
     double* racc;        // [2][64 * 64] accumulated R (CTA 0), row-major
     unsigned* bar;       // grid barrier word (generation bit flips every barrier)
@@ -261,8 +261,8 @@ __device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne, bool to
 #pragma unroll
         for (int u = 0; u < NB; ++u) {
             const int b = lane + 32 * u;
-            p0[u] = (v0 && b < grid) ? __ldcg(a.part + (int64_t)b * LF_PART + e0) : 0.0;
-            p1[u] = (v1 && b < grid) ? __ldcg(a.part + (int64_t)b * LF_PART + e1) : 0.0;
+            p0[u] = (v0 && b < grid) ? __ldcg(a.part + (int64_t)e0 * LF_MAX_GRID + b) : 0.0;
+            p1[u] = (v1 && b < grid) ? __ldcg(a.part + (int64_t)e1 * LF_MAX_GRID + b) : 0.0;
         }
         double s0 = p0[0], s1 = p1[0];
 #pragma unroll
@@ -387,7 +387,7 @@ __device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int rp) {
             if (e < LF_NENT) run[i] += s.scr[e];
         }
     }
-    double* out = a.part + (int64_t)blockIdx.x * LF_PART;
+    double* out = a.part + blockIdx.x;   // entry e at out[e * LF_MAX_GRID]
 #pragma unroll
     for (int i = 0; i < NQ; ++i) {
         const int e = threadIdx.x + LF_THREADS * i;
@@ -396,7 +396,7 @@ __device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int rp) {
             const int t = qq + 4 * u;
             const int bi = lf_blk_i(t), bj = lf_blk_j(t);
             const int ii = 8 * bi + (ln >> 2), jj = 8 * bj + 2 * (ln & 3) + v;
-            if (ii <= jj) __stcg(out + jj * (jj + 1) / 2 + ii, run[i]);
+            if (ii <= jj) __stcg(out + (int64_t)(jj * (jj + 1) / 2 + ii) * LF_MAX_GRID, run[i]);
         }
     }
 }
@@ -505,7 +505,7 @@ __device__ void lf_gram16(const LeafArgs& a, const LfSmem& s, int rp16) {
     LF_MARK(25);
     __syncthreads();
     // the four k-quarters in fixed order -> fp64 packed upper triangle of the CTA partial
-    double* out = a.part + (int64_t)blockIdx.x * LF_PART;
+    double* out = a.part + blockIdx.x;   // entry e at out[e * LF_MAX_GRID]
 #pragma unroll 2
     for (int e = threadIdx.x; e < 64 * 64; e += LF_THREADS) {
         const int i = e >> 6, j = e & 63;
@@ -513,7 +513,7 @@ __device__ void lf_gram16(const LeafArgs& a, const LfSmem& s, int rp16) {
             const int o = i * LF_G16LD + j;
             constexpr int S = 64 * LF_G16LD;
             const float sum = ((slabs[o] + slabs[S + o]) + slabs[2 * S + o]) + slabs[3 * S + o];
-            __stcg(out + j * (j + 1) / 2 + i, (double)sum);
+            __stcg(out + (int64_t)(j * (j + 1) / 2 + i) * LF_MAX_GRID, (double)sum);
         }
     }
 }
@@ -1139,13 +1139,13 @@ __device__ void lf_pro_k1(const LeafArgs& a, const LfSmem& s, int rp16) {
 #pragma unroll
         for (int nt = 0; nt < 2; ++nt) lf_mma16816(acc[nt], af, bfr[nt], BF);
     }
-    double* out = a.part + (int64_t)blockIdx.x * LF_PART;
+    double* out = a.part + blockIdx.x;   // entry e at out[e * LF_MAX_GRID]
 #pragma unroll
     for (int nt = 0; nt < 2; ++nt)
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
             const int i = 16 * bi + g + 8 * (u >> 1), j = 16 * bj + 8 * nt + 2 * c + (u & 1);
-            __stcg(out + i * 64 + j, (double)acc[nt][u]);
+            __stcg(out + (int64_t)(i * 64 + j) * LF_MAX_GRID, (double)acc[nt][u]);
         }
 }
 
