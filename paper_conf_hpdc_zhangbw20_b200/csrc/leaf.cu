@@ -48,6 +48,12 @@ constexpr int LF_NENT = 36 * 64;             // Gram fragment entries (36 8x8 bl
 constexpr int LF_PART = 4096;                // doubles per CTA partial in the workspace (64 x 64 prologue)
 constexpr int LF_ABLD = 72;                  // 16-bit -R_AB image [n][k] row stride (halves)
 constexpr int LF_MAX_GRID = 160;
+// Partial layout: entries in chunks of 8 consecutive doubles (64 B) per CTA, the CTAs' chunks of one
+// entry range adjacent -- a CTA writes whole 64 B chunks, a reducing warp reads 32 CTAs x 64 B
+// contiguously (one chunk = 8 entries per warp).
+__host__ __device__ constexpr int64_t lf_pidx(int e, int b) {
+    return (int64_t)(e >> 3) * (LF_MAX_GRID * 8) + b * 8 + (e & 7);
+}
 constexpr size_t LF_REGION = 33792;          // bytes of each of the two aliased scratch regions
 
 struct LeafArgs {
@@ -60,7 +66,7 @@ struct LeafArgs {
     int nc;              // block columns, 1..64
     float* R;            // nc x nc diagonal block of R, ldr (upper written, lower zeroed)
     int64_t ldr;
-    double* part;        // [LF_PART][LF_MAX_GRID] CTA partials, entry-major (coalesced reduce reads)
+    double* part;        // CTA partials in chunks of 8 entries: lf_pidx(e, b) (coalesced both ways)
     double* red;         // [LF_PART] reduced result
     double* racc;        // [2][64 * 64] accumulated R (CTA 0), row-major
     unsigned* bar;       // grid barrier word (generation bit flips every barrier)
@@ -249,35 +255,44 @@ __device__ void lf_allreduce(const LeafArgs& a, const LfSmem& s, int ne, bool to
     lf_grid_sync(a.bar);
     if (mk) LF_MARK(mk);
     const int grid = gridDim.x;
-    const int slice = (ne + grid - 1) / grid;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    // two entries per warp per round, all 2 NB loads in flight (the 4096-entry prologue reduction
-    // has ~28 entries per CTA: one round instead of two dependent ones)
-    for (int q = warp; q < slice; q += 2 * LF_NW) {
-        constexpr int NB = (LF_MAX_GRID + 31) / 32;   // summed in CTA order (deterministic)
-        const int e0 = blockIdx.x * slice + q, e1 = e0 + LF_NW;
-        const bool v0 = e0 < ne, v1 = (q + LF_NW < slice) && e1 < ne;
-        double p0[NB], p1[NB];
+    const int nch = (ne + 7) >> 3;
+    // chunk c is reduced by warp c / grid of CTA c % grid: lanes over CTAs lane, lane + 32, ... in
+    // order, then a fixed xor-shuffle tree per entry (deterministic)
+    for (int c = blockIdx.x + grid * warp; c < nch; c += grid * LF_NW) {
+        constexpr int NB = (LF_MAX_GRID + 31) / 32;
+        const double* src = a.part + (int64_t)c * (LF_MAX_GRID * 8);
+        double2 p[NB][4];
 #pragma unroll
         for (int u = 0; u < NB; ++u) {
             const int b = lane + 32 * u;
-            p0[u] = (v0 && b < grid) ? __ldcg(a.part + (int64_t)e0 * LF_MAX_GRID + b) : 0.0;
-            p1[u] = (v1 && b < grid) ? __ldcg(a.part + (int64_t)e1 * LF_MAX_GRID + b) : 0.0;
-        }
-        double s0 = p0[0], s1 = p1[0];
 #pragma unroll
-        for (int u = 1; u < NB; ++u) {
-            s0 += p0[u];
-            s1 += p1[u];
+            for (int k = 0; k < 4; ++k)
+                p[u][k] = b < grid ? __ldcg(reinterpret_cast<const double2*>(src + b * 8) + k) : make_double2(0.0, 0.0);
+        }
+        double sm[8];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            sm[2 * k] = p[0][k].x;
+            sm[2 * k + 1] = p[0][k].y;
         }
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            s0 += __shfl_xor_sync(0xffffffffu, s0, o);
-            s1 += __shfl_xor_sync(0xffffffffu, s1, o);
-        }
-        if (lane == 0) {
-            if (v0) __stcg(a.red + e0, s0);
-            if (v1) __stcg(a.red + e1, s1);
+        for (int u = 1; u < NB; ++u)
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                sm[2 * k] += p[u][k].x;
+                sm[2 * k + 1] += p[u][k].y;
+            }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1)
+#pragma unroll
+            for (int k = 0; k < 8; ++k) sm[k] += __shfl_xor_sync(0xffffffffu, sm[k], o);
+        if (lane < 8) {
+            double v = sm[0];
+#pragma unroll
+            for (int k = 1; k < 8; ++k) v = lane == k ? sm[k] : v;
+            const int e = 8 * c + lane;
+            if (e < ne) __stcg(a.red + e, v);
         }
     }
     if (mk) LF_MARK(mk + 1);
@@ -387,7 +402,6 @@ __device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int rp) {
             if (e < LF_NENT) run[i] += s.scr[e];
         }
     }
-    double* out = a.part + blockIdx.x;   // entry e at out[e * LF_MAX_GRID]
 #pragma unroll
     for (int i = 0; i < NQ; ++i) {
         const int e = threadIdx.x + LF_THREADS * i;
@@ -396,7 +410,7 @@ __device__ void lf_gram(const LeafArgs& a, const LfSmem& s, int rp) {
             const int t = qq + 4 * u;
             const int bi = lf_blk_i(t), bj = lf_blk_j(t);
             const int ii = 8 * bi + (ln >> 2), jj = 8 * bj + 2 * (ln & 3) + v;
-            if (ii <= jj) __stcg(out + (int64_t)(jj * (jj + 1) / 2 + ii) * LF_MAX_GRID, run[i]);
+            if (ii <= jj) __stcg(a.part + lf_pidx(jj * (jj + 1) / 2 + ii, blockIdx.x), run[i]);
         }
     }
 }
@@ -505,16 +519,17 @@ __device__ void lf_gram16(const LeafArgs& a, const LfSmem& s, int rp16) {
     LF_MARK(25);
     __syncthreads();
     // the four k-quarters in fixed order -> fp64 packed upper triangle of the CTA partial
-    double* out = a.part + blockIdx.x;   // entry e at out[e * LF_MAX_GRID]
+    // packed index p = j (j + 1) / 2 + i walked by consecutive threads: whole 64 B chunks per warp
 #pragma unroll 2
-    for (int e = threadIdx.x; e < 64 * 64; e += LF_THREADS) {
-        const int i = e >> 6, j = e & 63;
-        if (i <= j) {
-            const int o = i * LF_G16LD + j;
-            constexpr int S = 64 * LF_G16LD;
-            const float sum = ((slabs[o] + slabs[S + o]) + slabs[2 * S + o]) + slabs[3 * S + o];
-            __stcg(out + (int64_t)(j * (j + 1) / 2 + i) * LF_MAX_GRID, (double)sum);
-        }
+    for (int p = threadIdx.x; p < LF_NE; p += LF_THREADS) {
+        int j = (int)((sqrtf(8.f * (float)p + 1.f) - 1.f) * 0.5f);
+        if ((j + 1) * (j + 2) / 2 <= p) ++j;
+        if (j * (j + 1) / 2 > p) --j;
+        const int i = p - j * (j + 1) / 2;
+        const int o = i * LF_G16LD + j;
+        constexpr int S = 64 * LF_G16LD;
+        const float sum = ((slabs[o] + slabs[S + o]) + slabs[2 * S + o]) + slabs[3 * S + o];
+        __stcg(a.part + lf_pidx(p, blockIdx.x), (double)sum);
     }
 }
 
@@ -1139,13 +1154,13 @@ __device__ void lf_pro_k1(const LeafArgs& a, const LfSmem& s, int rp16) {
 #pragma unroll
         for (int nt = 0; nt < 2; ++nt) lf_mma16816(acc[nt], af, bfr[nt], BF);
     }
-    double* out = a.part + blockIdx.x;   // entry e at out[e * LF_MAX_GRID]
 #pragma unroll
     for (int nt = 0; nt < 2; ++nt)
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
-            const int i = 16 * bi + g + 8 * (u >> 1), j = 16 * bj + 8 * nt + 2 * c + (u & 1);
-            __stcg(out + (int64_t)(i * 64 + j) * LF_MAX_GRID, (double)acc[nt][u]);
+        for (int h = 0; h < 2; ++h) {
+            const int i = 16 * bi + g + 8 * h, j = 16 * bj + 8 * nt + 2 * c;   // (j, j + 1): one 16 B store
+            __stcg(reinterpret_cast<double2*>(a.part + lf_pidx(i * 64 + j, blockIdx.x)),
+                   make_double2((double)acc[nt][2 * h], (double)acc[nt][2 * h + 1]));
         }
 }
 
