@@ -79,6 +79,8 @@ struct GemmArgs {
     int vec_ok;            // C / Ch / Cl accesses may use 16-byte (8-byte) vectors
     int overwrite;         // K2 only: C = D instead of C -= D (plain product, lowrank_approx)
     int h0;                // K2 only: 16-bit image written for columns >= h0 only
+    int c_ef;              // K2 TMA epilogue: C read / written with the L2 evict_first policy (streamed
+                           // once; keeps the next leaf's code and operands resident)
 };
 
 __device__ __forceinline__ uint16_t f2h_bits(float x, int bf16) {
@@ -301,7 +303,11 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
                         mbar_arrive(&cfull_bar[s]);
                     } else {
                         mbar_arrive_expect_tx(&cfull_bar[s], C::kCSlot);
-                        tma_load_2d(epi_buf + s * (C::kCSlot / 4), &tmC, &cfull_bar[s], t0, tj * BN + ch * 32);
+                        if (args.c_ef)
+                            tma_load_2d_hint(epi_buf + s * (C::kCSlot / 4), &tmC, &cfull_bar[s], t0, tj * BN + ch * 32,
+                                             policy_evict_first());
+                        else
+                            tma_load_2d(epi_buf + s * (C::kCSlot / 4), &tmC, &cfull_bar[s], t0, tj * BN + ch * 32);
                     }
                 }
             }
@@ -320,7 +326,11 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
                     uint32_t round;
                     te_slot<kChunks, EPI_WG, kNcw>(cnt, ch, s, round);
                     mbar_wait(&cready_bar[s], round & 1u);
-                    tma_store_2d(&tmC, epi_buf + s * (C::kCSlot / 4), t0, tj * BN + ch * 32);
+                    if (args.c_ef)
+                        tma_store_2d_hint(&tmC, epi_buf + s * (C::kCSlot / 4), t0, tj * BN + ch * 32,
+                                          policy_evict_first());
+                    else
+                        tma_store_2d(&tmC, epi_buf + s * (C::kCSlot / 4), t0, tj * BN + ch * 32);
                     bulk_commit();
                     bulk_wait_read<1>();   // the previous chunk's slot has been read out: recycle it
                     if (prev >= 0) mbar_arrive(&cempty_bar[prev]);
@@ -798,6 +808,8 @@ cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, cons
     GemmArgs args{};
     args.overwrite = overwrite;
     args.h0 = h0;
+    static const bool c_ef = !getenv("RGSQR_K2_NO_EF");
+    args.c_ef = c_ef ? 1 : 0;
     args.C = C;
     args.ldc = ldc;
     args.Ch = Ch;

@@ -80,6 +80,7 @@ struct LeafArgs {
     const uint16_t* pq;  // Q_A, 16-bit image (ld ldh), m x ph; null: no prologue
     int ph;              // columns of Q_A (<= 64)
     int fast;            // first Gram on the 16-bit tensor cores (split fp16, see lf_gram16)
+    int chol;            // fast-path Cholesky + inverse: 1 lf_chol_inv_b4 (default), 0 lf_chol_inv32
     unsigned long long* stats;   // [0] launches, [1] fast-Gram fallbacks, [2] CholQR passes (CTA 0)
 };
 
@@ -90,7 +91,7 @@ struct LeafArgs {
         if (blockIdx.x == 0 && threadIdx.x == 0) a.stats[(i) + 1] += (v);     \
     } while (0)
 #ifdef LF_TRACE
-__device__ unsigned long long lf_trace[32];
+__device__ unsigned long long lf_trace[48];
 __device__ long long lf_clk[2];
 #define LF_MARK(i)                                                                     \
     do {                                                                               \
@@ -646,6 +647,9 @@ constexpr int LF_PUB = 129;   // published rows: S (0..63) | W (64..127), odd st
 #ifndef LF_CHOL_WARPS
 #define LF_CHOL_WARPS 16
 #endif
+#ifndef LF_CHOL_BLOCKED
+#define LF_CHOL_BLOCKED 1   // 1: 4 x 4-block LDL (lf_chol_inv_b4); 0: the 64-pivot loop (lf_chol_inv32)
+#endif
 
 __device__ __forceinline__ float lf_rcp32(float x) {
     float y;
@@ -722,6 +726,7 @@ __device__ int lf_chol_inv32(const LfSmem& s, int nc, double* keq) {
         }
     }
     __syncthreads();
+    LF_MARK(28);
     if (t < 64) {
         const float d = pub[t * LF_PUB + t];
         const bool good = (d > (float)s.gdiag[t] * 1e-4f) && isfinite(d);
@@ -757,6 +762,193 @@ __device__ int lf_chol_inv32(const LfSmem& s, int nc, double* keq) {
     }
     __syncthreads();
     return min(s_bad2[0], s_bad2[1]);
+}
+
+// Fast path, 4 x 4-block form: G = L_b D_b L_b^T with 4 x 4 diagonal blocks, 16 block steps instead
+// of 64 pivots.  Four warps, lane = one column: warp 0 G(:, 0..31), warp 1 G(:, 32..63), warp 2
+// W(:, 0..31), warp 3 W(:, 32..63) (W = L_b^-1, starting from I).  Block step K (rows / columns
+// 4K..4K+3), every lane:
+//   A_KK  <- the 4 x 4 pivot block (published by the G lanes, 4 floats per column, one STS.128)
+//   R_KK  = chol(A_KK) in registers (every lane redundantly: 4 rsqrt on the chain)
+//   z     = R_KK^-T x_K,  y = R_KK^-1 z       (x_K: the lane's column at rows 4K..4K+3)
+//   x_i  -= A(i, 4K..4K+3) y  for the trailing rows i
+// so one publish + one named barrier + a 4 x 4 factorisation per FOUR pivots.  z is final output:
+// for a G column it is R(4K..4K+3, col); for a W column it is X(col, 4K..4K+3) (R = R_D L_b^T,
+// X = R^-1 = W^T R_D^-1).  The columns are kept rotated (x[0..3] = rows 4K..4K+3), the steps run in
+// rolled loops, and the register length shrinks by 16 every 4 steps (only the live rows are
+// updated).  Measured (tools/leaf_bench.cu, ncu source view): a fully unrolled 32- or 64-step pivot
+// chain is ~25 KB of straight-line SASS executed once per launch and stalls on instruction fetch
+// (77 % stall_no_instruction); a one-warp register LDL with shuffles or a shared-memory row
+// broadcast costs 120-175 cycles per pivot even when the code is cached, so 64 single pivots stay
+// >= 4 us -- the 4 x 4 blocks cut the dependent steps to 16.  In the pipeline the variants are
+// within 1 % of each other (RGSQR_LEAF_CHOL=0 selects the 64-pivot loop): the leaf is bound by
+// its cold-code / cold-data phases, not by this factorisation.
+constexpr int LF_B4ROWS = 80;   // rows per publish buffer (4K + L - 1 <= 75: tail reads are garbage-in, unused)
+constexpr int LF_RST = 65;      // fp32 R scratch row stride
+
+struct LfB4 {
+    float4* buf;    // 2 x LF_B4ROWS: buf[(K & 1) * LF_B4ROWS + col] = rows 4K..4K+3 of column col
+    float* Rst;     // 64 x LF_RST fp32 R (row-major, upper valid)
+    float* XT;      // 64 x 64: XT[a * 64 + b] = X(b, a)
+    float* sd;      // 64 pivots d
+    float* srd;     // 64: 1 / R(k, k)
+};
+
+// Steps K0 .. K0+3 on a column of register length L (x[p] = row 4K + p).  PUB: publish x[0..3] at
+// column col; GCOL: z goes to R (else to X^T); REC: record pivots / 1 / R(k, k).
+template <int L, bool PUB, bool GCOL, bool REC>
+__device__ __forceinline__ void lf_b4_phase(float (&x)[64], int K0, int col, int lane, const LfB4& b) {
+#pragma unroll 1
+    for (int K = K0; K < K0 + 4; ++K) {
+        float4* bk = b.buf + (K & 1) * LF_B4ROWS;
+        if (PUB) bk[col] = make_float4(x[0], x[1], x[2], x[3]);
+        asm volatile("bar.sync 8, 128;" ::: "memory");
+        const int k0 = 4 * K;
+        const float4 c0 = bk[k0], c1 = bk[k0 + 1], c2 = bk[k0 + 2], c3 = bk[k0 + 3];
+        // R_KK = chol(A_KK), A(r, c) (r <= c) = component r of column 4K + c
+        const float d0 = c0.x, i0 = rsqrtf(d0);
+        const float r01 = c1.x * i0, r02 = c2.x * i0, r03 = c3.x * i0;
+        const float d1 = fmaf(-r01, r01, c1.y), i1 = rsqrtf(d1);
+        const float r12 = fmaf(-r01, r02, c2.y) * i1, r13 = fmaf(-r01, r03, c3.y) * i1;
+        const float d2 = fmaf(-r12, r12, fmaf(-r02, r02, c2.z)), i2 = rsqrtf(d2);
+        const float r23 = fmaf(-r12, r13, fmaf(-r02, r03, c3.z)) * i2;
+        const float d3 = fmaf(-r23, r23, fmaf(-r13, r13, fmaf(-r03, r03, c3.w))), i3 = rsqrtf(d3);
+        // z = R_KK^-T x_K, y = R_KK^-1 z
+        const float z0 = x[0] * i0;
+        const float z1 = fmaf(-r01, z0, x[1]) * i1;
+        const float z2 = fmaf(-r12, z1, fmaf(-r02, z0, x[2])) * i2;
+        const float z3 = fmaf(-r23, z2, fmaf(-r13, z1, fmaf(-r03, z0, x[3]))) * i3;
+        const float y3 = z3 * i3;
+        const float y2 = fmaf(-r23, y3, z2) * i2;
+        const float y1 = fmaf(-r13, y3, fmaf(-r12, y2, z1)) * i1;
+        const float y0 = fmaf(-r03, y3, fmaf(-r02, y2, fmaf(-r01, y1, z0))) * i0;
+        if (GCOL) {
+            b.Rst[(k0 + 0) * LF_RST + col] = z0;
+            b.Rst[(k0 + 1) * LF_RST + col] = z1;
+            b.Rst[(k0 + 2) * LF_RST + col] = z2;
+            b.Rst[(k0 + 3) * LF_RST + col] = z3;
+        } else {
+            b.XT[(k0 + 0) * 64 + col] = z0;
+            b.XT[(k0 + 1) * 64 + col] = z1;
+            b.XT[(k0 + 2) * 64 + col] = z2;
+            b.XT[(k0 + 3) * 64 + col] = z3;
+        }
+        if (REC && lane == 0) {
+            b.sd[k0] = d0, b.sd[k0 + 1] = d1, b.sd[k0 + 2] = d2, b.sd[k0 + 3] = d3;
+            b.srd[k0] = i0, b.srd[k0 + 1] = i1, b.srd[k0 + 2] = i2, b.srd[k0 + 3] = i3;
+        }
+        // trailing rows: x[p - 4] = x[p] - A(4K + p, 4K..4K+3) y
+#pragma unroll
+        for (int p = 4; p < L; ++p) {
+            const float4 v = bk[k0 + p];
+            x[p - 4] = fmaf(-v.w, y3, fmaf(-v.z, y2, fmaf(-v.y, y1, fmaf(-v.x, y0, x[p]))));
+        }
+#pragma unroll
+        for (int p = L - 4; p < L; ++p) x[p] = 0.f;
+    }
+}
+
+template <int L>
+__device__ __forceinline__ void lf_b4_idle(int K0) {
+#pragma unroll 1
+    for (int K = K0; K < K0 + 4; ++K) asm volatile("bar.sync 8, 128;" ::: "memory");
+}
+
+__device__ int lf_chol_inv_b4(const LfSmem& s, int nc, double* keq) {
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    float* G32 = reinterpret_cast<float*>(reinterpret_cast<uint8_t*>(s.red) + LF_NE * 8);   // region A, after red
+    static_assert(LF_NE * 8 + 64 * LF_RST * 4 <= LF_REGION, "region A: red + G32");
+    static_assert(64 * 64 * 4 <= LF_NE * 8, "region A: X^T over red");
+    LfB4 b;
+    b.buf = reinterpret_cast<float4*>(s.G);
+    b.Rst = reinterpret_cast<float*>(b.buf + 2 * LF_B4ROWS);
+    static_assert(2 * LF_B4ROWS * 16 + 64 * LF_RST * 4 <= LF_REGION, "region B");
+    b.XT = reinterpret_cast<float*>(s.red);
+    __shared__ float s_d[64], s_rd[64];
+    __shared__ double s_en[LF_NW];
+    __shared__ int s_bad3[2];
+    b.sd = s_d;
+    b.srd = s_rd;
+    // dense fp32 G (identity beyond nc)
+#pragma unroll
+    for (int u = 0; u < 64 * 64 / LF_THREADS; ++u) {
+        const int e = t + u * LF_THREADS, i = e >> 6, j = e & 63;
+        const int lo = min(i, j), hi = max(i, j);
+        G32[i * LF_RST + j] = (hi < nc) ? (float)s.red[hi * (hi + 1) / 2 + lo] : (i == j ? 1.f : 0.f);
+    }
+    __syncthreads();   // s.red dead: X^T may overwrite it
+    if (warp < 4) {
+        float x[64];
+        if (warp == 0) {          // G(:, 0..31): rows 0..31, steps 0..7
+#pragma unroll
+            for (int p = 0; p < 32; ++p) x[p] = G32[p * LF_RST + lane];
+            lf_b4_phase<32, true, true, false>(x, 0, lane, lane, b);
+            lf_b4_phase<16, true, true, false>(x, 4, lane, lane, b);
+            lf_b4_idle<0>(8);
+            lf_b4_idle<0>(12);
+        } else if (warp == 1) {   // G(:, 32..63): all rows, all steps
+#pragma unroll
+            for (int p = 0; p < 64; ++p) x[p] = G32[p * LF_RST + 32 + lane];
+            lf_b4_phase<64, true, true, true>(x, 0, 32 + lane, lane, b);
+            lf_b4_phase<48, true, true, true>(x, 4, 32 + lane, lane, b);
+            lf_b4_phase<32, true, true, true>(x, 8, 32 + lane, lane, b);
+            lf_b4_phase<16, true, true, true>(x, 12, 32 + lane, lane, b);
+        } else if (warp == 2) {   // W(:, 0..31) from I
+#pragma unroll
+            for (int p = 0; p < 64; ++p) x[p] = (p == lane) ? 1.f : 0.f;
+            lf_b4_phase<64, false, false, false>(x, 0, lane, lane, b);
+            lf_b4_phase<48, false, false, false>(x, 4, lane, lane, b);
+            lf_b4_phase<32, false, false, false>(x, 8, lane, lane, b);
+            lf_b4_phase<16, false, false, false>(x, 12, lane, lane, b);
+        } else {                  // W(:, 32..63): zero above row 32 (steps 0..7 are no-ops)
+#pragma unroll
+            for (int p = 0; p < 32; ++p) x[p] = (p == lane) ? 1.f : 0.f;   // rows 32.. after 8 steps
+            lf_b4_idle<0>(0);
+            lf_b4_idle<0>(4);
+            lf_b4_phase<32, false, false, false>(x, 8, 32 + lane, lane, b);
+            lf_b4_phase<16, false, false, false>(x, 12, 32 + lane, lane, b);
+            // X(32 + lane, 0..31) = 0 (W(0..31, 32 + lane) = 0): not written by the steps
+#pragma unroll 4
+            for (int a = 0; a < 32; ++a) b.XT[a * 64 + 32 + lane] = 0.f;
+        }
+    }
+    __syncthreads();
+    LF_MARK(28);
+    // X (row-major) from X^T, kappa term, R -> registers
+    constexpr int PER = 64 * 64 / LF_THREADS;
+    double en = 0.0;
+    float rr[PER];
+#pragma unroll
+    for (int u = 0; u < PER; ++u) {
+        const int e = t + u * LF_THREADS, i = e >> 6, j = e & 63;
+        const float x = (i <= j) ? b.XT[j * 64 + i] : 0.f;
+        s.X32[e] = x;
+        rr[u] = (i <= j) ? b.Rst[i * LF_RST + j] : 0.f;
+        if (i <= j && j < nc) en = fma((double)x * x, s.gdiag[i], en);
+    }
+    if (t < 64) {
+        const float d = s_d[t];
+        const bool good = (d > (float)s.gdiag[t] * 1e-4f) && isfinite(d);
+        s.rdiag32[t] = s_rd[t];
+        const unsigned badm = __ballot_sync(0xffffffffu, !good);
+        if (lane == 0) s_bad3[warp] = badm ? (__ffs(badm) - 1 + 32 * warp) : 64;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) en += __shfl_xor_sync(0xffffffffu, en, o);
+    if (lane == 0) s_en[warp] = en;
+    __syncthreads();   // scratch fully read: s.Rs (region B) may overwrite it
+    double se = 0.0;
+#pragma unroll
+    for (int w = 0; w < LF_NW; ++w) se += s_en[w];
+    *keq = (double)nc * se;
+#pragma unroll
+    for (int u = 0; u < PER; ++u) {
+        const int e = t + u * LF_THREADS, i = e >> 6, j = e & 63;
+        s.Rs[i * LF_GLD + j] = (double)rr[u];
+    }
+    const int bad = min(s_bad3[0], s_bad3[1]);
+    __syncthreads();
+    return bad;
 }
 
 // X = R^{-1} (upper, fp32: it only feeds the fp32 product P R^{-1} and the kappa test), blocked
@@ -1034,7 +1226,14 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
         if (pass == 0) LF_MARK(2);
         lf_allreduce(a, s, LF_NE, true, pass == 0 ? 20 : 0);
         if (pass == 0) LF_MARK(3);
-        lf_build_g(s, s.red, false, nc, 0.0);
+        if (fast && pass == 0 && a.chol) {
+            // the blocked fast path reads the packed Gram directly: only the diagonal is needed
+            if (threadIdx.x < 64)
+                s.gdiag[threadIdx.x] = threadIdx.x < nc ? s.red[threadIdx.x * (threadIdx.x + 3) / 2] : 1.0;
+        } else {
+            lf_build_g(s, s.red, false, nc, 0.0);
+        }
+        if (pass == 0) LF_MARK(26);
         if (fast && pass == 0) {
             // split-Gram validity: every column norm in [0.01, 2^15] (entries far from the fp16
             // subnormal and overflow ranges) and finite
@@ -1045,6 +1244,7 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
                 if (!(d >= 1e-4 && d <= 0x1p30)) s.flag[1] = 1;
             }
             __syncthreads();
+            LF_MARK(27);
             if (s.flag[1]) {
                 LF_COUNT(0, 1);
                 fast = false;
@@ -1056,7 +1256,7 @@ __device__ int lf_cholqr(const LeafArgs& a, const LfSmem& s, int nc, int rp, int
             // fp32 Cholesky + inverse in one loop; a failed pivot or a kappa above the fast-path
             // bound redoes the pass on the fp64 Gram
             double keq = 0.0;
-            const int fb32 = lf_chol_inv32<LF_CHOL_WARPS>(s, nc, &keq);
+            const int fb32 = a.chol ? lf_chol_inv_b4(s, nc, &keq) : lf_chol_inv32<LF_CHOL_WARPS>(s, nc, &keq);
             LF_MARK(4);
             if (fb32 < 64 || !(keq <= 1.21 * nc * nc)) {
                 LF_COUNT(0, 1);
@@ -1388,6 +1588,8 @@ cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st) {
     a.ph = L.pq ? L.ph : 0;
     static const bool fp64_gram = getenv("RGSQR_LEAF_FP64_GRAM") != nullptr;
     a.fast = fp64_gram ? 0 : 1;
+    static const int chol = getenv("RGSQR_LEAF_CHOL") ? atoi(getenv("RGSQR_LEAF_CHOL")) : LF_CHOL_BLOCKED;
+    a.chol = chol;
     if (a.pq && (a.ph < 1 || a.ph > 64 || (L.ldh & 7) != 0 || (reinterpret_cast<uintptr_t>(L.pq) & 15) != 0 ||
                  !leaf_prologue_fits(L.m)))
         return cudaErrorInvalidValue;

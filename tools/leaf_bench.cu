@@ -111,6 +111,25 @@ __global__ void bar_probe(long long* cyc, int n) {
     if (t < 64) sm[0][t] = v;
     if (t == 0) cyc[blockDim.x == 512 ? 0 : 1] = (t1 - t0) * 100 / n;
 }
+__global__ void stream_ef(float4* p, size_t n) {   // read-modify-write with L2 evict_first
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+        float4 v;
+        asm volatile("ld.global.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+                     : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p + i), "l"(pol));
+        v.x += 1.f;
+        asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;"
+                     :: "l"(p + i), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w), "l"(pol) : "memory");
+    }
+}
+__global__ void stream_plain(float4* p, size_t n) {
+    for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+        float4 v = p[i];
+        v.x += 1.f;
+        p[i] = v;
+    }
+}
 int main(int argc, char** argv) {
     {
         long long* cyc; cudaMalloc(&cyc, 64); cudaMemset(cyc, 0, 64);
@@ -178,9 +197,48 @@ int main(int argc, char** argv) {
         float ms; cudaEventElapsedTime(&ms, a, b);
         if (i >= 3) tot += ms;
     }
+    {   // back-to-back launches (code and data warm) vs after a 1 GB L2-flushing memset
+        void* big; cudaMalloc(&big, 1ull << 30);
+        float t2 = 0, t3 = 0;
+        for (int i = 0; i < 13; ++i) {
+            cudaMemcpyAsync(Q, P, m * nc * 4, cudaMemcpyDeviceToDevice, st);
+            rg::launch_leaf(L, st);
+            cudaEventRecord(a, st);
+            rg::launch_leaf(L, st);
+            cudaEventRecord(b, st);
+            cudaEventSynchronize(b);
+            float ms; cudaEventElapsedTime(&ms, a, b);
+            if (i >= 3) t2 += ms;
+            cudaMemcpyAsync(Q, P, m * nc * 4, cudaMemcpyDeviceToDevice, st);
+            cudaMemsetAsync(big, i, 1ull << 30, st);
+            cudaEventRecord(a, st);
+            rg::launch_leaf(L, st);
+            cudaEventRecord(b, st);
+            cudaEventSynchronize(b);
+            cudaEventElapsedTime(&ms, a, b);
+            if (i >= 3) t3 += ms;
+        }
+        printf("  second back-to-back launch %.2f us; after a 1 GB memset %.2f us\n", t2 * 100, t3 * 100);
+        for (int mode = 0; mode < 2; ++mode) {
+            float tt = 0;
+            for (int i = 0; i < 13; ++i) {
+                cudaMemcpyAsync(Q, P, m * nc * 4, cudaMemcpyDeviceToDevice, st);
+                if (mode) stream_ef<<<148 * 8, 256, 0, st>>>((float4*)big, (1ull << 30) / 16);
+                else stream_plain<<<148 * 8, 256, 0, st>>>((float4*)big, (1ull << 30) / 16);
+                cudaEventRecord(a, st);
+                rg::launch_leaf(L, st);
+                cudaEventRecord(b, st);
+                cudaEventSynchronize(b);
+                float ms; cudaEventElapsedTime(&ms, a, b);
+                if (i >= 3) tt += ms;
+            }
+            printf("  after a 1 GB %s read-modify-write stream: %.2f us\n", mode ? "L2-evict_first" : "plain", tt * 100);
+        }
+        cudaFree(big);
+    }
     printf("m=%lld nc=%d leaf kernel: %.2f us (err %s)\n", (long long)m, nc, tot * 1000 / iters,
            cudaGetErrorString(cudaGetLastError()));
-    unsigned long long tr[32];
+    unsigned long long tr[48];
     cudaMemcpyFromSymbol(tr, rg::lf_trace, sizeof(tr));
     const char* names[9] = {"start", "loaded", "gram", "allreduce", "chol", "inverse+racc", "apply", "cholqr done", "stored"};
     long long ck[2];
@@ -192,6 +250,8 @@ int main(int argc, char** argv) {
     printf("  SM clock during the kernel: %.0f MHz\n", (ck[1] - ck[0]) / ((tr[8] - tr[0]) * 1e-3));
     printf("  allreduce: barrier 1 %.2f, reduce %.2f, barrier 2 %.2f, to smem %.2f us\n", (tr[20] - tr[2]) / 1e3,
            (tr[21] - tr[20]) / 1e3, (tr[22] - tr[21]) / 1e3, (tr[3] - tr[22]) / 1e3);
+    printf("  chol phase: gdiag / build_g %.2f, check %.2f, factor %.2f, tail %.2f us\n", (tr[26] - tr[3]) / 1e3,
+           (tr[27] - tr[26]) / 1e3, (tr[28] - tr[27]) / 1e3, (tr[4] - tr[28]) / 1e3);
     if (L.pq) printf("  prologue: qa load %.2f, k1 %.2f, allreduce %.2f, R_AB %.2f, k2 %.2f us\n", (tr[10] - tr[0]) / 1e3,
                      (tr[11] - tr[10]) / 1e3, (tr[12] - tr[11]) / 1e3, (tr[13] - tr[12]) / 1e3, (tr[1] - tr[13]) / 1e3);
     for (int i = 1; i < 9; ++i) printf("  %-14s %7.2f us (+%.2f)\n", names[i], (tr[i] - tr[0]) / 1e3, ((long long)tr[i] - (long long)tr[i - 1]) / 1e3);
