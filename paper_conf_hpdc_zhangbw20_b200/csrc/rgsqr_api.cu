@@ -715,7 +715,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
         if (!pp || cend - pp->copied <= 0 || (!flush && cend - pp->copied < 256)) return RG_OK;
         // R(:, j) is final once column j's panel has run too (eq 6: R12 blocks of column j come
         // from K1s of levels where j lies in A2, all enqueued before that panel)
-        RG_CUDA(rg::launch_unscale_r(pl.R, pl.ldr, n, pl.scale ? h->scale.as<float>() : nullptr, st, pp->copied,
+        RG_CUDA(rg::launch_unscale_r(pl.R, pl.ldr, n, pl.scale > 0 ? h->scale.as<float>() : nullptr, st, pp->copied,
                                      cend - pp->copied));
         RG_CUDA(cudaEventRecord(pp->ev, st));
         RG_CUDA(cudaStreamWaitEvent(pp->cs_out, pp->ev, 0));
@@ -730,6 +730,12 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     };
     int panel_end = 0;   // columns left of this have had their panel enqueued
     if (pp) {
+        RG_CUDA(cudaMemset2DAsync(pl.R, pl.ldr * sizeof(float), 0, n * sizeof(float), n, st));
+    } else if (pl.scale < 0) {
+        // reorthogonalisation pass (reading #32): the input is the previous pass's Q, in place and
+        // unscaled -- no norm pass, no fp32 copy; only the 16-bit images are written
+        ProfScope _s(h, PC_SCALE, 0, (double)m * n * (pl.split ? 8 : 6));
+        RG_CUDA(rg::launch_scale_cast(pl.A, pl.lda, nullptr, 0, qh, ql, pl.ldh, m, n, nullptr, pl.bf16, st));
         RG_CUDA(cudaMemset2DAsync(pl.R, pl.ldr * sizeof(float), 0, n * sizeof(float), n, st));
     } else {
         ProfScope _s(h, PC_SCALE, 0, (double)m * n * (pl.split ? 16 : 14));
@@ -942,7 +948,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
     }
     {
         ProfScope _s(h, PC_OTHER);
-        RG_CUDA(rg::launch_unscale_r(pl.R, pl.ldr, n, pl.scale ? h->scale.as<float>() : nullptr, st));
+        RG_CUDA(rg::launch_unscale_r(pl.R, pl.ldr, n, pl.scale > 0 ? h->scale.as<float>() : nullptr, st));
     }
     return RG_OK;
 }
@@ -981,6 +987,7 @@ int check_status(rg_handle h) {
 int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq, float* R,
               int64_t ldr, const rg_opts& o, int split, bool local = false, HostPipe* pipe = nullptr) {
     if (!ensure_workspace(h, m, n, split)) return RG_ALLOC;
+    if (o.scale < 0 && (A != Q || lda != ldq || pipe)) return RG_CUDA_ERROR;   // reortho form: in place only
     const int nb = (o.nb <= 0 || o.nb > 32) ? 32 : o.nb;
     const int nranks = local ? 1 : h->nranks;
     Plan* pl = nullptr;
@@ -1103,7 +1110,9 @@ int factor_with_reortho(rg_handle h, int64_t m, int64_t n, const float* A, int64
         float* R2 = h->lsR.as<float>();
         // reading #8: for the CGLS preconditioner a plain 16-bit reortho pass suffices (kappa(A R^-1)
         // ~ 1.8 either way, SURVEY [EMU]); split precision only when the caller asks (opts.split)
-        rc = run_rgsqr(h, m, n, Q, ldq, Q, ldq, R2, n, o, o.split);
+        rg_opts o2 = o;
+        o2.scale = -1;   // in place, unscaled (reading #32)
+        rc = run_rgsqr(h, m, n, Q, ldq, Q, ldq, R2, n, o2, o.split);
         if (rc) return rc;
         rc = trmm_into(h, R2, n, R, ldr, (int)n);
     }
@@ -1620,6 +1629,7 @@ int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A, int64_
     if (!h) return -1;
     rg_opts o;
     if (opts) o = *opts; else rg_opts_default(&o);
+    o.scale = o.scale ? 1 : 0;   // (-1 is the internal in-place reortho form)
     if (m_local < 1 || (h->nranks <= 1 && m_local < n)) return -2;
     if (n < 1 || n > 65535) return -3;
     if (!A) return -4;
@@ -1697,6 +1707,7 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
     if (!h) return -1;
     rg_opts o;
     if (opts) o = *opts; else rg_opts_default(&o);
+    o.scale = o.scale ? 1 : 0;   // (-1 is the internal in-place reortho form)
     if (m_local < 1 || (h->nranks <= 1 && m_local < n)) return -2;
     if (n < 1 || n > 65535) return -3;
     if (!A) return -4;
@@ -1737,7 +1748,9 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
         // [Q2, R2] = RGSQR(Q) with split-precision GEMMs (reading #9); R <- R2 R
         if (!h->lsR.ensure((size_t)n * n * 4 + 256)) return RG_ALLOC;
         float* R2 = h->lsR.as<float>();
-        rc = run_rgsqr(h, m_local, n, dA, dlda, dA, dlda, R2, n, o, 1);
+        rg_opts o2 = o;
+        o2.scale = -1;   // in place, unscaled (reading #32)
+        rc = run_rgsqr(h, m_local, n, dA, dlda, dA, dlda, R2, n, o2, 1);
         if (rc) break;
         rc = trmm_into(h, R2, n, dR, n, (int)n);
         ++passes;
@@ -1768,6 +1781,7 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     if (!h) return -1;
     rg_opts o;
     if (opts) o = *opts; else rg_opts_default(&o);
+    o.scale = o.scale ? 1 : 0;   // (-1 is the internal in-place reortho form)
     if (m_local < 1 || (h->nranks <= 1 && m_local < n)) return -2;
     if (n < 1 || n > 16384) return -3;
     if (!A) return -4;
@@ -1927,6 +1941,7 @@ int lowrank_approx(rg_handle h, int64_t m_local, int64_t n, const float* A, int6
     if (!h) return -1;
     rg_opts o;
     if (opts) o = *opts; else rg_opts_default(&o);
+    o.scale = o.scale ? 1 : 0;   // (-1 is the internal in-place reortho form)
     if (m_local < 1) return -2;
     if (n < 1 || n > 65535) return -3;
     if (!A) return -4;
@@ -2065,6 +2080,7 @@ int lowrank_qrsvd(rg_handle h, int64_t m_local, int64_t n, const float* A, int64
     if (!h) return -1;
     rg_opts o;
     if (opts) o = *opts; else rg_opts_default(&o);
+    o.scale = o.scale ? 1 : 0;   // (-1 is the internal in-place reortho form)
     if (m_local < 1 || (h->nranks <= 1 && m_local < n)) return -2;
     if (n < 1 || n > 4096) return -3;
     if (!A) return -4;

@@ -110,7 +110,7 @@ __global__ void __launch_bounds__(256) scale_cast_kernel(const float* __restrict
     uint16_t* qh = Qh ? Qh + (int64_t)j * ldh : nullptr;
     uint16_t* ql = Ql ? Ql + (int64_t)j * ldh : nullptr;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    const bool vec = ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(q)) & 15) == 0 && q &&
+    const bool vec = ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(q)) & 15) == 0 &&
                      (!qh || (reinterpret_cast<uintptr_t>(qh) & 7) == 0) &&
                      (!ql || (reinterpret_cast<uintptr_t>(ql) & 7) == 0);
     if (vec) {
@@ -118,7 +118,7 @@ __global__ void __launch_bounds__(256) scale_cast_kernel(const float* __restrict
         for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < nv; v += stride) {
             float4 x = reinterpret_cast<const float4*>(a)[v];
             x.x *= s; x.y *= s; x.z *= s; x.w *= s;
-            reinterpret_cast<float4*>(q)[v] = x;
+            if (q) reinterpret_cast<float4*>(q)[v] = x;
             if (qh) {
                 ushort4 h;
                 h.x = s_to16(x.x, bf16); h.y = s_to16(x.y, bf16); h.z = s_to16(x.z, bf16); h.w = s_to16(x.w, bf16);
@@ -135,7 +135,7 @@ __global__ void __launch_bounds__(256) scale_cast_kernel(const float* __restrict
         }
         for (int64_t i = nv * 4 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += stride) {
             const float x = a[i] * s;
-            q[i] = x;
+            if (q) q[i] = x;
             if (qh) {
                 const uint16_t h = s_to16(x, bf16);
                 qh[i] = h;
