@@ -26,6 +26,7 @@
 #include <cstring>
 #include <memory>
 #include <string>
+#include <functional>
 #include <vector>
 
 #include "../../include/rgsqr.h"
@@ -159,7 +160,11 @@ struct Op {
     CUtensorMap mc;        // UPDATE: fp32 A2 for the TMA epilogue
     bool te = false;
     int h0 = 0;            // UPDATE: first output column whose 16-bit image a later K1 reads
+    int a0 = -1;           // PROJ/UPDATE: first A2 column when not c0 + h (a column chunk of a level)
+    int ref_w = 0;         // PROJ chunk: width of the whole level (its split-K decomposition is kept)
 };
+// first column of A2 (PROJ / UPDATE)
+static inline int op_a2(const Op& o) { return o.a0 >= 0 ? o.a0 : o.c0 + o.h; }
 
 // Host-pointer pipeline of rgsqr_factor (pinned host A/Q/R, one pass, one rank): A arrives in
 // column chunks on a copy stream and each chunk is scaled (section 3.5) just before the first op
@@ -185,6 +190,7 @@ struct Plan {
     float* Q = nullptr;
     float* R = nullptr;
     int nb = 0, bf16 = 0, split = 0, scale = 1, nranks = 1, rank = 0, panel = 0;
+    int lazy = 0;   // > 0: column-lazy schedule with this chunk width (host-pointer pipeline)
     bool leaf = false;       // last level runs as leaf.cu kernels
     int epoch = -1;          // handle allocation epoch the plan was built against
     // derived
@@ -503,7 +509,65 @@ const auto& ops = pl.ops;
 const Op& o = ops[oi];
 return pl.leaf && !no_fold64 && rg::leaf_prologue_fits(pl.m) && o.kind == Op::PROJ && o.h <= 64 && o.w <= 64 &&
        oi + 2 < ops.size() && ops[oi + 1].kind == Op::UPDATE && ops[oi + 1].c0 == o.c0 &&
-       ops[oi + 2].kind == Op::PAIR && ops[oi + 2].c0 == o.c0 + o.h && ops[oi + 2].h + ops[oi + 2].w == o.w;
+       ops[oi + 2].kind == Op::PAIR && ops[oi + 2].c0 == o.c0 + o.h && ops[oi + 2].h + ops[oi + 2].w == o.w &&
+       o.a0 < 0;
+}
+
+// Column-lazy schedule of the recursion for the host-pointer pipeline: the K1 / K2 pair of every
+// level wider than C is applied to its A2 in C-column chunks, each chunk just before the first op
+// that touches those columns (and after every earlier level's chunks on them), instead of all at
+// once.  Per column the updates are the same, in the same order (Alg 1's recursion); what changes is
+// only when they run -- so the factorization can follow the column-chunked H2D of A instead of
+// waiting for the whole right half before the top level's K1 (the e2e bound of the eager order:
+// H2D(A) + D2H(right half of Q)).
+void lazy_schedule(std::vector<Op>& ops, int C) {
+    struct Pend {
+        Op proj;
+        std::vector<char> done;
+    };
+    std::vector<Pend> pend;
+    std::vector<Op> out;
+    out.reserve(ops.size() * 2);
+    std::function<void(int, int, size_t)> flush = [&](int x0, int x1, size_t upto) {
+        for (size_t r = 0; r < upto && r < pend.size(); ++r) {
+            Pend& p = pend[r];
+            const int a = op_a2(p.proj);
+            for (size_t k = 0; k < p.done.size(); ++k) {
+                const int s0 = a + (int)k * C, s1 = std::min(a + p.proj.w, s0 + C);
+                if (p.done[k] || s1 <= x0 || s0 >= x1) continue;
+                flush(s0, s1, r);   // earlier levels first on these columns
+                p.done[k] = 1;
+                Op pr = p.proj;
+                pr.a0 = s0;
+                pr.w = s1 - s0;
+                pr.ref_w = p.proj.w;
+                out.push_back(pr);
+                Op up = pr;
+                up.kind = Op::UPDATE;
+                up.ref_w = 0;
+                out.push_back(up);
+            }
+        }
+    };
+    for (size_t i = 0; i < ops.size(); ++i) {
+        const Op& o = ops[i];
+        if (o.kind == Op::PROJ && o.w > C) {
+            Pend p;
+            p.proj = o;
+            p.done.assign((size_t)((o.w + C - 1) / C), 0);
+            pend.push_back(p);
+            ++i;   // its UPDATE
+            continue;
+        }
+        int x0, x1;
+        if (o.kind == Op::PANEL) x0 = o.c0, x1 = o.c0 + o.w;
+        else if (o.kind == Op::PAIR) x0 = o.c0, x1 = o.c0 + o.h + o.w;
+        else x0 = op_a2(o), x1 = op_a2(o) + o.w;
+        flush(x0, x1, pend.size());
+        out.push_back(o);
+    }
+    flush(0, INT_MAX, pend.size());
+    ops.swap(out);
 }
 
 int make_plan(rg_handle h, Plan& pl) {
@@ -526,6 +590,7 @@ int make_plan(rg_handle h, Plan& pl) {
                       (wide ? rg::cholqr_fused_fits(m, 64) : (rg::leaf_fits(m) && !pl.split));
     pl.leaf = pair && !wide;
     build_ops(pl.ops, 0, n, pl.nb, pair, pl.leaf);
+    if (pl.lazy > 0) lazy_schedule(pl.ops, pl.lazy);
     // 16-bit images written by K2 that nothing reads: a column's image is read only as A2 of a
     // later K1 before the leaf / panel that factors the column (those read fp32 and write the
     // image of Q).  In leaf mode that drops the image for the first 128 columns of every K2
@@ -536,10 +601,10 @@ int make_plan(rg_handle h, Plan& pl) {
         for (size_t i = 0; i < pl.ops.size(); ++i) {
             const Op& o = pl.ops[i];
             if (o.kind == Op::PROJ && !folded_into_leaf(pl, i)) {   // (a folded prologue reads fp32)
-                for (int c = o.c0 + o.h; c < o.c0 + o.h + o.w; ++c)
+                for (int c = op_a2(o); c < op_a2(o) + o.w; ++c)
                     if (last[c] >= 0) need[last[c]] = std::min(need[last[c]], c);
             } else if (o.kind == Op::UPDATE) {
-                for (int c = o.c0 + o.h; c < o.c0 + o.h + o.w; ++c) last[c] = (int)i;
+                for (int c = op_a2(o); c < op_a2(o) + o.w; ++c) last[c] = (int)i;
             } else {
                 const int c1 = o.kind == Op::PAIR ? o.c0 + o.h + o.w : o.c0 + o.w;
                 for (int c = o.c0; c < c1; ++c) last[c] = -2;
@@ -548,7 +613,7 @@ int make_plan(rg_handle h, Plan& pl) {
         for (size_t i = 0; i < pl.ops.size(); ++i)
             if (pl.ops[i].kind == Op::UPDATE) {
                 Op& o = pl.ops[i];
-                o.h0 = need[i] == INT_MAX ? o.w : std::max(0, need[i] - (o.c0 + o.h));
+                o.h0 = need[i] == INT_MAX ? o.w : std::max(0, need[i] - op_a2(o));
             }
     }
     int max_h = 0, max_w = 0;
@@ -567,16 +632,19 @@ int make_plan(rg_handle h, Plan& pl) {
     for (auto& o : pl.ops) {
         if (o.kind == Op::PANEL || o.kind == Op::PAIR) continue;
         const uint16_t* q1 = qh + (int64_t)o.c0 * pl.ldh;
-        const uint16_t* a2 = qh + (int64_t)(o.c0 + o.h) * pl.ldh;
+        const uint16_t* a2 = qh + (int64_t)op_a2(o) * pl.ldh;
         const uint16_t* q1l = pl.split ? ql + (int64_t)o.c0 * pl.ldh : q1;
-        const uint16_t* a2l = pl.split ? ql + (int64_t)(o.c0 + o.h) * pl.ldh : a2;
+        const uint16_t* a2l = pl.split ? ql + (int64_t)op_a2(o) * pl.ldh : a2;
         o.bn = pick_bn(o.w);
         if (o.kind == Op::UPDATE && getenv("RGSQR_K2_BN")) o.bn = std::min(o.bn, atoi(getenv("RGSQR_K2_BN")));
         if (o.kind == Op::PROJ) {
             o.tiles_i = (o.h + 127) / 128;
             o.tiles_j = (o.w + o.bn - 1) / o.bn;
             o.kb_total = (int)((m + 63) / 64);
-            const int tiles = o.tiles_i * o.tiles_j;
+            // a column chunk of a level keeps the whole level's split-K decomposition (the same
+            // partial sums in the same order: bit-identical R12 / Q to the unchunked plan)
+            const int sw = o.ref_w > 0 ? o.ref_w : o.w, sbn = pick_bn(sw);
+            const int tiles = o.tiles_i * ((sw + sbn - 1) / sbn);
             int splits = 1;
             if (tiles >= 32) {
                 // balance whole waves of 148 persistent CTAs against split-K partial traffic
@@ -602,7 +670,7 @@ int make_plan(rg_handle h, Plan& pl) {
                       encode_map(&o.mb_lo, a2l, m, o.w, pl.ldh, 64, o.bn, bf);
             if (!ok) return RG_CUDA_ERROR;
         } else {
-            o.te = !pl.split && encode_plain(&o.mc, pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq, m, o.w, pl.ldq, 4, bf, 128, 32);
+            o.te = !pl.split && encode_plain(&o.mc, pl.Q + (int64_t)op_a2(o) * pl.ldq, m, o.w, pl.ldq, 4, bf, 128, 32);
             bool ok = encode_map(&o.ma, q1, m, o.h, pl.ldh, 64, 64, bf) &&
                       encode_map(&o.mb, r12h, o.h, o.w, pl.ldr12, 64, o.bn, bf) &&
                       encode_map(&o.ma_lo, q1l, m, o.h, pl.ldh, 64, 64, bf) &&
@@ -755,7 +823,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
         const Op& o = pl.ops[oi];
         if (pp) {
             int rc = pipe_done(panel_end, false);
-            if (!rc) rc = pipe_need(o.c0 + (o.kind == Op::PANEL ? o.w : o.h + o.w));
+            if (!rc) rc = pipe_need(o.kind == Op::PANEL ? o.c0 + o.w : o.kind == Op::PAIR ? o.c0 + o.h + o.w : op_a2(o) + o.w);
             if (rc) return rc;
         }
         if (folded_into_leaf(pl, oi)) {
@@ -764,7 +832,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             continue;
         }
         if (o.kind == Op::UPDATE && !dist && pl.panel == 0 && o.h <= 64 && oi + 1 < pl.ops.size() &&
-            pl.ops[oi + 1].kind == Op::PANEL && pl.ops[oi + 1].c0 == o.c0 + o.h && pl.ops[oi + 1].w == o.w &&
+            pl.ops[oi + 1].kind == Op::PANEL && pl.ops[oi + 1].c0 == o.c0 + o.h && pl.ops[oi + 1].w == o.w && o.a0 < 0 &&
             rg::cholqr_fused_fits(m, 32) && getenv("RGSQR_NO_FOLD") == nullptr) {
             pending_update = &o;
             continue;
@@ -902,13 +970,13 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             }
         } else if (o.kind == Op::PROJ && no_tc) {
             ProfScope _s(h, PC_PROJ, 2.0 * m * o.h * o.w, (double)m * (o.h + o.w) * 4, o.w);
-            RG_CUDA(rg::launch_sgemm_proj(pl.Q + (int64_t)o.c0 * pl.ldq, pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq, pl.ldq, m,
-                                          o.h, o.w, pl.R + o.c0 + (int64_t)(o.c0 + o.h) * pl.ldr, pl.ldr,
+            RG_CUDA(rg::launch_sgemm_proj(pl.Q + (int64_t)o.c0 * pl.ldq, pl.Q + (int64_t)op_a2(o) * pl.ldq, pl.ldq, m,
+                                          o.h, o.w, pl.R + o.c0 + (int64_t)op_a2(o) * pl.ldr, pl.ldr,
                                           h->P.as<float>(), st));
         } else if (o.kind == Op::UPDATE && no_tc) {
             ProfScope _s(h, PC_UPDATE, 2.0 * m * o.h * o.w, (double)m * o.h * 4 + (double)m * o.w * 8, o.w);
-            RG_CUDA(rg::launch_sgemm_update(pl.Q + (int64_t)o.c0 * pl.ldq, pl.R + o.c0 + (int64_t)(o.c0 + o.h) * pl.ldr,
-                                            pl.ldr, pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq, pl.ldq, m, o.h, o.w, st));
+            RG_CUDA(rg::launch_sgemm_update(pl.Q + (int64_t)o.c0 * pl.ldq, pl.R + o.c0 + (int64_t)op_a2(o) * pl.ldr,
+                                            pl.ldr, pl.Q + (int64_t)op_a2(o) * pl.ldq, pl.ldq, m, o.h, o.w, st));
         } else if (o.kind == Op::PROJ) {
             ProfScope _s(h, PC_PROJ, 2.0 * m * o.h * o.w * (pl.split ? 3 : 1),
                              (double)m * (o.h + o.w) * (pl.split ? 4 : 2), o.w);
@@ -917,7 +985,7 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
             const int64_t pstride = ldp * o.tiles_j * o.bn;
             RG_CUDA(rg::launch_proj_gemm(o.bn, pl.split != 0, o.tiles_i, o.tiles_j, o.splits, o.ma, o.mb, o.ma_lo,
                                          o.mb_lo, P, ldp, pstride, o.kb_total, o.kb_per_split, pl.bf16, st));
-            float* Rblk = pl.R + o.c0 + (int64_t)(o.c0 + o.h) * pl.ldr;
+            float* Rblk = pl.R + o.c0 + (int64_t)op_a2(o) * pl.ldr;
             uint16_t* r12l = pl.split ? h->r12l.as<uint16_t>() : nullptr;
             if (!dist) {
                 RG_CUDA(rg::launch_proj_reduce(P, ldp, pstride, o.splits, o.h, o.w, Rblk, pl.ldr, nullptr, 0,
@@ -934,9 +1002,9 @@ int enqueue_rgsqr_impl(rg_handle h, Plan& pl) {
         } else {
             ProfScope _s(h, PC_UPDATE, 2.0 * m * o.h * o.w * (pl.split ? 3 : 1),
                              (double)m * o.h * (pl.split ? 4 : 2) + (double)m * o.w * (pl.split ? 12 : 10), o.w);
-            float* C = pl.Q + (int64_t)(o.c0 + o.h) * pl.ldq;
-            uint16_t* Ch = qh + (int64_t)(o.c0 + o.h) * pl.ldh;
-            uint16_t* Cl = ql ? ql + (int64_t)(o.c0 + o.h) * pl.ldh : nullptr;
+            float* C = pl.Q + (int64_t)op_a2(o) * pl.ldq;
+            uint16_t* Ch = qh + (int64_t)op_a2(o) * pl.ldh;
+            uint16_t* Cl = ql ? ql + (int64_t)op_a2(o) * pl.ldh : nullptr;
             RG_CUDA(rg::launch_update_gemm(o.bn, pl.split != 0, m, o.w, o.h, o.ma, o.mb, o.ma_lo, o.mb_lo, C, pl.ldq, Ch,
                                            Cl, pl.ldh, pl.bf16, st, 0, o.te ? &o.mc : nullptr, o.h0));
         }
@@ -990,12 +1058,14 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
     if (o.scale < 0 && (A != Q || lda != ldq || pipe)) return RG_CUDA_ERROR;   // reortho form: in place only
     const int nb = (o.nb <= 0 || o.nb > 32) ? 32 : o.nb;
     const int nranks = local ? 1 : h->nranks;
+    static const int pipe_chunk = getenv("RGSQR_PIPE_LAZY") ? atoi(getenv("RGSQR_PIPE_LAZY")) : 256;
+    const int lazy = pipe ? pipe_chunk : 0;
     Plan* pl = nullptr;
     for (size_t i = 0; i < h->plans.size(); ++i) {
         Plan* c = h->plans[i].get();
         if (c->m == m && c->n == n && c->lda == lda && c->ldq == ldq && c->ldr == ldr && c->A == A && c->Q == Q &&
             c->R == R && c->nb == nb && c->bf16 == o.precision && c->split == split && c->scale == o.scale &&
-            c->nranks == nranks && c->rank == h->rank && c->panel == o.panel) {
+            c->nranks == nranks && c->rank == h->rank && c->panel == o.panel && c->lazy == lazy) {
             if (c->epoch != h->alloc_epoch) {   // a workspace buffer moved: rebuild this plan
                 if (c->exec) cudaGraphExecDestroy(c->exec);
                 h->plans.erase(h->plans.begin() + i);
@@ -1011,7 +1081,7 @@ int run_rgsqr(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, fl
         np->m = m; np->n = n; np->lda = lda; np->ldq = ldq; np->ldr = ldr;
         np->A = A; np->Q = Q; np->R = R;
         np->nb = nb; np->bf16 = o.precision; np->split = split; np->scale = o.scale;
-        np->nranks = nranks; np->rank = h->rank; np->panel = o.panel;
+        np->nranks = nranks; np->rank = h->rank; np->panel = o.panel; np->lazy = lazy;
         int rc = make_plan(h, *np);
         if (rc) return rc;
         if (!h->P.ensure(np->p_floats * 4 + 4096)) return RG_ALLOC;

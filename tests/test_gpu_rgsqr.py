@@ -289,10 +289,13 @@ def test_rgsqr_invalid_arguments(rg):
     assert L.rgsqr_factor(h.ptr, 20, 10, p, 20, p, 20, p, 9, ctypes.byref(o)) == -9
 
 
-@pytest.mark.parametrize("m,n,pad", [(3000, 96, 0), (5000, 300, 7), (20000, 1000, 0), (4099, 640, 3)])
+@pytest.mark.parametrize("m,n,pad", [(3000, 96, 0), (5000, 300, 7), (20000, 1000, 0), (4099, 640, 3),
+                                     (6000, 1536, 0), (8192, 2048, 5)])
 def test_rgsqr_pinned_host_pipeline(rg, m, n, pad):
     """Pinned host A/Q/R take the pipelined path (column-chunked H2D, chunked scaling, Q columns
-    D2H as their panels finish); per-column scaling and per-column norms make it the same
+    D2H as their panels finish, and the column-lazy schedule: levels wider than 256 columns apply
+    their K1 / K2 in 256-column chunks as the columns arrive -- n >= 640 here); per-column
+    scaling, per-column norms and the chunk's unchanged split-K decomposition make it the same
     arithmetic as the device path, so Q and R must be bit-identical to it."""
     A = synth.gaussian(m, n, seed=synth.SEED_BASE + 31 + n).astype(np.float32)
     Ah = torch.zeros(n, m + pad, dtype=torch.float32, pin_memory=True)
