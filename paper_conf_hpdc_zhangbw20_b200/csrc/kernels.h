@@ -31,6 +31,17 @@ int dev_smem_optin();       // cudaDevAttrMaxSharedMemoryPerBlockOptin
 // size is needed on that device; the attribute is per device context.
 cudaError_t ensure_smem_attr(const void* kernel, size_t bytes);
 
+// ---- tall.cu (one CholQR pass of a tall block, n <= 256, on tcgen05; reading #33)
+size_t tall_ws_bytes();
+double* tall_gram_buffer(void* ws);          // n x n fp64 Gram (allreduced in place when row-sharded)
+int* tall_flag(void* ws);                    // nonzero after a failed pass (X untouched)
+double* tall_kout(void* ws);                 // [kappa_F(R^), first failed pivot]
+cudaError_t launch_tall_gram(const float* X, int64_t ldx, int64_t m, int n, float sig, int bf16, void* ws, double* G,
+                             cudaStream_t st);
+cudaError_t launch_tall_orth(const double* G, int n, double sig, double* out, cudaStream_t st);
+cudaError_t launch_tall_chol_apply(float* X, int64_t ldx, int64_t m, int n, const double* G, double sig_g, float sig_a,
+                                   int bf16, double kappa_max, float* R, int64_t ldr, void* ws, cudaStream_t st);
+
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
                             Args&&... args);

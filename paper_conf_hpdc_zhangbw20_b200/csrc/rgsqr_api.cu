@@ -344,13 +344,14 @@ struct rg_handle_s {
     int64_t cgls_key_mn[3] = {0, 0, 0};
     int cgls_solver = -1;                           // solver the captured block was built for
     DevBuf aux;                                     // misc (orthogonalize / lowrank)
+    DevBuf tallws;                                  // tall CholQR pass (tall.cu)
     DevBuf vscratch;                                // virtual-rank collectives (rank 0 of a group)
     int alloc_epoch = 0;                            // bumped whenever a workspace buffer moves
     std::vector<DevBuf*> bufs() {
         return {&qh, &ql, &P, &r12h, &r12l, &r12f, &partial, &norm2, &scale, &status, &pws, &pcnt,
                 &rgather, &rstackq, &stageA, &stageQ, &stageR, &stageB, &stageX, &cg, &aux, &lsQ, &lsR, &rinv,
                 &probeG, &probeW, &cq_ws, &cq_flags, &leaf_bar, &lrA16, &lrB16, &lrB16l, &lrY, &lrZ, &lrQ16,
-                &lrQ16l, &lrR, &lrW, &lrV, &lrUb, &lrVb, &lrSig, &lrOm, &lrScale, &lrFlags, &vscratch};
+                &lrQ16l, &lrR, &lrW, &lrV, &lrUb, &lrVb, &lrSig, &lrOm, &lrScale, &lrFlags, &vscratch, &tallws};
     }
     void bind_bufs() {
         for (DevBuf* b : bufs()) {
@@ -1166,6 +1167,61 @@ int orth_estimate(rg_handle h, const float* Q, int64_t ldq, int64_t m, int n, do
     return RG_OK;
 }
 
+// One tall CholQR pass (tall.cu, reading #33) in place on X (m_local x n, n <= 256): Gram on the
+// tensor cores (+ allreduce of the n x n Gram when row-sharded), Cholesky / inverse / kappa test,
+// X <- X R^-1; Rp (n x n, ld ldrp) = R.  *ok = false (X untouched) when the Cholesky broke down or
+// kappa_F of the equilibrated R exceeds 32 n: the caller falls back to an RGSQR pass.
+// first: the pass over the user's A (bf16 split, no column scaling needed); otherwise a
+// reorthogonalisation pass over unit columns (fp16 split at scale 2^14).
+bool tall_wanted(rg_handle h, int64_t m_local, int64_t n, const float* X, int64_t ldx) {
+    const char* e = getenv("RGSQR_TALL");
+    if (e && e[0] == '0') return false;
+    (void)X;
+    (void)ldx;
+    if (n < 1 || n > 256) return false;
+    if (e && e[0] == '1') return true;
+    return !rg::leaf_fits(m_local) && m_local >= 4 * n;
+}
+// Gram of X (tall.cu) into the workspace's G, allreduced when row-sharded.  first: the pass over
+// the user's A (bf16 split, no column scaling needed); otherwise unit columns (fp16 split, 2^14).
+constexpr float kTallSig = 16384.0f;
+int tall_gram(rg_handle h, int64_t m, int n, const float* X, int64_t ldx, bool first) {
+    if (!h->tallws.ensure(rg::tall_ws_bytes())) return RG_ALLOC;
+    double* G = rg::tall_gram_buffer(h->tallws.p);
+    RG_CUDA(rg::launch_tall_gram(X, ldx, m, n, first ? 1.0f : kTallSig, first ? 1 : 0, h->tallws.p, G, h->stream));
+    return nccl_allreduce(h, G, (size_t)n * n, ncclFloat64);
+}
+// ||I - X^T X||_F from the Gram just formed by tall_gram(first = false) (synchronous)
+int tall_orth(rg_handle h, int n, double* est) {
+    double* G = rg::tall_gram_buffer(h->tallws.p);
+    double* out = rg::tall_kout(h->tallws.p) + 2;
+    RG_CUDA(rg::launch_tall_orth(G, n, (double)kTallSig, out, h->stream));
+    RG_CUDA(cudaMemcpyAsync(est, out, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    RG_CUDA(cudaStreamSynchronize(h->stream));
+    return RG_OK;
+}
+// Cholesky / inverse / kappa test of the Gram from tall_gram, then X <- X R^-1 in place and
+// Rp (n x n, ld ldrp) = R.  *ok = false (X untouched) when the Cholesky broke down or kappa_F of the
+// equilibrated R exceeds 32 n: the caller falls back to an RGSQR pass.
+int tall_chol_apply(rg_handle h, int64_t m, int n, float* X, int64_t ldx, float* Rp, int64_t ldrp, bool first,
+                    bool* ok) {
+    void* ws = h->tallws.p;
+    const float sig = first ? 1.0f : kTallSig;
+    RG_CUDA(rg::launch_tall_chol_apply(X, ldx, m, n, rg::tall_gram_buffer(ws), (double)sig, sig, first ? 1 : 0,
+                                       32.0 * n, Rp, ldrp, ws, h->stream));
+    int flag = 0;
+    RG_CUDA(cudaMemcpyAsync(&flag, rg::tall_flag(ws), sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    RG_CUDA(cudaStreamSynchronize(h->stream));
+    *ok = flag == 0;
+    if (getenv("RGSQR_TALL_DEBUG")) {
+        double k[2] = {0, 0};
+        RG_CUDA(cudaMemcpy(k, rg::tall_kout(ws), sizeof(k), cudaMemcpyDeviceToHost));
+        fprintf(stderr, "[tall] m=%lld n=%d first=%d flag=%d kappa_F=%.4g (limit %.4g) pivot=%g\n", (long long)m, n,
+                (int)first, flag, k[0], 32.0 * n, k[1]);
+    }
+    return RG_OK;
+}
+
 // run RGSQR + `extra` reorthogonalisation passes (16-bit; split precision with opts.split) for the
 // least-squares preconditioner; Q (ldq) and R (ldr) outputs
 int factor_with_reortho(rg_handle h, int64_t m, int64_t n, const float* A, int64_t lda, float* Q, int64_t ldq, float* R,
@@ -1797,7 +1853,30 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
     }
     if (!h->stageR.ensure((size_t)n * n * 4 + 256)) return RG_ALLOC;
     float* dR = h->stageR.as<float>();   // accumulated R (n x n, ld n)
-    int rc = run_rgsqr(h, m_local, n, dA, dlda, dA, dlda, dR, n, o, o.split);
+    // tall blocks (n <= 256, too tall for the on-chip leaf): CholQR passes on the tensor cores
+    // (reading #33), each falling back to the RGSQR pass when its kappa test fails
+    bool tall = tall_wanted(h, m_local, n, dA, dlda);
+    bool tall_ok = false;
+    int rc = RG_OK;
+    if (h->dist()) {   // the ranks' row counts differ: take the path only if every rank wants it
+        if (!h->tallws.ensure(rg::tall_ws_bytes())) return RG_ALLOC;
+        double* v = rg::tall_kout(h->tallws.p) + 3;
+        const double mine = tall ? 1.0 : 0.0;
+        RG_CUDA(cudaMemcpyAsync(v, &mine, sizeof(double), cudaMemcpyHostToDevice, h->stream));
+        rc = nccl_allreduce(h, v, 1, ncclFloat64);
+        if (rc) return rc;
+        double all = 0;
+        RG_CUDA(cudaMemcpyAsync(&all, v, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+        RG_CUDA(cudaStreamSynchronize(h->stream));
+        tall = all > h->nranks - 0.5;
+    }
+    if (tall) {
+        if (!h->status.ensure(64)) return RG_ALLOC;
+        rc = reset_status(h);
+        if (rc == RG_OK) rc = tall_gram(h, m_local, (int)n, dA, dlda, true);
+        if (rc == RG_OK) rc = tall_chol_apply(h, m_local, (int)n, dA, dlda, dR, n, true, &tall_ok);
+    }
+    if (rc == RG_OK && !tall_ok) rc = run_rgsqr(h, m_local, n, dA, dlda, dA, dlda, dR, n, o, o.split);
     int passes = 1;
     double est = -1.0;
     while (rc == RG_OK && passes < max_passes) {
@@ -1810,8 +1889,14 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
         // pass 1 is skipped (the second pass runs anyway; only the estimate's cost is saved).
         const double u16 = o.precision ? 0x1p-8 : 0x1p-11;
         const double m_all = (double)m_local * std::max(1, h->nranks);
-        const bool skip_probe = passes == 1 && 0.25 * u16 * (double)n / std::sqrt(m_all) > orth_tol;
-        if (orth_tol > 0 && !skip_probe) {
+        const bool skip_probe = passes == 1 && !tall_ok && 0.25 * u16 * (double)n / std::sqrt(m_all) > orth_tol;
+        // tall: the Gram of the current Q is the next pass's Gram and gives ||I - Q^T Q||_F exactly
+        // (in its precision), so it replaces the Hutchinson probe
+        if (tall) {
+            rc = tall_gram(h, m_local, (int)n, dA, dlda, false);
+            if (rc == RG_OK) rc = tall_orth(h, (int)n, &est);
+            if (rc || (orth_tol > 0 && est <= orth_tol)) break;
+        } else if (orth_tol > 0 && !skip_probe) {
             rc = orth_estimate(h, dA, dlda, m_local, (int)n, &est);
             if (rc || est <= orth_tol) break;
         }
@@ -1820,7 +1905,9 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
         float* R2 = h->lsR.as<float>();
         rg_opts o2 = o;
         o2.scale = -1;   // in place, unscaled (reading #32)
-        rc = run_rgsqr(h, m_local, n, dA, dlda, dA, dlda, R2, n, o2, 1);
+        bool ok2 = false;
+        if (tall) rc = tall_chol_apply(h, m_local, (int)n, dA, dlda, R2, n, false, &ok2);
+        if (rc == RG_OK && !ok2) rc = run_rgsqr(h, m_local, n, dA, dlda, dA, dlda, R2, n, o2, 1);
         if (rc) break;
         rc = trmm_into(h, R2, n, dR, n, (int)n);
         ++passes;
@@ -1830,7 +1917,8 @@ int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda
     if (o.sync || host || orth_tol > 0 || orth_est_out) rc = check_status(h);
     if (rc) return rc;
     if ((orth_tol > 0 || orth_est_out) && est < 0) {
-        rc = orth_estimate(h, dA, dlda, m_local, (int)n, &est);
+        rc = tall ? tall_gram(h, m_local, (int)n, dA, dlda, false) : orth_estimate(h, dA, dlda, m_local, (int)n, &est);
+        if (rc == RG_OK && tall) rc = tall_orth(h, (int)n, &est);
         if (rc) return rc;
     }
     if (R) RG_CUDA(cudaMemcpy2DAsync(R, ldr * 4, dR, n * 4, n * 4, n,

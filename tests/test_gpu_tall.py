@@ -1,0 +1,136 @@
+"""Tall CholQR passes of `orthogonalize` (csrc/tall.cu, DESIGN reading #33) against the fp64
+oracle (-m gpu).
+
+The tall path (n <= 256, rows beyond the on-chip leaf) is forced on small shapes with
+RGSQR_TALL=1 so that the oracle's Householder QR finishes in seconds; the full config-4 size
+(2,097,152 x 256) takes it by default (tests/test_gpu_fullsize.py).  Checks: orthogonality
+||I - Q^T Q||_F <= 1e-5 (north_star), the backward error, the distance to the oracle's unique
+Q and R (reading #25), the exact Gram-based estimate against the fp64 one, the kappa-test
+fallback to the RGSQR pass, fixed pass counts, and the row-sharded path under virtual ranks.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def rg():
+    import paper_conf_hpdc_zhangbw20_b200 as rg
+    return rg
+
+
+@pytest.fixture
+def tall_on(monkeypatch):
+    monkeypatch.setenv("RGSQR_TALL", "1")
+
+
+def _dev(A):
+    return torch.from_numpy(np.ascontiguousarray(np.asarray(A, dtype=np.float32).T)).cuda().t()
+
+
+def _orth(rg, A, tol=1e-5, passes=3, handle=None):
+    n = A.shape[1]
+    Ad = _dev(A)
+    R = torch.zeros(n, n, device="cuda").t()
+    Q, R, p, est = rg.orthogonalize(Ad, R, orth_tol=tol, max_passes=passes, handle=handle)
+    torch.cuda.synchronize()
+    return Q.cpu().numpy().astype(np.float64), R.cpu().numpy().astype(np.float64), p, est
+
+
+@pytest.mark.parametrize("m,n,kind,kappa", [(20000, 256, "gauss", 1.0), (9001, 200, "geometric", 1e2),
+                                            (4099, 64, "gauss", 1.0), (777, 130, "gauss", 1.0),
+                                            (1000, 1, "gauss", 1.0), (5000, 33, "arithmetic", 10.0)])
+def test_tall_orthogonalize_parity(rg, tall_on, m, n, kind, kappa):
+    A = (synth.gaussian(m, n, seed=31 + n) if kind == "gauss" else
+         synth.svd_matrix(m, n, kind, kappa, seed=31 + n)).astype(np.float32)
+    A64 = A.astype(np.float64)
+    Q, R, p, est = _orth(rg, A)
+    orth = oracle.orthogonality(Q)
+    be = oracle.backward_error(A64, Q, R)
+    assert orth <= 1e-5, (orth, p, est)
+    assert be <= 1e-4, be            # bf16-split first pass: ~2^-17 per entry (reading #33)
+    assert np.all(np.tril(R, -1) == 0) and np.all(np.diag(R) > 0)
+    Qo, Ro, _ = oracle.householder(A64)
+    k = np.linalg.cond(A64)
+    dq = np.linalg.norm(Q - Qo) / np.linalg.norm(Qo)
+    dr = np.linalg.norm(R - Ro) / np.linalg.norm(Ro)
+    assert dq <= 10 * k * be + orth / np.sqrt(n) + 1e-6, (dq, be, orth)
+    assert dr <= 10 * k * be + orth + 1e-6, (dr, be, orth)
+    # the Gram-based estimate is ||I - Q^T Q||_F in the split Gram's precision
+    assert abs(est - orth) <= 0.05 * orth + 2e-7, (est, orth)
+
+
+def test_tall_kappa_fallback(rg, tall_on):
+    """kappa = 1e4: the first CholQR pass fails its kappa test (equilibrated kappa_F > 32 n), A is
+    left untouched and the RGSQR pass runs instead; the reorthogonalisation passes are CholQR."""
+    A = synth.svd_matrix(30000, 256, "geometric", 1e4, seed=37).astype(np.float32)
+    Q, R, p, est = _orth(rg, A)
+    orth = oracle.orthogonality(Q)
+    assert orth <= 1e-5 and p >= 2, (orth, p)
+    assert oracle.backward_error(A.astype(np.float64), Q, R) <= 5e-3
+
+
+def test_tall_fixed_two_passes(rg, tall_on):
+    """orth_tol = 0: exactly max_passes passes (CholQR2), the second a first-order closed-form
+    Cholesky (Gram within 4e-6 of I)."""
+    A = synth.gaussian(40000, 256, seed=41).astype(np.float32)
+    Q, R, p, est = _orth(rg, A, tol=0.0, passes=2)
+    assert p == 2
+    orth = oracle.orthogonality(Q)
+    assert orth <= 3e-6, orth
+    assert oracle.backward_error(A.astype(np.float64), Q, R) <= 1e-4
+
+
+def test_tall_matches_rgsqr_path(rg, monkeypatch):
+    """Same subspace and R up to the tolerances whether the passes are CholQR or RGSQR."""
+    A = synth.svd_matrix(16384, 192, "geometric", 50.0, seed=43).astype(np.float32)
+    monkeypatch.setenv("RGSQR_TALL", "1")
+    Q1, R1, _, _ = _orth(rg, A)
+    monkeypatch.setenv("RGSQR_TALL", "0")
+    Q2, R2, _, _ = _orth(rg, A)
+    assert np.linalg.norm(R1 - R2) / np.linalg.norm(R2) <= 1e-3
+    assert np.linalg.norm(Q1 - Q2) / np.linalg.norm(Q2) <= 1e-3
+
+
+@pytest.mark.parametrize("P", [2, 4])
+def test_tall_dist_virtual_ranks(rg, tall_on, P):
+    """Row-sharded tall passes: the n x n Gram is the only exchange (allreduce through the virtual
+    group); R and the estimate are identical on every rank, the gathered Q meets the tolerances
+    and matches the single-handle call (P-invariance up to the fp64 reduction order)."""
+    m, n = 24000, 256
+    A = synth.gaussian(m, n, seed=47).astype(np.float32)
+    w = np.linspace(1.0, 1.6, P)
+    c = np.concatenate([[0], np.cumsum(w / w.sum() * m)]).round().astype(int)
+    c[-1] = m
+    group = rg.VGroup(P)
+    streams = [torch.cuda.Stream() for _ in range(P)]
+    hs = [rg.Handle(0, stream=s.cuda_stream) for s in streams]
+    try:
+        for r, h in enumerate(hs):
+            h.set_vcomm(group, r)
+        blocks = [_dev(A[c[r]:c[r + 1]]) for r in range(P)]
+        Rs = [torch.zeros(n, n, device="cuda").t() for _ in range(P)]
+        torch.cuda.synchronize()
+        out = rg.run_ranks([lambda r=r: rg.orthogonalize(blocks[r], Rs[r], orth_tol=1e-5, max_passes=3,
+                                                         handle=hs[r]) for r in range(P)])
+        torch.cuda.synchronize()
+    finally:
+        for h in hs:
+            h.close()
+        group.close()
+    assert len({o[2] for o in out}) == 1 and len({o[3] for o in out}) == 1
+    for r in range(1, P):
+        np.testing.assert_array_equal(Rs[r].cpu().numpy(), Rs[0].cpu().numpy())
+    Q = np.vstack([b.cpu().numpy() for b in blocks]).astype(np.float64)
+    R = Rs[0].cpu().numpy().astype(np.float64)
+    orth = oracle.orthogonality(Q)
+    assert orth <= 1e-5
+    assert oracle.backward_error(A.astype(np.float64), Q, R) <= 1e-4
+    Q1, R1, _, _ = _orth(rg, A)
+    assert np.linalg.norm(R - R1) / np.linalg.norm(R1) <= 1e-5
+    assert np.linalg.norm(Q - Q1) / np.linalg.norm(Q1) <= 1e-5
