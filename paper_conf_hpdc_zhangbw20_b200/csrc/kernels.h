@@ -36,8 +36,10 @@ size_t tall_ws_bytes();
 double* tall_gram_buffer(void* ws);          // n x n fp64 Gram (allreduced in place when row-sharded)
 int* tall_flag(void* ws);                    // nonzero after a failed pass (X untouched)
 double* tall_kout(void* ws);                 // [kappa_F(R^), first failed pivot]
+double* tall_dbg(void* ws);                  // [TL_N] tensor-core Gram diagonal (RGSQR_TALL_DEBUG)
+// tmX: fp32 map of X (inner = rows, box 32 rows x 256 columns, no swizzle) or null (register-fed kernel)
 cudaError_t launch_tall_gram(const float* X, int64_t ldx, int64_t m, int n, float sig, int bf16, void* ws, double* G,
-                             cudaStream_t st);
+                             cudaStream_t st, const CUtensorMap* tmX = nullptr);
 cudaError_t launch_tall_orth(const double* G, int n, double sig, double* out, cudaStream_t st);
 cudaError_t launch_tall_chol_apply(float* X, int64_t ldx, int64_t m, int n, const double* G, double sig_g, float sig_a,
                                    int bf16, double kappa_max, float* R, int64_t ldr, void* ws, cudaStream_t st);

@@ -1188,7 +1188,24 @@ constexpr float kTallSig = 16384.0f;
 int tall_gram(rg_handle h, int64_t m, int n, const float* X, int64_t ldx, bool first) {
     if (!h->tallws.ensure(rg::tall_ws_bytes())) return RG_ALLOC;
     double* G = rg::tall_gram_buffer(h->tallws.p);
-    RG_CUDA(rg::launch_tall_gram(X, ldx, m, n, first ? 1.0f : kTallSig, first ? 1 : 0, h->tallws.p, G, h->stream));
+    CUtensorMap tm;
+    const bool tma = ensure_encode() && encode_plain(&tm, X, m, n, ldx, 4, false, 32, 256);
+    RG_CUDA(rg::launch_tall_gram(X, ldx, m, n, first ? 1.0f : kTallSig, first ? 1 : 0, h->tallws.p, G, h->stream,
+                                 tma ? &tm : nullptr));
+    if (getenv("RGSQR_TALL_DEBUG")) {   // tensor-core diagonal against the fp64 column sums
+        std::vector<double> dg((size_t)n), dt((size_t)n);
+        RG_CUDA(cudaStreamSynchronize(h->stream));
+        RG_CUDA(cudaMemcpy(dt.data(), rg::tall_dbg(h->tallws.p), n * 8, cudaMemcpyDeviceToHost));
+        RG_CUDA(cudaMemcpy2D(dg.data(), 8, G, (size_t)(n + 1) * 8, 8, n, cudaMemcpyDeviceToHost));
+        double mx = 0, sq = 0;
+        for (int i = 0; i < n; ++i) {
+            const double r = dt[i] / dg[i] - 1.0;
+            mx = std::max(mx, std::fabs(r));
+            sq += r * r;
+        }
+        fprintf(stderr, "[tall] gram m=%lld first=%d: tensor-core diagonal vs fp64 norms: max rel %.3g rms %.3g\n",
+                (long long)m, (int)first, mx, std::sqrt(sq / n));
+    }
     return nccl_allreduce(h, G, (size_t)n * n, ncclFloat64);
 }
 // ||I - X^T X||_F from the Gram just formed by tall_gram(first = false) (synchronous)

@@ -59,15 +59,23 @@ __device__ __forceinline__ float2 tl_unpack(uint32_t u, bool bf) {
     return __half22float2(*reinterpret_cast<__half2*>(&u));
 }
 
-// 4 consecutive rows (one float4, already scaled) -> 8 bytes of hi and of lo at byte `off` of the
-// line (off = 8 * (row group of 4), swizzled by the caller).
+__device__ __forceinline__ void tl_sts64(uint32_t addr, uint32_t a, uint32_t b) {
+    asm volatile("st.shared.v2.u32 [%0], {%1, %2};" ::"r"(addr), "r"(a), "r"(b) : "memory");
+}
+__device__ __forceinline__ float4 tl_lds128(uint32_t addr) {
+    float4 v;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(addr));
+    return v;
+}
+// 4 consecutive rows (one float4, already scaled) -> 8 bytes of hi at shared address hi_addr and
+// of lo at lo_addr (swizzled by the caller)
 template <bool BF>
-__device__ __forceinline__ void tl_split_store(float4 v, uint8_t* hi_line, uint8_t* lo_line, uint32_t off) {
+__device__ __forceinline__ void tl_split_sts(float4 v, uint32_t hi_addr, uint32_t lo_addr) {
     const uint32_t h0 = tl_pack(v.x, v.y, BF), h1 = tl_pack(v.z, v.w, BF);
     const float2 a = tl_unpack(h0, BF), b = tl_unpack(h1, BF);
     const uint32_t l0 = tl_pack(v.x - a.x, v.y - a.y, BF), l1 = tl_pack(v.z - b.x, v.w - b.y, BF);
-    *reinterpret_cast<uint2*>(hi_line + off) = make_uint2(h0, h1);
-    *reinterpret_cast<uint2*>(lo_line + off) = make_uint2(l0, l1);
+    tl_sts64(hi_addr, h0, h1);
+    tl_sts64(lo_addr, l0, l1);
 }
 
 // SWIZZLE_128B byte offset of the 8-byte piece g (0..15) of line `line` (1024-byte aligned tile)
@@ -161,8 +169,12 @@ __global__ void __launch_bounds__(TL_THREADS, 1) tl_gram_kernel(TlGramArgs a) {
         const int cw = warp - 4;
         const int g = lane & 15;
         double nrm[16];
+        float nf[16];
 #pragma unroll
-        for (int p = 0; p < 16; ++p) nrm[p] = 0.0;
+        for (int p = 0; p < 16; ++p) {
+            nrm[p] = 0.0;
+            nf[p] = 0.f;
+        }
         for (int it = 0; it < my; ++it) {
             const int s = it % TL_GSTAGES;
             const int64_t r0 = ((int64_t)blockIdx.x + (int64_t)it * gridDim.x) * 64 + 4 * g;
@@ -179,19 +191,26 @@ __global__ void __launch_bounds__(TL_THREADS, 1) tl_gram_kernel(TlGramArgs a) {
             for (int p = 0; p < 16; ++p) {
                 const int c = 2 * (16 * cw + p) + (lane >> 4);
                 float4 x = v[p];
-                nrm[p] += (double)fmaf(x.x, x.x, fmaf(x.y, x.y, fmaf(x.z, x.z, x.w * x.w)));
+                nf[p] = fmaf(x.x, x.x, fmaf(x.y, x.y, fmaf(x.z, x.z, fmaf(x.w, x.w, nf[p]))));
                 x.x *= a.sig; x.y *= a.sig; x.z *= a.sig; x.w *= a.sig;
                 const uint32_t off = tl_swz(c, g);
-                tl_split_store<BF>(x, hi + (off & ~127u), lo + (off & ~127u), off & 127u);
+                tl_split_sts<BF>(x, smem_u32(hi) + off, smem_u32(lo) + off);
             }
             fence_proxy_async_smem();
             __syncwarp();
             if (lane == 0) mbar_arrive(&full_bar[s]);
+            if ((it & 31) == 31) {
+#pragma unroll
+                for (int p = 0; p < 16; ++p) {
+                    nrm[p] += (double)nf[p];
+                    nf[p] = 0.f;
+                }
+            }
         }
         // column norms: 16 lanes share a column
 #pragma unroll
         for (int p = 0; p < 16; ++p) {
-            double x = nrm[p];
+            double x = nrm[p] + (double)nf[p];
 #pragma unroll
             for (int o = 1; o < 16; o <<= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
             if (g == 0) a.npart[(int64_t)blockIdx.x * TL_N + 2 * (16 * cw + p) + (lane >> 4)] = x * (double)a.sig * (double)a.sig;
@@ -221,10 +240,180 @@ __global__ void __launch_bounds__(TL_THREADS, 1) tl_gram_kernel(TlGramArgs a) {
     if (warp == 1) tmem_dealloc<512>(tmem);
 }
 
+// TMA-fed variant (16-byte aligned X and ldx): a producer warp streams 32-row x 256-column fp32
+// half-chunks of X into a ring of three 32 KB staging slots (HBM stays busy while the converters
+// work), the 8 converter warps split them from shared memory into the two operand stages.
+constexpr int TL_TSLOTS = 3;
+constexpr int TL_TSLOT = 32 * TL_N * 4;
+constexpr int TL_TSTAGES = 2;
+constexpr int TL_TCW = 16;                     // converter warps of the TMA-fed Gram
+constexpr int TL_TTHREADS = 128 + 32 * TL_TCW;
+constexpr int TL_GRAM_TMA_SMEM = TL_TSTAGES * TL_GSTAGE + TL_TSLOTS * TL_TSLOT + 256 + 1024;
+
+template <bool BF>
+__global__ void __launch_bounds__(TL_TTHREADS, 1) tl_gram_tma_kernel(const __grid_constant__ CUtensorMap tmX,
+                                                                    TlGramArgs a) {
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* stg = smem + TL_TSTAGES * TL_GSTAGE;
+    uint64_t* full_bar = reinterpret_cast<uint64_t*>(stg + TL_TSLOTS * TL_TSLOT);
+    uint64_t* empty_bar = full_bar + TL_TSTAGES;
+    uint64_t* sfull = empty_bar + TL_TSTAGES;
+    uint64_t* sempty = sfull + TL_TSLOTS;
+    uint64_t* done_bar = sempty + TL_TSLOTS;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(done_bar + 1);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int64_t nchunks = (a.m + 63) / 64;
+    const int my = nchunks > blockIdx.x ? (int)((nchunks - 1 - blockIdx.x) / gridDim.x + 1) : 0;
+
+    if (threadIdx.x == 0) {
+        tma_prefetch_desc(&tmX);
+        for (int s = 0; s < TL_TSTAGES; ++s) {
+            mbar_init(&full_bar[s], TL_TCW);
+            mbar_init(&empty_bar[s], 1);
+        }
+        for (int s = 0; s < TL_TSLOTS; ++s) {
+            mbar_init(&sfull[s], 1);
+            mbar_init(&sempty[s], TL_TCW);
+        }
+        mbar_init(done_bar, 1);
+        fence_barrier_init();
+    }
+    if (warp == 1) tmem_alloc<512>(tmem_slot);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+    RG_PDL_ENTRY();
+
+    if (warp == 0) {
+        if (elect_one()) {
+            const uint32_t id256 = umma_idesc_f16(128, 256, 0, 0, BF ? 1u : 0u);
+            const uint32_t id128 = umma_idesc_f16(128, 128, 0, 0, BF ? 1u : 0u);
+            for (int it = 0; it < my; ++it) {
+                const int s = it % TL_TSTAGES;
+                mbar_wait(&full_bar[s], (uint32_t)(it / TL_TSTAGES) & 1u);
+                tc_fence_after();
+                const uint32_t hi = smem_u32(smem + s * TL_GSTAGE);
+                const uint32_t lo = hi + TL_N * 128;
+#pragma unroll
+                for (int kk = 0; kk < 4; ++kk) {
+                    const uint32_t acc = (it > 0 || kk > 0) ? 1u : 0u;
+                    const uint64_t h0 = umma_desc_sw128(hi + kk * 32, 16, 1024);
+                    const uint64_t l0 = umma_desc_sw128(lo + kk * 32, 16, 1024);
+                    const uint64_t h1 = umma_desc_sw128(hi + 128 * 128 + kk * 32, 16, 1024);
+                    const uint64_t l1 = umma_desc_sw128(lo + 128 * 128 + kk * 32, 16, 1024);
+                    umma_f16(tmem, h0, h0, id256, acc);
+                    umma_f16(tmem, h0, l0, id256, 1u);
+                    umma_f16(tmem, l0, h0, id256, 1u);
+                    umma_f16(tmem + 256, h1, h1, id128, acc);
+                    umma_f16(tmem + 256, h1, l1, id128, 1u);
+                    umma_f16(tmem + 256, l1, h1, id128, 1u);
+                }
+                umma_commit(&empty_bar[s]);
+            }
+            umma_commit(done_bar);
+        }
+        __syncwarp();
+    } else if (warp == 2) {
+        if (elect_one()) {
+            // ---------------- TMA producer: half-chunk q = rows [64 (cta + grid (q >> 1)) + 32 (q & 1), +32)
+            for (int q = 0; q < 2 * my; ++q) {
+                const int sl = q % TL_TSLOTS;
+                mbar_wait(&sempty[sl], ((uint32_t)(q / TL_TSLOTS) & 1u) ^ 1u);
+                mbar_arrive_expect_tx(&sfull[sl], TL_TSLOT);
+                const int64_t r0 = ((int64_t)blockIdx.x + (int64_t)(q >> 1) * gridDim.x) * 64 + 32 * (q & 1);
+                tma_load_2d(stg + sl * TL_TSLOT, &tmX, &sfull[sl], (int32_t)r0, 0);
+            }
+        }
+        __syncwarp();
+    } else if (warp >= 4) {
+        // ---------------- converters: warp cw takes 16 columns (4 per instruction), rows
+        // 4 (lane & 7) .. + 3 of the half-chunk; staging layout [column][32 rows] fp32
+        // columns of instruction k: {b, b + 4, b + 1, b + 5}[lane >> 3], b = 8 (k >> 1) + 2 (k & 1): the
+        // two half-lines of each pair (c, c + 4) cover all 32 banks (swizzle chunk ^ (c & 7))
+        const int cw = warp - 4, g8 = lane & 7;
+        const int qsel = lane >> 3;
+        const int coff = (qsel & 1) * 4 + (qsel >> 1);
+        double nrm[4];
+        float nf[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            nrm[k] = 0.0;
+            nf[k] = 0.f;
+        }
+        for (int q = 0; q < 2 * my; ++q) {
+            const int sl = q % TL_TSLOTS, it = q >> 1, hf = q & 1, s = it % TL_TSTAGES;
+            mbar_wait(&sfull[sl], (uint32_t)(q / TL_TSLOTS) & 1u);
+            if (hf == 0) mbar_wait(&empty_bar[s], ((uint32_t)(it / TL_TSTAGES) & 1u) ^ 1u);
+            const uint32_t src = smem_u32(stg + sl * TL_TSLOT);
+            uint8_t* hi = smem + s * TL_GSTAGE;
+            uint8_t* lo = hi + TL_N * 128;
+            float4 v[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const int c = 16 * cw + 8 * (k >> 1) + 2 * (k & 1) + coff;
+                v[k] = tl_lds128(src + (uint32_t)(c * 128 + 16 * g8));
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&sempty[sl]);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const int c = 16 * cw + 8 * (k >> 1) + 2 * (k & 1) + coff;
+                float4 x = v[k];
+                nf[k] = fmaf(x.x, x.x, fmaf(x.y, x.y, fmaf(x.z, x.z, fmaf(x.w, x.w, nf[k]))));
+                x.x *= a.sig; x.y *= a.sig; x.z *= a.sig; x.w *= a.sig;
+                const uint32_t off = tl_swz(c, 8 * hf + g8);
+                tl_split_sts<BF>(x, smem_u32(hi) + off, smem_u32(lo) + off);
+            }
+            if (hf == 1) {
+                fence_proxy_async_smem();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&full_bar[s]);
+            }
+            if ((q & 31) == 31) {   // fp32 partial sums of <= 128 squares, then fp64
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    nrm[k] += (double)nf[k];
+                    nf[k] = 0.f;
+                }
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            double x = nrm[k] + (double)nf[k];
+#pragma unroll
+            for (int o = 1; o < 8; o <<= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+            if (g8 == 0) a.npart[(int64_t)blockIdx.x * TL_N + 16 * cw + 8 * (k >> 1) + 2 * (k & 1) + coff] = x * (double)a.sig * (double)a.sig;
+        }
+        const int qd = warp & 3, part = cw >> 2;
+        float* P = a.part + (int64_t)blockIdx.x * TL_PART;
+        if (my > 0) {
+            mbar_wait(done_bar, 0);
+            tc_fence_after();
+        }
+        for (int ch = part; ch < TL_GACC / 32; ch += TL_TCW / 4) {
+            uint32_t r[32];
+            if (my > 0) {
+                tmem_ld32(tmem + ((uint32_t)(32 * qd) << 16) + ch * 32, r);
+                tmem_ld_wait();
+            } else {
+#pragma unroll
+                for (int j = 0; j < 32; ++j) r[j] = 0u;
+            }
+#pragma unroll
+            for (int j = 0; j < 32; ++j) P[(int64_t)(ch * 32 + j) * 128 + 32 * qd + lane] = __uint_as_float(r[j]);
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 1) tmem_dealloc<512>(tmem);
+}
+
 // G (fp64, n x n, column-major ld n): strict upper triangle from the TMEM partials, diagonal from
 // the fp64 column sums, lower triangle zero; every entry summed over the CTAs in a fixed order.
 __global__ void __launch_bounds__(256) tl_reduce_kernel(const float* __restrict__ part, const double* __restrict__ npart,
-                                                         int nb, int n, double* G) {
+                                                         int nb, int n, double* G, double* dbg) {
     RG_PDL_ENTRY();
     const int e = blockIdx.x * blockDim.x + threadIdx.x;
     if (e < TL_PART) {
@@ -245,6 +434,8 @@ __global__ void __launch_bounds__(256) tl_reduce_kernel(const float* __restrict_
         if (row < col) {
             G[row + (int64_t)col * n] = s;
             G[col + (int64_t)row * n] = 0.0;
+        } else if (row == col && dbg) {
+            dbg[row] = s;   // the tensor-core diagonal (diagnostics: RGSQR_TALL_DEBUG)
         }
     } else if (e < TL_PART + TL_N) {
         const int c = e - TL_PART;
@@ -596,7 +787,8 @@ constexpr int TL_GRAM_SMEM = TL_GSTAGES * TL_GSTAGE + 128 + 1024;
 // first line of the K-block kc tile (lines j = 64 kc .. 255, one per output column)
 __host__ __device__ constexpr int tl_btile(int kc) { return kc == 0 ? 0 : kc == 1 ? 256 : kc == 2 ? 448 : 576; }
 
-constexpr int TL_ATHREADS = TL_THREADS + 128;   // + 4 epilogue warps (12..15)
+constexpr int TL_ACW = 16;                               // apply converter warps 4..19 (two groups)
+constexpr int TL_ATHREADS = 128 + 32 * TL_ACW + 128;   // + 4 epilogue warps (20..23)
 template <bool BF>
 __global__ void __launch_bounds__(TL_ATHREADS, 1) tl_apply_kernel(TlApplyArgs a) {
     extern __shared__ uint8_t smem_raw[];
@@ -616,7 +808,7 @@ __global__ void __launch_bounds__(TL_ATHREADS, 1) tl_apply_kernel(TlApplyArgs a)
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < TL_ASTAGES; ++s) {
-            mbar_init(&full_bar[s], TL_CW);
+            mbar_init(&full_bar[s], TL_ACW / 2);
             mbar_init(&empty_bar[s], 1);
         }
         for (int b = 0; b < 2; ++b) {
@@ -627,16 +819,16 @@ __global__ void __launch_bounds__(TL_ATHREADS, 1) tl_apply_kernel(TlApplyArgs a)
     }
     if (warp == 1) tmem_alloc<512>(tmem_slot);
     // resident B: for K-block kc, line j (output column, j >= 64 kc) = R^^-1[64 kc .. 64 kc + 63][j]
-    if (warp >= 4 && warp < 12) {
+    if (warp >= 4 && warp < 4 + TL_ACW) {
         const int cw = warp - 4, g = lane & 15;
-        for (int L = 2 * cw + (lane >> 4); L < 640; L += 2 * TL_CW) {
+        for (int L = 2 * cw + (lane >> 4); L < 640; L += 2 * TL_ACW) {
             const int kc = L < 256 ? 0 : L < 448 ? 1 : L < 576 ? 2 : 3;
             const int j = 64 * kc + (L - tl_btile(kc));
             float4 v = *reinterpret_cast<const float4*>(a.rinv + (int64_t)j * TL_N + 64 * kc + 4 * g);
             const uint32_t off = tl_swz(L, g);
-            tl_split_store<BF>(v, smem + (off & ~127u), smem + TL_BBYTES + (off & ~127u), off & 127u);
+            tl_split_sts<BF>(v, smem_u32(smem) + off, smem_u32(smem) + TL_BBYTES + off);
         }
-        for (int i = threadIdx.x - 128; i < TL_N; i += 32 * TL_CW) csc[i] = a.cscale[i];
+        for (int i = threadIdx.x - 128; i < TL_N; i += 32 * TL_ACW) csc[i] = a.cscale[i];
         fence_proxy_async_smem();
     }
     tc_fence_before();
@@ -679,40 +871,39 @@ __global__ void __launch_bounds__(TL_ATHREADS, 1) tl_apply_kernel(TlApplyArgs a)
             }
         }
         __syncwarp();
-    } else if (warp >= 4 && warp < 12) {
-        // ---------------- converters: line L = 2 pp + (lane >> 4): row half L >> 6, column 64 kc + (L & 63)
-        const int cw = warp - 4, g = lane & 15;
-        int it = 0;
-        for (int tt = 0; tt < my; ++tt) {
+    } else if (warp >= 4 && warp < 4 + TL_ACW) {
+        // ---------------- converters, two groups of 8 warps: group gr owns stage gr and converts
+        // the k-blocks it = 4 tt + kc with it % 2 == gr, so one group's loads are in flight while
+        // the other converts.  Line L = 2 pp + (lane >> 4): row half L >> 6, column 64 kc + (L & 63).
+        const int gr = (warp - 4) >> 3, cw = (warp - 4) & 7, g = lane & 15;
+        for (int it = gr; it < 4 * my; it += 2) {
+            const int tt = it >> 2, kc = it & 3;
             const int64_t t0 = ((int64_t)blockIdx.x + (int64_t)tt * gridDim.x) * 128;
-            for (int kc = 0; kc < 4; ++kc, ++it) {
-                const int s = it % TL_ASTAGES;
-                float4 v[8];
+            float4 v[8];
 #pragma unroll
-                for (int p = 0; p < 8; ++p) {
-                    const int L = 2 * (8 * cw + p) + (lane >> 4);
-                    const int c = 64 * kc + (L & 63);
-                    v[p] = c < a.n ? tl_load4(a.X + (int64_t)c * a.ldx, t0 + 64 * (L >> 6) + 4 * g, a.m, a.vec != 0)
-                                   : make_float4(0.f, 0.f, 0.f, 0.f);
-                }
-                mbar_wait(&empty_bar[s], ((uint32_t)(it / TL_ASTAGES) & 1u) ^ 1u);
-                uint8_t* ah = smem + TL_AOFF + s * TL_ASTAGE;
-#pragma unroll
-                for (int p = 0; p < 8; ++p) {
-                    const int L = 2 * (8 * cw + p) + (lane >> 4);
-                    const float sc = csc[64 * kc + (L & 63)];
-                    float4 x = v[p];
-                    x.x *= sc; x.y *= sc; x.z *= sc; x.w *= sc;
-                    // MN-major: row half at +8 KB, line = column within the k-block
-                    const uint32_t off = tl_swz(L & 63, g) + (uint32_t)(L >> 6) * 8192u;
-                    tl_split_store<BF>(x, ah + (off & ~127u), ah + TL_ASTAGE / 2 + (off & ~127u), off & 127u);
-                }
-                fence_proxy_async_smem();
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&full_bar[s]);
+            for (int p = 0; p < 8; ++p) {
+                const int L = 2 * (8 * cw + p) + (lane >> 4);
+                const int c = 64 * kc + (L & 63);
+                v[p] = c < a.n ? tl_load4(a.X + (int64_t)c * a.ldx, t0 + 64 * (L >> 6) + 4 * g, a.m, a.vec != 0)
+                               : make_float4(0.f, 0.f, 0.f, 0.f);
             }
+            mbar_wait(&empty_bar[gr], ((uint32_t)(it >> 1) & 1u) ^ 1u);
+            uint8_t* ah = smem + TL_AOFF + gr * TL_ASTAGE;
+#pragma unroll
+            for (int p = 0; p < 8; ++p) {
+                const int L = 2 * (8 * cw + p) + (lane >> 4);
+                const float sc = csc[64 * kc + (L & 63)];
+                float4 x = v[p];
+                x.x *= sc; x.y *= sc; x.z *= sc; x.w *= sc;
+                // MN-major: row half at +8 KB, line = column within the k-block
+                const uint32_t off = tl_swz(L & 63, g) + (uint32_t)(L >> 6) * 8192u;
+                tl_split_sts<BF>(x, smem_u32(ah) + off, smem_u32(ah) + TL_ASTAGE / 2 + off);
+            }
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&full_bar[gr]);
         }
-    } else if (warp >= 12) {
+    } else if (warp >= 4 + TL_ACW) {
         // ---------------- epilogue warps (TMEM lane quarter warp & 3): TMEM -> X in place.  A
         // tile's rows were all read (its four k-blocks converted) before its accumulator is full.
         const float es = *a.escale;
@@ -776,11 +967,12 @@ cudaError_t launch_tall_orth(const double* G, int n, double sig, double* out, cu
 // ======================================================================= launchers
 size_t tall_ws_bytes() {
     return (size_t)TL_MAX_GRID * TL_PART * 4 + (size_t)TL_MAX_GRID * TL_N * 8 + (size_t)TL_N * TL_N * 8 +
-           (size_t)TL_N * TL_N * 4 + TL_N * 4 + 128 + 64;
+           (size_t)TL_N * TL_N * 4 + TL_N * 4 + 128 + 64 + TL_N * 8;
 }
 
+double* tall_dbg(void* ws);
 cudaError_t launch_tall_gram(const float* X, int64_t ldx, int64_t m, int n, float sig, int bf16, void* ws,
-                             double* G, cudaStream_t st) {
+                             double* G, cudaStream_t st, const CUtensorMap* tmX) {
     uint8_t* w = reinterpret_cast<uint8_t*>(ws);
     float* part = reinterpret_cast<float*>(w);
     double* npart = reinterpret_cast<double*>(w + (size_t)TL_MAX_GRID * TL_PART * 4);
@@ -789,14 +981,23 @@ cudaError_t launch_tall_gram(const float* X, int64_t ldx, int64_t m, int n, floa
     TlGramArgs a{X, ldx, m, n, sig, ((reinterpret_cast<uintptr_t>(X) & 15) == 0 && (ldx & 3) == 0) ? 1 : 0, part,
                  npart};
     cudaError_t e;
-    if (bf16) {
+    if (tmX && !getenv("RGSQR_TALL_NO_TMA")) {
+        if (bf16) {
+            if ((e = ensure_smem_attr((const void*)tl_gram_tma_kernel<true>, TL_GRAM_TMA_SMEM))) return e;
+            RG_LAUNCH((tl_gram_tma_kernel<true>), grid, TL_TTHREADS, TL_GRAM_TMA_SMEM, st, *tmX, a);
+        } else {
+            if ((e = ensure_smem_attr((const void*)tl_gram_tma_kernel<false>, TL_GRAM_TMA_SMEM))) return e;
+            RG_LAUNCH((tl_gram_tma_kernel<false>), grid, TL_TTHREADS, TL_GRAM_TMA_SMEM, st, *tmX, a);
+        }
+    } else if (bf16) {
         if ((e = ensure_smem_attr((const void*)tl_gram_kernel<true>, TL_GRAM_SMEM))) return e;
         RG_LAUNCH((tl_gram_kernel<true>), grid, TL_THREADS, TL_GRAM_SMEM, st, a);
     } else {
         if ((e = ensure_smem_attr((const void*)tl_gram_kernel<false>, TL_GRAM_SMEM))) return e;
         RG_LAUNCH((tl_gram_kernel<false>), grid, TL_THREADS, TL_GRAM_SMEM, st, a);
     }
-    RG_LAUNCH(tl_reduce_kernel, (TL_PART + TL_N + 255) / 256, 256, 0, st, part, npart, grid, n, G);
+    RG_LAUNCH(tl_reduce_kernel, (TL_PART + TL_N + 255) / 256, 256, 0, st, part, npart, grid, n, G,
+              getenv("RGSQR_TALL_DEBUG") ? tall_dbg(ws) : nullptr);
     return cudaGetLastError();
 }
 
@@ -824,6 +1025,7 @@ double* tall_gram_buffer(void* ws) {
                                      (size_t)TL_MAX_GRID * TL_N * 8);
 }
 int* tall_flag(void* ws) { return tall_tail(ws).flag; }
+double* tall_dbg(void* ws) { return tall_tail(ws).kout + 8; }
 double* tall_kout(void* ws) { return tall_tail(ws).kout; }
 
 constexpr int TL_CHOL_SMEM = (36 + TC_NT) * TC_TILE * 4 + 2 * TL_N * 8;
