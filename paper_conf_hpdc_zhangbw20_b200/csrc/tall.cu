@@ -465,7 +465,7 @@ struct TlCholArgs {
 
 // Blocked on 32 x 32 tiles (8 x 8 tile grid, upper triangle: 36 tiles, row-major, row stride 36
 // floats so that rows are 16-byte aligned).  Tile products C op= A^T B ("TN") or A B ("NN") with a
-// 4 x 4 register tile per thread, 64 threads per output tile (16 tiles in flight on 1024 threads).
+// 4 x 4 register tile per thread, 64 threads per output tile (8 tiles in flight on 512 threads).
 constexpr int TC_LD = 36;
 constexpr int TC_TILE = 32 * TC_LD;
 constexpr int TC_NT = 8;
@@ -506,45 +506,55 @@ __device__ __forceinline__ void tc_store(float* C, int ti, int tj, const float (
             make_float4(alpha * c[r][0], alpha * c[r][1], alpha * c[r][2], alpha * c[r][3]);
 }
 
-// One warp: Cholesky of the 32 x 32 diagonal tile T (upper part; lane j holds column j), R into T,
-// its inverse into X.  Returns false (uniform) on a non-positive pivot.
+// One warp: Cholesky of the 32 x 32 diagonal tile T (upper part, row-major, stride TC_LD), R into T,
+// its inverse into X.  Lane j keeps column j in registers; the pivot row travels through shared
+// memory (no shuffles: inside a one-warp branch the compiler's collective shuffle sequence costs
+// ~300 cycles per pivot, tools/wchol_probe.cu):
+//   step k: p = T(k, k), r(k, j) = c_k / sqrt(p); every lane reads row k (T(k, i), i > k: the
+//   values lane i published at step k - 1) and updates c_i -= r(k, i) r(k, j); lane j then
+//   publishes its new c_{k+1} as T(k + 1, j).
+// X = R^-1 column-parallel (lane j: column j), right-looking: x_k /= r_kk, x_i -= r_ik x_k (i < k).
+// Returns false (uniform) on a non-positive pivot.
 __device__ __forceinline__ bool tc_diag(float* T, float* X, int lane) {
     float c[32];
 #pragma unroll
     for (int i = 0; i < 32; ++i) c[i] = T[i * TC_LD + lane];
     bool ok = true;
+    __syncwarp();
 #pragma unroll
     for (int k = 0; k < 32; ++k) {
-        const float p = __shfl_sync(0xffffffffu, c[k], k);
+        const float p = T[k * TC_LD + k];
         ok = ok && (p > 1e-30f);
-        const float r = __fdiv_rn(c[k], __fsqrt_rn(p));   // r_kj (lane j >= k), correctly rounded
-        c[k] = r;
+        const float rs = __frsqrt_rn(fmaxf(p, 1e-30f));
+        const float rk = c[k] * rs;   // r(k, lane), lane >= k
+        c[k] = rk;
 #pragma unroll
-        for (int i = k + 1; i < 32; ++i) c[i] = fmaf(-__shfl_sync(0xffffffffu, r, i), r, c[i]);
+        for (int i = k + 1; i < 32; ++i) c[i] = fmaf(-(T[k * TC_LD + i] * rs), rk, c[i]);
+        __syncwarp();
+        if (k < 31) T[(k + 1) * TC_LD + lane] = c[k + 1];
+        __syncwarp();
     }
 #pragma unroll
     for (int i = 0; i < 32; ++i) T[i * TC_LD + lane] = i <= lane ? c[i] : 0.f;
     __syncwarp();
-    // X = R^-1, column j on lane j: x_jj = 1 / r_jj, x_ij = -(sum_{i < l <= j} r_il x_lj) / r_ii
-    // (row i of R read from shared memory, the same address on every lane)
     float x[32];
 #pragma unroll
-    for (int i = 31; i >= 0; --i) {
-        float s0 = 0.f, s1 = 0.f;
+    for (int i = 0; i < 32; ++i) x[i] = i == lane ? 1.f : 0.f;
 #pragma unroll
-        for (int l = i + 1; l < 32; ++l) {
-            const float ril = T[i * TC_LD + l];
-            if ((l & 1) == 0) s0 = fmaf(ril, x[l], s0); else s1 = fmaf(ril, x[l], s1);
-        }
-        const float rii = T[i * TC_LD + i];
-        x[i] = lane == i ? __frcp_rn(rii) : (lane > i ? __fdiv_rn(-(s0 + s1), rii) : 0.f);
+    for (int k = 31; k >= 0; --k) {
+        x[k] = x[k] * __frcp_rn(T[k * TC_LD + k]);
+#pragma unroll
+        for (int i = 0; i < k; ++i) x[i] = fmaf(-T[i * TC_LD + k], x[k], x[i]);
     }
 #pragma unroll
     for (int i = 0; i < 32; ++i) X[i * TC_LD + lane] = x[i];
     return __all_sync(0xffffffffu, ok);
 }
 
-__global__ void __launch_bounds__(1024, 1) tl_chol_kernel(TlCholArgs a) {
+constexpr int TC_THREADS = 512;   // 128 registers per thread: the warp-register diagonal code does not spill
+constexpr int TC_NW = TC_THREADS / 32;
+constexpr int TC_TASKS = TC_THREADS / 64;
+__global__ void __launch_bounds__(TC_THREADS, 1) tl_chol_kernel(TlCholArgs a) {
     extern __shared__ __align__(16) float tsm[];
     float* Tl = tsm;                               // 36 tiles of the upper triangle
     float* XD = Tl + 36 * TC_TILE;                 // 8 inverted diagonal tiles
@@ -552,7 +562,7 @@ __global__ void __launch_bounds__(1024, 1) tl_chol_kernel(TlCholArgs a) {
     double* d = reinterpret_cast<double*>(XD + TC_NT * TC_TILE);   // [TL_N]
     __shared__ int bad;
     __shared__ float gmax;
-    __shared__ double red[3][32];
+    __shared__ double red[3][TC_NW];
     RG_PDL_ENTRY();
     const int n = a.n, t = threadIdx.x, warp = t >> 5, lane = t & 31;
     const int nt = (n + 31) / 32;
@@ -579,8 +589,8 @@ __global__ void __launch_bounds__(1024, 1) tl_chol_kernel(TlCholArgs a) {
     for (int i = t; i < TL_N; i += blockDim.x) dinv[i] = 1.0 / d[i];
     __syncthreads();
     float lmax = 0.f;
-    for (int j = warp; j < nt * 32; j += 32)
-        for (int i = lane; i < nt * 32; i += 32) {
+    for (int j = warp; j < nt * 32; j += TC_NW)
+        for (int i = lane; i <= j; i += 32) {
             const int ib = i >> 5, jb = j >> 5;
             if (ib > jb) continue;
             float v;
@@ -605,7 +615,7 @@ __global__ void __launch_bounds__(1024, 1) tl_chol_kernel(TlCholArgs a) {
         for (int e = t; e < nt * 32 * 32; e += blockDim.x) {
             const int kb = e >> 10, i = (e >> 5) & 31, j = e & 31;
             const float v = Tl[tc_idx(kb, kb) * TC_TILE + i * TC_LD + j];
-            XD[kb * TC_TILE + i * TC_LD + j] = i == j ? 1.0f : -v;
+            XD[kb * TC_TILE + i * TC_LD + j] = i == j ? 1.0f : (i < j ? -v : 0.f);
         }
         __syncthreads();
     } else {
@@ -632,7 +642,7 @@ __global__ void __launch_bounds__(1024, 1) tl_chol_kernel(TlCholArgs a) {
             __syncthreads();
             // trailing: S(ib, jb) -= R(kb, ib)^T R(kb, jb), kb < ib <= jb
             const int ntr = np * (np + 1) / 2;
-            for (int q = task; q < ntr; q += 16) {
+            for (int q = task; q < ntr; q += TC_TASKS) {
                 int jj = 0;
                 while ((jj + 1) * (jj + 2) / 2 <= q) ++jj;
                 const int ii = q - jj * (jj + 1) / 2;
@@ -657,7 +667,7 @@ __global__ void __launch_bounds__(1024, 1) tl_chol_kernel(TlCholArgs a) {
     }
     // R = R^ D (memory units), ||R^||_F^2
     double fr = 0.0;
-    for (int j = warp; j < n; j += 32) {
+    for (int j = warp; j < n; j += TC_NW) {
         const double dj = d[j] / a.sig_g;
         for (int i = lane; i < n; i += 32) {
             float v = 0.f;
@@ -710,7 +720,7 @@ __global__ void __launch_bounds__(1024, 1) tl_chol_kernel(TlCholArgs a) {
     // ||X||_F^2, max |X|
     double fx = 0.0;
     float mx = 0.f;
-    for (int j = warp; j < n; j += 32)
+    for (int j = warp; j < n; j += TC_NW)
         for (int i = lane; i <= j; i += 32) {
             const float v = Tl[tc_idx(i >> 5, j >> 5) * TC_TILE + (i & 31) * TC_LD + (j & 31)];
             fx += (double)v * v;
@@ -729,7 +739,7 @@ __global__ void __launch_bounds__(1024, 1) tl_chol_kernel(TlCholArgs a) {
     }
     __syncthreads();
     if (t < 32) {
-        double a0 = red[0][t], a1 = red[1][t], m0 = red[2][t];
+        double a0 = t < TC_NW ? red[0][t] : 0.0, a1 = t < TC_NW ? red[1][t] : 0.0, m0 = t < TC_NW ? red[2][t] : 0.0;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             a0 += __shfl_xor_sync(0xffffffffu, a0, o);
@@ -1037,7 +1047,7 @@ cudaError_t launch_tall_chol_apply(float* X, int64_t ldx, int64_t m, int n, cons
     if ((e = cudaMemsetAsync(t.flag, 0, sizeof(int), st))) return e;
     TlCholArgs c{G, n, sig_g, sig_a, bf16 ? 0 : 1, kappa_max, R, ldr, t.rinv, t.cscale, t.escale, t.flag, t.kout};
     if ((e = ensure_smem_attr((const void*)tl_chol_kernel, TL_CHOL_SMEM))) return e;
-    RG_LAUNCH(tl_chol_kernel, 1, 1024, TL_CHOL_SMEM, st, c);
+    RG_LAUNCH(tl_chol_kernel, 1, TC_THREADS, TL_CHOL_SMEM, st, c);
     const int64_t ntiles = (m + 127) / 128;
     const int grid = (int)std::min<int64_t>(dev_sms(), std::max<int64_t>(ntiles, 1));
     TlApplyArgs a{X, ldx, m, n, ((reinterpret_cast<uintptr_t>(X) & 15) == 0 && (ldx & 3) == 0) ? 1 : 0,
