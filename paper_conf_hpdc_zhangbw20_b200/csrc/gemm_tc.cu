@@ -81,6 +81,8 @@ struct GemmArgs {
     int h0;                // K2 only: 16-bit image written for columns >= h0 only
     int c_ef;              // K2 TMA epilogue: C read / written with the L2 evict_first policy (streamed
                            // once; keeps the next leaf's code and operands resident)
+    int mc;                // K2: cluster pair along M sharing the B tile (TMA multicast of its halves);
+                           // units are pair units, CTA rank blockIdx.x & 1 takes row block 2 (u / tiles_j) + rank
 };
 
 __device__ __forceinline__ uint16_t f2h_bits(float x, int bf16) {
@@ -113,7 +115,7 @@ __device__ __forceinline__ void unit_coords(const GemmArgs& a, int u, int& t0, i
         kb1 = min(kb0 + a.kb_per_split, a.kb_total);
     } else {
         z = 0;
-        t0 = (u / a.tiles_j) * kBM;
+        t0 = (a.mc ? 2 * (u / a.tiles_j) + (int)(blockIdx.x & 1) : u / a.tiles_j) * kBM;
         tj = u % a.tiles_j;
         kb0 = 0;
         kb1 = a.kb_h;
@@ -178,7 +180,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
         }
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(&full_bar[s], 1);
-            mbar_init(&empty_bar[s], 1);
+            mbar_init(&empty_bar[s], args.mc ? 2 : 1);   // both CTAs of a pair read every B stage
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(&tfull_bar[a], 1);
@@ -199,13 +201,16 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
+    if (args.mc) cluster_sync_all();   // the peer's barriers are initialised before any multicast
     RG_PDL_ENTRY();   // prologue above overlaps the previous kernel's tail
+    const int ubeg = args.mc ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+    const int ustep = args.mc ? (int)(gridDim.x >> 1) : (int)gridDim.x;
 
     if (warp == 0) {
         if (elect_one()) {
             // ---------------- TMA producer
             int it = 0;
-            for (int u = blockIdx.x; u < args.units; u += gridDim.x) {
+            for (int u = ubeg; u < args.units; u += ustep) {
                 int t0, tj, z, kb0, kb1;
                 unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
                 const int t1 = tj * BN;
@@ -227,7 +232,13 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
                         // MN-major A: two 64(row) x 64(k) boxes, the second at +8 KB (LBO)
                         tma_load_2d(sa, &tmA, &full_bar[s], t0, kb * kBK);
                         tma_load_2d(sa + C::kABytes / 2, &tmA, &full_bar[s], t0 + 64, kb * kBK);
-                        tma_load_2d(sb, &tmB, &full_bar[s], kb * kBK, t1);
+                        if (!SPLIT && args.mc) {   // this CTA's half of the B tile, into both CTAs of the pair
+                            const int rk = (int)(blockIdx.x & 1);
+                            tma_load_2d_mc(sb + rk * (C::kBBytes / 2), &tmB_lo, &full_bar[s], kb * kBK,
+                                           t1 + rk * (BN / 2), (uint16_t)3);
+                        } else {
+                            tma_load_2d(sb, &tmB, &full_bar[s], kb * kBK, t1);
+                        }
                         if (SPLIT) {
                             uint8_t* sal = sb + C::kBBytes;
                             tma_load_2d(sal, &tmA_lo, &full_bar[s], t0, kb * kBK);
@@ -244,7 +255,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
             // ---------------- MMA issuer (single thread)
             const uint32_t idesc = umma_idesc_f16(kBM, BN, MODE == 1 ? 1u : 0u, 0u, (uint32_t)args.bf16);
             int it = 0, cnt = 0;
-            for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+            for (int u = ubeg; u < args.units; u += ustep, ++cnt) {
                 int t0, tj, z, kb0, kb1;
                 unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
                 const int acc = cnt % C::kAcc;
@@ -280,7 +291,8 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
                             umma_f16(dtm + BN, adl, bd, idesc, 1u);      // lo * hi
                         }
                     }
-                    umma_commit(&empty_bar[s]);
+                    if (args.mc) umma_commit_mc(&empty_bar[s], (uint16_t)3);
+                    else umma_commit(&empty_bar[s]);
                 }
                 umma_commit(&tfull_bar[acc]);
             }
@@ -291,7 +303,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
             // ---------------- C producer: fp32 C chunks into the slot ring (chunk order = t)
             constexpr int kChunks = BN / 32;
             int cnt = 0;
-            for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+            for (int u = ubeg; u < args.units; u += ustep, ++cnt) {
                 int t0, tj, z, kb0, kb1;
                 unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
                 for (int ch = 0; ch < kChunks; ++ch) {
@@ -318,7 +330,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
             // ---------------- C store issuer: slot -> global (fp32 + 16-bit image), recycle
             constexpr int kChunks = BN / 32;
             int cnt = 0, prev = -1;
-            for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+            for (int u = ubeg; u < args.units; u += ustep, ++cnt) {
                 int t0, tj, z, kb0, kb1;
                 unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
                 for (int ch = 0; ch < kChunks; ++ch) {
@@ -348,7 +360,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
         const uint32_t lane_off = static_cast<uint32_t>(ew * 32) << 16;
         const bool hv = args.Ch != nullptr;
         int cnt = 0;
-        for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+        for (int u = ubeg; u < args.units; u += ustep, ++cnt) {
             int t0, tj, z, kb0, kb1;
             unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
             const int64_t row = (int64_t)t0 + ew * 32 + lane;
@@ -430,12 +442,12 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
             }
         };
         float4 old[8], nxt[8];
-        if (kAhead && rmw && blockIdx.x < args.units && wg < kChunks) {
+        if (kAhead && rmw && ubeg < args.units && wg < kChunks) {
             int t0, tj, z, kb0, kb1;
-            unit_coords<MODE>(args, blockIdx.x, t0, tj, z, kb0, kb1);
+            unit_coords<MODE>(args, ubeg, t0, tj, z, kb0, kb1);
             load_old(t0, tj * BN, wg, old);
         }
-        for (int u = blockIdx.x; u < args.units; u += gridDim.x, ++cnt) {
+        for (int u = ubeg; u < args.units; u += ustep, ++cnt) {
             int t0, tj, z, kb0, kb1;
             unit_coords<MODE>(args, u, t0, tj, z, kb0, kb1);
             const int t1 = tj * BN;
@@ -449,9 +461,9 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
                 if (kAhead && rmw) {
                     if (ch + EPI_WG < kChunks) {
                         load_old(t0, t1, ch + EPI_WG, nxt);
-                    } else if (u + (int)gridDim.x < args.units) {
+                    } else if (u + ustep < args.units) {
                         int t0n, tjn, zn, kb0n, kb1n;
-                        unit_coords<MODE>(args, u + gridDim.x, t0n, tjn, zn, kb0n, kb1n);
+                        unit_coords<MODE>(args, u + ustep, t0n, tjn, zn, kb0n, kb1n);
                         load_old(t0n, tjn * BN, wg, nxt);
                     }
                 }
@@ -548,6 +560,7 @@ __global__ void __launch_bounds__(GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>::kThrea
 
     tc_fence_before();
     __syncthreads();
+    if (args.mc) cluster_sync_all();   // no CTA exits while its peer may still signal its barriers
     if (warp == 2) tmem_dealloc<C::kTmemCols>(tmem_base);
 }
 
@@ -746,13 +759,54 @@ static cudaError_t launch_gemm(int units, const CUtensorMap& a, const CUtensorMa
     return cudaGetLastError();
 }
 
+// K2 on cluster pairs (args.mc): the two CTAs of a cluster take vertically adjacent 128-row tiles
+// with the same B tile, each loads one half of B (bh: box 64 k x BN / 2 rows) and multicasts it to
+// both, so the B operand -- the L2 traffic that bounds the wide top-level K2 (each R12 tile is
+// re-read for every row tile) -- is fetched once per pair.  Persistent grid of pairs.
+template <int MODE, int BN, int STAGES, bool SPLIT, int EPI_WG, int TE = 0>
+static cudaError_t launch_gemm_pair(int units, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& bh,
+                                    const GemmArgs& args, cudaStream_t st, const CUtensorMap* mc) {
+    using C = GemmCfg<BN, STAGES, SPLIT, EPI_WG, TE>;
+    auto kern = gemm_tc_kernel<MODE, BN, STAGES, SPLIT, EPI_WG, TE>;
+    {
+        cudaError_t e = ensure_smem_attr(reinterpret_cast<const void*>(kern), C::kTotal);
+        if (e != cudaSuccess) return e;
+    }
+    int grid = num_sms() & ~1;
+    if (grid > 2 * units) grid = 2 * units;
+    ++g_launches;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(C::kThreads);
+    cfg.dynamicSmemBytes = C::kTotal;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, a, b, a, bh, mc ? *mc : a, args);
+    return e != cudaSuccess ? e : cudaGetLastError();
+}
+
 // K2 with the TMA epilogue.  Shared memory (<= 227 KB) is split between the operand ring and
 // the C-chunk ring (16 KB per slot): the HBM-bound levels (few k-blocks per tile) trade operand
 // stages for C chunks in flight, the tensor-bound top level (K = 2048) keeps three stages.
 static cudaError_t dispatch_bn_te(int bn, int units, const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& args,
-                                  cudaStream_t st, const CUtensorMap* mc) {
+                                  cudaStream_t st, const CUtensorMap* mc, const CUtensorMap* bh) {
     static const int deep_kb = getenv("RGSQR_K2_DEEP_KB") ? atoi(getenv("RGSQR_K2_DEEP_KB")) : 8;
+    static const bool pair_off = getenv("RGSQR_K2_PAIR") && getenv("RGSQR_K2_PAIR")[0] == '0';
     const bool deep = args.kb_h <= deep_kb;
+    static const int pair_min_kb = getenv("RGSQR_K2_PAIR_KB") ? atoi(getenv("RGSQR_K2_PAIR_KB")) : 9;
+    if (bn == 256 && args.kb_h >= pair_min_kb && bh && !pair_off && args.tiles_i % 2 == 0) {
+        GemmArgs pa = args;
+        pa.mc = 1;
+        pa.units = (args.tiles_i / 2) * args.tiles_j;
+        if (deep) return launch_gemm_pair<1, 256, 2, false, 2, 8>(pa.units, a, b, *bh, pa, st, mc);
+        return launch_gemm_pair<1, 256, 3, false, 2, 4>(pa.units, a, b, *bh, pa, st, mc);
+    }
     switch (bn) {
         case 32: return launch_gemm<1, 32, 3, false, 2, 8>(units, a, b, a, b, args, st, mc);
         case 64: return launch_gemm<1, 64, 2, false, 2, 10>(units, a, b, a, b, args, st, mc);
@@ -825,7 +879,7 @@ cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, cons
     args.vec_ok = ((ldc & 3) == 0) && ((reinterpret_cast<uintptr_t>(C) & 15) == 0) && ((ldh & 3) == 0) &&
                   ((reinterpret_cast<uintptr_t>(Ch) & 7) == 0) && ((reinterpret_cast<uintptr_t>(Cl) & 7) == 0);
     if (!split && mc && !Cl && !getenv("RGSQR_NO_TMA_EPI"))
-        return dispatch_bn_te(bn, args.units, q1_mn, r12, args, st, mc);
+        return dispatch_bn_te(bn, args.units, q1_mn, r12, args, st, mc, &r12_lo);
     return split ? dispatch_bn<1, true>(bn, args.units, q1_mn, r12, q1_mn_lo, r12_lo, args, st)
                  : dispatch_bn<1, false>(bn, args.units, q1_mn, r12, q1_mn, r12, args, st);
 }

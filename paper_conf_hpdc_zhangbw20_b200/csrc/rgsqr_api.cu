@@ -675,7 +675,8 @@ int make_plan(rg_handle h, Plan& pl) {
             bool ok = encode_map(&o.ma, q1, m, o.h, pl.ldh, 64, 64, bf) &&
                       encode_map(&o.mb, r12h, o.h, o.w, pl.ldr12, 64, o.bn, bf) &&
                       encode_map(&o.ma_lo, q1l, m, o.h, pl.ldh, 64, 64, bf) &&
-                      encode_map(&o.mb_lo, pl.split ? r12l : r12h, o.h, o.w, pl.ldr12, 64, o.bn, bf);
+                      // non-split: the lo slot carries the half-width B box of the cluster-pair K2
+                      encode_map(&o.mb_lo, pl.split ? r12l : r12h, o.h, o.w, pl.ldr12, 64, pl.split ? o.bn : std::max(8, o.bn / 2), bf);
             if (!ok) return RG_CUDA_ERROR;
         }
     }
