@@ -1190,7 +1190,7 @@ int tall_gram(rg_handle h, int64_t m, int n, const float* X, int64_t ldx, bool f
     if (!h->tallws.ensure(rg::tall_ws_bytes())) return RG_ALLOC;
     double* G = rg::tall_gram_buffer(h->tallws.p);
     CUtensorMap tm;
-    const bool tma = ensure_encode() && encode_plain(&tm, X, m, n, ldx, 4, false, 32, 256);
+    const bool tma = ensure_encode() && encode_plain(&tm, X, m, n, ldx, 4, false, 64, 128);
     RG_CUDA(rg::launch_tall_gram(X, ldx, m, n, first ? 1.0f : kTallSig, first ? 1 : 0, h->tallws.p, G, h->stream,
                                  tma ? &tm : nullptr));
     if (getenv("RGSQR_TALL_DEBUG")) {   // tensor-core diagonal against the fp64 column sums

@@ -40,7 +40,9 @@ constexpr int TL_THREADS = 128 + 32 * TL_CW;
 constexpr int TL_GSTAGES = 3;
 constexpr int TL_GSTAGE = 2 * TL_N * 128;    // hi + lo tiles of one Gram stage (64 rows x 256 cols)
 constexpr int TL_GACC = 384;                 // TMEM columns: D0 (128 x 256) + D1 (128 x 128)
-constexpr int TL_PART = TL_GACC * 128;       // fp32 per CTA partial
+constexpr int TL_PART = TL_GACC * 128;       // fp32 per CTA partial (three-product Gram: D0 | D1)
+constexpr int TL_PART2 = 512 * 128;          // two-product Gram: full 256 x 256 D = H (H + 2L)^T
+constexpr int TL_PMAX = TL_PART2;
 constexpr int TL_ASTAGES = 2;
 constexpr int TL_ASTAGE = 2 * 64 * 256;      // hi + lo of one apply k-block (128 rows x 64 cols)
 constexpr int TL_BBYTES = (256 + 192 + 128 + 64) * 128;   // one of hi / lo of the resident R^-1 tiles
@@ -69,11 +71,13 @@ __device__ __forceinline__ float4 tl_lds128(uint32_t addr) {
 }
 // 4 consecutive rows (one float4, already scaled) -> 8 bytes of hi at shared address hi_addr and
 // of lo at lo_addr (swizzled by the caller)
-template <bool BF>
+// (LS: lo scale, 1 or 2 -- a power of two, so rn16(LS (x - hi)) = LS rn16(x - hi) exactly)
+template <bool BF, int LS = 1>
 __device__ __forceinline__ void tl_split_sts(float4 v, uint32_t hi_addr, uint32_t lo_addr) {
     const uint32_t h0 = tl_pack(v.x, v.y, BF), h1 = tl_pack(v.z, v.w, BF);
     const float2 a = tl_unpack(h0, BF), b = tl_unpack(h1, BF);
-    const uint32_t l0 = tl_pack(v.x - a.x, v.y - a.y, BF), l1 = tl_pack(v.z - b.x, v.w - b.y, BF);
+    const float ls = (float)LS;
+    const uint32_t l0 = tl_pack(ls * (v.x - a.x), ls * (v.y - a.y), BF), l1 = tl_pack(ls * (v.z - b.x), ls * (v.w - b.y), BF);
     tl_sts64(hi_addr, h0, h1);
     tl_sts64(lo_addr, l0, l1);
 }
@@ -240,9 +244,11 @@ __global__ void __launch_bounds__(TL_THREADS, 1) tl_gram_kernel(TlGramArgs a) {
     if (warp == 1) tmem_dealloc<512>(tmem);
 }
 
-// TMA-fed variant (16-byte aligned X and ldx): a producer warp streams 32-row x 256-column fp32
-// half-chunks of X into a ring of three 32 KB staging slots (HBM stays busy while the converters
-// work), the 8 converter warps split them from shared memory into the two operand stages.
+// TMA-fed variant (16-byte aligned X and ldx): a producer warp streams 64-row x 128-column fp32
+// half-chunks of X (256 contiguous bytes per column: 32-row boxes cap HBM reads at ~4.7 TB/s,
+// tools/colread_probe.cu) into a ring of three 32 KB staging slots, 16 converter warps split them
+// from shared memory into the two operand stages.  Two split products, D = H (H + 2L)^T over the
+// full 256 x 256 (512 TMEM columns); G = (D + D^T) / 2 = H H^T + H L^T + L H^T after the reduction.
 constexpr int TL_TSLOTS = 3;
 constexpr int TL_TSLOT = 32 * TL_N * 4;
 constexpr int TL_TSTAGES = 2;
@@ -288,8 +294,9 @@ __global__ void __launch_bounds__(TL_TTHREADS, 1) tl_gram_tma_kernel(const __gri
 
     if (warp == 0) {
         if (elect_one()) {
+            // D0 = rows 0..127, D1 = rows 128..255 of D = H H^T + H (2L)^T (all 256 columns; the
+            // symmetric part of D is G, formed after the reduction)
             const uint32_t id256 = umma_idesc_f16(128, 256, 0, 0, BF ? 1u : 0u);
-            const uint32_t id128 = umma_idesc_f16(128, 128, 0, 0, BF ? 1u : 0u);
             for (int it = 0; it < my; ++it) {
                 const int s = it % TL_TSTAGES;
                 mbar_wait(&full_bar[s], (uint32_t)(it / TL_TSTAGES) & 1u);
@@ -302,13 +309,10 @@ __global__ void __launch_bounds__(TL_TTHREADS, 1) tl_gram_tma_kernel(const __gri
                     const uint64_t h0 = umma_desc_sw128(hi + kk * 32, 16, 1024);
                     const uint64_t l0 = umma_desc_sw128(lo + kk * 32, 16, 1024);
                     const uint64_t h1 = umma_desc_sw128(hi + 128 * 128 + kk * 32, 16, 1024);
-                    const uint64_t l1 = umma_desc_sw128(lo + 128 * 128 + kk * 32, 16, 1024);
                     umma_f16(tmem, h0, h0, id256, acc);
                     umma_f16(tmem, h0, l0, id256, 1u);
-                    umma_f16(tmem, l0, h0, id256, 1u);
-                    umma_f16(tmem + 256, h1, h1, id128, acc);
-                    umma_f16(tmem + 256, h1, l1, id128, 1u);
-                    umma_f16(tmem + 256, l1, h1, id128, 1u);
+                    umma_f16(tmem + 256, h1, h0, id256, acc);
+                    umma_f16(tmem + 256, h1, l0, id256, 1u);
                 }
                 umma_commit(&empty_bar[s]);
             }
@@ -322,23 +326,21 @@ __global__ void __launch_bounds__(TL_TTHREADS, 1) tl_gram_tma_kernel(const __gri
                 const int sl = q % TL_TSLOTS;
                 mbar_wait(&sempty[sl], ((uint32_t)(q / TL_TSLOTS) & 1u) ^ 1u);
                 mbar_arrive_expect_tx(&sfull[sl], TL_TSLOT);
-                const int64_t r0 = ((int64_t)blockIdx.x + (int64_t)(q >> 1) * gridDim.x) * 64 + 32 * (q & 1);
-                tma_load_2d(stg + sl * TL_TSLOT, &tmX, &sfull[sl], (int32_t)r0, 0);
+                const int64_t r0 = ((int64_t)blockIdx.x + (int64_t)(q >> 1) * gridDim.x) * 64;
+                tma_load_2d(stg + sl * TL_TSLOT, &tmX, &sfull[sl], (int32_t)r0, 128 * (q & 1));
             }
         }
         __syncwarp();
     } else if (warp >= 4) {
-        // ---------------- converters: warp cw takes 16 columns (4 per instruction), rows
-        // 4 (lane & 7) .. + 3 of the half-chunk; staging layout [column][32 rows] fp32
-        // columns of instruction k: {b, b + 4, b + 1, b + 5}[lane >> 3], b = 8 (k >> 1) + 2 (k & 1): the
-        // two half-lines of each pair (c, c + 4) cover all 32 banks (swizzle chunk ^ (c & 7))
-        const int cw = warp - 4, g8 = lane & 7;
-        const int qsel = lane >> 3;
-        const int coff = (qsel & 1) * 4 + (qsel >> 1);
-        double nrm[4];
-        float nf[4];
+        // ---------------- converters: half-chunk q = 64 rows x 128 columns (128 hf + c), staging layout
+        // [column][64 rows] (256 contiguous bytes per column: 64-row segments stream at ~6.4 TB/s,
+        // 32-row ones at ~4.7, tools/colread_probe.cu); a half-warp takes one column (4 rows per
+        // lane), warp cw the column pairs 2 (4 cw + k) + (lane >> 4), k < 4: full 128-byte lines
+        const int cw = warp - 4, g = lane & 15, hsel = lane >> 4;
+        double nrm[8];
+        float nf[8];
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
+        for (int k = 0; k < 8; ++k) {
             nrm[k] = 0.0;
             nf[k] = 0.f;
         }
@@ -352,47 +354,48 @@ __global__ void __launch_bounds__(TL_TTHREADS, 1) tl_gram_tma_kernel(const __gri
             float4 v[4];
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
-                const int c = 16 * cw + 8 * (k >> 1) + 2 * (k & 1) + coff;
-                v[k] = tl_lds128(src + (uint32_t)(c * 128 + 16 * g8));
+                const int cl = 2 * (4 * cw + k) + hsel;   // column within the half
+                v[k] = tl_lds128(src + (uint32_t)(cl * 256 + 16 * g));
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&sempty[sl]);
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
-                const int c = 16 * cw + 8 * (k >> 1) + 2 * (k & 1) + coff;
+                const int c = 128 * hf + 2 * (4 * cw + k) + hsel;
                 float4 x = v[k];
-                nf[k] = fmaf(x.x, x.x, fmaf(x.y, x.y, fmaf(x.z, x.z, fmaf(x.w, x.w, nf[k]))));
+                nf[4 * hf + k] = fmaf(x.x, x.x, fmaf(x.y, x.y, fmaf(x.z, x.z, fmaf(x.w, x.w, nf[4 * hf + k]))));
                 x.x *= a.sig; x.y *= a.sig; x.z *= a.sig; x.w *= a.sig;
-                const uint32_t off = tl_swz(c, 8 * hf + g8);
-                tl_split_sts<BF>(x, smem_u32(hi) + off, smem_u32(lo) + off);
+                const uint32_t off = tl_swz(c, g);
+                tl_split_sts<BF, 2>(x, smem_u32(hi) + off, smem_u32(lo) + off);
             }
             if (hf == 1) {
                 fence_proxy_async_smem();
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&full_bar[s]);
             }
-            if ((q & 31) == 31) {   // fp32 partial sums of <= 128 squares, then fp64
+            if ((q & 31) == 31) {   // fp32 partial sums of <= 64 squares, then fp64
 #pragma unroll
-                for (int k = 0; k < 4; ++k) {
+                for (int k = 0; k < 8; ++k) {
                     nrm[k] += (double)nf[k];
                     nf[k] = 0.f;
                 }
             }
         }
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
+        for (int k = 0; k < 8; ++k) {
             double x = nrm[k] + (double)nf[k];
 #pragma unroll
-            for (int o = 1; o < 8; o <<= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
-            if (g8 == 0) a.npart[(int64_t)blockIdx.x * TL_N + 16 * cw + 8 * (k >> 1) + 2 * (k & 1) + coff] = x * (double)a.sig * (double)a.sig;
+            for (int o = 1; o < 16; o <<= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+            const int c = 128 * (k >> 2) + 2 * (4 * cw + (k & 3)) + hsel;
+            if (g == 0) a.npart[(int64_t)blockIdx.x * TL_N + c] = x * (double)a.sig * (double)a.sig;
         }
         const int qd = warp & 3, part = cw >> 2;
-        float* P = a.part + (int64_t)blockIdx.x * TL_PART;
+        float* P = a.part + (int64_t)blockIdx.x * TL_PART2;
         if (my > 0) {
             mbar_wait(done_bar, 0);
             tc_fence_after();
         }
-        for (int ch = part; ch < TL_GACC / 32; ch += TL_TCW / 4) {
+        for (int ch = part; ch < 512 / 32; ch += TL_TCW / 4) {
             uint32_t r[32];
             if (my > 0) {
                 tmem_ld32(tmem + ((uint32_t)(32 * qd) << 16) + ch * 32, r);
@@ -443,6 +446,55 @@ __global__ void __launch_bounds__(256) tl_reduce_kernel(const float* __restrict_
         double s = 0.0;
         for (int b = 0; b < nb; ++b) s += npart[(int64_t)b * TL_N + c];
         G[c + (int64_t)c * n] = s;
+    }
+}
+
+// Two-product layout: D (fp64 sum over the CTAs, fixed order) into G (n x n, both triangles),
+// diagonal from the fp64 column sums; then tl_sym_kernel sets G_ij = G_ji = (D_ij + D_ji) / 2.
+__global__ void __launch_bounds__(256) tl_reduce2_kernel(const float* __restrict__ part, const double* __restrict__ npart,
+                                                          int nb, int n, double* G) {
+    RG_PDL_ENTRY();
+    const int e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e < TL_PART2) {
+        const int jp = e >> 7, i = e & 127;
+        const int row = jp < 256 ? i : 128 + i;
+        const int col = jp & 255;
+        if (row >= n || col >= n || row == col) return;
+        double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+        int b = 0;
+        for (; b + 4 <= nb; b += 4) {
+            s0 += (double)part[(int64_t)b * TL_PART2 + e];
+            s1 += (double)part[(int64_t)(b + 1) * TL_PART2 + e];
+            s2 += (double)part[(int64_t)(b + 2) * TL_PART2 + e];
+            s3 += (double)part[(int64_t)(b + 3) * TL_PART2 + e];
+        }
+        for (; b < nb; ++b) s0 += (double)part[(int64_t)b * TL_PART2 + e];
+        G[row + (int64_t)col * n] = (s0 + s1) + (s2 + s3);
+    } else if (e < TL_PART2 + TL_N) {
+        const int c = e - TL_PART2;
+        if (c >= n) return;
+        double s = 0.0;
+        for (int b = 0; b < nb; ++b) s += npart[(int64_t)b * TL_N + c];
+        G[c + (int64_t)c * n] = s;
+    }
+}
+// 32 x 32 tile pairs (upper tile (I, J) with its transpose (J, I)) through shared memory
+__global__ void __launch_bounds__(1024) tl_sym_kernel(double* G, int n) {
+    RG_PDL_ENTRY();
+    __shared__ double tu[32][33], tl[32][33];
+    const int I = blockIdx.x, J = blockIdx.y;
+    if (I > J) return;
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    const int r = 32 * I + tx, c = 32 * J + ty;          // upper tile element (r, c)
+    const int r2 = 32 * J + tx, c2 = 32 * I + ty;        // lower tile element (r2, c2)
+    tu[ty][tx] = (r < n && c < n) ? G[r + (int64_t)c * n] : 0.0;
+    tl[ty][tx] = (r2 < n && c2 < n) ? G[r2 + (int64_t)c2 * n] : 0.0;
+    __syncthreads();
+    // upper (r, c) with lower (c, r): lower (c, r) = tl at (row c = 32 J + ty, col r = 32 I + tx)
+    if (r < n && c < n && r != c) {
+        const double v = 0.5 * (tu[ty][tx] + tl[tx][ty]);
+        G[r + (int64_t)c * n] = v;
+        G[c + (int64_t)r * n] = v;
     }
 }
 
@@ -976,7 +1028,7 @@ cudaError_t launch_tall_orth(const double* G, int n, double sig, double* out, cu
 
 // ======================================================================= launchers
 size_t tall_ws_bytes() {
-    return (size_t)TL_MAX_GRID * TL_PART * 4 + (size_t)TL_MAX_GRID * TL_N * 8 + (size_t)TL_N * TL_N * 8 +
+    return (size_t)TL_MAX_GRID * TL_PMAX * 4 + (size_t)TL_MAX_GRID * TL_N * 8 + (size_t)TL_N * TL_N * 8 +
            (size_t)TL_N * TL_N * 4 + TL_N * 4 + 128 + 64 + TL_N * 8;
 }
 
@@ -985,7 +1037,7 @@ cudaError_t launch_tall_gram(const float* X, int64_t ldx, int64_t m, int n, floa
                              double* G, cudaStream_t st, const CUtensorMap* tmX) {
     uint8_t* w = reinterpret_cast<uint8_t*>(ws);
     float* part = reinterpret_cast<float*>(w);
-    double* npart = reinterpret_cast<double*>(w + (size_t)TL_MAX_GRID * TL_PART * 4);
+    double* npart = reinterpret_cast<double*>(w + (size_t)TL_MAX_GRID * TL_PMAX * 4);
     const int64_t nchunks = (m + 63) / 64;
     const int grid = (int)std::min<int64_t>(std::min(dev_sms(), TL_MAX_GRID), std::max<int64_t>(nchunks, 1));
     TlGramArgs a{X, ldx, m, n, sig, ((reinterpret_cast<uintptr_t>(X) & 15) == 0 && (ldx & 3) == 0) ? 1 : 0, part,
@@ -1006,8 +1058,13 @@ cudaError_t launch_tall_gram(const float* X, int64_t ldx, int64_t m, int n, floa
         if ((e = ensure_smem_attr((const void*)tl_gram_kernel<false>, TL_GRAM_SMEM))) return e;
         RG_LAUNCH((tl_gram_kernel<false>), grid, TL_THREADS, TL_GRAM_SMEM, st, a);
     }
-    RG_LAUNCH(tl_reduce_kernel, (TL_PART + TL_N + 255) / 256, 256, 0, st, part, npart, grid, n, G,
-              getenv("RGSQR_TALL_DEBUG") ? tall_dbg(ws) : nullptr);
+    if (tmX && !getenv("RGSQR_TALL_NO_TMA")) {
+        RG_LAUNCH(tl_reduce2_kernel, (TL_PART2 + TL_N + 255) / 256, 256, 0, st, part, npart, grid, n, G);
+        RG_LAUNCH(tl_sym_kernel, dim3((n + 31) / 32, (n + 31) / 32), 1024, 0, st, G, n);
+    } else {
+        RG_LAUNCH(tl_reduce_kernel, (TL_PART + TL_N + 255) / 256, 256, 0, st, part, npart, grid, n, G,
+                  getenv("RGSQR_TALL_DEBUG") ? tall_dbg(ws) : nullptr);
+    }
     return cudaGetLastError();
 }
 
@@ -1020,7 +1077,7 @@ struct TallTail {
     double* kout;
 };
 static TallTail tall_tail(void* ws) {
-    uint8_t* w = reinterpret_cast<uint8_t*>(ws) + (size_t)TL_MAX_GRID * TL_PART * 4 + (size_t)TL_MAX_GRID * TL_N * 8 +
+    uint8_t* w = reinterpret_cast<uint8_t*>(ws) + (size_t)TL_MAX_GRID * TL_PMAX * 4 + (size_t)TL_MAX_GRID * TL_N * 8 +
                  (size_t)TL_N * TL_N * 8;
     TallTail t;
     t.rinv = reinterpret_cast<float*>(w);
@@ -1031,7 +1088,7 @@ static TallTail tall_tail(void* ws) {
     return t;
 }
 double* tall_gram_buffer(void* ws) {
-    return reinterpret_cast<double*>(reinterpret_cast<uint8_t*>(ws) + (size_t)TL_MAX_GRID * TL_PART * 4 +
+    return reinterpret_cast<double*>(reinterpret_cast<uint8_t*>(ws) + (size_t)TL_MAX_GRID * TL_PMAX * 4 +
                                      (size_t)TL_MAX_GRID * TL_N * 8);
 }
 int* tall_flag(void* ws) { return tall_tail(ws).flag; }
