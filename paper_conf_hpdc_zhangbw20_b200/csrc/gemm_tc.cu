@@ -797,7 +797,7 @@ static cudaError_t launch_gemm_pair(int units, const CUtensorMap& a, const CUten
 static cudaError_t dispatch_bn_te(int bn, int units, const CUtensorMap& a, const CUtensorMap& b, const GemmArgs& args,
                                   cudaStream_t st, const CUtensorMap* mc, const CUtensorMap* bh) {
     static const int deep_kb = getenv("RGSQR_K2_DEEP_KB") ? atoi(getenv("RGSQR_K2_DEEP_KB")) : 8;
-    static const bool pair_off = getenv("RGSQR_K2_PAIR") && getenv("RGSQR_K2_PAIR")[0] == '0';
+    const bool pair_off = getenv("RGSQR_K2_PAIR") && getenv("RGSQR_K2_PAIR")[0] == '0';   // read per plan (tests toggle it)
     const bool deep = args.kb_h <= deep_kb;
     static const int pair_min_kb = getenv("RGSQR_K2_PAIR_KB") ? atoi(getenv("RGSQR_K2_PAIR_KB")) : 9;
     if (bn == 256 && args.kb_h >= pair_min_kb && bh && !pair_off && args.tiles_i % 2 == 0) {

@@ -348,3 +348,25 @@ def test_rgsqr_pinned_host_options(rg, kw):
     np.testing.assert_array_equal(Rh.numpy(), Rd.cpu().numpy())
     _check_qr(A, Qh.numpy().astype(np.float64), Rh.numpy().astype(np.float64), kappa=np.linalg.cond(A),
               orth_scale=5e-2 if kw.get("precision") == "bf16" or kw.get("scale") is False else 1e-2)
+
+
+def test_rgsqr_k2_cluster_pair_bit_identical(rg, monkeypatch):
+    """The cluster-pair K2 (two CTAs share the multicast B tile; levels with >= 9 k-blocks, i.e.
+    h >= 576) runs the same MMAs in the same order per tile as the single-CTA K2: Q and R are
+    bit-identical with it on (default) and off (RGSQR_K2_PAIR=0)."""
+    A = synth.gaussian(8192, 1536, seed=51).astype(np.float32)
+    out = {}
+    for pair in ("1", "0"):
+        monkeypatch.setenv("RGSQR_K2_PAIR", pair)
+        h = rg.Handle(0)
+        try:
+            Ad = _dev(A)
+            Q, R = rg.rgsqr_factor(Ad, handle=h)
+            torch.cuda.synchronize()
+            out[pair] = (Q.cpu().numpy(), R.cpu().numpy())
+        finally:
+            h.close()
+    np.testing.assert_array_equal(out["1"][0], out["0"][0])
+    np.testing.assert_array_equal(out["1"][1], out["0"][1])
+    Q, R = (x.astype(np.float64) for x in out["1"])
+    _check_qr(A, Q, R, kappa=np.linalg.cond(A))
