@@ -147,10 +147,17 @@ RG_API int rgsqr_factor(rg_handle h, int64_t m_local, int64_t n, const float* A,
  * A (m_local x n, lda) is overwritten by Q.  One RGSQR pass, then while the orthogonality
  * estimate ||I - Q^T Q||_F > orth_tol and passes < max_passes: [Q2, R2] = RGSQR(Q) with the
  * split-precision GEMMs (reading #9) and R <- R2 R ("twice is enough").
+ * Tall blocks (n <= 256, rows beyond the on-chip leaf, e.g. config 4; every rank must agree when
+ * row-sharded): each pass is one CholQR pass over the whole block on the tensor cores (reading
+ * #33: split-16-bit Gram with fp64 column norms, n x n Gram allreduce when row-sharded, Cholesky
+ * of the equilibrated Gram, in-place X <- X R^-1); a pass whose Cholesky fails or whose
+ * equilibrated kappa_F(R) exceeds 32 n leaves A untouched and runs the RGSQR pass instead
+ * (RGSQR_TALL=0 / 1 forces the path off / on).
  * R (n x n, ldr) receives the accumulated triangular factor if non-NULL.  passes_out: number
- * of RGSQR passes run; orth_est_out: final ||I - Q^T Q||_F, a Hutchinson estimate with 8 fixed
- * Gaussian probes (E||M g||^2 = ||M||_F^2; within a few % of the exact value).
- * orth_tol <= 0 means "run exactly max_passes passes".
+ * of passes run; orth_est_out: final ||I - Q^T Q||_F -- on the tall path computed exactly (in the
+ * split Gram's precision) from the Gram of Q, which is also the next pass's Gram; otherwise a
+ * Hutchinson estimate with 8 fixed Gaussian probes (E||M g||^2 = ||M||_F^2; within a few % of the
+ * exact value).  orth_tol <= 0 means "run exactly max_passes passes".
  * Errors: -2..-6 as above (A is arg 4, lda arg 5, R arg 6, ldr arg 7 (< n with R non-NULL)),
  * -9 max_passes < 1; RG_NOT_CONVERGED if the final estimate is above orth_tol > 0. */
 RG_API int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int64_t lda, float* R, int64_t ldr,
