@@ -68,7 +68,7 @@ typedef struct {
     int scale;      /* 1 = automatic power-of-two column scaling (default, section 3.5 P:L357-361,
                        reading #4); 0 = off */
     int reortho;    /* extra reorthogonalisation passes: for rgsqr_factor default 0; for
-                       ls_solve_refined -1 = default 1 (reading #8) */
+                       ls_solve_refined -1 = default: one split-precision pass, no reortho (reading #8) */
     int split;      /* 1 = 3 x 16-bit split-precision tensor-core GEMMs (reading #9), default 0;
                        orthogonalize always uses it for its refinement passes */
     int sync;       /* 1 (default) = synchronise at the end of the call and return breakdown /
@@ -164,7 +164,9 @@ RG_API int orthogonalize(rg_handle h, int64_t m_local, int64_t n, float* A, int6
                   double orth_tol, int max_passes, int* passes_out, double* orth_est_out, const rg_opts* opts);
 
 /* ---- ls_solve_refined: x = argmin ||A x - b||_2 (eq 1; b in R^m, reading #14) ----
- * RGSQR (+ opts->reortho passes, default 1, reading #8), then CGLS preconditioned on the
+ * QR preconditioner (reading #8): by default (opts->reortho = -1) one RGSQR pass with split-
+ * precision (3 x 16-bit) K1 / K2, whose R leaves kappa(A R^-1) ~ 1; opts->reortho >= 0 runs
+ * RGSQR + that many reortho passes in opts->split precision.  Then CGLS preconditioned on the
  * right by R (Algorithm 3 as corrected by reading #5): vectors, reductions and scalars in
  * fp64, A read as fp32 (reading #7).  Stops when ||s_k|| <= tol ||s_0|| (reading #6) or after
  * maxit iterations.  b: m_local fp32; x: n fp64 (replicated).  iters_out / relres_out

@@ -13,9 +13,9 @@ bd = torch.from_numpy(b32).cuda()
 Q, R = np.linalg.qr(A32.astype(np.float64))
 xs = np.linalg.solve(R, Q.T @ b32.astype(np.float64))
 h = rg.Handle(0)
-for reo in (1, 0):
-    for solver in ("cgls", "lsqr"):
-        o = rg.make_opts(reortho=reo, solver=solver)
+for reo, split in ((1, 0), (0, 1), (1, 1), (0, 0)):
+    for solver in ("cgls",):
+        o = rg.make_opts(reortho=reo, solver=solver, split=bool(split))
         x = torch.zeros(n, dtype=torch.float64, device="cuda")
         for _ in range(2):
             rg.ls_solve_refined(Ad, bd, x, handle=h, opts=o)
@@ -26,4 +26,4 @@ for reo in (1, 0):
             _, it, rel, st = rg.ls_solve_refined(Ad, bd, x, handle=h, opts=o)
             torch.cuda.synchronize(); ts.append(time.perf_counter() - t0)
         xv = x.cpu().numpy()
-        print(f"reortho={reo} {solver}: {min(ts)*1e3:.2f} ms iters {it} relres {rel:.2e} fe {np.linalg.norm(xv-xs)/np.linalg.norm(xs):.2e} st {st}", flush=True)
+        print(f"reortho={reo} split={split} {solver}: {min(ts)*1e3:.2f} ms iters {it} relres {rel:.2e} fe {np.linalg.norm(xv-xs)/np.linalg.norm(xs):.2e} st {st}", flush=True)
