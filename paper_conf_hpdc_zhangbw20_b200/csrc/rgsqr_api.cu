@@ -100,6 +100,13 @@ bool encode_plain(CUtensorMap* map, const void* base, int64_t inner, int64_t out
 }
 
 int pick_bn(int w) { return w <= 32 ? 32 : w <= 64 ? 64 : w <= 128 ? 128 : 256; }
+// general GEMMs (lowrank): N > 256 takes 192-wide tiles when they waste fewer columns (N = 528:
+// 3 x 192 = 576 instead of 3 x 256 = 768)
+int pick_bn_general(int N) {
+    if (N <= 256) return pick_bn(N);
+    const int t256 = (N + 255) / 256 * 256, t192 = (N + 191) / 192 * 192;
+    return t192 < t256 ? 192 : 256;
+}
 
 enum ProfClass { PC_UPDATE = 0, PC_PROJ = 1, PC_PANEL = 2, PC_SCALE = 3, PC_CGLS = 4, PC_OTHER = 5, PC_N = 6 };
 
@@ -1353,7 +1360,7 @@ int enqueue_lsqr_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int 
 // split: A_lo / B_lo images give ~fp32 accuracy (reading #9).
 int gemm_nn(rg_handle h, int64_t m, int N, int K, const uint16_t* Ah, const uint16_t* Al, int64_t lda16,
             const uint16_t* Bh, const uint16_t* Bl, int64_t ldb16, float* C, int64_t ldc, int bf16) {
-    const int bn = pick_bn(N);
+    const int bn = pick_bn_general(N);
     CUtensorMap ma, mb, mal, mbl;
     const bool split = Al && Bl;
     if (!encode_map(&ma, Ah, m, K, lda16, 64, 64, bf16) || !encode_map(&mb, Bh, K, N, ldb16, 64, bn, bf16) ||
@@ -1369,7 +1376,7 @@ int gemm_nn(rg_handle h, int64_t m, int N, int K, const uint16_t* Ah, const uint
 // layout ldb16): split-K over the K = m rows + deterministic reduction (K1 kernels).
 int gemm_tn(rg_handle h, int64_t K, int M, int N, const uint16_t* Ah, int64_t lda16, const uint16_t* Bh,
             int64_t ldb16, float* O, int64_t ldo, int bf16) {
-    const int bn = pick_bn(N);
+    const int bn = pick_bn_general(N);
     CUtensorMap ma, mb;
     if (!encode_map(&ma, Ah, K, M, lda16, 64, 128, bf16) || !encode_map(&mb, Bh, K, N, ldb16, 64, bn, bf16))
         return RG_CUDA_ERROR;
