@@ -1231,9 +1231,12 @@ int tall_orth(rg_handle h, int n, double* est) {
 int tall_chol_apply(rg_handle h, int64_t m, int n, float* X, int64_t ldx, float* Rp, int64_t ldrp, bool first,
                     bool* ok) {
     void* ws = h->tallws.p;
-    const float sig = first ? 1.0f : kTallSig;
-    RG_CUDA(rg::launch_tall_chol_apply(X, ldx, m, n, rg::tall_gram_buffer(ws), (double)sig, sig, first ? 1 : 0,
-                                       32.0 * n, Rp, ldrp, ws, h->stream));
+    // the Gram's scale (bf16 split at 1 on the first pass: the column norms are unknown before it);
+    // the apply always splits in fp16 at 2^14: X D^-1 has unit columns once the Gram gave D
+    const float sig_g = first ? 1.0f : kTallSig;
+    const int apply_bf16 = getenv("RGSQR_TALL_APPLY_BF16") ? (first ? 1 : 0) : 0;
+    RG_CUDA(rg::launch_tall_chol_apply(X, ldx, m, n, rg::tall_gram_buffer(ws), (double)sig_g,
+                                       apply_bf16 ? 1.0f : kTallSig, apply_bf16, 32.0 * n, Rp, ldrp, ws, h->stream));
     int flag = 0;
     RG_CUDA(cudaMemcpyAsync(&flag, rg::tall_flag(ws), sizeof(int), cudaMemcpyDeviceToHost, h->stream));
     RG_CUDA(cudaStreamSynchronize(h->stream));

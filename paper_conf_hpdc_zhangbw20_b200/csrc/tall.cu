@@ -14,9 +14,9 @@
 //
 // The 16-bit split (reading #9, reading #33): x = hi + lo with hi = rn16(s x), lo = rn16(s x - hi)
 // (unscaled lo, so all three products accumulate into ONE accumulator; the per-column or per-pass
-// power-of-two scale s keeps lo in the normal 16-bit range).  bf16 on the first pass (fp32
-// exponent range: no column scaling pass needed before the Gram), fp16 (22-bit split) on the
-// reorthogonalisation passes, whose input columns have unit norm.
+// power-of-two scale s keeps lo in the normal 16-bit range).  The first pass's Gram in bf16 (fp32
+// exponent range: no column scaling pass needed before it), every other Gram and every apply in
+// fp16 (22-bit split) at 2^14 on unit columns (the apply scales X by D^-1 from the Gram).
 //
 // fp32 X is read straight from HBM by 8 converter warps (16-byte loads, 64 rows of a column per
 // half-warp) that write the swizzled 128-byte lines of the UMMA operands (SWIZZLE_128B: K-major
