@@ -53,7 +53,7 @@ def test_tall_orthogonalize_parity(rg, tall_on, m, n, kind, kappa):
     orth = oracle.orthogonality(Q)
     be = oracle.backward_error(A64, Q, R)
     assert orth <= 1e-5, (orth, p, est)
-    assert be <= 1e-4, be            # bf16-split first pass: ~2^-17 per entry (reading #33)
+    assert be <= 5e-6, be            # fp16-split applies (2^-22 per entry, reading #33): measured <= 7e-7
     assert np.all(np.tril(R, -1) == 0) and np.all(np.diag(R) > 0)
     Qo, Ro, _ = oracle.householder(A64)
     k = np.linalg.cond(A64)
@@ -83,7 +83,7 @@ def test_tall_fixed_two_passes(rg, tall_on):
     assert p == 2
     orth = oracle.orthogonality(Q)
     assert orth <= 3e-6, orth
-    assert oracle.backward_error(A.astype(np.float64), Q, R) <= 1e-4
+    assert oracle.backward_error(A.astype(np.float64), Q, R) <= 5e-6
 
 
 def test_tall_matches_rgsqr_path(rg, monkeypatch):
@@ -130,7 +130,7 @@ def test_tall_dist_virtual_ranks(rg, tall_on, P):
     R = Rs[0].cpu().numpy().astype(np.float64)
     orth = oracle.orthogonality(Q)
     assert orth <= 1e-5
-    assert oracle.backward_error(A.astype(np.float64), Q, R) <= 1e-4
+    assert oracle.backward_error(A.astype(np.float64), Q, R) <= 5e-6
     Q1, R1, _, _ = _orth(rg, A)
     assert np.linalg.norm(R - R1) / np.linalg.norm(R1) <= 1e-5
     assert np.linalg.norm(Q - Q1) / np.linalg.norm(Q1) <= 1e-5
