@@ -251,10 +251,14 @@ __global__ void __launch_bounds__(BJ_THREADS, 1) svd_bj_round_kernel(BjArgs a) {
     for (int o = 16; o > 0; o >>= 1) off = fmax(off, __shfl_xor_sync(0xffffffffu, off, o));
     if (lane == 0) s_off[warp] = off;
     __syncthreads();
-    if (tid == 0 && cr == 0) {
-        double mx = 0.0;
-        for (int w = 0; w < BJ_NW; ++w) mx = fmax(mx, s_off[w]);
-        atomicMax(a.maxoff + a.sweep, (unsigned long long)__double_as_longlong(mx));
+    double pair_off = 0.0;
+    for (int w = 0; w < BJ_NW; ++w) pair_off = fmax(pair_off, s_off[w]);
+    if (tid == 0 && cr == 0) atomicMax(a.maxoff + a.sweep, (unsigned long long)__double_as_longlong(pair_off));
+    // threshold Jacobi: a pair already orthogonal to the sweep tolerance is left as it is (every CTA
+    // of the cluster reduced the same Gram, so the decision is uniform over the cluster)
+    if (pair_off < a.tol) {
+        cl.sync();   // no CTA leaves while a cluster peer may still read its shared memory
+        return;
     }
     // ---- 4. one cyclic Jacobi sweep on M (64 indices, 63 rounds of 32 disjoint rotations);
     // every CTA of the cluster computes the same U
