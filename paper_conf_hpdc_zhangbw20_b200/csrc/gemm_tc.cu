@@ -81,6 +81,7 @@ struct GemmArgs {
     int h0;                // K2 only: 16-bit image written for columns >= h0 only
     int c_ef;              // K2 TMA epilogue: C read / written with the L2 evict_first policy (streamed
                            // once; keeps the next leaf's code and operands resident)
+    int jfast;             // K1: units enumerate the N tiles fastest (A is the operand too large for L2)
     int mc;                // K2: cluster pair along M sharing the B tile (TMA multicast of its halves);
                            // units are pair units, CTA rank blockIdx.x & 1 takes row block 2 (u / tiles_j) + rank
 };
@@ -109,8 +110,13 @@ __device__ __forceinline__ void unit_coords(const GemmArgs& a, int u, int& t0, i
         const int tiles = a.tiles_i * a.tiles_j;
         z = u / tiles;
         const int rem = u % tiles;
-        t0 = (rem % a.tiles_i) * kBM;
-        tj = rem / a.tiles_i;
+        if (a.jfast) {   // N tiles fastest: the concurrent CTAs share one A tile (read once from HBM)
+            t0 = (rem / a.tiles_j) * kBM;
+            tj = rem % a.tiles_j;
+        } else {          // M tiles fastest: the concurrent CTAs share one B tile
+            t0 = (rem % a.tiles_i) * kBM;
+            tj = rem / a.tiles_i;
+        }
         kb0 = z * a.kb_per_split;
         kb1 = min(kb0 + a.kb_per_split, a.kb_total);
     } else {
@@ -843,8 +849,9 @@ static cudaError_t dispatch_bn(int bn, int units, const CUtensorMap& a, const CU
 cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int splits, const CUtensorMap& q1,
                              const CUtensorMap& a2, const CUtensorMap& q1_lo, const CUtensorMap& a2_lo, float* P,
                              int64_t ldp, int64_t p_stride, int kb_total, int kb_per_split, int bf16,
-                             cudaStream_t st) {
+                             cudaStream_t st, int jfast) {
     GemmArgs args{};
+    args.jfast = jfast;
     args.units = tiles_i * tiles_j * splits;
     args.tiles_i = tiles_i;
     args.tiles_j = tiles_j;

@@ -166,7 +166,7 @@ cudaError_t launch_leaf(const LeafLaunch& L, cudaStream_t st);
 cudaError_t launch_proj_gemm(int bn, bool split, int tiles_i, int tiles_j, int splits, const CUtensorMap& q1,
                              const CUtensorMap& a2, const CUtensorMap& q1_lo, const CUtensorMap& a2_lo, float* P,
                              int64_t ldp, int64_t p_stride, int kb_total, int kb_per_split, int bf16,
-                             cudaStream_t st);
+                             cudaStream_t st, int jfast = 0);
 cudaError_t launch_update_gemm(int bn, bool split, int64_t m, int w, int h, const CUtensorMap& q1_mn,
                                const CUtensorMap& r12, const CUtensorMap& q1_mn_lo, const CUtensorMap& r12_lo,
                                float* C, int64_t ldc, void* Ch, void* Cl, int64_t ldh, int bf16, cudaStream_t st,

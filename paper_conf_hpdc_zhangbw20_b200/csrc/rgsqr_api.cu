@@ -1393,8 +1393,10 @@ int gemm_tn(rg_handle h, int64_t K, int M, int N, const uint16_t* Ah, int64_t ld
     const int64_t pstride = ldp * tiles_j * bn;
     if (!h->P.ensure((size_t)splits * pstride * 4 + 4096)) return RG_ALLOC;
     float* P = h->P.as<float>();
+    // A (M = the rows of the output: e.g. lowrank's 32768 columns of A, 2 GB) is the operand too large
+    // for L2: units enumerate the N tiles fastest so each A tile is read from HBM once
     RG_CUDA(rg::launch_proj_gemm(bn, false, tiles_i, tiles_j, splits, ma, mb, ma, mb, P, ldp, pstride, kb_total, kps,
-                                 bf16, h->stream));
+                                 bf16, h->stream, 1));
     RG_CUDA(rg::launch_proj_reduce(P, ldp, pstride, splits, M, N, nullptr, 0, O, ldo, nullptr, nullptr, 0, bf16,
                                    h->stream));
     return RG_OK;
