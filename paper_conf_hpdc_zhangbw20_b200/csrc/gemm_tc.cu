@@ -839,7 +839,7 @@ static cudaError_t dispatch_bn(int bn, int units, const CUtensorMap& a, const CU
             else
             return launch_gemm<MODE, 256, SPLIT ? 2 : 4, SPLIT, 1>(units, a, b, al, bl, args, st);
         case 192:   // general GEMMs with N = 3 x 176 .. 3 x 192 (lowrank l = 528): 3 tiles instead of 2 full + 1 nearly empty
-            if constexpr (MODE == 1 && !SPLIT) return launch_gemm<MODE, 192, 3, SPLIT, 2>(units, a, b, al, bl, args, st);
+            if constexpr (MODE == 1 && !SPLIT) return launch_gemm<MODE, 192, 4, SPLIT, 2>(units, a, b, al, bl, args, st);
             else
             return launch_gemm<MODE, 192, SPLIT ? 2 : 4, SPLIT, 1>(units, a, b, al, bl, args, st);
         default: return cudaErrorInvalidValue;
