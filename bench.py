@@ -556,10 +556,11 @@ def bench_ls(rg, torch, h, pk):
     x_ref32 = np.linalg.lstsq(A.astype(np.float32).astype(np.float64), b.astype(np.float32).astype(np.float64),
                               rcond=None)[0]
     xv = x.cpu().numpy()
-    # roofline: k CGLS iterations x 8mn bytes at the copy bandwidth + the one
-    # split-precision RGSQR pass of the default preconditioner (reading #8: three 16-bit products
-    # per K1 / K2) at the sustained tensor peak
-    roof_ms = (it * 8.0 * LS_M * LS_N / (pk["hbm_gbs"] * 1e9)
+    # roofline: one read of A per CGLS iteration (the one-pass product, reading
+    # #24) plus the initial A^T b, at the copy bandwidth, + the one split-precision RGSQR pass of
+    # the default preconditioner (reading #8: three 16-bit products per K1 / K2) at the sustained
+    # tensor peak
+    roof_ms = ((it + 1) * 4.0 * LS_M * LS_N / (pk["hbm_gbs"] * 1e9)
                + 3 * qr_flops(LS_M, LS_N) / (pk["bf16_tflops_sustained"] * 1e12)) * 1e3
     # LSQR (NEXT-4) on the same problem and preconditioner
     ol = rg.make_opts(solver="lsqr")
@@ -576,7 +577,7 @@ def bench_ls(rg, torch, h, pk):
     return {"workload": f"LS {LS_M}x{LS_N} cond 1e4 geometric, b ~ N(0,1) (BASELINE config 3)", "ms": ms,
             "lsqr": lsqr,
             "roofline": {"roofline_ms": roof_ms, "frac": roof_ms / ms,
-                         "note": "iters x 8mn bytes (A read twice per CGLS iteration) at the copy bandwidth "
+                         "note": "(iters + 1) x 4mn bytes (A read once per CGLS iteration) at the copy bandwidth "
                                  "+ one split-precision RGSQR pass (3 x 16-bit products) at the sustained tensor peak"},
             "preconditioner": "one RGSQR pass with split-precision K1/K2, no reortho pass (reading #8)",
             "iters": it, "relres": rel, "status": status,

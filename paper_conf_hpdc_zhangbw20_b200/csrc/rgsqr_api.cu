@@ -350,6 +350,8 @@ struct rg_handle_s {
     const void* cgls_key[4] = {nullptr, nullptr, nullptr, nullptr};
     int64_t cgls_key_mn[3] = {0, 0, 0};
     int cgls_solver = -1;                           // solver the captured block was built for
+    bool cgls_one_pass = false;                     // this solve's CGLS product (reading #24)
+    bool cgls_graph_one_pass = false;               // product the captured block was built with
     DevBuf aux;                                     // misc (orthogonalize / lowrank)
     DevBuf tallws;                                  // tall CholQR pass (tall.cu)
     DevBuf vscratch;                                // virtual-rank collectives (rank 0 of a group)
@@ -1289,7 +1291,7 @@ int enqueue_cgls_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int 
     double* sqp = work + std::max({rg::gemv_n_work_doubles(m, n), rg::gemv_t_work_doubles(m, n),
                                    rg::gemv_nt_work_doubles(n) + (size_t)n});
     const double* done = sc + 6;
-    if (rg::gemv_nt_ok(A, lda, n)) {
+    if (h->cgls_one_pass) {
         // one pass over A per iteration: q = A t and w = A^T q together; A^T r by recurrence
         double* w = work + rg::gemv_nt_work_doubles(n);
         for (int k = 0; k < iters; ++k) {
@@ -2022,12 +2024,25 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     double* sv = s + 2 * n;
     double* r = sv + n;
     double* wk = r + 2 * m_local;
+    const bool lsqr = o.solver == 1;
+    // the one-pass CGLS product needs 16 B aligned columns; the ranks' shards may differ, so under
+    // dist every rank takes it only if all can (the two forms issue different allreduces)
+    h->cgls_one_pass = !lsqr && rg::gemv_nt_ok(dA, dlda, (int)n);
+    if (!lsqr && h->dist()) {
+        const double mine = h->cgls_one_pass ? 1.0 : 0.0;
+        RG_CUDA(cudaMemcpyAsync(sc + 10, &mine, sizeof(double), cudaMemcpyHostToDevice, h->stream));
+        rc = nccl_allreduce(h, sc + 10, 1, ncclFloat64);
+        if (rc) return rc;
+        double all = 0;
+        RG_CUDA(cudaMemcpyAsync(&all, sc + 10, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+        RG_CUDA(cudaStreamSynchronize(h->stream));
+        h->cgls_one_pass = all > h->nranks - 0.5;
+    }
     {
         double init[16] = {0};
         init[8] = tol;
         RG_CUDA(cudaMemcpyAsync(sc, init, sizeof(init), cudaMemcpyHostToDevice, h->stream));
     }
-    const bool lsqr = o.solver == 1;
     if (lsqr) {
         // LSQR start: u = b, beta_1 = |b|, p = R^-T A^T u, alpha_1 v_1 = p / beta_1, w = v, y = 0
         double* y = sc + 16;
@@ -2065,7 +2080,8 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
         if (use_graph && cnt == blk) {
             const bool same = h->cgls_exec && h->cgls_key[0] == dA && h->cgls_key[1] == base &&
                               h->cgls_key[2] == h->rinv.p && h->cgls_key_mn[0] == m_local && h->cgls_key_mn[1] == n &&
-                              h->cgls_key_mn[2] == dlda && h->cgls_solver == o.solver;
+                              h->cgls_key_mn[2] == dlda && h->cgls_solver == o.solver &&
+                              h->cgls_graph_one_pass == h->cgls_one_pass;
             if (!same) {
                 if (h->cgls_exec) cudaGraphExecDestroy(h->cgls_exec);
                 h->cgls_exec = nullptr;
@@ -2077,6 +2093,7 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
                 rc = lsqr ? enqueue_lsqr_iters(h, dA, dlda, m_local, (int)n, blk, base)
                           : enqueue_cgls_iters(h, dA, dlda, m_local, (int)n, blk, base);
                 h->cgls_solver = o.solver;
+                h->cgls_graph_one_pass = h->cgls_one_pass;
                 const long long captured = rg::g_launches - before;
                 rg::g_launches = before;
                 h->cgls_key_mn[2] = dlda;
