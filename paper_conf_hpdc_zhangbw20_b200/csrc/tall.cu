@@ -838,6 +838,7 @@ struct TlApplyArgs {
     const float* cscale;
     const float* escale;
     const int* flag;    // nonzero: the Cholesky failed, leave X untouched
+    int pf;             // L2 prefetch distance in the group's k-blocks (0: none)
 };
 
 // smem: B hi (TL_BBYTES) | B lo | TL_ASTAGES x (A hi 16 KB | A lo 16 KB) | cscale | barriers
@@ -938,9 +939,20 @@ __global__ void __launch_bounds__(TL_ATHREADS, 1) tl_apply_kernel(TlApplyArgs a)
         // the k-blocks it = 4 tt + kc with it % 2 == gr, so one group's loads are in flight while
         // the other converts.  Line L = 2 pp + (lane >> 4): row half L >> 6, column 64 kc + (L & 63).
         const int gr = (warp - 4) >> 3, cw = (warp - 4) & 7, g = lane & 15;
+        const int ti = 32 * cw + lane;   // 0..255 within the group
         for (int it = gr; it < 4 * my; it += 2) {
             const int tt = it >> 2, kc = it & 3;
             const int64_t t0 = ((int64_t)blockIdx.x + (int64_t)tt * gridDim.x) * 128;
+            // the group's k-block pf steps ahead into L2, one 128 B line per thread (no registers held:
+            // the register-staged loads alone keep ~64 KB per SM in flight; 1.31 -> 1.21 ms at config
+            // 4 for pf = 1..3, slower from 4 on; 32 B-sector granularity was slower)
+            if (a.pf > 0 && it + 2 * a.pf < 4 * my) {
+                const int itp = it + 2 * a.pf;
+                const int64_t tp = ((int64_t)blockIdx.x + (int64_t)(itp >> 2) * gridDim.x) * 128;
+                const int c = 64 * (itp & 3) + (ti >> 2);
+                const int64_t r = tp + 32 * (ti & 3);
+                if (c < a.n && r < a.m) asm volatile("prefetch.global.L2 [%0];" ::"l"(a.X + (int64_t)c * a.ldx + r));
+            }
             float4 v[8];
 #pragma unroll
             for (int p = 0; p < 8; ++p) {
@@ -1108,7 +1120,8 @@ cudaError_t launch_tall_chol_apply(float* X, int64_t ldx, int64_t m, int n, cons
     const int64_t ntiles = (m + 127) / 128;
     const int grid = (int)std::min<int64_t>(dev_sms(), std::max<int64_t>(ntiles, 1));
     TlApplyArgs a{X, ldx, m, n, ((reinterpret_cast<uintptr_t>(X) & 15) == 0 && (ldx & 3) == 0) ? 1 : 0,
-                  t.rinv, t.cscale, t.escale, t.flag};
+                  t.rinv, t.cscale, t.escale, t.flag, 2};
+    if (const char* s = getenv("RGSQR_TALL_PF")) a.pf = atoi(s);
     if (bf16) {
         if ((e = ensure_smem_attr((const void*)tl_apply_kernel<true>, TL_APPLY_SMEM))) return e;
         RG_LAUNCH((tl_apply_kernel<true>), grid, TL_ATHREADS, TL_APPLY_SMEM, st, a);
