@@ -137,6 +137,20 @@ def test_ls_one_pass_cgls_matches_two_pass(rg, monkeypatch, m, n, kappa):
     assert np.linalg.norm(x1 - x_star) / np.linalg.norm(x_star) <= 1e-5
 
 
+@pytest.mark.parametrize("m,n", [(60, 13), (64, 1), (100, 7), (1028, 64), (4100, 1000)])
+def test_ls_one_pass_cgls_edges(rg, m, n):
+    """Edge shapes of the one-pass product's 64-row blocks (reading #24): a single partial block,
+    one column, exact and ragged block counts, n near the kernel's 1024-column limit; every lda
+    a multiple of 4 so the one-pass form is the one taken."""
+    A = synth.svd_matrix(m, n, "geometric", 1e3, seed=71 + n).astype(np.float32)
+    b = synth.rhs(A.astype(np.float64), seed=71 + n, consistent=False).astype(np.float32)
+    x_star, _ = oracle.ls_qr(A.astype(np.float64), b.astype(np.float64))
+    x, it, rel, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), tol=1e-12, maxit=200)
+    assert st == rg.RG_OK, (st, it, rel)
+    xe = x.cpu().numpy()
+    assert np.linalg.norm(xe - x_star) / np.linalg.norm(x_star) <= 1e-5, it
+
+
 @pytest.mark.parametrize("kind,kappa", [("geometric", 1e2), ("geometric", 1e4), ("arithmetic", 1e4)])
 @pytest.mark.parametrize("consistent", [False, True])
 def test_ls_lsqr_parity(rg, kind, kappa, consistent):
