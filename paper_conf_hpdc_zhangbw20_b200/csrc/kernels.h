@@ -228,6 +228,7 @@ cudaError_t launch_cgls_xr(double* x, const double* t, double* r, const double* 
 cudaError_t launch_cgls_p(const double* s, double* p, int n, double* sc, int first, cudaStream_t st);
 // LSQR (right-preconditioned by R, same passes as CGLS): u = q - (alpha / beta) u, sc[1] = |u|^2
 cudaError_t launch_lsqr_u(double* u, const double* q, int64_t m, double* sc, double* sqp, cudaStream_t st);
+cudaError_t launch_lsqr_sv(double* sv, const double* w, int n, const double* sc, cudaStream_t st);
 cudaError_t launch_lsqr_step(const double* p, double* v, double* w, double* y, int n, double* sc, int first,
                              cudaStream_t st);
 cudaError_t launch_gaussian_philox(int64_t total, uint64_t seed, double* out64, float* out32, cudaStream_t st);

@@ -1341,19 +1341,31 @@ int enqueue_lsqr_iters(rg_handle h, const float* A, int64_t lda, int64_t m, int 
     double* u = p + n;
     double* q = u + m;
     double* work = q + m;
-    double* sqp = work + std::max(rg::gemv_n_work_doubles(m, n), rg::gemv_t_work_doubles(m, n));
+    double* wnt = work + rg::gemv_nt_work_doubles(n);   // one-pass: A^T q
+    double* sqp = work + std::max({rg::gemv_n_work_doubles(m, n), rg::gemv_t_work_doubles(m, n),
+                                   rg::gemv_nt_work_doubles(n) + (size_t)n});
     double* Rinv = h->rinv.as<double>();
     const double* done = sc + 6;
+    const bool one = h->cgls_one_pass;
     for (int k = 0; k < iters; ++k) {
-        ProfScope _s(h, PC_CGLS, 4.0 * m * n, 8.0 * m * n);
+        ProfScope _s(h, PC_CGLS, 4.0 * m * n, (one ? 4.0 : 8.0) * m * n);
         RG_CUDA(rg::launch_trmv(Rinv, n, v, t, 0, done, st));                       // t = R^-1 v
-        RG_CUDA(rg::launch_gemv_n(A, lda, m, n, t, q, work, done, st));            // q = A t = M v
+        if (one)   // q = A t and A^T q in one sweep of A (reading #24)
+            RG_CUDA(rg::launch_gemv_nt(A, lda, m, n, t, q, wnt, work, sc, st));
+        else
+            RG_CUDA(rg::launch_gemv_n(A, lda, m, n, t, q, work, done, st));        // q = A t = M v
         RG_CUDA(rg::launch_lsqr_u(u, q, m, sc, sqp, st));                          // u = q - alpha u, |u|^2
         int rc = nccl_allreduce(h, sc + 1, 1, ncclFloat64);
         if (rc) return rc;
-        RG_CUDA(rg::launch_gemv_t(A, lda, m, n, u, sv, work, done, st));           // A^T u
-        rc = nccl_allreduce(h, sv, n, ncclFloat64);
-        if (rc) return rc;
+        if (one) {
+            rc = nccl_allreduce(h, wnt, n, ncclFloat64);
+            if (rc) return rc;
+            RG_CUDA(rg::launch_lsqr_sv(sv, wnt, n, sc, st));                       // A^T u by recurrence
+        } else {
+            RG_CUDA(rg::launch_gemv_t(A, lda, m, n, u, sv, work, done, st));       // A^T u
+            rc = nccl_allreduce(h, sv, n, ncclFloat64);
+            if (rc) return rc;
+        }
         RG_CUDA(rg::launch_trmv(Rinv, n, sv, p, 1, done, st));                     // p = R^-T A^T u
         RG_CUDA(rg::launch_lsqr_step(p, v, w, y, n, sc, 0, st));                   // v, alpha, Givens, y, w
     }
@@ -2025,10 +2037,10 @@ int ls_solve_refined(rg_handle h, int64_t m_local, int64_t n, const float* A, in
     double* r = sv + n;
     double* wk = r + 2 * m_local;
     const bool lsqr = o.solver == 1;
-    // the one-pass CGLS product needs 16 B aligned columns; the ranks' shards may differ, so under
+    // the one-pass product (CGLS and LSQR) needs 16 B aligned columns; the ranks' shards may differ, so under
     // dist every rank takes it only if all can (the two forms issue different allreduces)
-    h->cgls_one_pass = !lsqr && rg::gemv_nt_ok(dA, dlda, (int)n);
-    if (!lsqr && h->dist()) {
+    h->cgls_one_pass = rg::gemv_nt_ok(dA, dlda, (int)n);
+    if (h->dist()) {
         const double mine = h->cgls_one_pass ? 1.0 : 0.0;
         RG_CUDA(cudaMemcpyAsync(sc + 10, &mine, sizeof(double), cudaMemcpyHostToDevice, h->stream));
         rc = nccl_allreduce(h, sc + 10, 1, ncclFloat64);

@@ -111,11 +111,12 @@ def test_orthogonalize_fixed_two_passes(rg):
     assert oracle.orthogonality(Q.cpu().numpy().astype(np.float64)) <= 1e-5
 
 
+@pytest.mark.parametrize("solver", ["cgls", "lsqr"])
 @pytest.mark.parametrize("m,n,kappa", [(16384, 512, 1e2), (16384, 512, 1e4), (12300, 1000, 1e4)])
-def test_ls_one_pass_cgls_matches_two_pass(rg, monkeypatch, m, n, kappa):
-    """The one-pass CGLS product (q = A t and A^T q in one sweep of A, A^T r by recurrence) and the
-    two-pass form (A^T r recomputed from r, RGSQR_CGLS_TWO_PASS=1) reach the same solution (reading #24).  12300 x 1000:
-    a ragged 64-row tail block and two columns per thread in the sweep."""
+def test_ls_one_pass_cgls_matches_two_pass(rg, monkeypatch, m, n, kappa, solver):
+    """The one-pass product (q = A t and A^T q in one sweep of A; A^T r, for LSQR A^T u, by
+    recurrence) and the two-pass form (recomputed from r / u, RGSQR_CGLS_TWO_PASS=1) reach the same
+    solution (reading #24).  12300 x 1000: a ragged 64-row tail block."""
     A = synth.svd_matrix(m, n, "geometric", kappa, seed=61).astype(np.float32)
     b = synth.rhs(A.astype(np.float64), seed=61, consistent=False).astype(np.float32)
     x_star, _ = oracle.ls_qr(A.astype(np.float64), b.astype(np.float64))
@@ -126,7 +127,8 @@ def test_ls_one_pass_cgls_matches_two_pass(rg, monkeypatch, m, n, kappa):
         else:
             monkeypatch.delenv("RGSQR_CGLS_TWO_PASS", raising=False)
         h = rg.Handle(0)   # fresh handle: its captured CGLS graph follows the current mode
-        x, it, rel, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), tol=1e-10, maxit=200, handle=h)
+        x, it, rel, st = rg.ls_solve_refined(_dev(A), torch.from_numpy(b).cuda(), tol=1e-10, maxit=200, handle=h,
+                                             opts=rg.make_opts(solver=solver))
         torch.cuda.synchronize()
         out.append((x.cpu().numpy(), it, rel, st))
         h.close()
