@@ -97,6 +97,18 @@ def test_tall_matches_rgsqr_path(rg, monkeypatch):
     assert np.linalg.norm(Q1 - Q2) / np.linalg.norm(Q2) <= 1e-3
 
 
+@pytest.mark.parametrize("pf", ["0", "1", "3"])
+def test_tall_apply_prefetch_bit_identical(rg, tall_on, monkeypatch, pf):
+    """The apply's L2 prefetch distance (RGSQR_TALL_PF, default 2) only moves data into L2 earlier:
+    Q and R are bit-identical for every distance, ragged row tail included."""
+    A = synth.gaussian(70001, 256, seed=47).astype(np.float32)
+    Q0, R0, _, _ = _orth(rg, A)
+    monkeypatch.setenv("RGSQR_TALL_PF", pf)
+    Q1, R1, _, _ = _orth(rg, A)
+    np.testing.assert_array_equal(Q1, Q0)
+    np.testing.assert_array_equal(R1, R0)
+
+
 @pytest.mark.parametrize("P", [2, 4])
 def test_tall_dist_virtual_ranks(rg, tall_on, P):
     """Row-sharded tall passes: the n x n Gram is the only exchange (allreduce through the virtual
